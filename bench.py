@@ -1,0 +1,349 @@
+"""Benchmark of the AM hot path (driver contract: one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl ours|reference]
+
+A step is one accessibility map -- the whole hot path (a1-a8 of SURVEY.md 8(a))
+for one pivot of the seeded 1 mm path over the resident voxel model.  Default
+workload: C3 (head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096
+orientations), the configuration BASELINE.json's metric is quoted on.
+For N > 1 (torchrun), every rank computes its own pivots of the toolpath batch
+(pivot sharding): no data-path collective, weak scaling.
+
+value = voxel.orientation tests / s = N_vox * m * n * maps / max-over-ranks time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "ms per accessibility map (27M voxels, 64×64 orientations) and voxel·orientation tests/s"
+UNIT = "voxel-orientation tests/s"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+
+    def __init__(self, device=0, period=0.005):
+        self.period = period
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            idx = device
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            if vis:
+                try:
+                    idx = int(vis.split(",")[device])
+                except ValueError:
+                    idx = device
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self._ok = True
+        except Exception:
+            pass
+
+    _REASONS = {
+        0x0000000000000008: "hw_slowdown", 0x0000000000000040: "hw_thermal_slowdown",
+        0x0000000000000020: "sw_thermal_slowdown", 0x0000000000000004: "sw_power_cap",
+        0x0000000000000080: "hw_power_brake_slowdown", 0x0000000000000002: "applications_clocks_setting",
+    }
+
+    def _run(self):
+        nv = self._nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                for bit, name in self._REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self._ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self._ok:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def _dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _scene(cfg_name):
+    import scenes
+    cfg = scenes.CONFIGS[cfg_name]
+    t = time.time()
+    C, H = cfg.leaves()
+    gen_s = time.time() - t
+    return cfg, C, H, gen_s
+
+
+def cpu_oracle_sample(cfg, C, H, pivot, seconds=12.0, seed=0, max_cells=None):
+    """Time the fp64 oracle (as it stands) on a bounded sample of one map's cells."""
+    import oracle
+    rng = np.random.default_rng(seed)
+    cells_all = rng.permutation(cfg.m * cfg.n)
+    done = 0
+    t0 = time.perf_counter()
+    used = 0
+    chunk = 8
+    while True:
+        cells = cells_all[done: done + chunk]
+        if len(cells) == 0:
+            break
+        _, used = oracle.am_states(C, H, cfg.tool, pivot, cfg.m, cfg.n, cells=cells, return_threads=True)
+        done += len(cells)
+        el = time.perf_counter() - t0
+        if el >= seconds or (max_cells and done >= max_cells):
+            break
+        chunk = min(256, chunk * 2)
+    el = time.perf_counter() - t0
+    return {"tests": float(len(H)) * done, "cells": done, "seconds": el, "threads": used}
+
+
+def run_reference(args):
+    ws, rank, _ = _dist_env()
+    if rank != 0:
+        return 0
+    cfg, C, H, _ = _scene(args.config)
+    piv = cfg.pivots(max(args.steps + args.warmup, 1))
+    # each step: the oracle on a bounded sample of that step's map (per-step budget)
+    per_step = max(1.0, args.ref_seconds / max(args.steps, 1))
+    for k in range(args.warmup):
+        cpu_oracle_sample(cfg, C, H, piv[k], seconds=0.2, seed=k, max_cells=8)
+    tests = 0.0
+    secs = 0.0
+    cells = 0
+    threads = 0
+    for k in range(args.steps):
+        r = cpu_oracle_sample(cfg, C, H, piv[args.warmup + k], seconds=per_step, seed=100 + k)
+        tests += r["tests"]
+        secs += r["seconds"]
+        cells += r["cells"]
+        threads = r["threads"]
+    value = tests / secs
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": _config_dict(cfg, len(H)),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                         "sample": f"{cells} cells of {args.steps} maps (seeded cells, pivots of the 1 mm path), "
+                                   f"every voxel per cell, fp64 clip-project-hull test with exact-safe shortcuts"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def _config_dict(cfg, N):
+    return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
+                        f"pivots on the {cfg.offset:g} mm path",
+            "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
+            "l2": f"inputs ({16 * N / 1e6:.0f} MB) {'exceed' if 16 * N > L2_BYTES else 'fit in'} L2 (126 MB); no flush",
+            "parallelism": "pivot-sharded (weak)"}
+
+
+def run_ours(args):
+    import torch
+    ws, rank, local = _dist_env()
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl")
+    dev = torch.device("cuda", local if ws > 1 else 0)
+    torch.cuda.set_device(dev)
+    import paper_conf_icpp_chenktkv19_b200 as am
+
+    cfg, C, H, gen_s = _scene(args.config)
+    N = len(H)
+    npiv = args.pivots
+    piv_all = cfg.pivots(npiv * ws)
+    piv = piv_all[rank::ws]  # pivot sharding: rank r takes pivots r, r + G, ...
+    ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
+    t0 = time.time()
+    ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
+    torch.cuda.synchronize(dev)
+    upload_s = time.time() - t0
+    stream = torch.cuda.Stream(dev)
+    out = torch.zeros((len(piv), ctx.words), dtype=torch.int32, device=dev)
+    # warm-up
+    for k in range(args.warmup):
+        ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
+    stream.synchronize()
+    # stats of one map (outside the timed region)
+    _, st = ctx.compute(piv[0], stats=True)
+    ctx.set_option(am.binding.OPT_KERNEL_TIMING, 1)
+    ctx.kernel_time()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    with ClockSampler(dev.index) as clk:
+        ev0.record(stream)
+        for k in range(args.steps):
+            ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
+        ev1.record(stream)
+        stream.synchronize()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    ms = ev0.elapsed_time(ev1)
+    kms, klaunch = ctx.kernel_time()
+    ctx.set_option(am.binding.OPT_KERNEL_TIMING, 0)
+    # e2e: the public API with HOST buffers (pivot in, packed AM out), synchronous per step
+    host_out = np.zeros(ctx.words, dtype=np.uint32)
+    for k in range(min(args.warmup, 3)):
+        ctx.compute(piv[k % len(piv)], out=host_out)
+    ke = max(1, min(args.steps, args.e2e_steps))
+    if dist:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for k in range(ke):
+        ctx.compute(piv[k % len(piv)], out=host_out)
+    e2e_s = time.perf_counter() - t0
+    t = torch.tensor([ms, e2e_s, kms / max(klaunch, 1)], dtype=torch.float64, device=dev)
+    if dist:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max, e2e_max, kavg_ms = t.tolist()
+    maps = args.steps * ws
+    tests_per_map = float(N) * cfg.m * cfg.n
+    value = tests_per_map * maps / (ms_max / 1e3)
+    e2e_value = tests_per_map * ke * ws / e2e_max
+    peak, peak_src = _peaks()
+    alg_bytes = 16.0 * N + cfg.m * cfg.n / 8.0
+    achieved = alg_bytes / (kavg_ms / 1e3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(prof):
+        try:
+            d = json.load(open(prof))
+            if d.get("config") == cfg.name and d.get("build") == _build_id():
+                traffic = d.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    baseline_ms = None
+    if args.baseline and rank == 0:
+        ctx.set_option(am.binding.OPT_BASELINE_REJECT, 1)
+        bo = torch.zeros(ctx.words, dtype=torch.int32, device=dev)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        ctx.compute_baseline(piv[0], out=bo, stream=stream)
+        e1.record(stream)
+        stream.synchronize()
+        baseline_ms = e0.elapsed_time(e1)
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        r = cpu_oracle_sample(cfg, C, H, piv[0], seconds=args.cpu_seconds)
+        cpu = {"value": r["tests"] / r["seconds"], "unit": UNIT, "cores": r["threads"], "kind": "oracle",
+               "sample": f"{r['cells']} seeded cells of one {cfg.name} map (pivot 0), every voxel per cell, "
+                         f"{r['seconds']:.1f} s"}
+    if rank == 0:
+        ncpu = os.cpu_count()
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": _config_dict(cfg, N),
+            "ms_per_am": ms_max / args.steps,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "aica_stream_kernel", "kernel_ms_avg": kavg_ms,
+                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12, "d2h_bytes_per_step": 4 * ctx.words,
+                    "ms_per_am": 1e3 * e2e_max / ke, "steps": ke,
+                    "note": "am_compute with a host pivot (12 B, passed in the launch) and a host AM buffer; "
+                            "synchronous per step; voxels resident (upload excluded, PAPER.md L313)"},
+            "gpu_launches": 2 * args.steps,
+            "clocks": clk.summary(),
+            "cpu_baseline": cpu,
+            "detail": {"stats_pivot0": st.__dict__, "upload_s": upload_s, "scene_gen_s": gen_s,
+                       "pivots_per_rank": len(piv), "baseline_ms_per_am": baseline_ms,
+                       "host_cpus": ncpu,
+                       "paper_context": "PAPER.md L32/L75: <18 ms per AM, 27M octree nodes x 4096 orientations, "
+                                        "GTX 1080(Ti); 'over 23x' vs PBox"},
+        }
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if dist:
+        dist.destroy_process_group()
+    return 0
+
+
+def _build_id():
+    lib = os.path.join(ROOT, "paper_conf_icpp_chenktkv19_b200", "libam.so")
+    try:
+        import hashlib
+        return hashlib.sha1(open(lib, "rb").read()).hexdigest()[:12]
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--pivots", type=int, default=64, help="pivots per rank (cycled over the steps)")
+    ap.add_argument("--e2e-steps", type=int, default=100)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--ref-seconds", type=float, default=60.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--baseline", action="store_true", help="also time am_compute_baseline once")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,163 @@
+/*
+ * am.h -- C ABI of the B200-native accessibility-map (AM) engine.
+ *
+ * One call computes the AM of one pivot: for every orientation (phi_i, gamma_j)
+ * of an m x n grid, whether the tool -- N_c coaxial closed solid cylinders fixed
+ * at the pivot -- collides with any of N voxels (axis-aligned cubes, centre +
+ * half size).  PAPER.md L86-88 (problem statement), L56/L60 (orientation grid
+ * and AM, Fig. 1-2), L311 (tool made of cylinders).  The method is AICA
+ * (section 3-4, Alg. 1): per voxel, the inaccessible cone of
+ * its inscribed sphere (radius h) is certainly blocked, everything outside the
+ * cone of its circumscribed sphere (sqrt(3) h) is certainly clear, and the exact
+ * cylinder-box test (CHECKBOX, L97) runs only in the band between the two.
+ *
+ * Conventions:
+ *   - lengths in any consistent unit (mm in every config);
+ *   - cylinder k spans axial [z_k, z_k + height_k] along the tool direction d,
+ *     z_0 = 0 at the pivot, z_{k+1} = z_k + height_k (reading G3/G4);
+ *   - cell (i, j): phi_i = (i + 1/2) pi / m measured from +z, gamma_j =
+ *     (j + 1/2) 2 pi / n measured from +x toward +y,
+ *     d = (sin phi cos gamma, sin phi sin gamma, cos phi)  (reading G1);
+ *   - AM layout: W = ceil(n / 32) uint32 words per row, row-major in i; cell
+ *     (i, j) is bit (j & 31) of word i * W + (j >> 5); LSB-first; padding bits
+ *     are 0; 1 = collision ("black", L60)  (reading G2).
+ *
+ * Exactness: every cell whose oracle state is robust (exact-test margin above
+ * 1e-5 rad) equals the exact definition; cells inside the 1e-5 rad
+ * band may take either value.
+ *
+ * Ownership: the library copies whatever it is given; caller buffers are never
+ * retained.  Errors: every int-returning call returns AM_OK (0) or a negative
+ * AM_E* code, and am_last_error() describes the last failure on that context.
+ * Threading: calls on one context are not thread-safe; use one context per
+ * device (per rank).  No call falls back to the CPU: a missing or failing GPU
+ * is reported as AM_ECUDA.
+ */
+#ifndef AM_H_
+#define AM_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct am_ctx am_ctx; /* opaque; owns all device memory of one context */
+
+/* One bounding cylinder of the tool, ordered from the pivot outward. */
+typedef struct {
+    float radius; /* > 0, finite */
+    float height; /* > 0, finite */
+} am_cylinder;
+
+/* Per-call counters of the AICA path (filled by am_compute when stats != NULL). */
+typedef struct {
+    int64_t voxels_streamed;   /* voxels read by the streaming kernel                          */
+    int64_t voxels_culled;     /* beyond the tool's reach rho_max (step a2)                      */
+    int64_t voxels_skipped;    /* cheap outer cone lies entirely in already-full rows (a5)      */
+    int64_t voxels_live;       /* voxels whose exact cones were computed and rasterised (a4-a5) */
+    int64_t rows_rasterised;   /* (voxel, phi-row) pairs rasterised                             */
+    int64_t band_pairs;        /* (voxel, cell) pairs queued in the ambiguous band (a6)         */
+    int64_t exact_tests;       /* exact cylinder-box tests actually run (CHECKBOX, L97)         */
+    int64_t exact_hits;        /* of which collided                                             */
+    int64_t queue_overflow;    /* band pairs resolved inline because the queue was full         */
+    int64_t early_exit;        /* 1 if the AM filled up and the stream stopped early (a7)       */
+} am_stats;
+
+enum {
+    AM_OK = 0,
+    AM_EINVAL = -1, /* invalid argument (see each call)                       */
+    AM_ENOMEM = -2, /* device or host allocation failed                       */
+    AM_ECUDA = -3,  /* CUDA runtime error (no device, launch failure, ...)    */
+    AM_ESTATE = -4  /* call out of order (e.g. compute before upload)         */
+};
+
+/* Tunables (am_set_option).  Defaults are chosen at am_create. */
+enum {
+    AM_OPT_GRID_CTAS = 1,        /* persistent CTAs of the streaming kernel (0 = SMs x occupancy) */
+    AM_OPT_REFRESH_TILES = 2,    /* tiles between shared-AM <-> global-AM merges (>= 1)          */
+    AM_OPT_MORTON_SORT = 3,      /* 1 = Morton-sort voxels at upload (default), 0 = keep order   */
+    AM_OPT_BASELINE_REJECT = 4,  /* 1 = baseline uses an exact-safe bounding-sphere reject        */
+    AM_OPT_BAND_QUEUE = 5,       /* capacity of the deferred band queue, in (voxel, cell) pairs  */
+    AM_OPT_KERNEL_TIMING = 6     /* 1 = bracket every streaming-kernel launch with CUDA events   */
+};
+
+/*
+ * Create a context on CUDA device `device` for the tool `tool[0..n_cyl)` and an
+ * m x n orientation grid.  AM_EINVAL unless 1 <= n_cyl <= 8, every radius and
+ * height is finite and > 0, 1 <= m <= 1024, 1 <= n <= 1024 and out != NULL.
+ * AM_ECUDA if the device cannot be used.  On success *out owns the context.
+ */
+int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_ctx** out);
+
+/*
+ * Upload the voxel model: N voxels with centres centers_xyz[3*N] (x, y, z
+ * interleaved) and half sizes half_sizes[N], both float32, on the host
+ * (src_is_device = 0) or on `device` (1).  Replaces any previous model.  The
+ * library may reorder voxels (Morton sort); the AM is order-independent.
+ * AM_EINVAL if N < 0, a pointer is NULL while N > 0, or any value is non-finite
+ * or a half size is <= 0.  N = 0 is legal (every AM is then all-zero).
+ * Synchronous: returns after the model is resident (upload time is excluded
+ * from AM timings).
+ */
+int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_sizes, int64_t N,
+                     int src_is_device);
+
+/*
+ * AICA accessibility map of one pivot (host array pivot[3], finite).
+ * am_out receives am_words_per_map(ctx) uint32 words in the layout above, in
+ * host memory (dst_is_device = 0; the call then synchronises the stream) or in
+ * device memory (1; the call is asynchronous on `cuda_stream`).  cuda_stream is
+ * a cudaStream_t (NULL = legacy default stream).  stats, if non-NULL, is filled
+ * (this synchronises the stream).  AM_ESTATE before am_upload_voxels.
+ */
+int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_device,
+               void* cuda_stream, am_stats* stats);
+
+/*
+ * AMs of P pivots (host array pivots[3*P]); am_out receives P consecutive maps
+ * of am_words_per_map(ctx) words each (host or device as above).  Equivalent
+ * to P calls of am_compute (the toolpath batch of SURVEY.md 8(e)(2)).
+ */
+int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_out,
+                     int dst_is_device, void* cuda_stream);
+
+/*
+ * Baseline AM of one pivot: the exact cylinder-box test (CHECKBOX, PAPER.md
+ * L97, Fig. 4 L82) for every (voxel, orientation) pair, without cones -- the
+ * non-pruned analogue of the paper's PBox (L269).  Per orientation the scan
+ * stops at the first collision (Alg. 2).  Same output contract as
+ * am_compute.
+ */
+int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_device,
+                        void* cuda_stream);
+
+/* Set a tunable (AM_OPT_*).  AM_EINVAL for an unknown key or an out-of-range value. */
+int am_set_option(am_ctx* ctx, int key, int64_t value);
+
+/*
+ * Device time of the voxel-streaming kernel (steps a1-a5, the dominant kernel)
+ * summed over its launches since the previous call, measured with CUDA events
+ * recorded on the launching stream while AM_OPT_KERNEL_TIMING is 1.  Waits for
+ * the recorded events, then resets the accumulator.  *total_ms and *launches
+ * must be non-NULL.
+ */
+int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches);
+
+/* m * ceil(n / 32): words per AM.  -1 if ctx is NULL. */
+int am_words_per_map(const am_ctx* ctx);
+
+/* Number of voxels currently resident (-1 if ctx is NULL). */
+int64_t am_num_voxels(const am_ctx* ctx);
+
+/* Human-readable description of the last error on ctx (never NULL). */
+const char* am_last_error(const am_ctx* ctx);
+
+/* Free the context and all its device memory.  NULL is a no-op. */
+void am_destroy(am_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* AM_H_ */

@@ -1,0 +1,247 @@
+"""ctypes binding of include/am.h (argument marshalling only).
+
+Host data are numpy arrays; device data are ``torch`` CUDA tensors (PyTorch is
+used for device memory and streams only).  Names follow the C ABI:
+``am_create`` -> :class:`Context`, ``am_upload_voxels`` -> :meth:`Context.upload`,
+``am_compute`` -> :meth:`Context.compute`, ``am_compute_batch`` ->
+:meth:`Context.compute_batch`, ``am_compute_baseline`` ->
+:meth:`Context.compute_baseline`.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libam.so")
+
+AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
+OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
+OPT_KERNEL_TIMING = 6
+
+# every symbol include/am.h declares
+EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",
+           "am_set_option", "am_kernel_time", "am_words_per_map", "am_num_voxels", "am_last_error",
+           "am_destroy")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"{LIB_PATH} is missing: build the CUDA library first (python -c 'import __graft_entry__ as g; g.build()'). "
+        "There is no CPU fallback.")
+
+
+class _Cyl(ctypes.Structure):
+    _fields_ = [("radius", ctypes.c_float), ("height", ctypes.c_float)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int64) for k in (
+        "voxels_streamed", "voxels_culled", "voxels_skipped", "voxels_live", "rows_rasterised",
+        "band_pairs", "exact_tests", "exact_hits", "queue_overflow", "early_exit")]
+
+
+@dataclass
+class Stats:
+    voxels_streamed: int
+    voxels_culled: int
+    voxels_skipped: int
+    voxels_live: int
+    rows_rasterised: int
+    band_pairs: int
+    exact_tests: int
+    exact_hits: int
+    queue_overflow: int
+    early_exit: int
+
+
+lib = ctypes.CDLL(LIB_PATH)
+_P = ctypes.c_void_p
+lib.am_create.restype = ctypes.c_int
+lib.am_create.argtypes = [ctypes.POINTER(_Cyl), ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                          ctypes.POINTER(_P)]
+lib.am_upload_voxels.restype = ctypes.c_int
+lib.am_upload_voxels.argtypes = [_P, _P, _P, ctypes.c_int64, ctypes.c_int]
+lib.am_compute.restype = ctypes.c_int
+lib.am_compute.argtypes = [_P, ctypes.POINTER(ctypes.c_float), _P, ctypes.c_int, _P, ctypes.POINTER(_Stats)]
+lib.am_compute_batch.restype = ctypes.c_int
+lib.am_compute_batch.argtypes = [_P, ctypes.POINTER(ctypes.c_float), ctypes.c_int64, _P, ctypes.c_int, _P]
+lib.am_compute_baseline.restype = ctypes.c_int
+lib.am_compute_baseline.argtypes = [_P, ctypes.POINTER(ctypes.c_float), _P, ctypes.c_int, _P]
+lib.am_set_option.restype = ctypes.c_int
+lib.am_set_option.argtypes = [_P, ctypes.c_int, ctypes.c_int64]
+lib.am_kernel_time.restype = ctypes.c_int
+lib.am_kernel_time.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+lib.am_words_per_map.restype = ctypes.c_int
+lib.am_words_per_map.argtypes = [_P]
+lib.am_num_voxels.restype = ctypes.c_int64
+lib.am_num_voxels.argtypes = [_P]
+lib.am_last_error.restype = ctypes.c_char_p
+lib.am_last_error.argtypes = [_P]
+lib.am_destroy.restype = None
+lib.am_destroy.argtypes = [_P]
+
+
+def exported_symbols():
+    """Names of include/am.h entry points found in libam.so."""
+    return [s for s in EXPORTS if hasattr(lib, s)]
+
+
+class AMError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"AM error {code}: {msg}")
+        self.code = code
+
+
+def words_per_map(m: int, n: int) -> int:
+    return m * ((n + 31) // 32)
+
+
+def unpack(words, m: int, n: int) -> np.ndarray:
+    """uint32 words (ABI layout, include/am.h) -> uint8[m, n] collision map."""
+    W = (n + 31) // 32
+    w = np.asarray(words).view(np.uint32).reshape(m, W)
+    j = np.arange(n)
+    return ((w[:, j >> 5] >> (j & 31).astype(np.uint32)) & np.uint32(1)).astype(np.uint8)
+
+
+def _is_torch_cuda(x):
+    return hasattr(x, "is_cuda") and x.is_cuda
+
+
+def _stream_handle(stream):
+    if stream is None:
+        return None
+    if hasattr(stream, "cuda_stream"):
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(int(stream))
+
+
+def _f3(p):
+    a = np.ascontiguousarray(np.asarray(p, dtype=np.float32).reshape(3))
+    return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_float))
+
+
+class Context:
+    """One am_ctx: a tool, an m x n orientation grid and a resident voxel model on one GPU."""
+
+    def __init__(self, tool, m: int, n: int, device: int = 0):
+        t = list(tool)
+        arr = (_Cyl * max(len(t), 1))(*[_Cyl(float(r), float(h)) for r, h in t])
+        h = _P()
+        rc = lib.am_create(arr, len(t), int(m), int(n), int(device), ctypes.byref(h))
+        if rc != AM_OK:
+            raise AMError(rc, "am_create failed (tool / grid invalid or no usable CUDA device)")
+        self._h = h
+        self.m, self.n, self.device = int(m), int(n), int(device)
+        self.words = lib.am_words_per_map(h)
+        self.tool = tuple((float(r), float(hh)) for r, hh in t)
+
+    # ------------------------------------------------------------------ helpers
+    def _check(self, rc):
+        if rc != AM_OK:
+            raise AMError(rc, lib.am_last_error(self._h).decode())
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.am_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def set_option(self, key: int, value: int):
+        self._check(lib.am_set_option(self._h, int(key), int(value)))
+
+    def kernel_time(self):
+        """am_kernel_time: (total ms, launches) of the streaming kernel since the last call."""
+        ms = ctypes.c_double()
+        n = ctypes.c_int64()
+        self._check(lib.am_kernel_time(self._h, ctypes.byref(ms), ctypes.byref(n)))
+        return ms.value, n.value
+
+    @property
+    def num_voxels(self) -> int:
+        return int(lib.am_num_voxels(self._h))
+
+    # ------------------------------------------------------------------ calls
+    def upload(self, centers, half_sizes):
+        """am_upload_voxels: centres [N,3] + half sizes [N] (numpy host or torch CUDA float32)."""
+        if _is_torch_cuda(centers):
+            c = centers.contiguous()
+            hs = half_sizes.contiguous()
+            N = int(hs.numel())
+            self._check(lib.am_upload_voxels(self._h, _P(c.data_ptr()), _P(hs.data_ptr()), N, 1))
+        else:
+            c = np.ascontiguousarray(np.asarray(centers, dtype=np.float32).reshape(-1, 3))
+            hs = np.ascontiguousarray(np.asarray(half_sizes, dtype=np.float32).reshape(-1))
+            if len(c) != len(hs):
+                raise ValueError("centres and half sizes differ in length")
+            self._check(lib.am_upload_voxels(self._h, _P(c.ctypes.data), _P(hs.ctypes.data), len(hs), 0))
+
+    def compute(self, pivot, out=None, stream=None, stats: bool = False):
+        """am_compute for one pivot.
+
+        out=None -> host numpy uint32[words]; out = torch CUDA int32/uint32
+        tensor of >= words elements -> written on the device (asynchronous on
+        `stream`, default torch's current stream).  Returns (out, Stats|None).
+        """
+        _, pp = _f3(pivot)
+        st = _Stats() if stats else None
+        sp = ctypes.byref(st) if st is not None else None
+        if out is not None and _is_torch_cuda(out):
+            if stream is None:
+                import torch
+                stream = torch.cuda.current_stream(out.device)
+            self._check(lib.am_compute(self._h, pp, _P(out.data_ptr()), 1, _stream_handle(stream), sp))
+        else:
+            if out is None:
+                out = np.zeros(self.words, dtype=np.uint32)
+            self._check(lib.am_compute(self._h, pp, _P(out.ctypes.data), 0, _stream_handle(stream), sp))
+        return out, (Stats(*[getattr(st, f[0]) for f in _Stats._fields_]) if st is not None else None)
+
+    def compute_batch(self, pivots, out=None, stream=None):
+        """am_compute_batch: P pivots -> P maps (host numpy uint32[P, words] or torch CUDA)."""
+        pv = np.ascontiguousarray(np.asarray(pivots, dtype=np.float32).reshape(-1, 3))
+        P = len(pv)
+        pp = pv.ctypes.data_as(ctypes.POINTER(ctypes.c_float))
+        if out is not None and _is_torch_cuda(out):
+            if stream is None:
+                import torch
+                stream = torch.cuda.current_stream(out.device)
+            self._check(lib.am_compute_batch(self._h, pp, P, _P(out.data_ptr()), 1, _stream_handle(stream)))
+        else:
+            if out is None:
+                out = np.zeros((P, self.words), dtype=np.uint32)
+            self._check(lib.am_compute_batch(self._h, pp, P, _P(out.ctypes.data), 0, _stream_handle(stream)))
+        return out
+
+    def compute_baseline(self, pivot, out=None, stream=None):
+        """am_compute_baseline: all-pairs exact test (PBox analogue)."""
+        _, pp = _f3(pivot)
+        if out is not None and _is_torch_cuda(out):
+            if stream is None:
+                import torch
+                stream = torch.cuda.current_stream(out.device)
+            self._check(lib.am_compute_baseline(self._h, pp, _P(out.data_ptr()), 1, _stream_handle(stream)))
+        else:
+            if out is None:
+                out = np.zeros(self.words, dtype=np.uint32)
+            self._check(lib.am_compute_baseline(self._h, pp, _P(out.ctypes.data), 0, _stream_handle(stream)))
+        return out
+
+    def am(self, pivot) -> np.ndarray:
+        """Convenience: uint8[m, n] AICA map of one pivot (host)."""
+        w, _ = self.compute(pivot)
+        return unpack(w, self.m, self.n)

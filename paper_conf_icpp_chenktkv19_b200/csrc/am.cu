@@ -1,0 +1,532 @@
+// am.cu -- host side of the C ABI declared in include/am.h (L1 of SURVEY.md 1).
+//
+// Owns the device state of one context: the resident voxel list (float4,
+// Morton-sorted at upload), the orientation tables, the band queue, a scratch
+// AM and the per-call counters.  Every entry point validates its arguments,
+// launches sm_100a kernels on the caller's stream and reports CUDA failures as
+// AM_ECUDA.  There is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <cub/device/device_radix_sort.cuh>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/am.h"
+#include "kernels.cuh"
+
+using namespace am;
+
+struct am_ctx {
+    int device = 0;
+    int sms = 0;
+    ToolDev tool{};
+    GridDev grid{};
+    int MW = 0;
+    // resident model
+    float4* d_vox = nullptr;
+    long long N = 0;
+    long long vox_cap = 0;
+    bool uploaded = false;
+    // per-call state
+    float* d_tab = nullptr;                // cos phi, sin phi, cos gamma, sin gamma
+    uint32_t* d_am = nullptr;              // scratch AM(s) for host destinations
+    long long am_cap_maps = 0;
+    unsigned long long* d_ctr = nullptr;   // [0] queue count, [1..] stats
+    unsigned long long* d_queue = nullptr;
+    long long qcap = 0;
+    // options
+    int grid_ctas = 0;
+    int refresh_tiles = 4;
+    int morton = 1;
+    int baseline_reject = 0;
+    size_t smem = 0;
+    int occ = 0;
+    // kernel timing (AM_OPT_KERNEL_TIMING)
+    int timing = 0;
+    std::vector<cudaEvent_t> ev_start, ev_stop;
+    size_t ev_used = 0;
+    std::string err;
+};
+
+namespace {
+
+constexpr int kCtrWords = 1 + ST_COUNT;
+
+int fail(am_ctx* c, int code, const char* fmt, ...) {
+    if (c) {
+        char buf[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(buf, sizeof buf, fmt, ap);
+        va_end(ap);
+        c->err = buf;
+    }
+    return code;
+}
+
+#define CK(call)                                                                              \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess) {                                                              \
+            cudaGetLastError();                                                               \
+            return fail(ctx, e_ == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA, "%s: %s (%s:%d)", \
+                        #call, cudaGetErrorString(e_), __FILE__, __LINE__);                  \
+        }                                                                                     \
+    } while (0)
+
+// Restores the caller's current device on scope exit.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = false;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) == cudaSuccess && cudaSetDevice(dev) == cudaSuccess) ok = true;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+bool is_finite_f(float x) { return std::isfinite(x); }
+
+StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
+    StreamParams p{};
+    p.tool = c->tool;
+    p.grid = c->grid;
+    p.px = pivot[0];
+    p.py = pivot[1];
+    p.pz = pivot[2];
+    p.vox = c->d_vox;
+    p.N = c->N;
+    p.gam = gam;
+    p.tab = c->d_tab;
+    p.qcount = c->d_ctr;
+    p.stats = c->d_ctr + 1;
+    p.queue = c->d_queue;
+    p.qcap = c->qcap;
+    p.refresh_tiles = c->refresh_tiles;
+    return p;
+}
+
+int ensure_queue(am_ctx* ctx, long long cap) {
+    if (ctx->d_queue && ctx->qcap == cap) return AM_OK;
+    if (ctx->d_queue) cudaFree(ctx->d_queue);
+    ctx->d_queue = nullptr;
+    ctx->qcap = 0;
+    CK(cudaMalloc(&ctx->d_queue, (size_t)cap * sizeof(unsigned long long)));
+    ctx->qcap = cap;
+    return AM_OK;
+}
+
+int configure_launch(am_ctx* ctx) {
+    const int m = ctx->grid.m;
+    ctx->smem = (size_t)(2 * ctx->MW + ((m + 31) >> 5)) * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
+    if (ctx->smem > 48 * 1024)
+        CK(cudaFuncSetAttribute(aica_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)ctx->smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel, kThreads, ctx->smem));
+    if (occ < 1) return fail(ctx, AM_EINVAL, "grid %dx%d does not fit in shared memory", m, ctx->grid.n);
+    ctx->occ = occ;
+    return AM_OK;
+}
+
+// One AICA map into device buffer gam (asynchronous on s).
+int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
+    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
+    if (ctx->N == 0) return AM_OK;
+    StreamParams p = make_params(ctx, pivot, gam);
+    const long long ntiles = (ctx->N + kTile - 1) / kTile;
+    long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
+    if (g > ntiles) g = ntiles;
+    if (g < 1) g = 1;
+    if (ctx->timing) {
+        if (ctx->ev_used == ctx->ev_start.size()) {
+            cudaEvent_t a, b;
+            CK(cudaEventCreate(&a));
+            CK(cudaEventCreate(&b));
+            ctx->ev_start.push_back(a);
+            ctx->ev_stop.push_back(b);
+        }
+        CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
+    }
+    aica_stream_kernel<<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
+    CK(cudaGetLastError());
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
+    CK(cudaGetLastError());
+    return AM_OK;
+}
+
+int check_pivot(am_ctx* ctx, const float* pivot) {
+    if (!pivot) return fail(ctx, AM_EINVAL, "pivot is NULL");
+    for (int k = 0; k < 3; ++k)
+        if (!is_finite_f(pivot[k])) return fail(ctx, AM_EINVAL, "pivot[%d] is not finite", k);
+    return AM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_ctx** out) {
+    if (!out) return AM_EINVAL;
+    *out = nullptr;
+    if (!tool || n_cyl < 1 || n_cyl > AM_MAX_CYL) return AM_EINVAL;
+    if (m < 1 || m > 1024 || n < 1 || n > 1024) return AM_EINVAL;
+    for (int k = 0; k < n_cyl; ++k) {
+        if (!is_finite_f(tool[k].radius) || !is_finite_f(tool[k].height) || tool[k].radius <= 0.f ||
+            tool[k].height <= 0.f)
+            return AM_EINVAL;
+    }
+    am_ctx* ctx = new am_ctx();
+    ctx->device = device;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+        cudaGetLastError();
+        delete ctx;
+        return AM_ECUDA;
+    }
+    DeviceGuard dg(device);
+    if (!dg.ok) {
+        delete ctx;
+        return AM_ECUDA;
+    }
+    // tool: cylinders from the pivot outward (readings G3/G4); radii in double
+    // then rounded, so the device sees the caller's float values
+    ToolDev& T = ctx->tool;
+    T.ncyl = n_cyl;
+    double z = 0.0, rho = 0.0, pm = 0.0;
+    for (int k = 0; k < n_cyl; ++k) {
+        T.z0[k] = (float)z;
+        z += tool[k].height;
+        T.z1[k] = (float)z;
+        T.R[k] = tool[k].radius;
+        pm = std::max(pm, (double)tool[k].radius);
+        T.Rpm[k] = (float)pm;
+        rho = std::max(rho, std::sqrt(z * z + (double)tool[k].radius * tool[k].radius));
+    }
+    for (int k = 0; k < n_cyl; ++k) {
+        float mn = tool[k].radius;
+        for (int j = k; j < n_cyl; ++j) mn = std::min(mn, tool[j].radius);
+        T.Rin[k] = mn;
+    }
+    T.L = (float)z;
+    T.rho_max = (float)rho;
+    GridDev& G = ctx->grid;
+    G.m = m;
+    G.n = n;
+    G.W = (n + 31) / 32;
+    const double PI = 3.14159265358979323846;
+    G.dphi = (float)(PI / m);
+    G.inv_dphi = (float)(m / PI);
+    G.dgam = (float)(2.0 * PI / n);
+    G.inv_dgam = (float)(n / (2.0 * PI));
+    ctx->MW = m * G.W;
+    int rc;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) {
+        cudaGetLastError();
+        delete ctx;
+        return AM_ECUDA;
+    }
+    ctx->sms = prop.multiProcessorCount;
+    std::vector<float> tab(2 * m + 2 * n);
+    for (int i = 0; i < m; ++i) {
+        const double ph = (i + 0.5) * PI / m;
+        tab[i] = (float)std::cos(ph);
+        tab[m + i] = (float)std::sin(ph);
+    }
+    for (int j = 0; j < n; ++j) {
+        const double ga = (j + 0.5) * 2.0 * PI / n;
+        tab[2 * m + j] = (float)std::cos(ga);
+        tab[2 * m + n + j] = (float)std::sin(ga);
+    }
+    auto bail = [&](int code) {
+        am_destroy(ctx);
+        return code;
+    };
+    if (cudaMalloc(&ctx->d_tab, tab.size() * sizeof(float)) != cudaSuccess ||
+        cudaMemcpy(ctx->d_tab, tab.data(), tab.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMalloc(&ctx->d_ctr, kCtrWords * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_am, (size_t)ctx->MW * sizeof(uint32_t)) != cudaSuccess) {
+        cudaGetLastError();
+        return bail(AM_ENOMEM);
+    }
+    ctx->am_cap_maps = 1;
+    if ((rc = ensure_queue(ctx, 1 << 22)) != AM_OK) return bail(rc);
+    if ((rc = configure_launch(ctx)) != AM_OK) return bail(rc);
+    *out = ctx;
+    return AM_OK;
+}
+
+int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_sizes, int64_t N,
+                     int src_is_device) {
+    if (!ctx) return AM_EINVAL;
+    if (N < 0) return fail(ctx, AM_EINVAL, "N < 0");
+    if (N > 0x7fffffffLL) return fail(ctx, AM_EINVAL, "N exceeds 2^31 - 1");
+    if (N > 0 && (!centers_xyz || !half_sizes)) return fail(ctx, AM_EINVAL, "NULL voxel array");
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    ctx->uploaded = false;
+    if (N == 0) {
+        ctx->N = 0;
+        ctx->uploaded = true;
+        return AM_OK;
+    }
+    const float* dc = centers_xyz;
+    const float* dh = half_sizes;
+    float* tmp_c = nullptr;
+    float* tmp_h = nullptr;
+    float4* raw = nullptr;
+    unsigned int* bbox = nullptr;
+    unsigned long long* bad = nullptr;
+    unsigned long long* keys = nullptr;
+    unsigned long long* keys2 = nullptr;
+    unsigned int* ids = nullptr;
+    unsigned int* ids2 = nullptr;
+    void* cubtmp = nullptr;
+    int rc = AM_OK;
+    auto cleanup = [&]() {
+        cudaFree(tmp_c);
+        cudaFree(tmp_h);
+        cudaFree(raw);
+        cudaFree(bbox);
+        cudaFree(bad);
+        cudaFree(keys);
+        cudaFree(keys2);
+        cudaFree(ids);
+        cudaFree(ids2);
+        cudaFree(cubtmp);
+    };
+#define UK(call)                                                                               \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess) {                                                               \
+            cudaGetLastError();                                                                \
+            cleanup();                                                                         \
+            return fail(ctx, e_ == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA, "%s: %s", #call, \
+                        cudaGetErrorString(e_));                                               \
+        }                                                                                      \
+    } while (0)
+    if (!src_is_device) {
+        UK(cudaMalloc(&tmp_c, (size_t)N * 3 * sizeof(float)));
+        UK(cudaMalloc(&tmp_h, (size_t)N * sizeof(float)));
+        UK(cudaMemcpy(tmp_c, centers_xyz, (size_t)N * 3 * sizeof(float), cudaMemcpyHostToDevice));
+        UK(cudaMemcpy(tmp_h, half_sizes, (size_t)N * sizeof(float), cudaMemcpyHostToDevice));
+        dc = tmp_c;
+        dh = tmp_h;
+    }
+    if (ctx->vox_cap < N) {
+        cudaFree(ctx->d_vox);
+        ctx->d_vox = nullptr;
+        ctx->vox_cap = 0;
+        UK(cudaMalloc(&ctx->d_vox, (size_t)N * sizeof(float4)));
+        ctx->vox_cap = N;
+    }
+    UK(cudaMalloc(&raw, (size_t)N * sizeof(float4)));
+    UK(cudaMalloc(&bbox, 6 * sizeof(unsigned int)));
+    UK(cudaMalloc(&bad, sizeof(unsigned long long)));
+    const unsigned int init[6] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0u, 0u, 0u};
+    UK(cudaMemcpy(bbox, init, sizeof init, cudaMemcpyHostToDevice));
+    UK(cudaMemset(bad, 0, sizeof(unsigned long long)));
+    const int blocks = ctx->sms * 8;
+    pack_validate_kernel<<<blocks, 256>>>(dc, dh, N, raw, bbox, bad);
+    UK(cudaGetLastError());
+    unsigned long long nbad = 0;
+    UK(cudaMemcpy(&nbad, bad, sizeof nbad, cudaMemcpyDeviceToHost));
+    if (nbad) {
+        cleanup();
+        return fail(ctx, AM_EINVAL, "%llu voxels with a non-finite value or half size <= 0", nbad);
+    }
+    if (ctx->morton) {
+        UK(cudaMalloc(&keys, (size_t)N * sizeof(unsigned long long)));
+        UK(cudaMalloc(&keys2, (size_t)N * sizeof(unsigned long long)));
+        UK(cudaMalloc(&ids, (size_t)N * sizeof(unsigned int)));
+        UK(cudaMalloc(&ids2, (size_t)N * sizeof(unsigned int)));
+        morton_keys_kernel<<<blocks, 256>>>(raw, N, bbox, keys, ids);
+        UK(cudaGetLastError());
+        size_t tb = 0;
+        UK(cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, ids, ids2, (int)N, 0, 63));
+        UK(cudaMalloc(&cubtmp, tb));
+        UK(cub::DeviceRadixSort::SortPairs(cubtmp, tb, keys, keys2, ids, ids2, (int)N, 0, 63));
+        gather_kernel<<<blocks, 256>>>(raw, ids2, N, ctx->d_vox);
+        UK(cudaGetLastError());
+    } else {
+        UK(cudaMemcpy(ctx->d_vox, raw, (size_t)N * sizeof(float4), cudaMemcpyDeviceToDevice));
+    }
+    UK(cudaDeviceSynchronize());
+#undef UK
+    cleanup();
+    ctx->N = N;
+    ctx->uploaded = true;
+    return rc;
+}
+
+int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_device,
+               void* cuda_stream, am_stats* stats) {
+    if (!ctx) return AM_EINVAL;
+    int rc = check_pivot(ctx, pivot);
+    if (rc) return rc;
+    if (!am_out) return fail(ctx, AM_EINVAL, "am_out is NULL");
+    if (!ctx->uploaded) return fail(ctx, AM_ESTATE, "am_compute before am_upload_voxels");
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
+    if ((rc = launch_aica(ctx, pivot, gam, s)) != AM_OK) return rc;
+    if (!dst_is_device)
+        CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if (stats) {
+        unsigned long long h[kCtrWords];
+        CK(cudaMemcpyAsync(h, ctx->d_ctr, sizeof h, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        int64_t* o = reinterpret_cast<int64_t*>(stats);
+        for (int k = 0; k < ST_COUNT; ++k) o[k] = (int64_t)h[1 + k];
+        // band pairs resolved inline are counted as exact tests too
+    } else if (!dst_is_device) {
+        CK(cudaStreamSynchronize(s));
+    }
+    return AM_OK;
+}
+
+int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_out, int dst_is_device,
+                     void* cuda_stream) {
+    if (!ctx) return AM_EINVAL;
+    if (P < 0) return fail(ctx, AM_EINVAL, "P < 0");
+    if (P > 0 && (!pivots || !am_out)) return fail(ctx, AM_EINVAL, "NULL pivots or am_out");
+    for (int64_t k = 0; k < 3 * P; ++k)
+        if (!is_finite_f(pivots[k])) return fail(ctx, AM_EINVAL, "pivot %lld is not finite", (long long)(k / 3));
+    if (!ctx->uploaded) return fail(ctx, AM_ESTATE, "am_compute_batch before am_upload_voxels");
+    if (P == 0) return AM_OK;
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    uint32_t* dst = am_out;
+    if (!dst_is_device) {
+        if (ctx->am_cap_maps < P) {
+            cudaFree(ctx->d_am);
+            ctx->d_am = nullptr;
+            ctx->am_cap_maps = 0;
+            CK(cudaMalloc(&ctx->d_am, (size_t)P * ctx->MW * sizeof(uint32_t)));
+            ctx->am_cap_maps = P;
+        }
+        dst = ctx->d_am;
+    }
+    int rc;
+    for (int64_t k = 0; k < P; ++k)
+        if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
+    if (!dst_is_device) {
+        CK(cudaMemcpyAsync(am_out, dst, (size_t)P * ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return AM_OK;
+}
+
+int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_device,
+                        void* cuda_stream) {
+    if (!ctx) return AM_EINVAL;
+    int rc = check_pivot(ctx, pivot);
+    if (rc) return rc;
+    if (!am_out) return fail(ctx, AM_EINVAL, "am_out is NULL");
+    if (!ctx->uploaded) return fail(ctx, AM_ESTATE, "am_compute_baseline before am_upload_voxels");
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
+    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
+    if (ctx->N > 0) {
+        StreamParams p = make_params(ctx, pivot, gam);
+        const int ncell = ctx->grid.m * ctx->grid.n;
+        int g = ctx->sms * 8;
+        if (g > ncell) g = ncell;
+        baseline_kernel<<<g, kThreads, 0, s>>>(p, ctx->baseline_reject);
+        CK(cudaGetLastError());
+    }
+    if (!dst_is_device) {
+        CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return AM_OK;
+}
+
+int am_set_option(am_ctx* ctx, int key, int64_t value) {
+    if (!ctx) return AM_EINVAL;
+    DeviceGuard dg(ctx->device);
+    switch (key) {
+    case AM_OPT_GRID_CTAS:
+        if (value < 0 || value > (1 << 20)) return fail(ctx, AM_EINVAL, "grid_ctas out of range");
+        ctx->grid_ctas = (int)value;
+        return AM_OK;
+    case AM_OPT_REFRESH_TILES:
+        if (value < 1 || value > (1 << 20)) return fail(ctx, AM_EINVAL, "refresh_tiles out of range");
+        ctx->refresh_tiles = (int)value;
+        return AM_OK;
+    case AM_OPT_MORTON_SORT:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "morton_sort must be 0 or 1");
+        ctx->morton = (int)value;
+        return AM_OK;
+    case AM_OPT_BASELINE_REJECT:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "baseline_reject must be 0 or 1");
+        ctx->baseline_reject = (int)value;
+        return AM_OK;
+    case AM_OPT_BAND_QUEUE:
+        if (value < 1 || value > (1LL << 28)) return fail(ctx, AM_EINVAL, "band queue out of range");
+        return ensure_queue(ctx, value);
+    case AM_OPT_KERNEL_TIMING:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "kernel_timing must be 0 or 1");
+        ctx->timing = (int)value;
+        return AM_OK;
+    default:
+        return fail(ctx, AM_EINVAL, "unknown option %d", key);
+    }
+}
+
+int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches) {
+    if (!ctx) return AM_EINVAL;
+    if (!total_ms || !launches) return fail(ctx, AM_EINVAL, "NULL output");
+    DeviceGuard dg(ctx->device);
+    double tot = 0.0;
+    for (size_t k = 0; k < ctx->ev_used; ++k) {
+        float ms = 0.f;
+        CK(cudaEventSynchronize(ctx->ev_stop[k]));
+        CK(cudaEventElapsedTime(&ms, ctx->ev_start[k], ctx->ev_stop[k]));
+        tot += ms;
+    }
+    *total_ms = tot;
+    *launches = (int64_t)ctx->ev_used;
+    ctx->ev_used = 0;
+    return AM_OK;
+}
+
+int am_words_per_map(const am_ctx* ctx) { return ctx ? ctx->MW : -1; }
+
+int64_t am_num_voxels(const am_ctx* ctx) { return ctx ? (int64_t)ctx->N : -1; }
+
+const char* am_last_error(const am_ctx* ctx) {
+    if (!ctx) return "NULL context";
+    return ctx->err.empty() ? "no error" : ctx->err.c_str();
+}
+
+void am_destroy(am_ctx* ctx) {
+    if (!ctx) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(ctx->device);
+    cudaFree(ctx->d_vox);
+    cudaFree(ctx->d_tab);
+    cudaFree(ctx->d_am);
+    cudaFree(ctx->d_ctr);
+    cudaFree(ctx->d_queue);
+    for (auto e : ctx->ev_start) cudaEventDestroy(e);
+    for (auto e : ctx->ev_stop) cudaEventDestroy(e);
+    cudaGetLastError();
+    if (prev >= 0) cudaSetDevice(prev);
+    delete ctx;
+}
+
+}  // extern "C"

@@ -1,0 +1,368 @@
+// geometry.cuh -- device geometry of the AICA hot path (fp32, sm_100a).
+//
+// Three pieces, each citing the passage it implements:
+//   * tool_cones():  the two inaccessible cone angles of a voxel (GETTOOLICA for
+//     the inscribed radius h and the circumscribed radius sqrt(3) h, PAPER.md
+//     Alg. 1; crossed points on the 5 components of every expanded
+//     cylinder rectangle, L163-169, L175, Fig. 7), in the cosine domain,
+//     with reading G8 (inner cone on the monotone-shrunk tool; ring voxels).
+//   * gamma_interval(): one phi-row of a cone as a gamma interval -- Alg. 1
+//     L149-155 ("angle <= ica") evaluated for all cells of a row at once.
+//   * exact_hit(): the exact cylinder-box test (CHECKBOX, L97, Fig. 4 L82).
+//
+// Nothing here is shared with oracle/ (independent implementation; the oracle
+// uses a clip -> convex-hull formulation in fp64, this file a min-over-edges
+// formulation in fp32).
+#pragma once
+#include <cstdint>
+
+#define AM_MAX_CYL 8
+
+namespace am {
+
+constexpr float kSqrt3 = 1.7320508075688772f;
+constexpr float kPi = 3.14159265358979323846f;
+
+struct ToolDev {
+    int ncyl;
+    float z0[AM_MAX_CYL];   // axial start of cylinder k (z0[0] = 0 at the pivot)
+    float z1[AM_MAX_CYL];   // axial end
+    float R[AM_MAX_CYL];    // radius
+    float Rin[AM_MAX_CYL];  // monotone-shrunk radius min_{j >= k} R_j (reading G8)
+    float Rpm[AM_MAX_CYL];  // prefix max max_{j <= k} R_j (cheap outer bound)
+    float L;                // total length z1[ncyl-1]
+    float rho_max;          // max_k |(z1_k, R_k)|: reach of the tool from the pivot
+};
+
+struct GridDev {
+    int m, n, W;            // rows (phi), columns (gamma), words per row
+    float dphi, inv_dphi;   // pi / m
+    float dgam, inv_dgam;   // 2 pi / n
+};
+
+// Guards: the inner cone is shrunk and the outer cone
+// grown so that every fp32 rounding error lands in the band, which is resolved
+// by the exact test.  None of them can change a robust cell; they only add a
+// few band cells.
+constexpr float kCosGuard = 2e-6f;     // cosine-domain cone guard
+constexpr float kRadRel = 4e-6f;       // relative sphere-radius guard (x (D + r))
+constexpr float kGamGuard = 4e-6f;     // gamma-domain interval guard (rad)
+constexpr float kCellSlack = 1e-4f;    // interval ends, in cells
+constexpr float kRowSlack = 1e-4f;     // phi-row range slack (rad); loop bound only
+
+// Blocked-angle candidates of a sphere of radius r whose centre is at distance D
+// from the pivot, against ONE cylinder's meridian rectangle [z0, z1] x [0, R]
+// expanded by r ("crossed points" of the arc of radius D with
+// the expanded rectangle; five components, L175: bottom edge, top edge, side,
+// and the two rounded corners).  Every candidate is a point of the expanded
+// rectangle, and every boundary crossing is a candidate, so
+//   cmin = cos(largest blocked angle)   (2 if nothing is blocked)
+//   cmax = cos(smallest blocked angle)  (-2 if nothing is blocked).
+__device__ __forceinline__ void ica_cylinder(float D, float D2, float invD, float r, float z0,
+                                             float z1, float R, float& cmin, float& cmax) {
+    cmin = 2.f;
+    cmax = -2.f;
+    if (D + z0 <= r) cmin = -1.f;               // theta = pi lies inside
+    if (D >= z0 - r && D <= z1 + r) cmax = 1.f; // theta = 0 lies inside
+    const float R2 = R * R;
+    {   // bottom edge: a = z0 - r, 0 <= rho <= R
+        const float a = z0 - r;
+        const float t = D2 - a * a;
+        if (t >= 0.f && t <= R2) {
+            const float c = a * invD;
+            cmin = fminf(cmin, c);
+            cmax = fmaxf(cmax, c);
+        }
+    }
+    {   // top edge: a = z1 + r, 0 <= rho <= R
+        const float a = z1 + r;
+        const float t = D2 - a * a;
+        if (t >= 0.f && t <= R2) {
+            const float c = a * invD;
+            cmin = fminf(cmin, c);
+            cmax = fmaxf(cmax, c);
+        }
+    }
+    {   // side: rho = R + r, z0 <= a <= z1 (a >= 0 because z0 >= 0)
+        const float s = R + r;
+        const float t = D2 - s * s;
+        if (t >= 0.f) {
+            const float a = sqrtf(t);
+            if (a >= z0 && a <= z1) {
+                const float c = a * invD;
+                cmin = fminf(cmin, c);
+                cmax = fmaxf(cmax, c);
+            }
+        }
+    }
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {  // rounded corners centred (zc, R), radius r
+        const float zc = e ? z1 : z0;
+        const float Dc = sqrtf(zc * zc + R2);
+        const float dd = D - Dc;
+        if (fabsf(dd) <= r) {
+            // arc of radius D meets the corner circle at theta_c +- beta with
+            // cos(beta) = (D^2 + Dc^2 - r^2) / (2 D Dc); 1 -+ cos(beta) factored
+            // so sin(beta) keeps its relative accuracy near tangency
+            const float inv2 = 0.5f / (D * Dc);
+            const float omc = (r - dd) * (r + dd) * inv2;               // 1 - cos(beta)
+            const float sp = D + Dc;
+            const float opc = (sp - r) * (sp + r) * inv2;               // 1 + cos(beta)
+            const float cb = 0.5f * (opc - omc);
+            const float sb = sqrtf(fmaxf(omc * opc, 0.f));
+            const float ct = zc / Dc, st = R / Dc;
+            const float s_hi = st * cb + ct * sb;                       // sin(theta_c + beta)
+            const float c_hi = (s_hi < 0.f) ? -1.f : (ct * cb - st * sb);
+            const float s_lo = st * cb - ct * sb;                       // sin(theta_c - beta)
+            const float c_lo = (s_lo < 0.f) ? 1.f : (ct * cb + st * sb);
+            cmin = fminf(cmin, c_hi);
+            cmax = fmaxf(cmax, c_lo);
+        }
+    }
+}
+
+struct Cones {
+    float cin;   // inner cone: cells with cos(theta) >= cin are certainly blocked (> 1: none)
+    float cout;  // outer cone: cells with cos(theta) <  cout are certainly clear  (> 1: none)
+    float clo;   // ring voxels: cells with cos(theta) >  clo are certainly clear (> 1: no ring)
+};
+
+// GETTOOLICA(r = h) on the monotone-shrunk tool and GETTOOLICA(r = sqrt(3) h) on
+// the true tool (Alg. 1), guarded.  Reading G8: for the shrunk tool
+// (radii non-decreasing away from the pivot) the blocked set is exactly
+// [0, ica1] whenever D <= L + r; beyond the tool end (D > L + r) the blocked set
+// is a ring [lo, hi], so the inner cone is empty and the outer set is the ring.
+__device__ __forceinline__ Cones tool_cones(float D, float h, const ToolDev& T) {
+    const float r1 = fmaxf(h - kRadRel * (D + h), 0.f);
+    const float r2 = kSqrt3 * h + kRadRel * (D + kSqrt3 * h);
+    const float D2 = D * D;
+    const float invD = 1.f / D;
+    Cones c;
+    c.cin = 2.f;
+    if (D * (1.f + kRadRel) <= T.L + r1 && r1 > 0.f) {
+        float cm = 2.f;
+        for (int k = 0; k < T.ncyl; ++k) {
+            float a, b;
+            ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], a, b);
+            cm = fminf(cm, a);
+        }
+        c.cin = (cm <= 1.f) ? cm + kCosGuard : 2.f;
+    }
+    float co = 2.f, cx = -2.f;
+    for (int k = 0; k < T.ncyl; ++k) {
+        float a, b;
+        ica_cylinder(D, D2, invD, r2, T.z0[k], T.z1[k], T.R[k], a, b);
+        co = fminf(co, a);
+        cx = fmaxf(cx, b);
+    }
+    c.cout = (co <= 1.f) ? co - kCosGuard : 2.f;
+    c.clo = 2.f;
+    if (D * (1.f - kRadRel) > T.L + r2 && cx >= -1.f) c.clo = cx + kCosGuard;
+    return c;
+}
+
+// Cells j of one phi-row with base + den * cos(gamma_j - gv) >= cthr, as the
+// cyclic range [lo, lo + len) (mod n).  grow = +1 widens the interval by the
+// guards (outer cone), grow = -1 narrows it (inner cone / ring exclusion).
+struct Interval {
+    int lo, len;  // len == 0: empty; len == n: full row
+};
+
+__device__ __forceinline__ Interval gamma_interval(float cthr, float base, float den, float gv,
+                                                   int grow, const GridDev& g) {
+    Interval I{0, 0};
+    if (cthr > 1.5f) return I;
+    float dl;
+    if (den <= 1e-20f) {
+        if (base < cthr) return I;
+        I.len = g.n;
+        return I;
+    }
+    const float x = (cthr - base) / den;
+    if (x <= -1.f) { I.len = g.n; return I; }
+    if (x > 1.f) return I;
+    dl = acosf(x) + (grow > 0 ? kGamGuard : -kGamGuard);
+    if (dl < 0.f) return I;
+    if (dl >= kPi) { I.len = g.n; return I; }
+    const float slack = grow > 0 ? kCellSlack : -kCellSlack;
+    const float a = (gv - dl) * g.inv_dgam - 0.5f - slack;
+    const float b = (gv + dl) * g.inv_dgam - 0.5f + slack;
+    int lo = (int)ceilf(a);
+    const int hi = (int)floorf(b);
+    if (hi < lo) return I;
+    int len = hi - lo + 1;
+    if (len >= g.n) { I.len = g.n; return I; }
+    lo %= g.n;
+    if (lo < 0) lo += g.n;
+    I.lo = lo;
+    I.len = len;
+    return I;
+}
+
+// Bits of word w (cells 32w .. 32w+31) covered by the cyclic range I.
+__device__ __forceinline__ uint32_t interval_bits(const Interval& I, int w, int n) {
+    if (I.len == 0) return 0u;
+    const int c0 = w << 5;
+    const int c1 = min(c0 + 31, n - 1);
+    uint32_t valid = (c1 - c0 == 31) ? 0xffffffffu : ((1u << (c1 - c0 + 1)) - 1u);
+    if (I.len >= n) return valid;
+    uint32_t bits = 0u;
+    // first segment [lo, min(lo+len-1, n-1)], second [0, lo+len-1-n]
+    int a = I.lo, b = min(I.lo + I.len - 1, n - 1);
+    {
+        const int x = max(a, c0), y = min(b, c1);
+        if (x <= y) bits |= ((y - x == 31) ? 0xffffffffu : (((1u << (y - x + 1)) - 1u))) << (x - c0);
+    }
+    const int e = I.lo + I.len - 1 - n;
+    if (e >= 0) {
+        const int x = c0, y = min(e, c1);
+        if (x <= y) bits |= ((y - x == 31) ? 0xffffffffu : (((1u << (y - x + 1)) - 1u))) << (x - c0);
+    }
+    return bits;
+}
+
+// ---------------------------------------------------------------------------
+// Exact closed cylinder vs closed box (CHECKBOX, Fig. 4 L82).
+//
+// Q = box cap slab{z0 <= w.d <= z1}.  The tool cylinder meets the box iff the
+// distance rho from the axis line to Q is <= R.  rho^2 is convex on Q; it is 0
+// iff the axis segment [z0, z1] d crosses the box; otherwise its minimum is on
+// an edge of Q (it is a positive-definite quadratic on every facet that is not
+// parallel to d, and constant along d on the others).  The edges of Q are the
+// box edges clipped to the slab (decomposition: 12 segments) and, on each cap
+// plane, the segments between the crossing points of one box face's edges.
+// All geometry is expressed in the cylinder frame (rotation) and the distance
+// is taken in the plane normal to d (projection).
+// ---------------------------------------------------------------------------
+
+__device__ __forceinline__ float seg_dist2(float ax, float ay, float bx, float by) {
+    const float ux = bx - ax, uy = by - ay;
+    const float uu = ux * ux + uy * uy;
+    float t = 0.f;
+    if (uu > 0.f) t = fminf(fmaxf(-(ax * ux + ay * uy) / uu, 0.f), 1.f);
+    const float x = fmaf(t, ux, ax), y = fmaf(t, uy, ay);
+    return x * x + y * y;
+}
+
+// Edge e in 0..11: axis = e >> 2, the other two vertex bits from e & 3.
+// Vertex index bits: bit0 = x side, bit1 = y side, bit2 = z side.
+__device__ __forceinline__ void edge_vertices(int e, int& a, int& b) {
+    const int ax = e >> 2, q = e & 3;
+    int v = 0;
+    if (ax == 0) v = (q & 1) << 1 | (q >> 1) << 2;  // y, z bits
+    if (ax == 1) v = (q & 1) | (q >> 1) << 2;       // x, z bits
+    if (ax == 2) v = (q & 1) | (q >> 1) << 1;       // x, y bits
+    a = v;
+    b = v | (1 << ax);
+}
+
+__device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, float dx, float dy,
+                                       float dz, const ToolDev& T) {
+    // frame: e1 = normalize(d x a), a = the world axis least aligned with d; e2 = d x e1
+    const float adx = fabsf(dx), ady = fabsf(dy), adz = fabsf(dz);
+    float e1x, e1y, e1z;
+    if (adx <= ady && adx <= adz) { e1x = 0.f; e1y = dz; e1z = -dy; }      // d x (1,0,0)
+    else if (ady <= adz)          { e1x = -dz; e1y = 0.f; e1z = dx; }      // d x (0,1,0)
+    else                          { e1x = dy; e1y = -dx; e1z = 0.f; }      // d x (0,0,1)
+    const float in1 = rsqrtf(e1x * e1x + e1y * e1y + e1z * e1z);
+    e1x *= in1; e1y *= in1; e1z *= in1;
+    const float e2x = dy * e1z - dz * e1y, e2y = dz * e1x - dx * e1z, e2z = dx * e1y - dy * e1x;
+
+    // rotated vertices (x, y) in the plane normal to d, z along d
+    float X[8], Y[8], Z[8];
+    const float cX = vx * e1x + vy * e1y + vz * e1z;
+    const float cY = vx * e2x + vy * e2y + vz * e2z;
+    const float cZ = vx * dx + vy * dy + vz * dz;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const float sx = (k & 1) ? h : -h, sy = (k & 2) ? h : -h, sz = (k & 4) ? h : -h;
+        X[k] = cX + sx * e1x + sy * e1y + sz * e1z;
+        Y[k] = cY + sx * e2x + sy * e2y + sz * e2z;
+        Z[k] = cZ + sx * dx + sy * dy + sz * dz;
+    }
+    for (int c = 0; c < T.ncyl; ++c) {
+        const float z0 = T.z0[c], z1 = T.z1[c], R = T.R[c], R2 = R * R;
+        // (0) the axis segment crosses the box: slab test in world coordinates
+        {
+            float tlo = z0, thi = z1;
+            const float dv[3] = {dx, dy, dz}, vv[3] = {vx, vy, vz};
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+                if (dv[a] != 0.f) {
+                    const float inv = 1.f / dv[a];
+                    float t0 = (vv[a] - h) * inv, t1 = (vv[a] + h) * inv;
+                    if (t0 > t1) { const float t = t0; t0 = t1; t1 = t; }
+                    tlo = fmaxf(tlo, t0);
+                    thi = fminf(thi, t1);
+                } else if (fabsf(vv[a]) > h) {
+                    thi = -1e30f;
+                }
+            }
+            if (tlo <= thi) return true;
+        }
+        // (1) box edges clipped to the slab
+#pragma unroll
+        for (int e = 0; e < 12; ++e) {
+            int a, b;
+            edge_vertices(e, a, b);
+            const float za = Z[a], zb = Z[b];
+            float t0, t1;
+            if (za == zb) {
+                if (za < z0 || za > z1) continue;
+                t0 = 0.f; t1 = 1.f;
+            } else {
+                const float inv = 1.f / (zb - za);
+                float ta = (z0 - za) * inv, tb = (z1 - za) * inv;
+                t0 = fmaxf(fminf(ta, tb), 0.f);
+                t1 = fminf(fmaxf(ta, tb), 1.f);
+                if (t0 > t1) continue;
+            }
+            const float ux = X[b] - X[a], uy = Y[b] - Y[a];
+            if (seg_dist2(fmaf(t0, ux, X[a]), fmaf(t0, uy, Y[a]), fmaf(t1, ux, X[a]), fmaf(t1, uy, Y[a])) <= R2)
+                return true;
+        }
+        // (2) on each cap plane, segments between crossing points of one face's edges
+        for (int cap = 0; cap < 2; ++cap) {
+            const float zc = cap ? z1 : z0;
+            float PX[12], PY[12];
+            bool ok[12];
+#pragma unroll
+            for (int e = 0; e < 12; ++e) {
+                int a, b;
+                edge_vertices(e, a, b);
+                const float za = Z[a], zb = Z[b];
+                ok[e] = (za != zb) && ((za - zc) * (zb - zc) <= 0.f);
+                const float t = ok[e] ? (zc - za) / (zb - za) : 0.f;
+                PX[e] = fmaf(t, X[b] - X[a], X[a]);
+                PY[e] = fmaf(t, Y[b] - Y[a], Y[a]);
+            }
+#pragma unroll
+            for (int f = 0; f < 6; ++f) {
+                const int fa = f >> 1, fs = f & 1;
+                // the 4 edges of face (fa, fs): edges along the other two axes whose fa-bit == fs
+                int ids[4];
+                int k = 0;
+#pragma unroll
+                for (int e = 0; e < 12; ++e) {
+                    if ((e >> 2) == fa) continue;
+                    int a, b;
+                    edge_vertices(e, a, b);
+                    if (((a >> fa) & 1) == fs) ids[k++] = e;
+                }
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    if (!ok[ids[p]]) continue;
+                    if (PX[ids[p]] * PX[ids[p]] + PY[ids[p]] * PY[ids[p]] <= R2) return true;
+#pragma unroll
+                    for (int q = p + 1; q < 4; ++q) {
+                        if (!ok[ids[q]]) continue;
+                        if (seg_dist2(PX[ids[p]], PY[ids[p]], PX[ids[q]], PY[ids[q]]) <= R2) return true;
+                    }
+                }
+            }
+        }
+    }
+    return false;
+}
+
+}  // namespace am

@@ -1,0 +1,448 @@
+// kernels.cuh -- the AICA hot path on sm_100a: voxel-streaming kernel, deferred
+// band kernel, all-pairs baseline kernel, and upload helpers.
+//
+// Map of SURVEY.md 8(a) steps to code:
+//   a1 voxel stream ........ aica_stream_kernel: persistent CTAs, float4 LDG.128
+//                             streaming loads (ld.global.cs), kVPT voxels/thread
+//   a2 reach cull .......... process_voxel(): D - sqrt3 h > rho_max
+//   a3 cone axis ........... process_voxel(): v, D, phi_v, gamma_v
+//   a4 cone half-angles .... am::tool_cones() (geometry.cuh)
+//   a5 rasterise ........... process_voxel(): per phi-row gamma intervals ->
+//                             32-bit masks OR-ed into the per-CTA shared AM
+//   a6 band resolution ..... band pairs pushed to a global queue; band_exact_kernel
+//                             runs CHECKBOX only where the final AM bit is still 0
+//   a7 merge/flush/exit .... cta_merge(): one atomicOr per changed word, global AM
+//                             read back into smem, row-full bits, early exit
+//   a8 output .............. bit-packed AM (layout in include/am.h)
+//   a9 baseline ............ baseline_kernel: CHECKBOX for every (voxel, cell)
+#pragma once
+#include <cstdint>
+
+#include "geometry.cuh"
+
+namespace am {
+
+constexpr int kThreads = 256;
+constexpr int kVPT = 4;                  // voxels per thread per tile (MLP for the HBM stream)
+constexpr int kTile = kThreads * kVPT;   // voxels per tile
+
+enum StatIdx {
+    ST_STREAMED = 0, ST_CULLED, ST_SKIPPED, ST_LIVE, ST_ROWS, ST_BAND, ST_EXACT, ST_EXACT_HIT,
+    ST_OVERFLOW, ST_EARLY, ST_COUNT
+};
+
+struct StreamParams {
+    ToolDev tool;
+    GridDev grid;
+    float px, py, pz;
+    const float4* __restrict__ vox;
+    long long N;
+    uint32_t* gam;                 // global AM, m * W words, zeroed before launch
+    const float* __restrict__ tab; // cos phi[m], sin phi[m], cos gamma[n], sin gamma[n]
+    unsigned long long* qcount;    // band queue fill counter (zeroed)
+    unsigned long long* queue;     // band pairs: (voxel << 32) | cell
+    long long qcap;
+    unsigned long long* stats;     // ST_COUNT counters (zeroed)
+    int refresh_tiles;
+};
+
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ uint32_t ld_vol_shared(const uint32_t* p) {
+    return *reinterpret_cast<const volatile uint32_t*>(p);
+}
+
+__device__ __forceinline__ uint32_t row_word_mask(int w, int n) {
+    const int rem = n - (w << 5);
+    return rem >= 32 ? 0xffffffffu : ((1u << rem) - 1u);
+}
+
+// Exact test of one (voxel, cell) pair with directions from the global tables.
+__device__ __forceinline__ bool exact_pair(const StreamParams& p, float4 q, int cell) {
+    const int i = cell / p.grid.n, j = cell - i * p.grid.n;
+    const float* t = p.tab;
+    const float cph = __ldg(t + i), sph = __ldg(t + p.grid.m + i);
+    const float cg = __ldg(t + 2 * p.grid.m + j), sg = __ldg(t + 2 * p.grid.m + p.grid.n + j);
+    return exact_hit(q.x - p.px, q.y - p.py, q.z - p.pz, q.w, sph * cg, sph * sg, cph, p.tool);
+}
+
+struct Counters {
+    unsigned long long streamed = 0, culled = 0, skipped = 0, live = 0, rows = 0, band = 0,
+                       overflow = 0;
+};
+
+// Are all rows i0..i1 full (bit set in sRowFull)?
+__device__ __forceinline__ bool rows_all_full(const uint32_t* sRowFull, int i0, int i1) {
+    for (int w = i0 >> 5; w <= (i1 >> 5); ++w) {
+        uint32_t need = 0xffffffffu;
+        if (w == (i0 >> 5)) need &= 0xffffffffu << (i0 & 31);
+        if (w == (i1 >> 5)) need &= 0xffffffffu >> (31 - (i1 & 31));
+        if ((ld_vol_shared(sRowFull + w) & need) != need) return false;
+    }
+    return true;
+}
+
+__device__ void fill_all(const StreamParams& p, uint32_t* sAM) {
+    const int W = p.grid.W;
+    for (int i = 0; i < p.grid.m; ++i)
+        for (int w = 0; w < W; ++w) atomicOr(sAM + i * W + w, row_word_mask(w, p.grid.n));
+}
+
+__device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, unsigned int vidx,
+                                          float4 q, int cell, uint32_t* wp, uint32_t bit,
+                                          Counters& cnt) {
+    cnt.band++;
+    const unsigned long long slot = atomicAdd(p.qcount, 1ULL);
+    if ((long long)slot < p.qcap) {
+        p.queue[slot] = ((unsigned long long)vidx << 32) | (unsigned int)cell;
+    } else {
+        // queue full: resolve inline (rare; keeps the result exact)
+        cnt.overflow++;
+        if (exact_pair(p, q, cell)) atomicOr(wp, bit);
+    }
+}
+
+// Steps a2-a5 for one voxel.
+__device__ __forceinline__ void process_voxel(const StreamParams& p, unsigned int vidx, float4 q,
+                                              uint32_t* sAM, const uint32_t* sRowFull,
+                                              const float* sCos, const float* sSin, Counters& cnt) {
+    const ToolDev& T = p.tool;
+    const GridDev& g = p.grid;
+    const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
+    cnt.streamed++;
+    // the pivot lies in the closed box: the tool (which contains the pivot) hits it everywhere
+    if (fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
+        fill_all(p, sAM);
+        return;
+    }
+    const float D2 = vx * vx + vy * vy + vz * vz;
+    const float D = sqrtf(D2);
+    const float r2 = kSqrt3 * h;
+    // a2: reach cull -- every tool point is within rho_max of the pivot
+    if (D - r2 > T.rho_max + kRadRel * (D + r2)) {
+        cnt.culled++;
+        return;
+    }
+    // a3: cone axis
+    const float rxy = sqrtf(vx * vx + vy * vy);
+    const float phv = atan2f(rxy, vz);
+    // cheap outer bound: a sphere of radius r2 at distance D can only touch
+    // cylinders that start within D + r2, all of radius <= Reff, so its blocked
+    // angles satisfy sin(theta) <= (Reff + r2) / D
+    const float reach = D + r2 + kRadRel * (D + r2);
+    float Reff = 0.f;
+    for (int k = 0; k < T.ncyl; ++k)
+        if (T.z0[k] <= reach) Reff = T.Rpm[k];
+    const float s = (Reff + r2) / D * (1.f + 8e-6f) + 1e-6f;
+    const float ac = (s >= 1.f) ? kPi : asinf(s);
+    int i0 = max(0, (int)ceilf((phv - ac - kRowSlack) * g.inv_dphi - 0.5f));
+    int i1 = min(g.m - 1, (int)floorf((phv + ac + kRowSlack) * g.inv_dphi - 0.5f));
+    if (i0 > i1 || rows_all_full(sRowFull, i0, i1)) {
+        cnt.skipped++;
+        return;
+    }
+    // a4: the two cones
+    cnt.live++;
+    const Cones c = tool_cones(D, h, T);
+    if (c.cout > 1.f) return;
+    const float ao = acosf(fmaxf(c.cout, -1.f));
+    i0 = max(i0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+    i1 = min(i1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+    const float invD = 1.f / D;
+    const float cphv = vz * invD, sphv = rxy * invD;
+    const float gv = atan2f(vy, vx);
+    const int W = g.W;
+    // a5: rasterise row by row
+    for (int i = i0; i <= i1; ++i) {
+        if ((ld_vol_shared(sRowFull + (i >> 5)) >> (i & 31)) & 1u) continue;
+        const float base = sCos[i] * cphv, den = sSin[i] * sphv;
+        const Interval O = gamma_interval(c.cout, base, den, gv, +1, g);
+        if (O.len == 0) continue;
+        cnt.rows++;
+        const Interval In = gamma_interval(c.cin, base, den, gv, -1, g);
+        const Interval X = gamma_interval(c.clo, base, den, gv, -1, g);
+        for (int w = 0; w < W; ++w) {
+            uint32_t ob = interval_bits(O, w, g.n);
+            if (!ob) continue;
+            const uint32_t xb = interval_bits(X, w, g.n);
+            const uint32_t ib = interval_bits(In, w, g.n) & ~xb;
+            ob &= ~xb;
+            uint32_t* wp = sAM + i * W + w;
+            uint32_t cur = ld_vol_shared(wp);
+            if (ib & ~cur) {
+                atomicOr(wp, ib);
+                cur |= ib;
+            }
+            uint32_t band = ob & ~ib & ~cur;
+            while (band) {
+                const int b = __ffs(band) - 1;
+                band &= band - 1u;
+                push_band(p, sAM, vidx, q, i * g.n + (w << 5) + b, wp, 1u << b, cnt);
+            }
+        }
+    }
+}
+
+// a7: merge the CTA's shared AM with the global AM (one atomicOr per word that
+// gained bits), read the union back, recompute the row-full bits.  Returns
+// true when the whole AM is blocked (early exit).
+__device__ bool cta_merge(const StreamParams& p, uint32_t* sAM, uint32_t* sShadow,
+                          uint32_t* sRowFull, int* sCount) {
+    const int MW = p.grid.m * p.grid.W;
+    const int W = p.grid.W;
+    __syncthreads();
+    if (threadIdx.x == 0) *sCount = 0;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        const uint32_t s = sAM[w];
+        uint32_t gv;
+        if (s & ~sShadow[w])
+            gv = atomicOr(p.gam + w, s) | s;
+        else
+            gv = ld_cg(p.gam + w) | s;
+        sAM[w] = gv;
+        sShadow[w] = gv;
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int base = 0; base < p.grid.m; base += blockDim.x) {
+        const int i = base + threadIdx.x;
+        bool full = false;
+        if (i < p.grid.m) {
+            full = true;
+            for (int w = 0; w < W; ++w)
+                if (sAM[i * W + w] != row_word_mask(w, p.grid.n)) full = false;
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, full);
+        if (lane == 0 && base + warp * 32 < p.grid.m) {
+            sRowFull[(base + warp * 32) >> 5] = bal;
+            atomicAdd(sCount, __popc(bal));
+        }
+    }
+    __syncthreads();
+    return *sCount == p.grid.m;
+}
+
+__global__ void __launch_bounds__(kThreads, 4) aica_stream_kernel(const StreamParams p) {
+    extern __shared__ uint32_t smem[];
+    __shared__ int sCount;
+    const int m = p.grid.m;
+    const int MW = m * p.grid.W;
+    uint32_t* sAM = smem;
+    uint32_t* sShadow = sAM + MW;
+    uint32_t* sRowFull = sShadow + MW;
+    float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
+    float* sSin = sCos + m;
+    for (int i = threadIdx.x; i < m; i += blockDim.x) {
+        sCos[i] = p.tab[i];
+        sSin[i] = p.tab[m + i];
+    }
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        sAM[w] = 0u;
+        sShadow[w] = 0u;
+    }
+    Counters cnt;
+    bool early = cta_merge(p, sAM, sShadow, sRowFull, &sCount);
+    const long long ntiles = (p.N + kTile - 1) / kTile;
+    int since = 0;
+    for (long long t = blockIdx.x; t < ntiles && !early; t += gridDim.x) {
+        if (since == p.refresh_tiles) {
+            since = 0;
+            early = cta_merge(p, sAM, sShadow, sRowFull, &sCount);
+            if (early) break;
+        }
+        ++since;
+        float4 q[kVPT];
+        const long long base = t * kTile + threadIdx.x;
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) {
+            const long long idx = base + (long long)k * kThreads;
+            q[k] = idx < p.N ? __ldcs(p.vox + idx) : make_float4(0.f, 0.f, 0.f, -1.f);
+        }
+#pragma unroll 1
+        for (int k = 0; k < kVPT; ++k) {
+            if (q[k].w > 0.f)
+                process_voxel(p, (unsigned int)(base + (long long)k * kThreads), q[k], sAM, sRowFull,
+                              sCos, sSin, cnt);
+        }
+    }
+    // final flush of words that gained bits
+    __syncthreads();
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        const uint32_t s = sAM[w];
+        if (s & ~sShadow[w]) atomicOr(p.gam + w, s);
+    }
+    // counters: warp-reduce then one atomic per warp
+    unsigned long long vals[7] = {cnt.streamed, cnt.culled, cnt.skipped, cnt.live, cnt.rows,
+                                  cnt.band, cnt.overflow};
+    const int idx[7] = {ST_STREAMED, ST_CULLED, ST_SKIPPED, ST_LIVE, ST_ROWS, ST_BAND, ST_OVERFLOW};
+#pragma unroll
+    for (int k = 0; k < 7; ++k) {
+        unsigned long long v = vals[k];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if ((threadIdx.x & 31) == 0 && v) atomicAdd(p.stats + idx[k], v);
+    }
+    if (early && threadIdx.x == 0) atomicMax(reinterpret_cast<unsigned long long*>(p.stats + ST_EARLY), 1ULL);
+}
+
+// a6: exact test for queued band pairs whose AM bit is still clear.
+__global__ void __launch_bounds__(kThreads) band_exact_kernel(const StreamParams p) {
+    const unsigned long long cnt = *p.qcount;
+    const long long n = (long long)(cnt < (unsigned long long)p.qcap ? cnt : (unsigned long long)p.qcap);
+    unsigned long long tests = 0, hits = 0;
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < n;
+         k += (long long)gridDim.x * blockDim.x) {
+        const unsigned long long e = p.queue[k];
+        const unsigned int vidx = (unsigned int)(e >> 32);
+        const int cell = (int)(e & 0xffffffffu);
+        const int i = cell / p.grid.n, j = cell - i * p.grid.n;
+        uint32_t* wp = p.gam + i * p.grid.W + (j >> 5);
+        const uint32_t bit = 1u << (j & 31);
+        if (ld_cg(wp) & bit) continue;
+        ++tests;
+        if (exact_pair(p, p.vox[vidx], cell)) {
+            ++hits;
+            atomicOr(wp, bit);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        tests += __shfl_xor_sync(0xffffffffu, tests, o);
+        hits += __shfl_xor_sync(0xffffffffu, hits, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (tests) atomicAdd(p.stats + ST_EXACT, tests);
+        if (hits) atomicAdd(p.stats + ST_EXACT_HIT, hits);
+    }
+}
+
+// a9: baseline -- CHECKBOX for every (voxel, cell) pair, one CTA per cell,
+// stopping at the first collision (Alg. 2).  `reject` enables an
+// exact-safe bounding-sphere reject (circumscribed ball vs each cylinder).
+__global__ void __launch_bounds__(kThreads) baseline_kernel(const StreamParams p, int reject) {
+    const int ncell = p.grid.m * p.grid.n;
+    for (int cell = blockIdx.x; cell < ncell; cell += gridDim.x) {
+        const int i = cell / p.grid.n, j = cell - i * p.grid.n;
+        const float cph = __ldg(p.tab + i), sph = __ldg(p.tab + p.grid.m + i);
+        const float cg = __ldg(p.tab + 2 * p.grid.m + j), sg = __ldg(p.tab + 2 * p.grid.m + p.grid.n + j);
+        const float dx = sph * cg, dy = sph * sg, dz = cph;
+        int found = 0;
+        for (long long b = 0; b < p.N; b += blockDim.x) {
+            const long long idx = b + threadIdx.x;
+            int hit = 0;
+            if (idx < p.N) {
+                const float4 q = __ldg(p.vox + idx);
+                const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz;
+                bool cand = true;
+                if (reject) {
+                    // circumscribed ball (grown) vs each cylinder, 2-D meridian distance
+                    const float a = vx * dx + vy * dy + vz * dz;
+                    const float ex = vx - a * dx, ey = vy - a * dy, ez = vz - a * dz;
+                    const float rho = sqrtf(ex * ex + ey * ey + ez * ez);
+                    const float r2 = kSqrt3 * q.w * (1.f + 1e-5f) + 1e-5f * (fabsf(a) + rho);
+                    cand = false;
+                    for (int k = 0; k < p.tool.ncyl; ++k) {
+                        const float da = a < p.tool.z0[k] ? p.tool.z0[k] - a
+                                                          : (a > p.tool.z1[k] ? a - p.tool.z1[k] : 0.f);
+                        const float dr = fmaxf(rho - p.tool.R[k], 0.f);
+                        if (da * da + dr * dr <= r2 * r2) cand = true;
+                    }
+                }
+                hit = cand && exact_hit(vx, vy, vz, q.w, dx, dy, dz, p.tool);
+            }
+            if (__syncthreads_or(hit)) { found = 1; break; }
+        }
+        if (threadIdx.x == 0 && found) atomicOr(p.gam + i * p.grid.W + (j >> 5), 1u << (j & 31));
+    }
+}
+
+// ---------------------------------------------------------------- upload helpers
+
+__device__ __forceinline__ unsigned int float_to_ordered(float f) {
+    const unsigned int u = __float_as_uint(f);
+    return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__device__ __forceinline__ float ordered_to_float(unsigned int u) {
+    return __uint_as_float((u & 0x80000000u) ? (u & 0x7fffffffu) : ~u);
+}
+
+// Validate, pack to float4 and take the bounding box (ordered-int atomics).
+__global__ void pack_validate_kernel(const float* __restrict__ c, const float* __restrict__ h,
+                                     long long N, float4* __restrict__ out, unsigned int* bbox,
+                                     unsigned long long* bad) {
+    unsigned int lo[3] = {0xffffffffu, 0xffffffffu, 0xffffffffu}, hi[3] = {0u, 0u, 0u};
+    unsigned long long nbad = 0;
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < N;
+         k += (long long)gridDim.x * blockDim.x) {
+        const float x = c[3 * k], y = c[3 * k + 1], z = c[3 * k + 2], s = h[k];
+        const bool ok = isfinite(x) && isfinite(y) && isfinite(z) && isfinite(s) && s > 0.f;
+        nbad += !ok;
+        out[k] = make_float4(x, y, z, s);
+        if (ok) {
+            const unsigned int o[3] = {float_to_ordered(x), float_to_ordered(y), float_to_ordered(z)};
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+                lo[a] = min(lo[a], o[a]);
+                hi[a] = max(hi[a], o[a]);
+            }
+        }
+    }
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            lo[a] = min(lo[a], __shfl_xor_sync(0xffffffffu, lo[a], o));
+            hi[a] = max(hi[a], __shfl_xor_sync(0xffffffffu, hi[a], o));
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) nbad += __shfl_xor_sync(0xffffffffu, nbad, o);
+    if ((threadIdx.x & 31) == 0) {
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            atomicMin(bbox + a, lo[a]);
+            atomicMax(bbox + 3 + a, hi[a]);
+        }
+        if (nbad) atomicAdd(bad, nbad);
+    }
+}
+
+__device__ __forceinline__ unsigned long long spread3(unsigned int v) {
+    unsigned long long x = v & 0x1fffffu;
+    x = (x | x << 32) & 0x1f00000000ffffULL;
+    x = (x | x << 16) & 0x1f0000ff0000ffULL;
+    x = (x | x << 8) & 0x100f00f00f00f00fULL;
+    x = (x | x << 4) & 0x10c30c30c30c30c3ULL;
+    x = (x | x << 2) & 0x1249249249249249ULL;
+    return x;
+}
+
+__global__ void morton_keys_kernel(const float4* __restrict__ v, long long N, const unsigned int* bbox,
+                                   unsigned long long* keys, unsigned int* ids) {
+    const float lx = ordered_to_float(bbox[0]), ly = ordered_to_float(bbox[1]), lz = ordered_to_float(bbox[2]);
+    const float hx = ordered_to_float(bbox[3]), hy = ordered_to_float(bbox[4]), hz = ordered_to_float(bbox[5]);
+    const float ext = fmaxf(fmaxf(hx - lx, hy - ly), fmaxf(hz - lz, 1e-30f));
+    const float sc = 2097151.f / ext;
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < N;
+         k += (long long)gridDim.x * blockDim.x) {
+        const float4 q = v[k];
+        const unsigned int qx = (unsigned int)fminf(fmaxf((q.x - lx) * sc, 0.f), 2097151.f);
+        const unsigned int qy = (unsigned int)fminf(fmaxf((q.y - ly) * sc, 0.f), 2097151.f);
+        const unsigned int qz = (unsigned int)fminf(fmaxf((q.z - lz) * sc, 0.f), 2097151.f);
+        keys[k] = spread3(qx) | spread3(qy) << 1 | spread3(qz) << 2;
+        ids[k] = (unsigned int)k;
+    }
+}
+
+__global__ void gather_kernel(const float4* __restrict__ src, const unsigned int* __restrict__ ids,
+                              long long N, float4* __restrict__ dst) {
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < N;
+         k += (long long)gridDim.x * blockDim.x)
+        dst[k] = src[ids[k]];
+}
+
+}  // namespace am

@@ -1,0 +1,223 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Rule (north_star): every cell the oracle calls robust
+(state 0 or 2) must match exactly -- zero mismatches; band cells (state 1)
+accept either value and are counted.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import scenes
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def am(gpu):
+    import paper_conf_icpp_chenktkv19_b200 as am
+    return am
+
+
+def _compare(gpu_map, states):
+    robust = states != 1
+    mism = int(((gpu_map == 1) != (states == 2))[robust].sum())
+    return mism, int((~robust).sum())
+
+
+def _ctx(am, cfg, C, H, m=None, n=None, tool=None):
+    ctx = am.Context(tool or cfg.tool, m or cfg.m, n or cfg.n, device=0)
+    ctx.upload(C, H)
+    return ctx
+
+
+@pytest.mark.parametrize("name,npiv", [("C1", 2), ("T_head", 4), ("T_head4", 3), ("T_blade", 2), ("T_imp", 2)])
+def test_small_configs_full_am(am, name, npiv):
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    for p in cfg.pivots(npiv):
+        gmap = ctx.am(p)
+        S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n)
+        mism, band = _compare(gmap, S)
+        assert mism == 0, (name, p, mism, band)
+        base = am.unpack(ctx.compute_baseline(p), cfg.m, cfg.n)
+        mism_b, _ = _compare(base, S)
+        assert mism_b == 0, (name, p, mism_b)
+    ctx.close()
+
+
+def _random_scene(rng, nvox, spread, hmin, hmax):
+    piv = rng.uniform(-5, 5, 3).astype(np.float32)
+    dirs = rng.normal(size=(nvox, 3))
+    dirs /= np.linalg.norm(dirs, axis=1, keepdims=True)
+    dist = spread * rng.random(nvox) ** 0.7
+    C = (piv[None, :] + dirs * dist[:, None]).astype(np.float32)
+    H = np.exp(rng.uniform(math.log(hmin), math.log(hmax), nvox)).astype(np.float32)
+    # keep the pivot outside every voxel (that case has its own test)
+    inside = np.all(np.abs(C - piv[None, :]) <= H[:, None], axis=1)
+    return piv, C[~inside], H[~inside]
+
+
+TOOLS = {
+    "3cyl": scenes.TOOL_3CYL,
+    "paper4": scenes.TOOL_PAPER4,
+    "nonmono": ((3.0, 10.0), (1.5, 20.0), (5.0, 15.0), (2.0, 30.0)),  # radii go down and up
+    "short": ((4.0, 6.0),),
+}
+
+
+@pytest.mark.parametrize("tool_name", list(TOOLS))
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_random_scenes(am, tool_name, seed):
+    """Scattered voxels of mixed sizes at all distances, including beyond the
+    tool end (ring voxels) and next to the pivot (cones wider than 90 deg)."""
+    rng = np.random.default_rng(100 + seed)
+    tool = TOOLS[tool_name]
+    L = sum(t[1] for t in tool)
+    piv, C, H = _random_scene(rng, 150, 1.3 * L, 0.05, 3.0)
+    m, n = (40, 48) if seed != 2 else (17, 70)
+    ctx = am.Context(tool, m, n, device=0)
+    ctx.upload(C, H)
+    gmap = ctx.am(piv)
+    S = oracle.am_states(C, H, tool, piv, m, n)
+    mism, band = _compare(gmap, S)
+    assert mism == 0, (tool_name, seed, mism, band)
+    base = am.unpack(ctx.compute_baseline(piv), m, n)
+    assert _compare(base, S)[0] == 0
+    ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_single_voxels(am, seed):
+    """One voxel per map: every cone and band path in isolation."""
+    rng = np.random.default_rng(7 + seed)
+    tool = TOOLS[["3cyl", "paper4", "nonmono", "short"][seed]]
+    L = sum(t[1] for t in tool)
+    ctx = am.Context(tool, 32, 64, device=0)
+    for k in range(40):
+        piv, C, H = _random_scene(rng, 1, 1.2 * L, 0.02, 4.0)
+        if len(H) == 0:
+            continue
+        ctx.upload(C, H)
+        gmap = ctx.am(piv)
+        S = oracle.am_states(C, H, tool, piv, 32, 64)
+        assert _compare(gmap, S)[0] == 0, (seed, k, C, H, piv)
+    ctx.close()
+
+
+def test_edge_cases(am):
+    tool = scenes.TOOL_3CYL
+    ctx = am.Context(tool, 16, 33, device=0)
+    # empty model
+    ctx.upload(np.zeros((0, 3), np.float32), np.zeros(0, np.float32))
+    assert (ctx.am((0, 0, 0)) == 0).all()
+    # out of reach
+    ctx.upload(np.array([[400.0, 0, 0]], np.float32), np.array([1.0], np.float32))
+    assert (ctx.am((0, 0, 0)) == 0).all()
+    # pivot inside a voxel
+    ctx.upload(np.array([[0.3, -0.2, 0.1]], np.float32), np.array([0.5], np.float32))
+    assert (ctx.am((0, 0, 0)) == 1).all()
+    # padding bits stay zero
+    w, _ = ctx.compute((0, 0, 0))
+    assert (w.reshape(16, 2)[:, 1] == 1).all()
+    ctx.close()
+
+
+def test_enclosing_shell_early_exit(am):
+    C, H = scenes.octree_leaves("shell", (24.0, 20.0), (-32, -32, -32), 64.0, 6)
+    ctx = am.Context(scenes.TOOL_3CYL, 64, 64, device=0)
+    ctx.upload(C, H)
+    w, st = ctx.compute((0.5, -0.25, 0.3), stats=True)
+    assert (am.unpack(w, 64, 64) == 1).all()
+    assert st.voxels_streamed <= len(H)
+    ctx.close()
+
+
+@pytest.mark.parametrize("m,n", [(1, 1), (1, 64), (5, 1), (33, 95), (64, 1024), (200, 32)])
+def test_grid_shapes(am, m, n):
+    cfg = scenes.CONFIGS["T_head"]
+    C, H = cfg.leaves()
+    p = cfg.pivots(1)[0]
+    ctx = am.Context(cfg.tool, m, n, device=0)
+    ctx.upload(C, H)
+    S = oracle.am_states(C, H, cfg.tool, p, m, n)
+    assert _compare(ctx.am(p), S)[0] == 0
+    ctx.close()
+
+
+def test_batch_device_host_and_sort_invariance(am):
+    import torch
+    cfg = scenes.CONFIGS["T_head"]
+    C, H = cfg.leaves()
+    P = cfg.pivots(5)
+    ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=0)
+    ctx.upload(torch.from_numpy(C).cuda(), torch.from_numpy(H).cuda())
+    single = np.stack([ctx.compute(p)[0] for p in P])
+    batch = ctx.compute_batch(P)
+    assert np.array_equal(single, batch)
+    dev = torch.zeros((len(P), ctx.words), dtype=torch.int32, device="cuda:0")
+    ctx.compute_batch(P, out=dev)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy().view(np.uint32), batch)
+    # unsorted upload and a permuted model give the same maps
+    ctx2 = am.Context(cfg.tool, cfg.m, cfg.n, device=0)
+    ctx2.set_option(am.binding.OPT_MORTON_SORT, 0)
+    perm = np.random.default_rng(0).permutation(len(H))
+    ctx2.upload(C[perm], H[perm])
+    assert np.array_equal(ctx2.compute_batch(P), batch)
+    ctx.close()
+    ctx2.close()
+
+
+def test_small_queue_overflow_is_exact(am):
+    cfg = scenes.CONFIGS["T_head"]
+    C, H = cfg.leaves()
+    p = cfg.pivots(1)[0]
+    ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=0)
+    ctx.upload(C, H)
+    ref, st = ctx.compute(p, stats=True)
+    ctx.set_option(am.binding.OPT_BAND_QUEUE, 3)
+    out, st2 = ctx.compute(p, stats=True)
+    assert st2.queue_overflow > 0 or st.band_pairs <= 3
+    S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n)
+    assert _compare(am.unpack(out, cfg.m, cfg.n), S)[0] == 0
+    ctx.close()
+
+
+def test_sphere_cap_bounds_gpu(am):
+    """P3 directly on the GPU map (not only via the oracle)."""
+    cfg = scenes.CONFIGS["C1"]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    g = ctx.am((0, 0, 31.0))
+
+    def thc(Rs, Dp, R):
+        if math.sqrt(Dp * Dp - Rs * Rs) <= R:
+            return math.acos(Rs / Dp)
+        return math.asin((Dp * Dp + R * R - Rs * Rs) / (2 * Dp * R))
+    lo, hi = thc(28 + 2 * math.sqrt(3) * 0.5, 31, 6.35), thc(28, 31, 6.35)
+    phi = (np.arange(32) + 0.5) * math.pi / 32
+    assert (g[phi < lo - 1e-4] == 0).all() and (g[phi > hi + 1e-4] == 1).all()
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", ["C2"])
+def test_c2_full_size_sampled(am, name):
+    """C2 (~2M leaves) at full size: all GPU-clear cells plus a seeded sample of
+    blocked cells are checked cell by cell against the oracle."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    rng = np.random.default_rng(11)
+    for p in cfg.pivots(2):
+        g = ctx.am(p).reshape(-1)
+        clear = np.nonzero(g == 0)[0]
+        blocked = np.nonzero(g == 1)[0]
+        cells = np.concatenate([clear[:48], rng.choice(blocked, size=min(48, len(blocked)), replace=False)])
+        S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n, cells=cells)
+        robust = S != 1
+        assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
+    ctx.close()
