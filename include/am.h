@@ -79,7 +79,9 @@ enum {
     AM_OPT_MORTON_SORT = 3,      /* 1 = Morton-sort voxels at upload (default), 0 = keep order   */
     AM_OPT_BASELINE_REJECT = 4,  /* 1 = baseline uses an exact-safe bounding-sphere reject        */
     AM_OPT_BAND_QUEUE = 5,       /* capacity of the deferred band queue, in (voxel, cell) pairs  */
-    AM_OPT_KERNEL_TIMING = 6     /* 1 = bracket every streaming-kernel launch with CUDA events   */
+    AM_OPT_KERNEL_TIMING = 6,    /* 1 = bracket every full-stream kernel launch with CUDA events */
+    AM_OPT_PHASES = 7            /* 1 = coarse levels + clear-direction map before the full
+                                    stream (default); 0 = one plain stream.  Same map either way */
 };
 
 /*

@@ -45,6 +45,13 @@ struct am_ctx {
     int baseline_reject = 0;
     size_t smem = 0;
     int occ = 0;
+    // coarse levels (largest voxels + a strided sample) and the clear-direction map
+    float4* d_coarse = nullptr;
+    long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
+    float4* d_texels = nullptr;            // cube-map texel centres (xyz) + angular radius (w)
+    float* d_cmap = nullptr;
+    int cmapT = 32;
+    int phases = 1;
     // kernel timing (AM_OPT_KERNEL_TIMING)
     int timing = 0;
     std::vector<cudaEvent_t> ev_start, ev_stop;
@@ -108,7 +115,50 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.queue = c->d_queue;
     p.qcap = c->qcap;
     p.refresh_tiles = c->refresh_tiles;
+    p.vox_main = c->d_vox;
+    p.vox_coarse = c->d_coarse;
+    p.cmapT = c->cmapT;
     return p;
+}
+
+// Cube-map texels: centre direction and an angular radius bounding every
+// direction cube_texel() maps into the texel (max angle to the 4 corners of a
+// convex spherical quadrilateral, plus slack for fp32 rounding at the edges).
+std::vector<float> make_texels(int T) {
+    std::vector<float> out((size_t)6 * T * T * 4);
+    auto dir = [](int face, double u, double w, double* d) {
+        const int a = face >> 1;
+        const double sg = (face & 1) ? -1.0 : 1.0;
+        double v[3];
+        if (a == 0) { v[0] = sg; v[1] = u; v[2] = w; }
+        else if (a == 1) { v[0] = u; v[1] = sg; v[2] = w; }
+        else { v[0] = u; v[1] = w; v[2] = sg; }
+        const double nn = std::sqrt(v[0] * v[0] + v[1] * v[1] + v[2] * v[2]);
+        for (int k = 0; k < 3; ++k) d[k] = v[k] / nn;
+    };
+    for (int f = 0; f < 6; ++f)
+        for (int iw = 0; iw < T; ++iw)
+            for (int iu = 0; iu < T; ++iu) {
+                const double u0 = -1.0 + 2.0 * iu / T, u1 = -1.0 + 2.0 * (iu + 1) / T;
+                const double w0 = -1.0 + 2.0 * iw / T, w1 = -1.0 + 2.0 * (iw + 1) / T;
+                double c[3];
+                dir(f, 0.5 * (u0 + u1), 0.5 * (w0 + w1), c);
+                double r = 0.0;
+                const double us[2] = {u0, u1}, ws[2] = {w0, w1};
+                for (double uu : us)
+                    for (double ww : ws) {
+                        double d[3];
+                        dir(f, uu, ww, d);
+                        const double dp = std::min(1.0, c[0] * d[0] + c[1] * d[1] + c[2] * d[2]);
+                        r = std::max(r, std::acos(dp));
+                    }
+                const size_t t = ((size_t)(f * T + iw) * T + iu) * 4;
+                out[t] = (float)c[0];
+                out[t + 1] = (float)c[1];
+                out[t + 2] = (float)c[2];
+                out[t + 3] = (float)(r + 2e-5);
+            }
+    return out;
 }
 
 int ensure_queue(am_ctx* ctx, long long cap) {
@@ -134,17 +184,21 @@ int configure_launch(am_ctx* ctx) {
     return AM_OK;
 }
 
-// One AICA map into device buffer gam (asynchronous on s).
-int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
-    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
-    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
-    if (ctx->N == 0) return AM_OK;
-    StreamParams p = make_params(ctx, pivot, gam);
-    const long long ntiles = (ctx->N + kTile - 1) / kTile;
+// One launch of the voxel-streaming kernel over vox[0, n).
+int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, unsigned int vbase,
+                  unsigned int vtag, const float* cmap, bool timed, cudaStream_t s) {
+    if (n <= 0) return AM_OK;
+    p.vox = vox;
+    p.N = n;
+    p.vbase = vbase;
+    p.vtag = vtag;
+    p.cmap = cmap;
+    const long long ntiles = (n + kTile - 1) / kTile;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
     if (g > ntiles) g = ntiles;
     if (g < 1) g = 1;
-    if (ctx->timing) {
+    timed = timed && ctx->timing;
+    if (timed) {
         if (ctx->ev_used == ctx->ev_start.size()) {
             cudaEvent_t a, b;
             CK(cudaEventCreate(&a));
@@ -156,7 +210,42 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     }
     aica_stream_kernel<<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
     CK(cudaGetLastError());
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    return AM_OK;
+}
+
+int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
+    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+    clear_map_kernel<<<(ntex + 7) / 8, 256, 0, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_texels, ntex,
+                                                    ctx->d_cmap);
+    CK(cudaGetLastError());
+    return AM_OK;
+}
+
+// One AICA map into device buffer gam (asynchronous on s):
+//   level 0 (largest voxels) -> clear map -> level 1 (next largest + strided
+//   sample) -> clear map -> every voxel, skipping those whose cheap cone misses
+//   every still-clear cell -> deferred band.  The coarse levels only make the
+//   skip test effective; each level is a subset of the model, so the map is the
+//   same with or without them (AM_OPT_PHASES).
+int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
+    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
+    if (ctx->N == 0) return AM_OK;
+    StreamParams p = make_params(ctx, pivot, gam);
+    int rc;
+    const float* cm = nullptr;
+    if (ctx->phases && ctx->n_l0 > 0) {
+        constexpr unsigned int kCoarse = 0x80000000u;
+        if ((rc = launch_stream(ctx, p, ctx->d_coarse, ctx->n_l0, 0, kCoarse, nullptr, false, s))) return rc;
+        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
+        if ((rc = launch_stream(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0,
+                                (unsigned int)ctx->n_l0, kCoarse, ctx->d_cmap, false, s)))
+            return rc;
+        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
+        cm = ctx->d_cmap;
+    }
+    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, 0, 0, cm, true, s))) return rc;
     band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     return AM_OK;
@@ -258,6 +347,15 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         return bail(AM_ENOMEM);
     }
     ctx->am_cap_maps = 1;
+    {
+        const std::vector<float> tex = make_texels(ctx->cmapT);
+        if (cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)) != cudaSuccess ||
+            cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
+            cudaMalloc(&ctx->d_cmap, tex.size() / 4 * sizeof(float)) != cudaSuccess) {
+            cudaGetLastError();
+            return bail(AM_ENOMEM);
+        }
+    }
     if ((rc = ensure_queue(ctx, 1 << 22)) != AM_OK) return bail(rc);
     if ((rc = configure_launch(ctx)) != AM_OK) return bail(rc);
     *out = ctx;
@@ -358,6 +456,56 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
         UK(cudaGetLastError());
     } else {
         UK(cudaMemcpy(ctx->d_vox, raw, (size_t)N * sizeof(float4), cudaMemcpyDeviceToDevice));
+    }
+    // coarse levels for the clear-direction map: level 0 = the n0 largest
+    // voxels, level 1 = the next ones up to n1 plus every 512th voxel
+    cudaFree(ctx->d_coarse);
+    ctx->d_coarse = nullptr;
+    ctx->n_l0 = ctx->n_l1 = 0;
+    if (N >= 2048) {
+        const long long n0 = std::min<long long>(N, std::max<long long>(1024, N / 2048));
+        const long long n1 = std::min<long long>(N, std::max<long long>(8192, N / 256));
+        const long long stride = 512, ns = N / stride;
+        unsigned int *sk = nullptr, *sk2 = nullptr, *si = nullptr, *si2 = nullptr, *cid = nullptr;
+        void* ct = nullptr;
+        auto cfree = [&]() {
+            cudaFree(sk); cudaFree(sk2); cudaFree(si); cudaFree(si2); cudaFree(cid); cudaFree(ct);
+        };
+#define CUK(call)                                                                              \
+        do {                                                                                   \
+            cudaError_t e_ = (call);                                                           \
+            if (e_ != cudaSuccess) {                                                           \
+                cudaGetLastError();                                                            \
+                cfree();                                                                       \
+                cleanup();                                                                     \
+                return fail(ctx, e_ == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA, "%s: %s", #call, \
+                            cudaGetErrorString(e_));                                           \
+            }                                                                                  \
+        } while (0)
+        CUK(cudaMalloc(&sk, (size_t)N * 4));
+        CUK(cudaMalloc(&sk2, (size_t)N * 4));
+        CUK(cudaMalloc(&si, (size_t)N * 4));
+        CUK(cudaMalloc(&si2, (size_t)N * 4));
+        CUK(cudaMalloc(&cid, (size_t)(n1 + ns) * 4));
+        size_keys_kernel<<<blocks, 256>>>(ctx->d_vox, N, sk, si);
+        CUK(cudaGetLastError());
+        size_t tb = 0;
+        CUK(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, sk, sk2, si, si2, (int)N, 0, 32));
+        CUK(cudaMalloc(&ct, tb));
+        CUK(cub::DeviceRadixSort::SortPairsDescending(ct, tb, sk, sk2, si, si2, (int)N, 0, 32));
+        CUK(cudaMemcpy(cid, si2, (size_t)n1 * 4, cudaMemcpyDeviceToDevice));
+        if (ns > 0) {
+            strided_ids_kernel<<<blocks, 256>>>(cid + n1, ns, stride);
+            CUK(cudaGetLastError());
+        }
+        CUK(cudaMalloc(&ctx->d_coarse, (size_t)(n1 + ns) * sizeof(float4)));
+        gather_kernel<<<blocks, 256>>>(ctx->d_vox, cid, n1 + ns, ctx->d_coarse);
+        CUK(cudaGetLastError());
+        CUK(cudaDeviceSynchronize());
+#undef CUK
+        cfree();
+        ctx->n_l0 = n0;
+        ctx->n_l1 = n1 + ns;
     }
     UK(cudaDeviceSynchronize());
 #undef UK
@@ -481,6 +629,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "kernel_timing must be 0 or 1");
         ctx->timing = (int)value;
         return AM_OK;
+    case AM_OPT_PHASES:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "phases must be 0 or 1");
+        ctx->phases = (int)value;
+        return AM_OK;
     default:
         return fail(ctx, AM_EINVAL, "unknown option %d", key);
     }
@@ -522,6 +674,9 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_am);
     cudaFree(ctx->d_ctr);
     cudaFree(ctx->d_queue);
+    cudaFree(ctx->d_coarse);
+    cudaFree(ctx->d_texels);
+    cudaFree(ctx->d_cmap);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

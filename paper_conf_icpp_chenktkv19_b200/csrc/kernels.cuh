@@ -44,7 +44,32 @@ struct StreamParams {
     long long qcap;
     unsigned long long* stats;     // ST_COUNT counters (zeroed)
     int refresh_tiles;
+    // band-queue voxel references: bit 31 of the queued index selects vox_coarse
+    const float4* __restrict__ vox_main;
+    const float4* __restrict__ vox_coarse;
+    unsigned int vtag;             // OR-ed into queued indices by this launch
+    unsigned int vbase;            // index of vox[0] within its array
+    // clear-direction map; nullptr = not yet built
+    const float* __restrict__ cmap;
+    int cmapT;                     // texels per cube-face side
 };
+
+// Cube-map texel of direction v (any length): face = dominant axis and sign,
+// (u, w) = the other two components over the dominant one.  The host computes
+// each texel's centre and an angular radius that bounds every direction this
+// exact function maps into the texel.
+__device__ __forceinline__ int cube_texel(float vx, float vy, float vz, int T) {
+    const float ax = fabsf(vx), ay = fabsf(vy), az = fabsf(vz);
+    int face;
+    float a, u, w;
+    if (ax >= ay && ax >= az) { face = vx >= 0.f ? 0 : 1; a = ax; u = vy; w = vz; }
+    else if (ay >= az)        { face = vy >= 0.f ? 2 : 3; a = ay; u = vx; w = vz; }
+    else                      { face = vz >= 0.f ? 4 : 5; a = az; u = vx; w = vy; }
+    const float s = 0.5f * (float)T / a;
+    const int iu = min(T - 1, max(0, (int)((u + a) * s)));
+    const int iw = min(T - 1, max(0, (int)((w + a) * s)));
+    return (face * T + iw) * T + iu;
+}
 
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) {
     uint32_t v;
@@ -127,9 +152,6 @@ __device__ __forceinline__ void process_voxel(const StreamParams& p, unsigned in
         cnt.culled++;
         return;
     }
-    // a3: cone axis
-    const float rxy = sqrtf(vx * vx + vy * vy);
-    const float phv = atan2f(rxy, vz);
     // cheap outer bound: a sphere of radius r2 at distance D can only touch
     // cylinders that start within D + r2, all of radius <= Reff, so its blocked
     // angles satisfy sin(theta) <= (Reff + r2) / D
@@ -138,6 +160,23 @@ __device__ __forceinline__ void process_voxel(const StreamParams& p, unsigned in
     for (int k = 0; k < T.ncyl; ++k)
         if (T.z0[k] <= reach) Reff = T.Rpm[k];
     const float s = (Reff + r2) / D * (1.f + 8e-6f) + 1e-6f;
+    if (p.cmap) {
+        // clear-direction map: U >= cos of the angle from any direction of this
+        // texel to the nearest still-clear cell.  The cone touches no clear cell
+        // when cos(cone) > U, i.e. U < 0 <= cos or U^2 < 1 - s^2 (s < 1).
+        const float U = __ldg(p.cmap + cube_texel(vx, vy, vz, p.cmapT));
+        if (s < 1.f && (U < 0.f || U * U < 1.f - s * s)) {
+            cnt.skipped++;
+            return;
+        }
+        if (s >= 1.f && U < -1.5f) {  // no clear cell left at all
+            cnt.skipped++;
+            return;
+        }
+    }
+    // a3: cone axis
+    const float rxy = sqrtf(vx * vx + vy * vy);
+    const float phv = atan2f(rxy, vz);
     const float ac = (s >= 1.f) ? kPi : asinf(s);
     int i0 = max(0, (int)ceilf((phv - ac - kRowSlack) * g.inv_dphi - 0.5f));
     int i1 = min(g.m - 1, (int)floorf((phv + ac + kRowSlack) * g.inv_dphi - 0.5f));
@@ -265,7 +304,7 @@ __global__ void __launch_bounds__(kThreads, 4) aica_stream_kernel(const StreamPa
 #pragma unroll 1
         for (int k = 0; k < kVPT; ++k) {
             if (q[k].w > 0.f)
-                process_voxel(p, (unsigned int)(base + (long long)k * kThreads), q[k], sAM, sRowFull,
+                process_voxel(p, (p.vbase + (unsigned int)(base + (long long)k * kThreads)) | p.vtag, q[k], sAM, sRowFull,
                               sCos, sSin, cnt);
         }
     }
@@ -289,6 +328,52 @@ __global__ void __launch_bounds__(kThreads, 4) aica_stream_kernel(const StreamPa
     if (early && threadIdx.x == 0) atomicMax(reinterpret_cast<unsigned long long*>(p.stats + ST_EARLY), 1ULL);
 }
 
+// Clear-direction map: for every cube-map texel t with centre c_t
+// and angular radius r_t, U_t >= cos(max(0, angle(c_t, nearest clear cell) - r_t)),
+// so any direction mapped to t is at least acos(U_t) away from every cell that
+// is still clear in `gam`; U_t = -2 when no cell is clear.  Cells only ever get
+// blocked, so a map built from a partial AM stays valid for the final one.
+// One warp per texel; lanes scan the AM words.
+__global__ void __launch_bounds__(256) clear_map_kernel(const uint32_t* __restrict__ gam, GridDev g,
+                                                        const float* __restrict__ tab,
+                                                        const float4* __restrict__ texels, int ntex,
+                                                        float* __restrict__ U) {
+    const int lane = threadIdx.x & 31;
+    const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * blockDim.x) >> 5;
+    const int MW = g.m * g.W;
+    for (int t = warp; t < ntex; t += nwarps) {
+        const float4 c = texels[t];
+        float best = -2.f;
+        for (int w = lane; w < MW; w += 32) {
+            const int i = w / g.W, wj = w - i * g.W;
+            uint32_t clear = ~ld_cg(gam + w) & row_word_mask(wj, g.n);
+            if (!clear) continue;
+            const float cph = __ldg(tab + i), sph = __ldg(tab + g.m + i);
+            const float zc = c.z * cph;
+            while (clear) {
+                const int b = __ffs(clear) - 1;
+                clear &= clear - 1u;
+                const int j = (wj << 5) + b;
+                const float xy = fmaf(c.x, __ldg(tab + 2 * g.m + j), c.y * __ldg(tab + 2 * g.m + g.n + j));
+                best = fmaxf(best, fmaf(sph, xy, zc));
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, o));
+        if (lane == 0) {
+            float u = -2.f;
+            if (best >= -1.5f) {
+                // round the nearest-cell angle down and the bound up (fp32 guards)
+                const float th = acosf(fminf(best + 2e-6f, 1.f));
+                const float r = c.w;
+                u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+            }
+            U[t] = u;
+        }
+    }
+}
+
 // a6: exact test for queued band pairs whose AM bit is still clear.
 __global__ void __launch_bounds__(kThreads) band_exact_kernel(const StreamParams p) {
     const unsigned long long cnt = *p.qcount;
@@ -304,7 +389,8 @@ __global__ void __launch_bounds__(kThreads) band_exact_kernel(const StreamParams
         const uint32_t bit = 1u << (j & 31);
         if (ld_cg(wp) & bit) continue;
         ++tests;
-        if (exact_pair(p, p.vox[vidx], cell)) {
+        const float4 q = (vidx & 0x80000000u) ? p.vox_coarse[vidx & 0x7fffffffu] : p.vox_main[vidx];
+        if (exact_pair(p, q, cell)) {
             ++hits;
             atomicOr(wp, bit);
         }
@@ -436,6 +522,22 @@ __global__ void morton_keys_kernel(const float4* __restrict__ v, long long N, co
         keys[k] = spread3(qx) | spread3(qy) << 1 | spread3(qz) << 2;
         ids[k] = (unsigned int)k;
     }
+}
+
+// Sort keys for the coarse levels: half-size bits (positive floats order as uints).
+__global__ void size_keys_kernel(const float4* __restrict__ v, long long N, unsigned int* keys,
+                                 unsigned int* ids) {
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < N;
+         k += (long long)gridDim.x * blockDim.x) {
+        keys[k] = __float_as_uint(v[k].w);
+        ids[k] = (unsigned int)k;
+    }
+}
+
+__global__ void strided_ids_kernel(unsigned int* ids, long long count, long long stride) {
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < count;
+         k += (long long)gridDim.x * blockDim.x)
+        ids[k] = (unsigned int)(k * stride);
 }
 
 __global__ void gather_kernel(const float4* __restrict__ src, const unsigned int* __restrict__ ids,

@@ -221,3 +221,43 @@ def test_c2_full_size_sampled(am, name):
         robust = S != 1
         assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "T_imp", "C2"])
+def test_phases_and_tunables_give_identical_maps(am, name):
+    """The coarse levels / clear-direction map, the grid size and the merge
+    period only decide which work is skipped: the map is a deterministic
+    function of the per-(voxel, cell) decisions, so it must be bit-identical."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    P = cfg.pivots(3)
+    ctx = _ctx(am, cfg, C, H)
+    ref = ctx.compute_batch(P)
+    ctx.set_option(am.binding.OPT_PHASES, 0)
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_PHASES, 1)
+    ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
+    ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.close()
+
+
+def test_c3_bench_config_sampled(am):
+    """C3 (~27M leaves) in the launch configuration bench.py times: every
+    GPU-clear cell (up to 64) and a seeded sample of blocked cells against the
+    oracle, one by one."""
+    cfg = scenes.CONFIGS["C3"]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    rng = np.random.default_rng(3)
+    p = cfg.pivots(1)[0]
+    g = ctx.am(p).reshape(-1)
+    clear = np.nonzero(g == 0)[0]
+    blocked = np.nonzero(g == 1)[0]
+    assert len(clear) > 0 and len(blocked) > 0
+    cells = np.concatenate([rng.choice(clear, size=min(64, len(clear)), replace=False),
+                            rng.choice(blocked, size=min(32, len(blocked)), replace=False)])
+    S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n, cells=cells)
+    robust = S != 1
+    assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
+    ctx.close()
