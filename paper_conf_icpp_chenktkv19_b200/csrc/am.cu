@@ -17,6 +17,7 @@
 
 #include "../../include/am.h"
 #include "kernels.cuh"
+#include "stream.cuh"
 
 using namespace am;
 
@@ -61,7 +62,8 @@ struct am_ctx {
 
 namespace {
 
-constexpr int kCtrWords = 1 + ST_COUNT;
+constexpr int kCtrTiles = 1 + ST_COUNT;      // first dynamic tile counter
+constexpr int kCtrWords = kCtrTiles + 3;
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -118,6 +120,7 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.vox_main = c->d_vox;
     p.vox_coarse = c->d_coarse;
     p.cmapT = c->cmapT;
+    p.cull_dist = c->tool.rho_max * (1.f + 1e-5f) + 1e-6f;
     return p;
 }
 
@@ -173,27 +176,38 @@ int ensure_queue(am_ctx* ctx, long long cap) {
 
 int configure_launch(am_ctx* ctx) {
     const int m = ctx->grid.m;
-    ctx->smem = (size_t)(2 * ctx->MW + ((m + 31) >> 5)) * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
-    if (ctx->smem > 48 * 1024)
-        CK(cudaFuncSetAttribute(aica_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)ctx->smem));
+    ctx->smem = stream_smem_bytes(m, ctx->grid.W);
+    CK(cudaFuncSetAttribute(aica_stream_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)std::min<size_t>(ctx->smem, 232448)));
+    CK(cudaFuncSetAttribute(aica_stream_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)std::min<size_t>(ctx->smem, 232448)));
     int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel, kThreads, ctx->smem));
-    if (occ < 1) return fail(ctx, AM_EINVAL, "grid %dx%d does not fit in shared memory", m, ctx->grid.n);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel<false>, kThreads,
+                                                                  ctx->smem);
+    if (e != cudaSuccess || occ < 1) {
+        cudaGetLastError();
+        return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
+                    ctx->grid.n, ctx->smem);
+    }
     ctx->occ = occ;
     return AM_OK;
 }
 
-// One launch of the voxel-streaming kernel over vox[0, n).
+// One launch of the voxel-streaming kernel over vox[0, n): `slot` selects the
+// dynamic tile counter, `tile` the voxels per tile (small tiles spread the
+// few, heavy coarse voxels over every SM).
 int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, unsigned int vbase,
-                  unsigned int vtag, const float* cmap, bool timed, cudaStream_t s) {
+                  unsigned int vtag, const float* cmap, bool coarse, int tile, int slot, bool timed,
+                  cudaStream_t s) {
     if (n <= 0) return AM_OK;
     p.vox = vox;
     p.N = n;
     p.vbase = vbase;
     p.vtag = vtag;
     p.cmap = cmap;
-    const long long ntiles = (n + kTile - 1) / kTile;
+    p.tile = tile;
+    p.tile_ctr = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles + slot);
+    const long long ntiles = (n + tile - 1) / tile;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
     if (g > ntiles) g = ntiles;
     if (g < 1) g = 1;
@@ -208,7 +222,10 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, u
         }
         CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
     }
-    aica_stream_kernel<<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
+    if (coarse)
+        aica_stream_kernel<true><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
+    else
+        aica_stream_kernel<false><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
     return AM_OK;
@@ -223,11 +240,11 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
 }
 
 // One AICA map into device buffer gam (asynchronous on s):
-//   level 0 (largest voxels) -> clear map -> level 1 (next largest + strided
-//   sample) -> clear map -> every voxel, skipping those whose cheap cone misses
-//   every still-clear cell -> deferred band.  The coarse levels only make the
-//   skip test effective; each level is a subset of the model, so the map is the
-//   same with or without them (AM_OPT_PHASES).
+//   level 0 (largest voxels, inner cones) -> clear map -> level 1 (next largest
+//   + strided sample, inner cones, filtered) -> clear map -> every voxel,
+//   filtered by the clear map, both cones -> deferred band.  The coarse levels
+//   only make the filter effective; each level is a subset of the model, so
+//   the map is the same with or without them (AM_OPT_PHASES).
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
@@ -237,15 +254,16 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     const float* cm = nullptr;
     if (ctx->phases && ctx->n_l0 > 0) {
         constexpr unsigned int kCoarse = 0x80000000u;
-        if ((rc = launch_stream(ctx, p, ctx->d_coarse, ctx->n_l0, 0, kCoarse, nullptr, false, s))) return rc;
+        if ((rc = launch_stream(ctx, p, ctx->d_coarse, ctx->n_l0, 0, kCoarse, nullptr, true, 16, 0, false, s)))
+            return rc;
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         if ((rc = launch_stream(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0,
-                                (unsigned int)ctx->n_l0, kCoarse, ctx->d_cmap, false, s)))
+                                (unsigned int)ctx->n_l0, kCoarse, ctx->d_cmap, true, 256, 1, false, s)))
             return rc;
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         cm = ctx->d_cmap;
     }
-    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, 0, 0, cm, true, s))) return rc;
+    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, 0, 0, cm, false, kTile, 2, true, s))) return rc;
     band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     return AM_OK;
@@ -303,6 +321,13 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         float mn = tool[k].radius;
         for (int j = k; j < n_cyl; ++j) mn = std::min(mn, tool[j].radius);
         T.Rin[k] = mn;
+    }
+    for (int k = n_cyl; k < AM_MAX_CYL; ++k) {  // padding read by the unrolled cheap-cone select
+        T.z0[k] = 3.0e38f;
+        T.z1[k] = 3.0e38f;
+        T.R[k] = T.R[n_cyl - 1];
+        T.Rin[k] = T.Rin[n_cyl - 1];
+        T.Rpm[k] = T.Rpm[n_cyl - 1];
     }
     T.L = (float)z;
     T.rho_max = (float)rho;

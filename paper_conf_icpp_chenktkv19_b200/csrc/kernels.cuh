@@ -1,18 +1,19 @@
-// kernels.cuh -- the AICA hot path on sm_100a: voxel-streaming kernel, deferred
-// band kernel, all-pairs baseline kernel, and upload helpers.
+// kernels.cuh -- shared device state and the non-streaming kernels of the AICA
+// hot path on sm_100a: deferred band kernel, clear-direction map, all-pairs
+// baseline kernel, upload helpers.  The voxel-streaming kernel is stream.cuh.
 //
 // Map of SURVEY.md 8(a) steps to code:
-//   a1 voxel stream ........ aica_stream_kernel: persistent CTAs, float4 LDG.128
-//                             streaming loads (ld.global.cs), kVPT voxels/thread
-//   a2 reach cull .......... process_voxel(): D - sqrt3 h > rho_max
-//   a3 cone axis ........... process_voxel(): v, D, phi_v, gamma_v
+//   a1 voxel stream ........ stream.cuh aica_stream_kernel: persistent CTAs, dynamic
+//                             tiles, 1-D TMA (cp.async.bulk) into a 2-stage smem ring
+//   a2 reach cull .......... stream.cuh fast_filter(): D - sqrt3 h > rho_max
+//   a3 cone axis ........... stream.cuh process_live(): v, D, phi_v, gamma_v
 //   a4 cone half-angles .... am::tool_cones() (geometry.cuh)
-//   a5 rasterise ........... process_voxel(): per phi-row gamma intervals ->
-//                             32-bit masks OR-ed into the per-CTA shared AM
+//   a5 rasterise ........... stream.cuh process_live(): per phi-row gamma
+//                             intervals -> 32-bit masks OR-ed into the per-CTA smem AM
 //   a6 band resolution ..... band pairs pushed to a global queue; band_exact_kernel
 //                             runs CHECKBOX only where the final AM bit is still 0
-//   a7 merge/flush/exit .... cta_merge(): one atomicOr per changed word, global AM
-//                             read back into smem, row-full bits, early exit
+//   a7 merge/flush/exit .... stream.cuh cta_merge(): one atomicOr per changed word,
+//                             global AM read back into smem, row-full bits, early exit
 //   a8 output .............. bit-packed AM (layout in include/am.h)
 //   a9 baseline ............ baseline_kernel: CHECKBOX for every (voxel, cell)
 #pragma once
@@ -52,6 +53,9 @@ struct StreamParams {
     // clear-direction map; nullptr = not yet built
     const float* __restrict__ cmap;
     int cmapT;                     // texels per cube-face side
+    float cull_dist;               // rho_max, grown by the fp32 guard (reach cull)
+    int tile;                      // voxels per tile of this launch (<= kTile, multiple of 4)
+    unsigned int* tile_ctr;        // dynamic tile counter of this launch (zeroed)
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,
@@ -60,14 +64,16 @@ struct StreamParams {
 // exact function maps into the texel.
 __device__ __forceinline__ int cube_texel(float vx, float vy, float vz, int T) {
     const float ax = fabsf(vx), ay = fabsf(vy), az = fabsf(vz);
-    int face;
-    float a, u, w;
-    if (ax >= ay && ax >= az) { face = vx >= 0.f ? 0 : 1; a = ax; u = vy; w = vz; }
-    else if (ay >= az)        { face = vy >= 0.f ? 2 : 3; a = ay; u = vx; w = vz; }
-    else                      { face = vz >= 0.f ? 4 : 5; a = az; u = vx; w = vy; }
-    const float s = 0.5f * (float)T / a;
-    const int iu = min(T - 1, max(0, (int)((u + a) * s)));
-    const int iw = min(T - 1, max(0, (int)((w + a) * s)));
+    const bool xm = ax >= fmaxf(ay, az);
+    const bool ym = !xm && ay >= az;
+    const float a = fmaxf(ax, fmaxf(ay, az));
+    const float u = xm ? vy : vx;
+    const float w = (xm || ym) ? vz : vy;
+    const int face = xm ? (vx < 0.f) : (ym ? 2 + (vy < 0.f) : 4 + (vz < 0.f));
+    const float hs = 0.5f * (float)T;
+    const float s = hs * __frcp_rn(a);
+    const int iu = min(T - 1, max(0, __float2int_rz(fmaf(u, s, hs))));
+    const int iw = min(T - 1, max(0, __float2int_rz(fmaf(w, s, hs))));
     return (face * T + iw) * T + iu;
 }
 
@@ -95,10 +101,12 @@ __device__ __forceinline__ bool exact_pair(const StreamParams& p, float4 q, int 
     return exact_hit(q.x - p.px, q.y - p.py, q.z - p.pz, q.w, sph * cg, sph * sg, cph, p.tool);
 }
 
+// Cold-path counters of one CTA, kept in shared memory (32-bit; flushed to the
+// 64-bit global stats when the CTA retires) so they cost no registers.
 struct Counters {
-    unsigned long long streamed = 0, culled = 0, skipped = 0, live = 0, rows = 0, band = 0,
-                       overflow = 0;
+    unsigned int* c;  // [CT_LIVE, CT_ROWS, CT_BAND, CT_OVERFLOW]
 };
+enum { CT_LIVE = 0, CT_ROWS, CT_BAND, CT_OVERFLOW, CT_COUNT };
 
 // Are all rows i0..i1 full (bit set in sRowFull)?
 __device__ __forceinline__ bool rows_all_full(const uint32_t* sRowFull, int i0, int i1) {
@@ -120,213 +128,18 @@ __device__ void fill_all(const StreamParams& p, uint32_t* sAM) {
 __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, unsigned int vidx,
                                           float4 q, int cell, uint32_t* wp, uint32_t bit,
                                           Counters& cnt) {
-    cnt.band++;
+    atomicAdd(cnt.c + CT_BAND, 1u);
     const unsigned long long slot = atomicAdd(p.qcount, 1ULL);
     if ((long long)slot < p.qcap) {
         p.queue[slot] = ((unsigned long long)vidx << 32) | (unsigned int)cell;
     } else {
         // queue full: resolve inline (rare; keeps the result exact)
-        cnt.overflow++;
+        atomicAdd(cnt.c + CT_OVERFLOW, 1u);
         if (exact_pair(p, q, cell)) atomicOr(wp, bit);
     }
 }
 
-// Steps a2-a5 for one voxel.
-__device__ __forceinline__ void process_voxel(const StreamParams& p, unsigned int vidx, float4 q,
-                                              uint32_t* sAM, const uint32_t* sRowFull,
-                                              const float* sCos, const float* sSin, Counters& cnt) {
-    const ToolDev& T = p.tool;
-    const GridDev& g = p.grid;
-    const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
-    cnt.streamed++;
-    // the pivot lies in the closed box: the tool (which contains the pivot) hits it everywhere
-    if (fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
-        fill_all(p, sAM);
-        return;
-    }
-    const float D2 = vx * vx + vy * vy + vz * vz;
-    const float D = sqrtf(D2);
-    const float r2 = kSqrt3 * h;
-    // a2: reach cull -- every tool point is within rho_max of the pivot
-    if (D - r2 > T.rho_max + kRadRel * (D + r2)) {
-        cnt.culled++;
-        return;
-    }
-    // cheap outer bound: a sphere of radius r2 at distance D can only touch
-    // cylinders that start within D + r2, all of radius <= Reff, so its blocked
-    // angles satisfy sin(theta) <= (Reff + r2) / D
-    const float reach = D + r2 + kRadRel * (D + r2);
-    float Reff = 0.f;
-    for (int k = 0; k < T.ncyl; ++k)
-        if (T.z0[k] <= reach) Reff = T.Rpm[k];
-    const float s = (Reff + r2) / D * (1.f + 8e-6f) + 1e-6f;
-    if (p.cmap) {
-        // clear-direction map: U >= cos of the angle from any direction of this
-        // texel to the nearest still-clear cell.  The cone touches no clear cell
-        // when cos(cone) > U, i.e. U < 0 <= cos or U^2 < 1 - s^2 (s < 1).
-        const float U = __ldg(p.cmap + cube_texel(vx, vy, vz, p.cmapT));
-        if (s < 1.f && (U < 0.f || U * U < 1.f - s * s)) {
-            cnt.skipped++;
-            return;
-        }
-        if (s >= 1.f && U < -1.5f) {  // no clear cell left at all
-            cnt.skipped++;
-            return;
-        }
-    }
-    // a3: cone axis
-    const float rxy = sqrtf(vx * vx + vy * vy);
-    const float phv = atan2f(rxy, vz);
-    const float ac = (s >= 1.f) ? kPi : asinf(s);
-    int i0 = max(0, (int)ceilf((phv - ac - kRowSlack) * g.inv_dphi - 0.5f));
-    int i1 = min(g.m - 1, (int)floorf((phv + ac + kRowSlack) * g.inv_dphi - 0.5f));
-    if (i0 > i1 || rows_all_full(sRowFull, i0, i1)) {
-        cnt.skipped++;
-        return;
-    }
-    // a4: the two cones
-    cnt.live++;
-    const Cones c = tool_cones(D, h, T);
-    if (c.cout > 1.f) return;
-    const float ao = acosf(fmaxf(c.cout, -1.f));
-    i0 = max(i0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-    i1 = min(i1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-    const float invD = 1.f / D;
-    const float cphv = vz * invD, sphv = rxy * invD;
-    const float gv = atan2f(vy, vx);
-    const int W = g.W;
-    // a5: rasterise row by row
-    for (int i = i0; i <= i1; ++i) {
-        if ((ld_vol_shared(sRowFull + (i >> 5)) >> (i & 31)) & 1u) continue;
-        const float base = sCos[i] * cphv, den = sSin[i] * sphv;
-        const Interval O = gamma_interval(c.cout, base, den, gv, +1, g);
-        if (O.len == 0) continue;
-        cnt.rows++;
-        const Interval In = gamma_interval(c.cin, base, den, gv, -1, g);
-        const Interval X = gamma_interval(c.clo, base, den, gv, -1, g);
-        for (int w = 0; w < W; ++w) {
-            uint32_t ob = interval_bits(O, w, g.n);
-            if (!ob) continue;
-            const uint32_t xb = interval_bits(X, w, g.n);
-            const uint32_t ib = interval_bits(In, w, g.n) & ~xb;
-            ob &= ~xb;
-            uint32_t* wp = sAM + i * W + w;
-            uint32_t cur = ld_vol_shared(wp);
-            if (ib & ~cur) {
-                atomicOr(wp, ib);
-                cur |= ib;
-            }
-            uint32_t band = ob & ~ib & ~cur;
-            while (band) {
-                const int b = __ffs(band) - 1;
-                band &= band - 1u;
-                push_band(p, sAM, vidx, q, i * g.n + (w << 5) + b, wp, 1u << b, cnt);
-            }
-        }
-    }
-}
-
-// a7: merge the CTA's shared AM with the global AM (one atomicOr per word that
-// gained bits), read the union back, recompute the row-full bits.  Returns
-// true when the whole AM is blocked (early exit).
-__device__ bool cta_merge(const StreamParams& p, uint32_t* sAM, uint32_t* sShadow,
-                          uint32_t* sRowFull, int* sCount) {
-    const int MW = p.grid.m * p.grid.W;
-    const int W = p.grid.W;
-    __syncthreads();
-    if (threadIdx.x == 0) *sCount = 0;
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
-        const uint32_t s = sAM[w];
-        uint32_t gv;
-        if (s & ~sShadow[w])
-            gv = atomicOr(p.gam + w, s) | s;
-        else
-            gv = ld_cg(p.gam + w) | s;
-        sAM[w] = gv;
-        sShadow[w] = gv;
-    }
-    __syncthreads();
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    for (int base = 0; base < p.grid.m; base += blockDim.x) {
-        const int i = base + threadIdx.x;
-        bool full = false;
-        if (i < p.grid.m) {
-            full = true;
-            for (int w = 0; w < W; ++w)
-                if (sAM[i * W + w] != row_word_mask(w, p.grid.n)) full = false;
-        }
-        const uint32_t bal = __ballot_sync(0xffffffffu, full);
-        if (lane == 0 && base + warp * 32 < p.grid.m) {
-            sRowFull[(base + warp * 32) >> 5] = bal;
-            atomicAdd(sCount, __popc(bal));
-        }
-    }
-    __syncthreads();
-    return *sCount == p.grid.m;
-}
-
-__global__ void __launch_bounds__(kThreads, 4) aica_stream_kernel(const StreamParams p) {
-    extern __shared__ uint32_t smem[];
-    __shared__ int sCount;
-    const int m = p.grid.m;
-    const int MW = m * p.grid.W;
-    uint32_t* sAM = smem;
-    uint32_t* sShadow = sAM + MW;
-    uint32_t* sRowFull = sShadow + MW;
-    float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
-    float* sSin = sCos + m;
-    for (int i = threadIdx.x; i < m; i += blockDim.x) {
-        sCos[i] = p.tab[i];
-        sSin[i] = p.tab[m + i];
-    }
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
-        sAM[w] = 0u;
-        sShadow[w] = 0u;
-    }
-    Counters cnt;
-    bool early = cta_merge(p, sAM, sShadow, sRowFull, &sCount);
-    const long long ntiles = (p.N + kTile - 1) / kTile;
-    int since = 0;
-    for (long long t = blockIdx.x; t < ntiles && !early; t += gridDim.x) {
-        if (since == p.refresh_tiles) {
-            since = 0;
-            early = cta_merge(p, sAM, sShadow, sRowFull, &sCount);
-            if (early) break;
-        }
-        ++since;
-        float4 q[kVPT];
-        const long long base = t * kTile + threadIdx.x;
-#pragma unroll
-        for (int k = 0; k < kVPT; ++k) {
-            const long long idx = base + (long long)k * kThreads;
-            q[k] = idx < p.N ? __ldcs(p.vox + idx) : make_float4(0.f, 0.f, 0.f, -1.f);
-        }
-#pragma unroll 1
-        for (int k = 0; k < kVPT; ++k) {
-            if (q[k].w > 0.f)
-                process_voxel(p, (p.vbase + (unsigned int)(base + (long long)k * kThreads)) | p.vtag, q[k], sAM, sRowFull,
-                              sCos, sSin, cnt);
-        }
-    }
-    // final flush of words that gained bits
-    __syncthreads();
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
-        const uint32_t s = sAM[w];
-        if (s & ~sShadow[w]) atomicOr(p.gam + w, s);
-    }
-    // counters: warp-reduce then one atomic per warp
-    unsigned long long vals[7] = {cnt.streamed, cnt.culled, cnt.skipped, cnt.live, cnt.rows,
-                                  cnt.band, cnt.overflow};
-    const int idx[7] = {ST_STREAMED, ST_CULLED, ST_SKIPPED, ST_LIVE, ST_ROWS, ST_BAND, ST_OVERFLOW};
-#pragma unroll
-    for (int k = 0; k < 7; ++k) {
-        unsigned long long v = vals[k];
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if ((threadIdx.x & 31) == 0 && v) atomicAdd(p.stats + idx[k], v);
-    }
-    if (early && threadIdx.x == 0) atomicMax(reinterpret_cast<unsigned long long*>(p.stats + ST_EARLY), 1ULL);
-}
+// (the voxel-streaming kernel lives in stream.cuh)
 
 // Clear-direction map: for every cube-map texel t with centre c_t
 // and angular radius r_t, U_t >= cos(max(0, angle(c_t, nearest clear cell) - r_t)),
