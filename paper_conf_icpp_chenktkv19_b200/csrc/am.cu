@@ -41,16 +41,17 @@ struct am_ctx {
     long long qcap = 0;
     // options
     int grid_ctas = 0;
-    int refresh_tiles = 4;
+    int refresh_tiles = 8;
     int morton = 1;
     int baseline_reject = 0;
-    size_t smem = 0;
+    size_t smem = 0, smem_coarse = 0;
     int occ = 0;
     // coarse levels (largest voxels + a strided sample) and the clear-direction map
     float4* d_coarse = nullptr;
     long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
     float4* d_texels = nullptr;            // cube-map texel centres (xyz) + angular radius (w)
     float* d_cmap = nullptr;
+    float* d_cmap_ones = nullptr;          // the all-clear map (no voxel can be dropped)
     int cmapT = 32;
     int phases = 1;
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -63,7 +64,7 @@ struct am_ctx {
 namespace {
 
 constexpr int kCtrTiles = 1 + ST_COUNT;      // first dynamic tile counter
-constexpr int kCtrWords = kCtrTiles + 3;
+constexpr int kCtrWords = kCtrTiles + 1;
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -177,13 +178,14 @@ int ensure_queue(am_ctx* ctx, long long cap) {
 int configure_launch(am_ctx* ctx) {
     const int m = ctx->grid.m;
     ctx->smem = stream_smem_bytes(m, ctx->grid.W);
-    CK(cudaFuncSetAttribute(aica_stream_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)std::min<size_t>(ctx->smem, 232448)));
-    CK(cudaFuncSetAttribute(aica_stream_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)std::min<size_t>(ctx->smem, 232448)));
+    ctx->smem_coarse = (size_t)ctx->MW * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
+    if (ctx->smem > 232448 || ctx->smem_coarse > 232448)
+        return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
+                    ctx->grid.n, ctx->smem);
+    CK(cudaFuncSetAttribute(aica_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(coarse_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_coarse));
     int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel<false>, kThreads,
-                                                                  ctx->smem);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel, kThreads, ctx->smem);
     if (e != cudaSuccess || occ < 1) {
         cudaGetLastError();
         return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
@@ -193,23 +195,20 @@ int configure_launch(am_ctx* ctx) {
     return AM_OK;
 }
 
-// One launch of the voxel-streaming kernel over vox[0, n): `slot` selects the
-// dynamic tile counter, `tile` the voxels per tile (small tiles spread the
-// few, heavy coarse voxels over every SM).
-int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, unsigned int vbase,
-                  unsigned int vtag, const float* cmap, bool coarse, int tile, int slot, bool timed,
+// The full voxel stream over vox[0, n) with clear-direction map `cmap`.
+int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, bool timed,
                   cudaStream_t s) {
     if (n <= 0) return AM_OK;
     p.vox = vox;
     p.N = n;
-    p.vbase = vbase;
-    p.vtag = vtag;
+    p.vbase = 0;
+    p.vtag = 0;
     p.cmap = cmap;
-    p.tile = tile;
-    p.tile_ctr = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles + slot);
-    const long long ntiles = (n + tile - 1) / tile;
+    p.tile_ctr = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
+    const long long nchunks = (n + kChunk - 1) / kChunk;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
-    if (g > ntiles) g = ntiles;
+    const long long need = (nchunks + (long long)kWarps * kSuper - 1) / ((long long)kWarps * kSuper);
+    if (g > need) g = need;
     if (g < 1) g = 1;
     timed = timed && ctx->timing;
     if (timed) {
@@ -222,12 +221,26 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, u
         }
         CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
     }
-    if (coarse)
-        aica_stream_kernel<true><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
-    else
-        aica_stream_kernel<false><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
+    aica_stream_kernel<<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    return AM_OK;
+}
+
+// A coarse level: inner cones of vox[0, n), `batch` voxels per warp iteration.
+int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, int batch,
+                  cudaStream_t s) {
+    if (n <= 0) return AM_OK;
+    p.vox = vox;
+    p.N = n;
+    p.cmap = cmap;
+    p.tile = batch;
+    const long long warps = (n + batch - 1) / batch;
+    long long g = (warps + kWarps - 1) / kWarps;
+    const long long gmax = (long long)ctx->sms * 8;
+    if (g > gmax) g = gmax;
+    coarse_kernel<<<(unsigned)g, kThreads, ctx->smem_coarse, s>>>(p);
+    CK(cudaGetLastError());
     return AM_OK;
 }
 
@@ -240,30 +253,28 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
 }
 
 // One AICA map into device buffer gam (asynchronous on s):
-//   level 0 (largest voxels, inner cones) -> clear map -> level 1 (next largest
-//   + strided sample, inner cones, filtered) -> clear map -> every voxel,
-//   filtered by the clear map, both cones -> deferred band.  The coarse levels
-//   only make the filter effective; each level is a subset of the model, so
-//   the map is the same with or without them (AM_OPT_PHASES).
+//   level 0 (largest voxels, inner cones, one warp each) -> clear map ->
+//   level 1 (next largest + strided sample, filtered, inner cones) -> clear map
+//   -> the full stream of every voxel, filtered by the map, both cones ->
+//   deferred band.  The coarse levels only make the filter effective; they are
+//   subsets of the model, so the map is the same with or without them
+//   (AM_OPT_PHASES).
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     if (ctx->N == 0) return AM_OK;
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
-    const float* cm = nullptr;
+    const float* cm = ctx->d_cmap_ones;
     if (ctx->phases && ctx->n_l0 > 0) {
-        constexpr unsigned int kCoarse = 0x80000000u;
-        if ((rc = launch_stream(ctx, p, ctx->d_coarse, ctx->n_l0, 0, kCoarse, nullptr, true, 16, 0, false, s)))
-            return rc;
+        if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 1, s))) return rc;
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
-        if ((rc = launch_stream(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0,
-                                (unsigned int)ctx->n_l0, kCoarse, ctx->d_cmap, true, 256, 1, false, s)))
+        if ((rc = launch_coarse(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, 32, s)))
             return rc;
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         cm = ctx->d_cmap;
     }
-    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, 0, 0, cm, false, kTile, 2, true, s))) return rc;
+    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, cm, true, s))) return rc;
     band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     return AM_OK;
@@ -329,6 +340,18 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         T.Rin[k] = T.Rin[n_cyl - 1];
         T.Rpm[k] = T.Rpm[n_cyl - 1];
     }
+    T.R_first = T.Rpm[0];
+    T.nbp = 0;
+    for (int k = 0; k < AM_MAX_CYL; ++k) {
+        T.bp_z[k] = 3.0e38f;
+        T.bp_R[k] = T.Rpm[n_cyl - 1];
+    }
+    for (int k = 1; k < n_cyl; ++k)
+        if (T.Rpm[k] > T.Rpm[k - 1]) {
+            T.bp_z[T.nbp] = T.z0[k];
+            T.bp_R[T.nbp] = T.Rpm[k];
+            ++T.nbp;
+        }
     T.L = (float)z;
     T.rho_max = (float)rho;
     GridDev& G = ctx->grid;
@@ -376,9 +399,18 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         const std::vector<float> tex = make_texels(ctx->cmapT);
         if (cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)) != cudaSuccess ||
             cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMalloc(&ctx->d_cmap, tex.size() / 4 * sizeof(float)) != cudaSuccess) {
+            cudaMalloc(&ctx->d_cmap, tex.size() / 4 * sizeof(float)) != cudaSuccess ||
+            cudaMalloc(&ctx->d_cmap_ones, tex.size() / 4 * sizeof(float)) != cudaSuccess) {
             cudaGetLastError();
             return bail(AM_ENOMEM);
+        }
+    }
+    {
+        const std::vector<float> ones((size_t)6 * ctx->cmapT * ctx->cmapT, 1.0f);
+        if (cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            return bail(AM_ECUDA);
         }
     }
     if ((rc = ensure_queue(ctx, 1 << 22)) != AM_OK) return bail(rc);
@@ -702,6 +734,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_coarse);
     cudaFree(ctx->d_texels);
     cudaFree(ctx->d_cmap);
+    cudaFree(ctx->d_cmap_ones);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

@@ -32,7 +32,27 @@ struct ToolDev {
     float Rpm[AM_MAX_CYL];  // prefix max max_{j <= k} R_j (cheap outer bound)
     float L;                // total length z1[ncyl-1]
     float rho_max;          // max_k |(z1_k, R_k)|: reach of the tool from the pivot
+    // cheap-cone radius as a step function of the reach D + sqrt3 h: R_first up
+    // to bp_z[0], then bp_R[k] from bp_z[k] on (only where the prefix max grows;
+    // unused entries are +inf)
+    int nbp;
+    float R_first;
+    float bp_z[AM_MAX_CYL];
+    float bp_R[AM_MAX_CYL];
 };
+
+// Largest radius of any cylinder that starts within `reach` of the pivot.
+__device__ __forceinline__ float reach_radius(const ToolDev& T, float reach) {
+    float R = T.R_first;
+#pragma unroll
+    for (int k = 0; k < 3; ++k)
+        if (T.bp_z[k] <= reach) R = T.bp_R[k];
+    if (T.nbp > 3) {
+        for (int k = 3; k < T.nbp; ++k)
+            if (T.bp_z[k] <= reach) R = T.bp_R[k];
+    }
+    return R;
+}
 
 struct GridDev {
     int m, n, W;            // rows (phi), columns (gamma), words per row
@@ -161,6 +181,23 @@ __device__ __forceinline__ Cones tool_cones(float D, float h, const ToolDev& T) 
     return c;
 }
 
+// Inner cone only (GETTOOLICA(r = h) on the monotone-shrunk tool), guarded;
+// > 1 when empty.  Used by the coarse levels, which only need certainly-blocked
+// cells.
+__device__ __forceinline__ float inner_cone(float D, float h, const ToolDev& T) {
+    const float r1 = fmaxf(h - kRadRel * (D + h), 0.f);
+    if (!(D * (1.f + kRadRel) <= T.L + r1 && r1 > 0.f)) return 2.f;
+    const float D2 = D * D;
+    const float invD = 1.f / D;
+    float cm = 2.f;
+    for (int k = 0; k < T.ncyl; ++k) {
+        float a, b;
+        ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], a, b);
+        cm = fminf(cm, a);
+    }
+    return (cm <= 1.f) ? cm + kCosGuard : 2.f;
+}
+
 // Cells j of one phi-row with base + den * cos(gamma_j - gv) >= cthr, as the
 // cyclic range [lo, lo + len) (mod n).  grow = +1 widens the interval by the
 // guards (outer cone), grow = -1 narrows it (inner cone / ring exclusion).
@@ -192,8 +229,9 @@ __device__ __forceinline__ Interval gamma_interval(float cthr, float base, float
     if (hi < lo) return I;
     int len = hi - lo + 1;
     if (len >= g.n) { I.len = g.n; return I; }
-    lo %= g.n;
+    // gv in (-pi, pi] and dl in [0, pi) keep lo within [-n, n): one wrap suffices
     if (lo < 0) lo += g.n;
+    if (lo >= g.n) lo -= g.n;
     I.lo = lo;
     I.len = len;
     return I;
