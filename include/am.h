@@ -80,8 +80,15 @@ enum {
     AM_OPT_BASELINE_REJECT = 4,  /* 1 = baseline uses an exact-safe bounding-sphere reject        */
     AM_OPT_BAND_QUEUE = 5,       /* capacity of the deferred band queue, in (voxel, cell) pairs  */
     AM_OPT_KERNEL_TIMING = 6,    /* 1 = bracket every full-stream kernel launch with CUDA events */
-    AM_OPT_PHASES = 7            /* 1 = coarse levels + clear-direction map before the full
+    AM_OPT_PHASES = 7,           /* 1 = coarse levels + clear-direction map before the full
                                     stream (default); 0 = one plain stream.  Same map either way */
+    AM_OPT_DIAG = 8,             /* diagnostics, 0 in production: bit 0 = stop after the coarse
+                                    levels (partial map); bit 1 = seed the map and the clear-
+                                    direction map with the previous map of this context instead
+                                    of the coarse levels (a lower-bound probe of the filter; the
+                                    result is exact only when that map had the same pivot)       */
+    AM_OPT_CMAP_T = 9            /* clear-direction map resolution: texels per cube-face side
+                                    (4..256, default 32)                                         */
 };
 
 /*

@@ -48,10 +48,13 @@ struct am_ctx {
     int occ = 0;
     // coarse levels (largest voxels + a strided sample) and the clear-direction map
     float4* d_coarse = nullptr;
+    unsigned int* d_live = nullptr;        // live-voxel list of the full stream (capacity N)
     long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
     float4* d_texels = nullptr;            // cube-map texel centres (xyz) + angular radius (w)
     float* d_cmap = nullptr;
     float* d_cmap_ones = nullptr;          // the all-clear map (no voxel can be dropped)
+    uint32_t* d_prev = nullptr;            // diagnostics: copy of the last map
+    int diag = 0;
     int cmapT = 32;
     int phases = 1;
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -177,15 +180,15 @@ int ensure_queue(am_ctx* ctx, long long cap) {
 
 int configure_launch(am_ctx* ctx) {
     const int m = ctx->grid.m;
-    ctx->smem = stream_smem_bytes(m, ctx->grid.W);
+    ctx->smem = live_smem_bytes(m, ctx->grid.W);
     ctx->smem_coarse = (size_t)ctx->MW * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
     if (ctx->smem > 232448 || ctx->smem_coarse > 232448)
         return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
                     ctx->grid.n, ctx->smem);
-    CK(cudaFuncSetAttribute(aica_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(live_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
     CK(cudaFuncSetAttribute(coarse_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_coarse));
     int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, aica_stream_kernel, kThreads, ctx->smem);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, filter_kernel, kThreads, 0);
     if (e != cudaSuccess || occ < 1) {
         cudaGetLastError();
         return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
@@ -204,11 +207,11 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     p.vbase = 0;
     p.vtag = 0;
     p.cmap = cmap;
-    p.tile_ctr = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
-    const long long nchunks = (n + kChunk - 1) / kChunk;
+    p.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
+    p.live_idx = ctx->d_live;
+    const long long ntiles = (n + kTile - 1) / kTile;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
-    const long long need = (nchunks + (long long)kWarps * kSuper - 1) / ((long long)kWarps * kSuper);
-    if (g > need) g = need;
+    if (g > ntiles) g = ntiles;
     if (g < 1) g = 1;
     timed = timed && ctx->timing;
     if (timed) {
@@ -221,9 +224,11 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
         }
         CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
     }
-    aica_stream_kernel<<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
+    filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    live_kernel<<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
+    CK(cudaGetLastError());
     return AM_OK;
 }
 
@@ -266,7 +271,13 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
     const float* cm = ctx->d_cmap_ones;
-    if (ctx->phases && ctx->n_l0 > 0) {
+    if (ctx->diag & 2) {
+        // diagnostic: clear map from the previous map computed on this context
+        // (exact only when the previous call used the same pivot)
+        CK(cudaMemcpyAsync(gam, ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
+        cm = ctx->d_cmap;
+    } else if (ctx->phases && ctx->n_l0 > 0) {
         if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 1, s))) return rc;
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         if ((rc = launch_coarse(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, 32, s)))
@@ -274,9 +285,13 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         cm = ctx->d_cmap;
     }
-    if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, cm, true, s))) return rc;
-    band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
-    CK(cudaGetLastError());
+    if (!(ctx->diag & 1)) {
+        if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, cm, true, s))) return rc;
+        band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
+        CK(cudaGetLastError());
+    }
+    if (ctx->d_prev)  // allocated once diagnostics were enabled
+        CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
     return AM_OK;
 }
 
@@ -478,9 +493,12 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     }
     if (ctx->vox_cap < N) {
         cudaFree(ctx->d_vox);
+        cudaFree(ctx->d_live);
         ctx->d_vox = nullptr;
+        ctx->d_live = nullptr;
         ctx->vox_cap = 0;
         UK(cudaMalloc(&ctx->d_vox, (size_t)N * sizeof(float4)));
+        UK(cudaMalloc(&ctx->d_live, (size_t)N * sizeof(unsigned int)));
         ctx->vox_cap = N;
     }
     UK(cudaMalloc(&raw, (size_t)N * sizeof(float4)));
@@ -690,6 +708,32 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "phases must be 0 or 1");
         ctx->phases = (int)value;
         return AM_OK;
+    case AM_OPT_DIAG:
+        if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "diag must be in [0, 3]");
+        if (value && !ctx->d_prev) {
+            CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
+            CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
+        }
+        ctx->diag = (int)value;
+        return AM_OK;
+    case AM_OPT_CMAP_T:
+        if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
+        {
+            const std::vector<float> tex = make_texels((int)value);
+            const std::vector<float> ones(tex.size() / 4, 1.0f);
+            cudaFree(ctx->d_texels);
+            cudaFree(ctx->d_cmap);
+            cudaFree(ctx->d_cmap_ones);
+            ctx->d_texels = nullptr;
+            ctx->d_cmap = ctx->d_cmap_ones = nullptr;
+            CK(cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)));
+            CK(cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
+            CK(cudaMalloc(&ctx->d_cmap, ones.size() * sizeof(float)));
+            CK(cudaMalloc(&ctx->d_cmap_ones, ones.size() * sizeof(float)));
+            CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice));
+            ctx->cmapT = (int)value;
+        }
+        return AM_OK;
     default:
         return fail(ctx, AM_EINVAL, "unknown option %d", key);
     }
@@ -732,9 +776,11 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_ctr);
     cudaFree(ctx->d_queue);
     cudaFree(ctx->d_coarse);
+    cudaFree(ctx->d_live);
     cudaFree(ctx->d_texels);
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);
+    cudaFree(ctx->d_prev);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

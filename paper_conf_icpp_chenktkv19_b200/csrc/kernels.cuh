@@ -56,6 +56,8 @@ struct StreamParams {
     float cull_dist;               // rho_max, grown by the fp32 guard (reach cull)
     int tile;                      // voxels per tile of this launch (<= kTile, multiple of 4)
     unsigned int* tile_ctr;        // dynamic tile counter of this launch (zeroed)
+    unsigned int* live_count;      // live voxels found by the filter (zeroed)
+    unsigned int* live_idx;        // their indices into vox (capacity N)
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,

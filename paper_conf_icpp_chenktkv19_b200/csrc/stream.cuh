@@ -1,70 +1,38 @@
-// stream.cuh -- the voxel-streaming AICA kernels (SURVEY.md 8(a) steps a1-a5, a7).
+// stream.cuh -- the voxel-streaming AICA kernels (SURVEY.md 8(a) steps a1-a7).
 //
-// aica_stream_kernel (the full stream, every voxel):
-//   Every warp is an independent worker with its own 3-stage ring in shared
-//   memory.  Lane 0 claims chunks of 128 voxels (4 chunks per atomic) and pulls
-//   them global -> shared with the 1-D TMA engine (cp.async.bulk + mbarrier
-//   complete_tx; SASS UBLKCP), so the HBM stream runs ahead of the arithmetic
-//   without registers and without CTA-wide barriers.  Per voxel the warp runs a
-//   cheap, exact-safe FILTER (fast_filter): reach cull, then the cheap outer cone
-//   -- a sphere of radius sqrt(3) h at distance D only touches cylinders that
-//   start within D + sqrt(3) h, of radius at most Reff, so its blocked directions
-//   satisfy sin(theta) <= (Reff + sqrt3 h) / D -- against the clear-direction map
+// The full stream is split in two launches so the part that touches every
+// voxel stays lean:
+//
+// filter_kernel (a1, a2, cheap cones; every voxel): coalesced 16-byte float4
+//   loads (4 independent LDG.128 per thread in flight, streaming cache hint),
+//   then an exact-safe FILTER per voxel: reach cull, then a cheap outer cone --
+//   a sphere of radius sqrt(3) h at distance D only touches cylinders starting
+//   within D + sqrt(3) h, of radius at most Reff, so its blocked directions
+//   satisfy sin(theta) <= (Reff + sqrt3 h) / D, and none lies more than r2 behind
+//   the tool's end face at the pivot -- against the clear-direction map
 //   (kernels.cuh clear_map_kernel).  A voxel whose cheap cone holds no
-//   still-clear cell cannot change the AM and is dropped.  Survivors ("live",
-//   ~1-2 % at the paper's 1 mm offset) go to a per-warp queue (ballot) and are
-//   processed 32 at a time, one per lane (process_live): the paper's two ICA
-//   cones (Alg. 1) rasterised row by row into the CTA's shared AM,
-//   band cells deferred to the global band queue.  Each warp merges the shared
-//   AM with the global AM on its own (a7).
+//   still-clear cell cannot change the AM and is dropped after ~60
+//   instructions; the survivors ("live") are appended to a global list with one
+//   warp-aggregated atomic.
 //
-// coarse_kernel (levels 0/1, the largest voxels):
-//   one warp per voxel, phi-rows across lanes, inner cones only -- these few
-//   voxels have cones spanning most rows, so row parallelism is what they need.
+// live_kernel (a3-a6; the live voxels only, ~0.1-1 %): one voxel per thread,
+//   the paper's two ICA cones (Alg. 1) checked against the map once
+//   more, then rasterised row by row into the CTA's shared AM; band cells are
+//   deferred to the global band queue; the shared AM is OR-ed into the global
+//   AM at the end (a7).
+//
+// coarse_kernel (levels 0/1, the largest voxels): one warp per voxel, phi-rows
+//   across lanes, inner cones only -- these few voxels have cones spanning most
+//   rows, so row parallelism is what they need.
 #pragma once
 #include "kernels.cuh"
 
 namespace am {
 
 constexpr int kWarps = kThreads / 32;
-constexpr int kChunk = 128;     // voxels per TMA copy (4 per lane)
-constexpr int kWStages = 3;     // per-warp ring depth
-constexpr int kSuper = 4;       // chunks claimed per atomic
-constexpr int kWQ = 64;         // per-warp live queue (drained at 32)
+constexpr int kLiveBlocksPerSM = 4;
 static_assert(sizeof(StreamParams) % 4 == 0 && sizeof(StreamParams) / 4 <= kThreads,
               "StreamParams is copied to shared memory one word per thread");
-
-__device__ __forceinline__ unsigned int smem_u32(const void* p) {
-    return static_cast<unsigned int>(__cvta_generic_to_shared(p));
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, unsigned int count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, unsigned int bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned int parity) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
-        "r"(parity)
-        : "memory");
-}
-
-// 1-D bulk copy global -> shared, completion signalled on `bar` (bytes % 16 == 0).
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, unsigned int bytes, uint64_t* bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
-}
 
 __device__ __forceinline__ float rcp_approx(float x) {
     float r;
@@ -74,17 +42,19 @@ __device__ __forceinline__ float rcp_approx(float x) {
 
 enum { F_DROP = 0, F_LIVE = 1, F_CULLED = 2 };
 
+__device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T);
+
 // a2 + cheap cone vs clear-direction map (p.cmap is never null: before any map
 // is built it is the all-clear map, U = 1).  F_LIVE when the voxel may still
-// change the AM, F_CULLED beyond reach, F_DROP otherwise.
-__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* sAM) {
+// change the AM, F_CULLED beyond reach, F_DROP otherwise.  A voxel holding the
+// pivot blocks every orientation: it fills `am` (shared or global) directly.
+__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am) {
     const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
     const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
     const float r2 = kSqrt3 * h;
     if (D2 <= 3.0001f * h * h) {
-        // the pivot may lie in the closed box: then every orientation collides
         if (fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
-            fill_all(p, sAM);
+            fill_all(p, am);
             return F_DROP;
         }
         return F_LIVE;
@@ -94,8 +64,20 @@ __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint
     if (D - r2 > p.cull_dist) return F_CULLED;
     const float Reff = reach_radius(p.tool, (D + r2) * (1.f + kRadRel));
     const float s = fmaf((Reff + r2) * invD, 1.f + 1.6e-5f, 1e-6f);
-    // cube-map texel of v (cube_texel with an approximate reciprocal; the texel
-    // radii carry 2e-5 rad of slack for the rounding at texel edges)
+    const float U = __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT));
+    // U bounds cos(angle to the nearest clear cell) from above for every
+    // direction of the texel: drop when cos(cheap cone) > U.  Far voxels
+    // (s < 1): sin(theta) <= s.  Near voxels: the tool has nothing behind the
+    // plane of its end face at the pivot, so a blocked direction keeps the
+    // sphere centre within r2 of that plane: cos(theta) >= -r2 / D.
+    const bool drop = (s < 1.f) ? (U < 0.f || U * U < 1.f - s * s)
+                                : (U < -fmaf(r2 * invD, 1.f + 1.6e-5f, 1e-6f));
+    return drop ? F_DROP : F_LIVE;
+}
+
+// Cube-map texel of v (cube_texel of kernels.cuh with an approximate
+// reciprocal; the texel radii carry 2e-5 rad of slack for rounding at edges).
+__device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
     const float ax = fabsf(vx), ay = fabsf(vy), az = fabsf(vz);
     const bool xm = ax >= fmaxf(ay, az);
     const bool ym = !xm && ay >= az;
@@ -103,16 +85,11 @@ __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint
     const float u = xm ? vy : vx;
     const float w = (xm || ym) ? vz : vy;
     const int face = xm ? (vx < 0.f) : (ym ? 2 + (vy < 0.f) : 4 + (vz < 0.f));
-    const int T = p.cmapT;
     const float hs = 0.5f * (float)T;
     const float sc = hs * rcp_approx(a);
     const int iu = min(T - 1, max(0, __float2int_rz(fmaf(u, sc, hs))));
     const int iw = min(T - 1, max(0, __float2int_rz(fmaf(w, sc, hs))));
-    const float U = __ldg(p.cmap + (face * T + iw) * T + iu);
-    // U bounds cos(angle to the nearest clear cell) from above for every
-    // direction of the texel: drop when cos(cheap cone) > U.
-    const bool drop = (s < 1.f) ? (U < 0.f || U * U < 1.f - s * s) : (U < -1.5f);
-    return drop ? F_DROP : F_LIVE;
+    return (face * T + iw) * T + iu;
 }
 
 // a3-a6 for one live voxel: both cones, rasterised row by row, band deferred.
@@ -131,6 +108,9 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
     atomicAdd(cnt.c + CT_LIVE, 1u);
     const Cones c = tool_cones(D, h, T);
     if (c.cout > 1.f) return;
+    // the exact outer cone against the clear-direction map: no clear cell
+    // within it means this voxel cannot change the map
+    if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout) return;
     const float ao = acosf(fmaxf(c.cout, -1.f));
     const int i0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
     const int i1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
@@ -172,212 +152,113 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
     if (rows) atomicAdd(cnt.c + CT_ROWS, rows);
 }
 
-// a7 by one warp: OR the shared AM into the global AM (one atomicOr per word
-// with bits the global AM may lack), OR the global AM back into shared memory,
-// refresh the row-full bits.  Races between warps are benign: every update is
-// an OR of bits that are certainly blocked.  Returns true when the AM is full.
-__device__ __noinline__ bool warp_merge(const StreamParams& p, uint32_t* sAM, uint32_t* sShadow,
-                                        uint32_t* sRowFull) {
-    const int lane = threadIdx.x & 31;
-    const int m = p.grid.m, W = p.grid.W, MW = m * W;
-    for (int w = lane; w < MW; w += 32) {
-        const uint32_t s = ld_vol_shared(sAM + w);
-        const uint32_t sh = ld_vol_shared(sShadow + w);
-        const uint32_t gv = (s & ~sh) ? (atomicOr(p.gam + w, s) | s) : ld_cg(p.gam + w);
-        if (gv & ~s) atomicOr(sAM + w, gv);
-        if (gv & ~sh) atomicOr(sShadow + w, gv | s);
-    }
-    __syncwarp();
-    int nfull = 0;
-    for (int i = lane; i < m; i += 32) {
-        bool full = true;
-        for (int w = 0; w < W; ++w)
-            if (ld_vol_shared(sAM + i * W + w) != row_word_mask(w, p.grid.n)) full = false;
-        if (full) {
-            atomicOr(sRowFull + (i >> 5), 1u << (i & 31));
-            ++nfull;
-        }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) nfull += __shfl_xor_sync(0xffffffffu, nfull, o);
-    return nfull == m;
+
+// Dynamic shared memory of live_kernel for an m x n grid.
+__host__ __device__ inline size_t live_smem_bytes(int m, int W) {
+    return (size_t)(m * W + ((m + 31) >> 5)) * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
 }
 
-// Dynamic shared memory of aica_stream_kernel for an m x n grid.
-__host__ __device__ inline size_t stream_smem_bytes(int m, int W) {
-    size_t b = (size_t)kWarps * kWStages * kChunk * sizeof(float4);  // per-warp TMA rings
-    b += (size_t)kWarps * kWQ * sizeof(float4);                         // live queue voxels
-    b += (size_t)kWarps * kWQ * sizeof(unsigned int);                   // live queue indices
-    b += (size_t)(2 * m * W + ((m + 31) >> 5)) * sizeof(uint32_t);    // AM, shadow, row-full bits
-    b += (size_t)2 * m * sizeof(float);                                 // cos / sin phi rows
-    return b;
-}
-
-__global__ void __launch_bounds__(kThreads, 3) aica_stream_kernel(const __grid_constant__ StreamParams p) {
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    __shared__ uint64_t bar[kWarps][kWStages];
-    __shared__ long long sChunk[kWarps][kWStages];
-    __shared__ unsigned int sCnt[CT_COUNT];
-    __shared__ unsigned long long sStreamed, sCulled, sPassed;
-    __shared__ int sExit;
-    // shared copy of the parameters for the out-of-line cold path (a reference
-    // to the kernel parameter would make every call copy it to local memory)
-    __shared__ StreamParams sP;
-    if (threadIdx.x < (int)(sizeof(StreamParams) / 4))
-        reinterpret_cast<unsigned int*>(&sP)[threadIdx.x] = reinterpret_cast<const unsigned int*>(&p)[threadIdx.x];
-    const int m = p.grid.m;
-    const int MW = m * p.grid.W;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    float4* ring = reinterpret_cast<float4*>(smem_raw) + warp * kWStages * kChunk;
-    float4* sQv = reinterpret_cast<float4*>(smem_raw) + kWarps * kWStages * kChunk;
-    unsigned int* sQi = reinterpret_cast<unsigned int*>(sQv + kWarps * kWQ);
-    uint32_t* sAM = sQi + kWarps * kWQ;
-    uint32_t* sShadow = sAM + MW;
-    uint32_t* sRowFull = sShadow + MW;
-    float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
-    float* sSin = sCos + m;
-    float4* wQv = sQv + warp * kWQ;
-    unsigned int* wQi = sQi + warp * kWQ;
-    const Counters cnt{sCnt};
-
-    for (int i = threadIdx.x; i < m; i += blockDim.x) {
-        sCos[i] = p.tab[i];
-        sSin[i] = p.tab[m + i];
-    }
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
-        sAM[w] = 0u;
-        sShadow[w] = 0u;
-    }
-    for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
-    if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
-    if (threadIdx.x == 0) {
-        sStreamed = sCulled = sPassed = 0ull;
-        sExit = 0;
-    }
-    const long long nchunks = (p.N + kChunk - 1) / kChunk;
-    long long nxt = 0, end = 0;  // lane 0's claimed chunk range
-    auto claim = [&]() -> long long {
-        if (nxt >= end) {
-            nxt = (long long)atomicAdd(p.tile_ctr, (unsigned int)kSuper);
-            end = nxt + kSuper;
-        }
-        return nxt++;
-    };
-    auto issue = [&](int s, long long c) {
-        sChunk[warp][s] = c;
-        if (c < nchunks) {
-            const long long first = c * kChunk;
-            const unsigned int bytes = (unsigned int)(min((long long)kChunk, p.N - first) * sizeof(float4));
-            mbar_expect_tx(&bar[warp][s], bytes);
-            tma_load_1d(ring + s * kChunk, p.vox + first, bytes, &bar[warp][s]);
-        }
-    };
-    if (lane == 0) {
-        for (int s = 0; s < kWStages; ++s) mbar_init(&bar[warp][s], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int s = 0; s < kWStages; ++s) issue(s, claim());
-    }
+// a1-a2 + cheap cones over vox[0, N): live indices go to p.live_idx.
+__global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant__ StreamParams p) {
+    __shared__ unsigned long long sCulled, sPassed;
+    if (threadIdx.x == 0) sCulled = sPassed = 0ull;
     __syncthreads();
-
-    unsigned int phase = 0;      // bit s = parity of stage s
+    const int lane = threadIdx.x & 31;
     unsigned int nculled = 0, npassed = 0;
     unsigned long long streamed = 0;
-    int qn = 0;                  // live entries in this warp's queue (warp-uniform)
-    int since = 0;
-    int s = 0;
-    bool early = false;
-    for (;;) {
-        const long long c = *reinterpret_cast<volatile long long*>(&sChunk[warp][s]);
-        if (c >= nchunks) break;
-        mbar_wait(&bar[warp][s], (phase >> s) & 1u);
-        phase ^= 1u << s;
-        const long long first = c * kChunk;
-        const int cntv = (int)min((long long)kChunk, p.N - first);
-        streamed += cntv;
-        const float4* tv = ring + s * kChunk;
+    const long long ntiles = (p.N + kTile - 1) / kTile;
+    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const long long base = t * kTile + threadIdx.x;
+        float4 q[kVPT];
 #pragma unroll
-        for (int k = 0; k < kChunk / 32; ++k) {
-            const int local = k * 32 + lane;
-            int f = F_DROP;
-            float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (local < cntv) {
-                q = tv[local];
-                f = fast_filter(p, q, sAM);
-            }
-            const unsigned int mlive = __ballot_sync(0xffffffffu, f == F_LIVE);
-            nculled += __popc(__ballot_sync(0xffffffffu, f == F_CULLED));
+        for (int k = 0; k < kVPT; ++k) {
+            const long long idx = base + (long long)k * kThreads;
+            q[k] = idx < p.N ? __ldcs(p.vox + idx) : make_float4(0.f, 0.f, 0.f, -1.f);
+        }
+        int f[kVPT];
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) f[k] = q[k].w > 0.f ? fast_filter(p, q[k], p.gam) : F_DROP;
+        if (lane == 0) streamed += (unsigned long long)min((long long)kTile, p.N - t * kTile);
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) {
+            const unsigned int mlive = __ballot_sync(0xffffffffu, f[k] == F_LIVE);
+            nculled += __popc(__ballot_sync(0xffffffffu, f[k] == F_CULLED));
             if (mlive) {
                 npassed += __popc(mlive);
-                if (f == F_LIVE) {
-                    const int pos = qn + __popc(mlive & ((1u << lane) - 1u));
-                    wQv[pos] = q;
-                    wQi[pos] = (p.vbase + (unsigned int)(first + local)) | p.vtag;
-                }
-                qn += __popc(mlive);
-                if (qn >= 32) {  // drain 32 entries, one per lane, then compact the rest
-                    __syncwarp();
-                    process_live(sP, wQi[lane], wQv[lane], sAM, sRowFull, sCos, sSin, cnt);
-                    const int rest = qn - 32;
-                    float4 rv;
-                    unsigned int ri = 0;
-                    if (lane < rest) {
-                        rv = wQv[32 + lane];
-                        ri = wQi[32 + lane];
-                    }
-                    __syncwarp();
-                    if (lane < rest) {
-                        wQv[lane] = rv;
-                        wQi[lane] = ri;
-                    }
-                    __syncwarp();
-                    qn = rest;
-                }
+                unsigned int pos = 0;
+                const int leader = __ffs(mlive) - 1;
+                if (lane == leader) pos = atomicAdd(p.live_count, (unsigned int)__popc(mlive));
+                pos = __shfl_sync(0xffffffffu, pos, leader) + __popc(mlive & ((1u << lane) - 1u));
+                if (f[k] == F_LIVE) p.live_idx[pos] = (unsigned int)(base + (long long)k * kThreads);
             }
         }
-        __syncwarp();  // the warp is done reading stage s
-        if (lane == 0) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            issue(s, claim());
-        }
-        __syncwarp();
-        if (++since >= p.refresh_tiles) {
-            since = 0;
-            if (warp_merge(sP, sAM, sShadow, sRowFull)) sExit = 1;
-        }
-        if (*reinterpret_cast<volatile int*>(&sExit)) {
-            early = true;
-            break;
-        }
-        s = (s + 1 == kWStages) ? 0 : s + 1;
-    }
-    if (lane < qn) process_live(sP, wQi[lane], wQv[lane], sAM, sRowFull, sCos, sSin, cnt);
-    // an early exit may leave bulk copies in flight: wait for them before the
-    // CTA retires (its shared memory must not be written after it exits)
-    if (early) {
-        for (int k = 0; k < kWStages; ++k)
-            if (*reinterpret_cast<volatile long long*>(&sChunk[warp][k]) < nchunks)
-                mbar_wait(&bar[warp][k], (phase >> k) & 1u);
     }
     if (lane == 0) {
         atomicAdd(&sCulled, (unsigned long long)nculled);
         atomicAdd(&sPassed, (unsigned long long)npassed);
-        atomicAdd(&sStreamed, streamed);
     }
-    // final flush of words that gained bits
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        // every warp saw the same tiles: thread 0's tally is the CTA's
+        atomicAdd(p.stats + ST_STREAMED, streamed);
+        atomicAdd(p.stats + ST_CULLED, sCulled);
+        atomicAdd(p.stats + ST_SKIPPED, streamed - sCulled - sPassed);
+    }
+}
+
+// a3-a6 over the live list, one voxel per thread, into a shared AM seeded from
+// the global AM; a7 at the end.
+__global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ StreamParams p) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ unsigned int sCnt[CT_COUNT];
+    // shared copy of the parameters for the out-of-line process_live (a
+    // reference to the kernel parameter would make every call copy it)
+    __shared__ StreamParams sP;
+    if (threadIdx.x < (int)(sizeof(StreamParams) / 4))
+        reinterpret_cast<unsigned int*>(&sP)[threadIdx.x] = reinterpret_cast<const unsigned int*>(&p)[threadIdx.x];
+    const int m = p.grid.m, W = p.grid.W, MW = m * W;
+    uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
+    uint32_t* sRowFull = sAM + MW;
+    float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
+    float* sSin = sCos + m;
+    const unsigned int nlive = *p.live_count;
+    if ((unsigned long long)blockIdx.x * kThreads >= nlive) return;
+    for (int i = threadIdx.x; i < m; i += blockDim.x) {
+        sCos[i] = p.tab[i];
+        sSin[i] = p.tab[m + i];
+    }
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
+    if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int base = 0; base < m; base += blockDim.x) {
+        const int i = base + threadIdx.x;
+        bool full = false;
+        if (i < m) {
+            full = true;
+            for (int w = 0; w < W; ++w)
+                if (sAM[i * W + w] != row_word_mask(w, p.grid.n)) full = false;
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, full);
+        if (lane == 0 && base + warp * 32 < m) sRowFull[(base + warp * 32) >> 5] = bal;
+    }
+    __syncthreads();
+    const Counters cnt{sCnt};
+    for (unsigned long long e = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; e < nlive;
+         e += (unsigned long long)gridDim.x * kThreads) {
+        const unsigned int vidx = p.live_idx[e];
+        process_live(sP, vidx, p.vox[vidx], sAM, sRowFull, sCos, sSin, cnt);
+    }
     __syncthreads();
     for (int w = threadIdx.x; w < MW; w += blockDim.x) {
         const uint32_t sv = sAM[w];
-        if (sv & ~sShadow[w]) atomicOr(p.gam + w, sv);
+        if (sv & ~ld_cg(p.gam + w)) atomicOr(p.gam + w, sv);
     }
     if (threadIdx.x == 0) {
-        atomicAdd(p.stats + ST_STREAMED, sStreamed);
-        atomicAdd(p.stats + ST_CULLED, sCulled);
-        atomicAdd(p.stats + ST_SKIPPED, sStreamed - sCulled - sPassed);
         atomicAdd(p.stats + ST_LIVE, (unsigned long long)sCnt[CT_LIVE]);
         atomicAdd(p.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
         atomicAdd(p.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
         atomicAdd(p.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
-        if (early) atomicMax(p.stats + ST_EARLY, 1ULL);
     }
 }
 
@@ -443,5 +324,6 @@ __global__ void __launch_bounds__(kThreads) coarse_kernel(const __grid_constant_
         if (sv) atomicOr(p.gam + w, sv);
     }
 }
+
 
 }  // namespace am
