@@ -56,7 +56,9 @@ struct am_ctx {
     uint32_t* d_prev = nullptr;            // diagnostics: copy of the last map
     int diag = 0;
     int cmapT = 32;
-    int phases = 1;
+    int phases = 2;
+    float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
+    float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
     int timing = 0;
     std::vector<cudaEvent_t> ev_start, ev_stop;
@@ -67,7 +69,8 @@ struct am_ctx {
 namespace {
 
 constexpr int kCtrTiles = 1 + ST_COUNT;      // first dynamic tile counter
-constexpr int kCtrWords = kCtrTiles + 1;
+constexpr int kCtrClear = kCtrTiles + 1;     // clear-cell counts of the (up to 3) maps of a call
+constexpr int kCtrWords = kCtrClear + 3;
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -125,6 +128,14 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.vox_coarse = c->d_coarse;
     p.cmapT = c->cmapT;
     p.cull_dist = c->tool.rho_max * (1.f + 1e-5f) + 1e-6f;
+    // the reach cull can only fire when some voxel centre lies farther than
+    // cull_dist from the pivot: compare with the farthest corner of the bbox
+    double far2 = 0.0;
+    for (int k = 0; k < 3; ++k) {
+        const double d = std::max(std::fabs((double)c->bbox[k] - pivot[k]), std::fabs((double)c->bbox[3 + k] - pivot[k]));
+        far2 += d * d;
+    }
+    p.may_cull = std::sqrt(far2) * (1.0 + 1e-6) + 1e-6 > (double)p.cull_dist;
     return p;
 }
 
@@ -249,10 +260,13 @@ int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     return AM_OK;
 }
 
-int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
+// Clear-direction map from `gam`; `slot` picks a zeroed counter of d_ctr.
+int launch_clear_map(am_ctx* ctx, const uint32_t* gam, int slot, cudaStream_t s) {
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
-    clear_map_kernel<<<(ntex + 7) / 8, 256, 0, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_texels, ntex,
-                                                    ctx->d_cmap);
+    unsigned int* n = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrClear + slot);
+    clear_list_kernel<<<1, 1024, 0, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_dirs, n);
+    CK(cudaGetLastError());
+    clear_map_kernel<<<(ntex + 255) / 256, 256, 0, s>>>(ctx->d_dirs, n, ctx->d_texels, ntex, ctx->d_cmap);
     CK(cudaGetLastError());
     return AM_OK;
 }
@@ -262,8 +276,8 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
 //   level 1 (next largest + strided sample, filtered, inner cones) -> clear map
 //   -> the full stream of every voxel, filtered by the map, both cones ->
 //   deferred band.  The coarse levels only make the filter effective; they are
-//   subsets of the model, so the map is the same with or without them
-//   (AM_OPT_PHASES).
+//   subsets of the model, so the map is the same with any number of them
+//   (AM_OPT_PHASES = 0, 1 or 2 levels).
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
@@ -275,14 +289,16 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         // diagnostic: clear map from the previous map computed on this context
         // (exact only when the previous call used the same pivot)
         CK(cudaMemcpyAsync(gam, ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
-        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
+        if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
         cm = ctx->d_cmap;
-    } else if (ctx->phases && ctx->n_l0 > 0) {
+    } else if (ctx->phases > 0 && ctx->n_l0 > 0) {
         if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 1, s))) return rc;
-        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
-        if ((rc = launch_coarse(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, 32, s)))
-            return rc;
-        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
+        if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
+        if (ctx->phases > 1) {
+            if ((rc = launch_coarse(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, 32, s)))
+                return rc;
+            if ((rc = launch_clear_map(ctx, gam, 1, s))) return rc;
+        }
         cm = ctx->d_cmap;
     }
     if (!(ctx->diag & 1)) {
@@ -428,6 +444,10 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
             return bail(AM_ECUDA);
         }
     }
+    if (cudaMalloc(&ctx->d_dirs, (size_t)m * n * sizeof(float4)) != cudaSuccess) {
+        cudaGetLastError();
+        return bail(AM_ENOMEM);
+    }
     if ((rc = ensure_queue(ctx, 1 << 22)) != AM_OK) return bail(rc);
     if ((rc = configure_launch(ctx)) != AM_OK) return bail(rc);
     *out = ctx;
@@ -515,6 +535,16 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     if (nbad) {
         cleanup();
         return fail(ctx, AM_EINVAL, "%llu voxels with a non-finite value or half size <= 0", nbad);
+    }
+    {
+        unsigned int hb[6];
+        UK(cudaMemcpy(hb, bbox, sizeof hb, cudaMemcpyDeviceToHost));
+        for (int k = 0; k < 6; ++k) {  // ordered-int encoding back to float (see float_to_ordered)
+            const unsigned int u = (hb[k] & 0x80000000u) ? (hb[k] & 0x7fffffffu) : ~hb[k];
+            float f;
+            std::memcpy(&f, &u, sizeof f);
+            ctx->bbox[k] = f;
+        }
     }
     if (ctx->morton) {
         UK(cudaMalloc(&keys, (size_t)N * sizeof(unsigned long long)));
@@ -609,8 +639,11 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         CK(cudaMemcpyAsync(h, ctx->d_ctr, sizeof h, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         int64_t* o = reinterpret_cast<int64_t*>(stats);
-        for (int k = 0; k < ST_COUNT; ++k) o[k] = (int64_t)h[1 + k];
-        // band pairs resolved inline are counted as exact tests too
+        static_assert(sizeof(am_stats) == ST_PASSED * sizeof(int64_t), "am_stats mirrors StatIdx");
+        for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
+        // every voxel goes through the filter once; the rest of it was dropped
+        o[ST_STREAMED] = (int64_t)ctx->N;
+        o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
     } else if (!dst_is_device) {
         CK(cudaStreamSynchronize(s));
     }
@@ -705,7 +738,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->timing = (int)value;
         return AM_OK;
     case AM_OPT_PHASES:
-        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "phases must be 0 or 1");
+        if (value < 0 || value > 2) return fail(ctx, AM_EINVAL, "phases must be 0, 1 or 2");
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
@@ -781,6 +814,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);
     cudaFree(ctx->d_prev);
+    cudaFree(ctx->d_dirs);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

@@ -41,16 +41,13 @@ struct ToolDev {
     float bp_R[AM_MAX_CYL];
 };
 
-// Largest radius of any cylinder that starts within `reach` of the pivot.
+// An upper bound on the radius of every cylinder that starts within `reach`
+// of the pivot: the leading radius up to the first growth point, the tool's
+// largest radius beyond it (exact for tools whose radius grows once, like the
+// 3-cylinder tip/shank/holder tool).
 __device__ __forceinline__ float reach_radius(const ToolDev& T, float reach) {
     float R = T.R_first;
-#pragma unroll
-    for (int k = 0; k < 3; ++k)
-        if (T.bp_z[k] <= reach) R = T.bp_R[k];
-    if (T.nbp > 3) {
-        for (int k = 3; k < T.nbp; ++k)
-            if (T.bp_z[k] <= reach) R = T.bp_R[k];
-    }
+    if (T.bp_z[0] <= reach) R = T.Rpm[AM_MAX_CYL - 1];
     return R;
 }
 

@@ -29,7 +29,7 @@ constexpr int kTile = kThreads * kVPT;   // voxels per tile
 
 enum StatIdx {
     ST_STREAMED = 0, ST_CULLED, ST_SKIPPED, ST_LIVE, ST_ROWS, ST_BAND, ST_EXACT, ST_EXACT_HIT,
-    ST_OVERFLOW, ST_EARLY, ST_COUNT
+    ST_OVERFLOW, ST_EARLY, ST_PASSED, ST_COUNT
 };
 
 struct StreamParams {
@@ -58,6 +58,7 @@ struct StreamParams {
     unsigned int* tile_ctr;        // dynamic tile counter of this launch (zeroed)
     unsigned int* live_count;      // live voxels found by the filter (zeroed)
     unsigned int* live_idx;        // their indices into vox (capacity N)
+    int may_cull;                  // some voxel may lie beyond the tool's reach (per pivot)
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,
@@ -146,46 +147,62 @@ __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, 
 // Clear-direction map: for every cube-map texel t with centre c_t
 // and angular radius r_t, U_t >= cos(max(0, angle(c_t, nearest clear cell) - r_t)),
 // so any direction mapped to t is at least acos(U_t) away from every cell that
-// is still clear in `gam`; U_t = -2 when no cell is clear.  Cells only ever get
-// blocked, so a map built from a partial AM stays valid for the final one.
-// One warp per texel; lanes scan the AM words.
-__global__ void __launch_bounds__(256) clear_map_kernel(const uint32_t* __restrict__ gam, GridDev g,
-                                                        const float* __restrict__ tab,
-                                                        const float4* __restrict__ texels, int ntex,
-                                                        float* __restrict__ U) {
-    const int lane = threadIdx.x & 31;
-    const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int nwarps = (gridDim.x * blockDim.x) >> 5;
+// is still clear in `gam`; U_t = -2 when no cell is clear.  The map stores
+// V_t = U_t |U_t| (monotone in U; lets the filter compare squared cosines).
+// Cells only ever get blocked, so a map built from a partial AM stays valid
+// for the final one.
+//
+// Step 1 (one CTA): the directions of the cells still clear, counted in *n.
+__global__ void __launch_bounds__(1024) clear_list_kernel(const uint32_t* __restrict__ gam, GridDev g,
+                                                          const float* __restrict__ tab,
+                                                          float4* __restrict__ dirs, unsigned int* n) {
     const int MW = g.m * g.W;
-    for (int t = warp; t < ntex; t += nwarps) {
-        const float4 c = texels[t];
-        float best = -2.f;
-        for (int w = lane; w < MW; w += 32) {
-            const int i = w / g.W, wj = w - i * g.W;
-            uint32_t clear = ~ld_cg(gam + w) & row_word_mask(wj, g.n);
-            if (!clear) continue;
-            const float cph = __ldg(tab + i), sph = __ldg(tab + g.m + i);
-            const float zc = c.z * cph;
-            while (clear) {
-                const int b = __ffs(clear) - 1;
-                clear &= clear - 1u;
-                const int j = (wj << 5) + b;
-                const float xy = fmaf(c.x, __ldg(tab + 2 * g.m + j), c.y * __ldg(tab + 2 * g.m + g.n + j));
-                best = fmaxf(best, fmaf(sph, xy, zc));
-            }
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        const int i = w / g.W, wj = w - i * g.W;
+        uint32_t clear = ~ld_cg(gam + w) & row_word_mask(wj, g.n);
+        if (!clear) continue;
+        unsigned int pos = atomicAdd(n, (unsigned int)__popc(clear));
+        const float cph = __ldg(tab + i), sph = __ldg(tab + g.m + i);
+        while (clear) {
+            const int j = (wj << 5) + __ffs(clear) - 1;
+            clear &= clear - 1u;
+            dirs[pos++] = make_float4(sph * __ldg(tab + 2 * g.m + j), sph * __ldg(tab + 2 * g.m + g.n + j), cph,
+                                      0.f);
         }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, o));
-        if (lane == 0) {
-            float u = -2.f;
-            if (best >= -1.5f) {
-                // round the nearest-cell angle down and the bound up (fp32 guards)
-                const float th = acosf(fminf(best + 2e-6f, 1.f));
-                const float r = c.w;
-                u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
-            }
-            U[t] = u;
+    }
+}
+
+// Step 2: one thread per texel, the clear directions staged through shared
+// memory in chunks.
+__global__ void __launch_bounds__(256) clear_map_kernel(const float4* __restrict__ dirs,
+                                                        const unsigned int* n,
+                                                        const float4* __restrict__ texels, int ntex,
+                                                        float* __restrict__ V) {
+    constexpr int kChunkDirs = 1024;
+    __shared__ float4 sd[kChunkDirs];
+    const unsigned int cnt = *n;
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    const float4 c = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
+    float best = -2.f;
+    for (unsigned int base = 0; base < cnt; base += kChunkDirs) {
+        const unsigned int k = min((unsigned int)kChunkDirs, cnt - base);
+        __syncthreads();
+        for (unsigned int e = threadIdx.x; e < k; e += blockDim.x) sd[e] = dirs[base + e];
+        __syncthreads();
+        for (unsigned int e = 0; e < k; ++e) {
+            const float4 d = sd[e];
+            best = fmaxf(best, fmaf(c.x, d.x, fmaf(c.y, d.y, c.z * d.z)));
         }
+    }
+    if (t < ntex) {
+        float u = -2.f;
+        if (best >= -1.5f) {
+            // round the nearest-cell angle down and the bound up (fp32 guards)
+            const float th = acosf(fminf(best + 2e-6f, 1.f));
+            const float r = c.w;
+            u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+        }
+        V[t] = u * fabsf(u);
     }
 }
 

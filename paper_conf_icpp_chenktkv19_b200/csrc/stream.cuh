@@ -45,9 +45,12 @@ enum { F_DROP = 0, F_LIVE = 1, F_CULLED = 2 };
 __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T);
 
 // a2 + cheap cone vs clear-direction map (p.cmap is never null: before any map
-// is built it is the all-clear map, U = 1).  F_LIVE when the voxel may still
-// change the AM, F_CULLED beyond reach, F_DROP otherwise.  A voxel holding the
-// pivot blocks every orientation: it fills `am` (shared or global) directly.
+// is built it is the all-clear map).  The map stores V = U |U|, where U bounds
+// from above the cosine of the angle from any direction of the texel to the
+// nearest still-clear cell; V is monotone in U, so U < x <=> V < x |x|.
+// F_LIVE when the voxel may still change the AM, F_CULLED beyond reach,
+// F_DROP otherwise.  A voxel holding the pivot blocks every orientation: it
+// fills `am` (shared or global) directly.
 __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am) {
     const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
     const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
@@ -61,30 +64,30 @@ __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint
     }
     const float invD = rsqrtf(D2);
     const float D = D2 * invD;
-    if (D - r2 > p.cull_dist) return F_CULLED;
+    if (p.may_cull && D - r2 > p.cull_dist) return F_CULLED;
     const float Reff = reach_radius(p.tool, (D + r2) * (1.f + kRadRel));
-    const float s = fmaf((Reff + r2) * invD, 1.f + 1.6e-5f, 1e-6f);
-    const float U = __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT));
-    // U bounds cos(angle to the nearest clear cell) from above for every
-    // direction of the texel: drop when cos(cheap cone) > U.  Far voxels
-    // (s < 1): sin(theta) <= s.  Near voxels: the tool has nothing behind the
+    // drop when cos(cheap cone) > U.  Far voxels (s < 1): sin(theta) <= s, so
+    // cos(cone) = sqrt(1 - s^2).  Near voxels: the tool has nothing behind the
     // plane of its end face at the pivot, so a blocked direction keeps the
-    // sphere centre within r2 of that plane: cos(theta) >= -r2 / D.
-    const bool drop = (s < 1.f) ? (U < 0.f || U * U < 1.f - s * s)
-                                : (U < -fmaf(r2 * invD, 1.f + 1.6e-5f, 1e-6f));
-    return drop ? F_DROP : F_LIVE;
+    // sphere centre within r2 of that plane: cos(cone) = -c with c = r2 / D.
+    const float s = fmaf((Reff + r2) * invD, 1.f + 1.6e-5f, 1e-6f);
+    const float c = fmaf(r2 * invD, 1.f + 1.6e-5f, 1e-6f);
+    const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
+    return __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < thr ? F_DROP : F_LIVE;
 }
 
 // Cube-map texel of v (cube_texel of kernels.cuh with an approximate
-// reciprocal; the texel radii carry 2e-5 rad of slack for rounding at edges).
+// reciprocal; ties between axes may pick either face, and the texel radii
+// carry 2e-5 rad of slack for rounding at texel edges).
 __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
     const float ax = fabsf(vx), ay = fabsf(vy), az = fabsf(vz);
-    const bool xm = ax >= fmaxf(ay, az);
-    const bool ym = !xm && ay >= az;
     const float a = fmaxf(ax, fmaxf(ay, az));
+    const bool xm = ax == a;
+    const bool ym = !xm && ay == a;
     const float u = xm ? vy : vx;
     const float w = (xm || ym) ? vz : vy;
-    const int face = xm ? (vx < 0.f) : (ym ? 2 + (vy < 0.f) : 4 + (vz < 0.f));
+    const float maj = xm ? vx : (ym ? vy : vz);
+    const int face = (xm ? 0 : (ym ? 2 : 4)) + (maj < 0.f);
     const float hs = 0.5f * (float)T;
     const float sc = hs * rcp_approx(a);
     const int iu = min(T - 1, max(0, __float2int_rz(fmaf(u, sc, hs))));
@@ -110,7 +113,7 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
     if (c.cout > 1.f) return;
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
-    if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout) return;
+    if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) return;
     const float ao = acosf(fmaxf(c.cout, -1.f));
     const int i0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
     const int i1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
@@ -158,51 +161,61 @@ __host__ __device__ inline size_t live_smem_bytes(int m, int W) {
     return (size_t)(m * W + ((m + 31) >> 5)) * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
 }
 
-// a1-a2 + cheap cones over vox[0, N): live indices go to p.live_idx.
+// Append the live voxels among one warp-row of 32 to the global live list.
+__device__ __forceinline__ void append_live(const StreamParams& p, bool live, unsigned int idx,
+                                            unsigned int& npassed) {
+    const unsigned int mlive = __ballot_sync(0xffffffffu, live);
+    if (mlive) {
+        const int lane = threadIdx.x & 31;
+        npassed += __popc(mlive);
+        unsigned int pos = 0;
+        const int leader = __ffs(mlive) - 1;
+        if (lane == leader) pos = atomicAdd(p.live_count, (unsigned int)__popc(mlive));
+        pos = __shfl_sync(0xffffffffu, pos, leader) + __popc(mlive & ((1u << lane) - 1u));
+        if (live) p.live_idx[pos] = idx;
+    }
+}
+
+// a1-a2 + cheap cones over vox[0, N): live indices go to p.live_idx.  Full
+// tiles of kTile voxels take the unguarded path (kVPT independent LDG.128 per
+// thread, streaming cache hint); the ragged last tile is guarded.
 __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant__ StreamParams p) {
-    __shared__ unsigned long long sCulled, sPassed;
-    if (threadIdx.x == 0) sCulled = sPassed = 0ull;
+    __shared__ unsigned int sCulled, sPassed;
+    if (threadIdx.x == 0) sCulled = sPassed = 0u;
     __syncthreads();
-    const int lane = threadIdx.x & 31;
     unsigned int nculled = 0, npassed = 0;
-    unsigned long long streamed = 0;
-    const long long ntiles = (p.N + kTile - 1) / kTile;
-    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        const long long base = t * kTile + threadIdx.x;
+    const unsigned int nfull = (unsigned int)(p.N / kTile);
+    for (unsigned int t = blockIdx.x; t < nfull; t += gridDim.x) {
+        const unsigned int base = t * kTile + threadIdx.x;
+        const float4* src = p.vox + base;
         float4 q[kVPT];
 #pragma unroll
-        for (int k = 0; k < kVPT; ++k) {
-            const long long idx = base + (long long)k * kThreads;
-            q[k] = idx < p.N ? __ldcs(p.vox + idx) : make_float4(0.f, 0.f, 0.f, -1.f);
-        }
+        for (int k = 0; k < kVPT; ++k) q[k] = __ldcs(src + k * kThreads);
         int f[kVPT];
 #pragma unroll
-        for (int k = 0; k < kVPT; ++k) f[k] = q[k].w > 0.f ? fast_filter(p, q[k], p.gam) : F_DROP;
-        if (lane == 0) streamed += (unsigned long long)min((long long)kTile, p.N - t * kTile);
+        for (int k = 0; k < kVPT; ++k) f[k] = fast_filter(p, q[k], p.gam);
 #pragma unroll
         for (int k = 0; k < kVPT; ++k) {
-            const unsigned int mlive = __ballot_sync(0xffffffffu, f[k] == F_LIVE);
-            nculled += __popc(__ballot_sync(0xffffffffu, f[k] == F_CULLED));
-            if (mlive) {
-                npassed += __popc(mlive);
-                unsigned int pos = 0;
-                const int leader = __ffs(mlive) - 1;
-                if (lane == leader) pos = atomicAdd(p.live_count, (unsigned int)__popc(mlive));
-                pos = __shfl_sync(0xffffffffu, pos, leader) + __popc(mlive & ((1u << lane) - 1u));
-                if (f[k] == F_LIVE) p.live_idx[pos] = (unsigned int)(base + (long long)k * kThreads);
-            }
+            nculled += f[k] >> 1;
+            append_live(p, f[k] == F_LIVE, base + k * kThreads, npassed);
         }
     }
-    if (lane == 0) {
-        atomicAdd(&sCulled, (unsigned long long)nculled);
-        atomicAdd(&sPassed, (unsigned long long)npassed);
+    if (blockIdx.x == nfull % gridDim.x && (long long)nfull * kTile < p.N) {  // ragged tail
+        const unsigned int base = nfull * kTile + threadIdx.x;
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) {
+            const unsigned int idx = base + k * kThreads;
+            const int f = idx < p.N ? fast_filter(p, p.vox[idx], p.gam) : F_DROP;
+            nculled += f >> 1;
+            append_live(p, f == F_LIVE, idx, npassed);
+        }
     }
+    if ((threadIdx.x & 31) == 0) atomicAdd(&sPassed, npassed);
+    if (nculled) atomicAdd(&sCulled, nculled);
     __syncthreads();
     if (threadIdx.x == 0) {
-        // every warp saw the same tiles: thread 0's tally is the CTA's
-        atomicAdd(p.stats + ST_STREAMED, streamed);
-        atomicAdd(p.stats + ST_CULLED, sCulled);
-        atomicAdd(p.stats + ST_SKIPPED, streamed - sCulled - sPassed);
+        atomicAdd(p.stats + ST_CULLED, (unsigned long long)sCulled);
+        atomicAdd(p.stats + ST_PASSED, (unsigned long long)sPassed);
     }
 }
 

@@ -29,10 +29,11 @@ def main():
     ctx.upload(torch.from_numpy(C).cuda(), torch.from_numpy(H).cuda())
     out = torch.zeros(ctx.words, dtype=torch.int32, device="cuda")
     res = []
-    for T in (16, 32, 64, 128):
+    for T, ph in ((32, 2), (64, 2), (128, 2), (32, 1), (64, 1), (128, 1)):
         ctx.set_option(B.OPT_CMAP_T, T)
+        ctx.set_option(B.OPT_PHASES, ph)
         for p in P:
-            row = {"T": T, "pivot": p.tolist()}
+            row = {"T": T, "levels": ph, "pivot": p.tolist()}
             ctx.set_option(B.OPT_DIAG, 1)
             w, _ = ctx.compute(p)
             row["coarse_bits"] = int(am.unpack(w, cfg.m, cfg.n).sum())
