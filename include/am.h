@@ -88,7 +88,7 @@ enum {
                                     of the coarse levels (a lower-bound probe of the filter; the
                                     result is exact only when that map had the same pivot)       */
     AM_OPT_CMAP_T = 9            /* clear-direction map resolution: texels per cube-face side
-                                    (4..256, default 32)                                         */
+                                    (4..256, default 128)                                        */
 };
 
 /*

@@ -55,7 +55,7 @@ struct am_ctx {
     float* d_cmap_ones = nullptr;          // the all-clear map (no voxel can be dropped)
     uint32_t* d_prev = nullptr;            // diagnostics: copy of the last map
     int diag = 0;
-    int cmapT = 32;
+    int cmapT = 128;
     int phases = 2;
     float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
@@ -70,7 +70,8 @@ namespace {
 
 constexpr int kCtrTiles = 1 + ST_COUNT;      // first dynamic tile counter
 constexpr int kCtrClear = kCtrTiles + 1;     // clear-cell counts of the (up to 3) maps of a call
-constexpr int kCtrWords = kCtrClear + 3;
+constexpr int kCtrWords = kCtrClear + 4;     // + the live count of the level-1 stream
+constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the level-1 stream
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -196,7 +197,8 @@ int configure_launch(am_ctx* ctx) {
     if (ctx->smem > 232448 || ctx->smem_coarse > 232448)
         return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
                     ctx->grid.n, ctx->smem);
-    CK(cudaFuncSetAttribute(live_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(live_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(live_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
     CK(cudaFuncSetAttribute(coarse_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_coarse));
     int occ = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, filter_kernel, kThreads, 0);
@@ -211,14 +213,15 @@ int configure_launch(am_ctx* ctx) {
 
 // The full voxel stream over vox[0, n) with clear-direction map `cmap`.
 int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, bool timed,
-                  cudaStream_t s) {
+                  cudaStream_t s, bool coarse = false) {
     if (n <= 0) return AM_OK;
     p.vox = vox;
     p.N = n;
     p.vbase = 0;
     p.vtag = 0;
     p.cmap = cmap;
-    p.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
+    p.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles + (coarse ? 4 : 0));
+    if (coarse) p.stats = ctx->d_ctr + kCtrWords;  // keep am_stats about the full stream
     p.live_idx = ctx->d_live;
     const long long ntiles = (n + kTile - 1) / kTile;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
@@ -238,7 +241,10 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
-    live_kernel<<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
+    if (coarse)
+        live_kernel<true><<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
+    else
+        live_kernel<false><<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
     CK(cudaGetLastError());
     return AM_OK;
 }
@@ -280,7 +286,7 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, int slot, cudaStream_t s)
 //   (AM_OPT_PHASES = 0, 1 or 2 levels).
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
-    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrAll * sizeof(unsigned long long), s));
     if (ctx->N == 0) return AM_OK;
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
@@ -295,7 +301,10 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 1, s))) return rc;
         if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
         if (ctx->phases > 1) {
-            if ((rc = launch_coarse(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, 32, s)))
+            // level 1 through the same filter + live pipeline as the full stream
+            // (inner cones only, no band)
+            if ((rc = launch_stream(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, false, s,
+                                    true)))
                 return rc;
             if ((rc = launch_clear_map(ctx, gam, 1, s))) return rc;
         }
@@ -420,7 +429,7 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
     };
     if (cudaMalloc(&ctx->d_tab, tab.size() * sizeof(float)) != cudaSuccess ||
         cudaMemcpy(ctx->d_tab, tab.data(), tab.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMalloc(&ctx->d_ctr, kCtrWords * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_ctr, kCtrAll * sizeof(unsigned long long)) != cudaSuccess ||
         cudaMalloc(&ctx->d_am, (size_t)ctx->MW * sizeof(uint32_t)) != cudaSuccess) {
         cudaGetLastError();
         return bail(AM_ENOMEM);

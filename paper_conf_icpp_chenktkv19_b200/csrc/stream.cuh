@@ -96,6 +96,10 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
 }
 
 // a3-a6 for one live voxel: both cones, rasterised row by row, band deferred.
+// COARSE (level 1 of the clear-direction map) rasterises the inner cone only:
+// the map needs certainly-blocked cells, and every coarse voxel is streamed
+// again, with its band, by the full stream.
+template <bool COARSE>
 __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vidx, float4 q, uint32_t* sAM,
                                           const uint32_t* sRowFull, const float* sCos, const float* sSin,
                                           Counters cnt) {
@@ -109,7 +113,13 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
     const float phv = atan2f(rxy, vz);
     // a4: the two cones (GETTOOLICA twice, Alg. 1)
     atomicAdd(cnt.c + CT_LIVE, 1u);
-    const Cones c = tool_cones(D, h, T);
+    Cones c;
+    if (COARSE) {
+        c.cin = c.cout = inner_cone(D, h, T);
+        c.clo = 2.f;
+    } else {
+        c = tool_cones(D, h, T);
+    }
     if (c.cout > 1.f) return;
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
@@ -127,6 +137,17 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
     for (int i = i0; i <= i1; ++i) {
         if ((ld_vol_shared(sRowFull + (i >> 5)) >> (i & 31)) & 1u) continue;
         const float base = sCos[i] * cphv, den = sSin[i] * sphv;
+        if (COARSE) {
+            const Interval In = gamma_interval(c.cin, base, den, gv, -1, g);
+            if (In.len == 0) continue;
+            ++rows;
+            for (int w = 0; w < W; ++w) {
+                const uint32_t ib = interval_bits(In, w, g.n);
+                uint32_t* wp = sAM + i * W + w;
+                if (ib & ~ld_vol_shared(wp)) atomicOr(wp, ib);
+            }
+            continue;
+        }
         const Interval O = gamma_interval(c.cout, base, den, gv, +1, g);
         if (O.len == 0) continue;
         ++rows;
@@ -221,6 +242,7 @@ __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant_
 
 // a3-a6 over the live list, one voxel per thread, into a shared AM seeded from
 // the global AM; a7 at the end.
+template <bool COARSE>
 __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ StreamParams p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ unsigned int sCnt[CT_COUNT];
@@ -260,7 +282,7 @@ __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ 
     for (unsigned long long e = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; e < nlive;
          e += (unsigned long long)gridDim.x * kThreads) {
         const unsigned int vidx = p.live_idx[e];
-        process_live(sP, vidx, p.vox[vidx], sAM, sRowFull, sCos, sSin, cnt);
+        process_live<COARSE>(sP, vidx, p.vox[vidx], sAM, sRowFull, sCos, sSin, cnt);
     }
     __syncthreads();
     for (int w = threadIdx.x; w < MW; w += blockDim.x) {

@@ -29,7 +29,7 @@ def main():
     ctx.upload(torch.from_numpy(C).cuda(), torch.from_numpy(H).cuda())
     out = torch.zeros(ctx.words, dtype=torch.int32, device="cuda")
     res = []
-    for T, ph in ((32, 2), (64, 2), (128, 2), (32, 1), (64, 1), (128, 1)):
+    for T, ph in ((64, 2), (128, 2), (256, 2), (128, 1)):
         ctx.set_option(B.OPT_CMAP_T, T)
         ctx.set_option(B.OPT_PHASES, ph)
         for p in P:
