@@ -199,7 +199,6 @@ int configure_launch(am_ctx* ctx) {
                     ctx->grid.n, ctx->smem);
     CK(cudaFuncSetAttribute(live_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
     CK(cudaFuncSetAttribute(live_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
-    CK(cudaFuncSetAttribute(coarse_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_coarse));
     int occ = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, filter_kernel, kThreads, 0);
     if (e != cudaSuccess || occ < 1) {
@@ -253,15 +252,17 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
 int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, int batch,
                   cudaStream_t s) {
     if (n <= 0) return AM_OK;
+    (void)batch;
     p.vox = vox;
     p.N = n;
     p.cmap = cmap;
-    p.tile = batch;
-    const long long warps = (n + batch - 1) / batch;
-    long long g = (warps + kWarps - 1) / kWarps;
-    const long long gmax = (long long)ctx->sms * 8;
+    p.live_idx = nullptr;  // every voxel of the level is live
+    p.live_count = nullptr;
+    p.stats = ctx->d_ctr + kCtrWords;  // keep am_stats about the full stream
+    long long g = (n + kThreads - 1) / kThreads;
+    const long long gmax = (long long)ctx->sms * kLiveBlocksPerSM;
     if (g > gmax) g = gmax;
-    coarse_kernel<<<(unsigned)g, kThreads, ctx->smem_coarse, s>>>(p);
+    live_kernel<true><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
     CK(cudaGetLastError());
     return AM_OK;
 }

@@ -15,15 +15,13 @@
 //   instructions; the survivors ("live") are appended to a global list with one
 //   warp-aggregated atomic.
 //
-// live_kernel (a3-a6; the live voxels only, ~0.1-1 %): one voxel per thread,
-//   the paper's two ICA cones (Alg. 1) checked against the map once
-//   more, then rasterised row by row into the CTA's shared AM; band cells are
-//   deferred to the global band queue; the shared AM is OR-ed into the global
-//   AM at the end (a7).
-//
-// coarse_kernel (levels 0/1, the largest voxels): one warp per voxel, phi-rows
-//   across lanes, inner cones only -- these few voxels have cones spanning most
-//   rows, so row parallelism is what they need.
+// live_kernel (a3-a6; the live voxels only, ~0.01-1 %): 32 voxels per warp,
+//   one per lane for the paper's two ICA cones (Alg. 1), checked
+//   against the map once more; the (voxel, phi-row) pairs of the warp are then
+//   dealt evenly over the lanes and rasterised into the CTA's shared AM; band
+//   cells are deferred to the global band queue; the shared AM is OR-ed into
+//   the global AM at the end (a7).  The clear-map levels use the same kernel
+//   with inner cones only (level 0: every voxel of the level is live).
 #pragma once
 #include "kernels.cuh"
 
@@ -95,50 +93,96 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
     return (face * T + iw) * T + iu;
 }
 
-// a3-a6 for one live voxel: both cones, rasterised row by row, band deferred.
-// COARSE (level 1 of the clear-direction map) rasterises the inner cone only:
-// the map needs certainly-blocked cells, and every coarse voxel is streamed
-// again, with its band, by the full stream.
+// a3-a6 for the live voxels of one warp (one per lane, `valid` lanes only).
+// Each lane first computes its own voxel's two cones (GETTOOLICA twice, Alg. 1
+// L147-148), checks the exact outer cone against the clear-direction map and
+// finds its phi-row range; the warp then shares out the (voxel, row) pairs of
+// all 32 voxels evenly over its lanes (a warp scan of the row counts), so a
+// voxel with a 64-row cone and one with a 2-row cone cost the same latency.
+// Per row (Alg. 1 L149-155 for all cells of a row at once): the inner-cone
+// interval is OR-ed into the shared AM, outer-minus-inner cells still clear go
+// to the band queue.  COARSE (clear-map levels) rasterises inner cones only.
 template <bool COARSE>
-__device__ __noinline__ void process_live(const StreamParams& p, unsigned int vidx, float4 q, uint32_t* sAM,
-                                          const uint32_t* sRowFull, const float* sCos, const float* sSin,
-                                          Counters cnt) {
+__device__ __noinline__ void process_live_warp(const StreamParams& p, bool valid, unsigned int vidx, float4 q,
+                                               uint32_t* sAM, const uint32_t* sRowFull, const float* sCos,
+                                               const float* sSin, Counters cnt) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
-    const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
-    const float D2 = vx * vx + vy * vy + vz * vz;
-    const float D = sqrtf(D2);
-    if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) return;  // filled already
-    const float rxy = sqrtf(vx * vx + vy * vy);
-    const float phv = atan2f(rxy, vz);
-    // a4: the two cones (GETTOOLICA twice, Alg. 1)
-    atomicAdd(cnt.c + CT_LIVE, 1u);
-    Cones c;
-    if (COARSE) {
-        c.cin = c.cout = inner_cone(D, h, T);
-        c.clo = 2.f;
-    } else {
-        c = tool_cones(D, h, T);
+    const int lane = threadIdx.x & 31;
+    float cin = 2.f, cout = 2.f, clo = 2.f, cphv = 0.f, sphv = 0.f, gv = 0.f;
+    int i0 = 0, nrows = 0;
+    if (valid) {
+        const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
+        const float D = sqrtf(vx * vx + vy * vy + vz * vz);
+        const bool inside = D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h;
+        if (!inside) {  // (a voxel holding the pivot was filled by the filter)
+            Cones c;
+            if (COARSE) {
+                c.cin = c.cout = inner_cone(D, h, T);
+                c.clo = 2.f;
+            } else {
+                c = tool_cones(D, h, T);
+            }
+            // the exact outer cone against the clear-direction map: no clear
+            // cell within it means this voxel cannot change the map
+            if (c.cout <= 1.f &&
+                __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) >= c.cout * fabsf(c.cout)) {
+                const float rxy = sqrtf(vx * vx + vy * vy);
+                const float phv = atan2f(rxy, vz);
+                const float ao = acosf(fmaxf(c.cout, -1.f));
+                const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+                const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+                if (a0 <= a1 && !rows_all_full(sRowFull, a0, a1)) {
+                    const float invD = 1.f / D;
+                    cin = c.cin;
+                    cout = c.cout;
+                    clo = c.clo;
+                    cphv = vz * invD;
+                    sphv = rxy * invD;
+                    gv = atan2f(vy, vx);
+                    i0 = a0;
+                    nrows = a1 - a0 + 1;
+                }
+            }
+        }
     }
-    if (c.cout > 1.f) return;
-    // the exact outer cone against the clear-direction map: no clear cell
-    // within it means this voxel cannot change the map
-    if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) return;
-    const float ao = acosf(fmaxf(c.cout, -1.f));
-    const int i0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-    const int i1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-    if (i0 > i1 || rows_all_full(sRowFull, i0, i1)) return;
-    const float invD = 1.f / D;
-    const float cphv = vz * invD, sphv = rxy * invD;
-    const float gv = atan2f(vy, vx);
+    if (valid) atomicAdd(cnt.c + CT_LIVE, 1u);
+    // warp scan of the row counts; (voxel, row) pairs are dealt round-robin
+    int incl = nrows;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const int total = __shfl_sync(0xffffffffu, incl, 31);
     const int W = g.W;
     unsigned int rows = 0;
-    // a5: rasterise row by row (Alg. 1 L149-155 for all cells of a row at once)
-    for (int i = i0; i <= i1; ++i) {
+    for (int base = 0; base < total; base += 32) {
+        const int k = base + lane;
+        // owner = number of lanes whose inclusive count is <= k
+        int owner = 0;
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+            const int cand = owner + step;
+            if (__shfl_sync(0xffffffffu, incl, cand - 1) <= k) owner = cand;
+        }
+        owner = min(owner, 31);
+        const int o_incl = __shfl_sync(0xffffffffu, incl, owner);
+        const int o_n = __shfl_sync(0xffffffffu, nrows, owner);
+        const int o_i0 = __shfl_sync(0xffffffffu, i0, owner);
+        const float o_cin = __shfl_sync(0xffffffffu, cin, owner);
+        const float o_cout = __shfl_sync(0xffffffffu, cout, owner);
+        const float o_clo = __shfl_sync(0xffffffffu, clo, owner);
+        const float o_c = __shfl_sync(0xffffffffu, cphv, owner);
+        const float o_s = __shfl_sync(0xffffffffu, sphv, owner);
+        const float o_gv = __shfl_sync(0xffffffffu, gv, owner);
+        const unsigned int o_vidx = __shfl_sync(0xffffffffu, vidx, owner);
+        if (k >= total) continue;
+        const int i = o_i0 + (k - (o_incl - o_n));
         if ((ld_vol_shared(sRowFull + (i >> 5)) >> (i & 31)) & 1u) continue;
-        const float base = sCos[i] * cphv, den = sSin[i] * sphv;
+        const float rb = sCos[i] * o_c, rd = sSin[i] * o_s;
         if (COARSE) {
-            const Interval In = gamma_interval(c.cin, base, den, gv, -1, g);
+            const Interval In = gamma_interval(o_cin, rb, rd, o_gv, -1, g);
             if (In.len == 0) continue;
             ++rows;
             for (int w = 0; w < W; ++w) {
@@ -148,11 +192,11 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
             }
             continue;
         }
-        const Interval O = gamma_interval(c.cout, base, den, gv, +1, g);
+        const Interval O = gamma_interval(o_cout, rb, rd, o_gv, +1, g);
         if (O.len == 0) continue;
         ++rows;
-        const Interval In = gamma_interval(c.cin, base, den, gv, -1, g);
-        const Interval X = gamma_interval(c.clo, base, den, gv, -1, g);
+        const Interval In = gamma_interval(o_cin, rb, rd, o_gv, -1, g);
+        const Interval X = gamma_interval(o_clo, rb, rd, o_gv, -1, g);
         for (int w = 0; w < W; ++w) {
             uint32_t ob = interval_bits(O, w, g.n);
             if (!ob) continue;
@@ -169,7 +213,7 @@ __device__ __noinline__ void process_live(const StreamParams& p, unsigned int vi
             while (band) {
                 const int b = __ffs(band) - 1;
                 band &= band - 1u;
-                push_band(p, sAM, vidx, q, i * g.n + (w << 5) + b, wp, 1u << b, cnt);
+                push_band(p, sAM, o_vidx, p.vox_main[o_vidx], i * g.n + (w << 5) + b, wp, 1u << b, cnt);
             }
         }
     }
@@ -240,13 +284,14 @@ __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant_
     }
 }
 
-// a3-a6 over the live list, one voxel per thread, into a shared AM seeded from
-// the global AM; a7 at the end.
+// a3-a6 over the live list, 32 voxels per warp, into a shared AM seeded from
+// the global AM; a7 (OR into the global AM) at the end.  With p.live_idx ==
+// nullptr every voxel of vox[0, N) is live (clear-map level 0).
 template <bool COARSE>
 __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ StreamParams p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ unsigned int sCnt[CT_COUNT];
-    // shared copy of the parameters for the out-of-line process_live (a
+    // shared copy of the parameters for the out-of-line process_live_warp (a
     // reference to the kernel parameter would make every call copy it)
     __shared__ StreamParams sP;
     if (threadIdx.x < (int)(sizeof(StreamParams) / 4))
@@ -256,7 +301,7 @@ __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ 
     uint32_t* sRowFull = sAM + MW;
     float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
     float* sSin = sCos + m;
-    const unsigned int nlive = *p.live_count;
+    const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
     if ((unsigned long long)blockIdx.x * kThreads >= nlive) return;
     for (int i = threadIdx.x; i < m; i += blockDim.x) {
         sCos[i] = p.tab[i];
@@ -279,10 +324,18 @@ __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ 
     }
     __syncthreads();
     const Counters cnt{sCnt};
-    for (unsigned long long e = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; e < nlive;
-         e += (unsigned long long)gridDim.x * kThreads) {
-        const unsigned int vidx = p.live_idx[e];
-        process_live<COARSE>(sP, vidx, p.vox[vidx], sAM, sRowFull, sCos, sSin, cnt);
+    // warps stride over groups of 32 entries (the loop bound is warp-uniform)
+    for (unsigned long long e0 = (blockIdx.x * (unsigned long long)kThreads) + warp * 32ull; e0 < nlive;
+         e0 += (unsigned long long)gridDim.x * kThreads) {
+        const unsigned long long e = e0 + lane;
+        const bool valid = e < nlive;
+        unsigned int vidx = 0;
+        float4 q = make_float4(0.f, 0.f, 0.f, 1.f);
+        if (valid) {
+            vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
+            q = p.vox[vidx];
+        }
+        process_live_warp<COARSE>(sP, valid, vidx, q, sAM, sRowFull, sCos, sSin, cnt);
     }
     __syncthreads();
     for (int w = threadIdx.x; w < MW; w += blockDim.x) {
@@ -296,69 +349,5 @@ __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ 
         atomicAdd(p.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
     }
 }
-
-// Coarse levels: inner cones of the largest voxels, one warp per voxel with
-// phi-rows across lanes, into a shared AM flushed to the global AM at the end.
-// Voxels whose cheap cone holds no clear cell of p.cmap are skipped.
-__global__ void __launch_bounds__(kThreads) coarse_kernel(const __grid_constant__ StreamParams p) {
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    const GridDev& g = p.grid;
-    const int m = g.m, W = g.W, MW = m * W;
-    uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
-    float* sCos = reinterpret_cast<float*>(sAM + MW);
-    float* sSin = sCos + m;
-    for (int i = threadIdx.x; i < m; i += blockDim.x) {
-        sCos[i] = p.tab[i];
-        sSin[i] = p.tab[m + i];
-    }
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = 0u;
-    __syncthreads();
-    const int lane = threadIdx.x & 31;
-    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
-    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    const int B = p.tile;  // voxels per warp iteration: 1 (level 0, all live) or 32 (level 1, filtered)
-    for (long long base = gw * B; base < p.N; base += nw * B) {
-        const long long idx = base + lane;
-        float4 q = make_float4(0.f, 0.f, 0.f, 1.f);
-        int f = F_DROP;
-        if (lane < B && idx < p.N) {
-            q = p.vox[idx];
-            f = fast_filter(p, q, sAM);
-        }
-        unsigned int live = __ballot_sync(0xffffffffu, f == F_LIVE);
-        while (live) {
-            const int src = __ffs(live) - 1;
-            live &= live - 1u;
-            const float4 v = make_float4(__shfl_sync(0xffffffffu, q.x, src), __shfl_sync(0xffffffffu, q.y, src),
-                                         __shfl_sync(0xffffffffu, q.z, src), __shfl_sync(0xffffffffu, q.w, src));
-            const float vx = v.x - p.px, vy = v.y - p.py, vz = v.z - p.pz, h = v.w;
-            const float D = sqrtf(vx * vx + vy * vy + vz * vz);
-            const float cin = inner_cone(D, h, p.tool);
-            if (cin > 1.f) continue;
-            const float rxy = sqrtf(vx * vx + vy * vy);
-            const float phv = atan2f(rxy, vz);
-            const float ai = acosf(fmaxf(cin, -1.f));
-            const int i0 = max(0, (int)ceilf((phv - ai - kRowSlack) * g.inv_dphi - 0.5f));
-            const int i1 = min(m - 1, (int)floorf((phv + ai + kRowSlack) * g.inv_dphi - 0.5f));
-            const float invD = 1.f / D;
-            const float cphv = vz * invD, sphv = rxy * invD;
-            const float gv = atan2f(vy, vx);
-            for (int i = i0 + lane; i <= i1; i += 32) {
-                const Interval In = gamma_interval(cin, sCos[i] * cphv, sSin[i] * sphv, gv, -1, g);
-                if (In.len == 0) continue;
-                for (int w = 0; w < W; ++w) {
-                    const uint32_t ib = interval_bits(In, w, g.n);
-                    if (ib & ~ld_vol_shared(sAM + i * W + w)) atomicOr(sAM + i * W + w, ib);
-                }
-            }
-        }
-    }
-    __syncthreads();
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
-        const uint32_t sv = sAM[w];
-        if (sv) atomicOr(p.gam + w, sv);
-    }
-}
-
 
 }  // namespace am
