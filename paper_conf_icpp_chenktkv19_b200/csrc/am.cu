@@ -49,6 +49,8 @@ struct am_ctx {
     // coarse levels (largest voxels + a strided sample) and the clear-direction map
     float4* d_coarse = nullptr;
     unsigned int* d_live = nullptr;        // live-voxel list of the full stream (capacity N)
+    ConeRec* d_recs = nullptr;             // cone records (kRecCap) and row tasks (kTaskCap)
+    unsigned long long* d_tasks = nullptr;
     long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
     float4* d_texels = nullptr;            // cube-map texel centres (xyz) + angular radius (w)
     float* d_cmap = nullptr;
@@ -68,10 +70,16 @@ struct am_ctx {
 
 namespace {
 
-constexpr int kCtrTiles = 1 + ST_COUNT;      // first dynamic tile counter
+// d_ctr layout (64-bit words, zeroed once per map): [0] band-queue count,
+// [1, 1 + ST_COUNT) am_stats of the full stream, then the per-stage counters,
+// then scratch stats for the clear-map levels.
+constexpr int kCtrTiles = 1 + ST_COUNT;      // live count: full stream (+0), level 1 (+4)
 constexpr int kCtrClear = kCtrTiles + 1;     // clear-cell counts of the (up to 3) maps of a call
-constexpr int kCtrWords = kCtrClear + 4;     // + the live count of the level-1 stream
-constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the level-1 stream
+constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, task count at +2s+1
+constexpr int kCtrWords = kCtrRT + 6;
+constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
+constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
+constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -197,8 +205,8 @@ int configure_launch(am_ctx* ctx) {
     if (ctx->smem > 232448 || ctx->smem_coarse > 232448)
         return fail(ctx, AM_EINVAL, "grid %dx%d needs %zu B of shared memory per CTA: too large", m,
                     ctx->grid.n, ctx->smem);
-    CK(cudaFuncSetAttribute(live_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
-    CK(cudaFuncSetAttribute(live_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(row_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    CK(cudaFuncSetAttribute(row_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
     int occ = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, filter_kernel, kThreads, 0);
     if (e != cudaSuccess || occ < 1) {
@@ -207,6 +215,29 @@ int configure_launch(am_ctx* ctx) {
                     ctx->grid.n, ctx->smem);
     }
     ctx->occ = occ;
+    return AM_OK;
+}
+
+// cone_kernel then row_kernel over the live list of p (stage s: its counters).
+int launch_cones_rows(am_ctx* ctx, StreamParams p, bool coarse, int stage, cudaStream_t s) {
+    p.recs = ctx->d_recs;
+    p.tasks = ctx->d_tasks;
+    p.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2 * stage);
+    p.task_count = ctx->d_ctr + kCtrRT + 2 * stage + 1;
+    p.rec_cap = kRecCap;
+    p.task_cap = kTaskCap;
+    const unsigned int gc = (unsigned int)(ctx->sms * 8);
+    const unsigned int gr = (unsigned int)(ctx->sms * kLiveBlocksPerSM);
+    if (coarse) {
+        cone_kernel<true><<<gc, kThreads, 0, s>>>(p);
+        CK(cudaGetLastError());
+        row_kernel<true><<<gr, kThreads, ctx->smem, s>>>(p);
+    } else {
+        cone_kernel<false><<<gc, kThreads, 0, s>>>(p);
+        CK(cudaGetLastError());
+        row_kernel<false><<<gr, kThreads, ctx->smem, s>>>(p);
+    }
+    CK(cudaGetLastError());
     return AM_OK;
 }
 
@@ -240,31 +271,20 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
-    if (coarse)
-        live_kernel<true><<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
-    else
-        live_kernel<false><<<(unsigned)(ctx->sms * kLiveBlocksPerSM), kThreads, ctx->smem, s>>>(p);
-    CK(cudaGetLastError());
-    return AM_OK;
+    return launch_cones_rows(ctx, p, coarse, coarse ? 1 : 2, s);
 }
 
-// A coarse level: inner cones of vox[0, n), `batch` voxels per warp iteration.
-int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, int batch,
+// A coarse level: inner cones of every voxel of vox[0, n) (no filter).
+int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, int stage,
                   cudaStream_t s) {
     if (n <= 0) return AM_OK;
-    (void)batch;
     p.vox = vox;
     p.N = n;
     p.cmap = cmap;
     p.live_idx = nullptr;  // every voxel of the level is live
     p.live_count = nullptr;
     p.stats = ctx->d_ctr + kCtrWords;  // keep am_stats about the full stream
-    long long g = (n + kThreads - 1) / kThreads;
-    const long long gmax = (long long)ctx->sms * kLiveBlocksPerSM;
-    if (g > gmax) g = gmax;
-    live_kernel<true><<<(unsigned)g, kThreads, ctx->smem, s>>>(p);
-    CK(cudaGetLastError());
-    return AM_OK;
+    return launch_cones_rows(ctx, p, true, stage, s);
 }
 
 // Clear-direction map from `gam`; `slot` picks a zeroed counter of d_ctr.
@@ -299,7 +319,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
         cm = ctx->d_cmap;
     } else if (ctx->phases > 0 && ctx->n_l0 > 0) {
-        if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 1, s))) return rc;
+        if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 0, s))) return rc;
         if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
         if (ctx->phases > 1) {
             // level 1 through the same filter + live pipeline as the full stream
@@ -454,7 +474,9 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
             return bail(AM_ECUDA);
         }
     }
-    if (cudaMalloc(&ctx->d_dirs, (size_t)m * n * sizeof(float4)) != cudaSuccess) {
+    if (cudaMalloc(&ctx->d_dirs, (size_t)m * n * sizeof(float4)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_recs, (size_t)kRecCap * sizeof(ConeRec)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_tasks, (size_t)kTaskCap * sizeof(unsigned long long)) != cudaSuccess) {
         cudaGetLastError();
         return bail(AM_ENOMEM);
     }
@@ -820,6 +842,8 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_queue);
     cudaFree(ctx->d_coarse);
     cudaFree(ctx->d_live);
+    cudaFree(ctx->d_recs);
+    cudaFree(ctx->d_tasks);
     cudaFree(ctx->d_texels);
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);

@@ -59,6 +59,13 @@ struct StreamParams {
     unsigned int* live_count;      // live voxels found by the filter (zeroed)
     unsigned int* live_idx;        // their indices into vox (capacity N)
     int may_cull;                  // some voxel may lie beyond the tool's reach (per pivot)
+    // cone records and (voxel, row) tasks between cone_kernel and row_kernel
+    struct ConeRec* recs;
+    unsigned long long* tasks;     // (record << 16) | row offset
+    unsigned int* rec_count;       // zeroed per launch pair
+    unsigned long long* task_count;
+    unsigned int rec_cap;
+    unsigned long long task_cap;
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,
@@ -131,13 +138,13 @@ __device__ void fill_all(const StreamParams& p, uint32_t* sAM) {
 __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, unsigned int vidx,
                                           float4 q, int cell, uint32_t* wp, uint32_t bit,
                                           Counters& cnt) {
-    atomicAdd(cnt.c + CT_BAND, 1u);
+    if (cnt.c) atomicAdd(cnt.c + CT_BAND, 1u);
     const unsigned long long slot = atomicAdd(p.qcount, 1ULL);
     if ((long long)slot < p.qcap) {
         p.queue[slot] = ((unsigned long long)vidx << 32) | (unsigned int)cell;
     } else {
         // queue full: resolve inline (rare; keeps the result exact)
-        atomicAdd(cnt.c + CT_OVERFLOW, 1u);
+        if (cnt.c) atomicAdd(cnt.c + CT_OVERFLOW, 1u);
         if (exact_pair(p, q, cell)) atomicOr(wp, bit);
     }
 }

@@ -15,13 +15,18 @@
 //   instructions; the survivors ("live") are appended to a global list with one
 //   warp-aggregated atomic.
 //
-// live_kernel (a3-a6; the live voxels only, ~0.01-1 %): 32 voxels per warp,
-//   one per lane for the paper's two ICA cones (Alg. 1), checked
-//   against the map once more; the (voxel, phi-row) pairs of the warp are then
-//   dealt evenly over the lanes and rasterised into the CTA's shared AM; band
-//   cells are deferred to the global band queue; the shared AM is OR-ed into
-//   the global AM at the end (a7).  The clear-map levels use the same kernel
-//   with inner cones only (level 0: every voxel of the level is live).
+// cone_kernel (a3-a4; the live voxels only, ~0.01-1 %): one voxel per thread,
+//   the paper's two ICA cones (Alg. 1), checked against the map once
+//   more; each survivor writes a cone record and one task per phi-row of its
+//   outer cone.
+//
+// row_kernel (a5-a7): one (voxel, row) task per thread -- perfectly balanced
+//   whatever the cone sizes -- rasterised into the CTA's shared AM (seeded from
+//   the global AM); band cells go to the global band queue; the shared AM is
+//   OR-ed into the global AM at the end.
+//
+// The clear-map levels use the same two kernels with inner cones only (level
+// 0 without the filter: every voxel of the level is live).
 #pragma once
 #include "kernels.cuh"
 
@@ -93,139 +98,6 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
     return (face * T + iw) * T + iu;
 }
 
-// a3-a6 for the live voxels of one warp (one per lane, `valid` lanes only).
-// Each lane first computes its own voxel's two cones (GETTOOLICA twice, Alg. 1
-// L147-148), checks the exact outer cone against the clear-direction map and
-// finds its phi-row range; the warp then shares out the (voxel, row) pairs of
-// all 32 voxels evenly over its lanes (a warp scan of the row counts), so a
-// voxel with a 64-row cone and one with a 2-row cone cost the same latency.
-// Per row (Alg. 1 L149-155 for all cells of a row at once): the inner-cone
-// interval is OR-ed into the shared AM, outer-minus-inner cells still clear go
-// to the band queue.  COARSE (clear-map levels) rasterises inner cones only.
-template <bool COARSE>
-__device__ __noinline__ void process_live_warp(const StreamParams& p, bool valid, unsigned int vidx, float4 q,
-                                               uint32_t* sAM, const uint32_t* sRowFull, const float* sCos,
-                                               const float* sSin, Counters cnt) {
-    const ToolDev& T = p.tool;
-    const GridDev& g = p.grid;
-    const int lane = threadIdx.x & 31;
-    float cin = 2.f, cout = 2.f, clo = 2.f, cphv = 0.f, sphv = 0.f, gv = 0.f;
-    int i0 = 0, nrows = 0;
-    if (valid) {
-        const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
-        const float D = sqrtf(vx * vx + vy * vy + vz * vz);
-        const bool inside = D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h;
-        if (!inside) {  // (a voxel holding the pivot was filled by the filter)
-            Cones c;
-            if (COARSE) {
-                c.cin = c.cout = inner_cone(D, h, T);
-                c.clo = 2.f;
-            } else {
-                c = tool_cones(D, h, T);
-            }
-            // the exact outer cone against the clear-direction map: no clear
-            // cell within it means this voxel cannot change the map
-            if (c.cout <= 1.f &&
-                __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) >= c.cout * fabsf(c.cout)) {
-                const float rxy = sqrtf(vx * vx + vy * vy);
-                const float phv = atan2f(rxy, vz);
-                const float ao = acosf(fmaxf(c.cout, -1.f));
-                const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-                const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-                if (a0 <= a1 && !rows_all_full(sRowFull, a0, a1)) {
-                    const float invD = 1.f / D;
-                    cin = c.cin;
-                    cout = c.cout;
-                    clo = c.clo;
-                    cphv = vz * invD;
-                    sphv = rxy * invD;
-                    gv = atan2f(vy, vx);
-                    i0 = a0;
-                    nrows = a1 - a0 + 1;
-                }
-            }
-        }
-    }
-    if (valid) atomicAdd(cnt.c + CT_LIVE, 1u);
-    // warp scan of the row counts; (voxel, row) pairs are dealt round-robin
-    int incl = nrows;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
-    }
-    const int total = __shfl_sync(0xffffffffu, incl, 31);
-    const int W = g.W;
-    unsigned int rows = 0;
-    for (int base = 0; base < total; base += 32) {
-        const int k = base + lane;
-        // owner = number of lanes whose inclusive count is <= k
-        int owner = 0;
-#pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-            const int cand = owner + step;
-            if (__shfl_sync(0xffffffffu, incl, cand - 1) <= k) owner = cand;
-        }
-        owner = min(owner, 31);
-        const int o_incl = __shfl_sync(0xffffffffu, incl, owner);
-        const int o_n = __shfl_sync(0xffffffffu, nrows, owner);
-        const int o_i0 = __shfl_sync(0xffffffffu, i0, owner);
-        const float o_cin = __shfl_sync(0xffffffffu, cin, owner);
-        const float o_cout = __shfl_sync(0xffffffffu, cout, owner);
-        const float o_clo = __shfl_sync(0xffffffffu, clo, owner);
-        const float o_c = __shfl_sync(0xffffffffu, cphv, owner);
-        const float o_s = __shfl_sync(0xffffffffu, sphv, owner);
-        const float o_gv = __shfl_sync(0xffffffffu, gv, owner);
-        const unsigned int o_vidx = __shfl_sync(0xffffffffu, vidx, owner);
-        if (k >= total) continue;
-        const int i = o_i0 + (k - (o_incl - o_n));
-        if ((ld_vol_shared(sRowFull + (i >> 5)) >> (i & 31)) & 1u) continue;
-        const float rb = sCos[i] * o_c, rd = sSin[i] * o_s;
-        if (COARSE) {
-            const Interval In = gamma_interval(o_cin, rb, rd, o_gv, -1, g);
-            if (In.len == 0) continue;
-            ++rows;
-            for (int w = 0; w < W; ++w) {
-                const uint32_t ib = interval_bits(In, w, g.n);
-                uint32_t* wp = sAM + i * W + w;
-                if (ib & ~ld_vol_shared(wp)) atomicOr(wp, ib);
-            }
-            continue;
-        }
-        const Interval O = gamma_interval(o_cout, rb, rd, o_gv, +1, g);
-        if (O.len == 0) continue;
-        ++rows;
-        const Interval In = gamma_interval(o_cin, rb, rd, o_gv, -1, g);
-        const Interval X = gamma_interval(o_clo, rb, rd, o_gv, -1, g);
-        for (int w = 0; w < W; ++w) {
-            uint32_t ob = interval_bits(O, w, g.n);
-            if (!ob) continue;
-            const uint32_t xb = interval_bits(X, w, g.n);
-            const uint32_t ib = interval_bits(In, w, g.n) & ~xb;
-            ob &= ~xb;
-            uint32_t* wp = sAM + i * W + w;
-            uint32_t cur = ld_vol_shared(wp);
-            if (ib & ~cur) {
-                atomicOr(wp, ib);
-                cur |= ib;
-            }
-            uint32_t band = ob & ~ib & ~cur;
-            while (band) {
-                const int b = __ffs(band) - 1;
-                band &= band - 1u;
-                push_band(p, sAM, o_vidx, p.vox_main[o_vidx], i * g.n + (w << 5) + b, wp, 1u << b, cnt);
-            }
-        }
-    }
-    if (rows) atomicAdd(cnt.c + CT_ROWS, rows);
-}
-
-
-// Dynamic shared memory of live_kernel for an m x n grid.
-__host__ __device__ inline size_t live_smem_bytes(int m, int W) {
-    return (size_t)(m * W + ((m + 31) >> 5)) * sizeof(uint32_t) + (size_t)2 * m * sizeof(float);
-}
-
 // Append the live voxels among one warp-row of 32 to the global live list.
 __device__ __forceinline__ void append_live(const StreamParams& p, bool live, unsigned int idx,
                                             unsigned int& npassed) {
@@ -284,29 +156,140 @@ __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant_
     }
 }
 
-// a3-a6 over the live list, 32 voxels per warp, into a shared AM seeded from
-// the global AM; a7 (OR into the global AM) at the end.  With p.live_idx ==
-// nullptr every voxel of vox[0, N) is live (clear-map level 0).
+// Dynamic shared memory of row_kernel for an m x n grid: AM + row-full bits.
+__host__ __device__ inline size_t live_smem_bytes(int m, int W) {
+    return (size_t)(m * W + ((m + 31) >> 5)) * sizeof(uint32_t);
+}
+
+// A live voxel's cones and phi-row range, as the row kernel needs them.
+struct ConeRec {
+    float cin, cout, clo;  // guarded cone cosines (geometry.cuh Cones)
+    float cphv, sphv, gv;  // cone axis: cos/sin of phi_v, gamma_v
+    unsigned int vidx;     // voxel index (band queue entries)
+    int i0;                // first phi-row of the outer cone
+};
+
+// Rows of a voxel processed inline when the record/task buffers are full
+// (correct, only slower).
 template <bool COARSE>
-__global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ StreamParams p) {
+__device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint32_t* am, Counters cnt);
+
+// a3-a4 for the live voxels (one per thread): the paper's two cones
+// (GETTOOLICA twice, Alg. 1; COARSE: the inner one only), the exact
+// outer cone checked against the clear-direction map, the phi-row range; one
+// record per surviving voxel and one task per (voxel, row).  With
+// p.live_idx == nullptr every voxel of vox[0, N) is live (clear-map level 0).
+template <bool COARSE>
+__global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
+    const ToolDev& T = p.tool;
+    const GridDev& g = p.grid;
+    const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
+    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < nlive;
+         e += (unsigned long long)gridDim.x * blockDim.x) {
+        const unsigned int vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
+        const float4 q = p.vox[vidx];
+        const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
+        const float D = sqrtf(vx * vx + vy * vy + vz * vz);
+        if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
+            fill_all(p, p.gam);  // the pivot lies in the closed box: every orientation collides
+            continue;
+        }
+        atomicAdd(p.stats + ST_LIVE, 1ull);
+        Cones c;
+        if (COARSE) {
+            c.cin = c.cout = inner_cone(D, h, T);
+            c.clo = 2.f;
+        } else {
+            c = tool_cones(D, h, T);
+        }
+        if (c.cout > 1.f) continue;
+        // the exact outer cone against the clear-direction map: no clear cell
+        // within it means this voxel cannot change the map
+        if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) continue;
+        const float rxy = sqrtf(vx * vx + vy * vy);
+        const float phv = atan2f(rxy, vz);
+        const float ao = acosf(fmaxf(c.cout, -1.f));
+        const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+        const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+        if (a0 > a1) continue;
+        const float invD = 1.f / D;
+        ConeRec r;
+        r.cin = c.cin;
+        r.cout = c.cout;
+        r.clo = c.clo;
+        r.cphv = vz * invD;
+        r.sphv = rxy * invD;
+        r.gv = atan2f(vy, vx);
+        r.vidx = vidx;
+        r.i0 = a0;
+        const int nrows = a1 - a0 + 1;
+        const unsigned int slot = atomicAdd(p.rec_count, 1u);
+        const unsigned long long t0 = atomicAdd(p.task_count, (unsigned long long)nrows);
+        if (slot < p.rec_cap && t0 + nrows <= p.task_cap) {
+            p.recs[slot] = r;
+            for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+        } else {
+            // buffers full: rasterise this voxel's rows here, straight into the global AM
+            for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, a0 + k, p.gam, Counters{nullptr});
+            if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
+        }
+    }
+}
+
+// One phi-row of one cone (Alg. 1 L149-155 for all cells of a row at once):
+// the inner-cone interval is OR-ed into `am`; outer-minus-inner cells still
+// clear go to the band queue (COARSE: inner cone only).
+template <bool COARSE>
+__device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint32_t* am, Counters cnt) {
+    const GridDev& g = p.grid;
+    const int W = g.W;
+    const float rb = __ldg(p.tab + i) * r.cphv, rd = __ldg(p.tab + g.m + i) * r.sphv;
+    if (COARSE) {
+        const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
+        if (In.len == 0) return;
+        for (int w = 0; w < W; ++w) {
+            const uint32_t ib = interval_bits(In, w, g.n);
+            uint32_t* wp = am + i * W + w;
+            if (ib & ~*reinterpret_cast<volatile uint32_t*>(wp)) atomicOr(wp, ib);
+        }
+        return;
+    }
+    const Interval O = gamma_interval(r.cout, rb, rd, r.gv, +1, g);
+    if (O.len == 0) return;
+    const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
+    const Interval X = gamma_interval(r.clo, rb, rd, r.gv, -1, g);
+    for (int w = 0; w < W; ++w) {
+        uint32_t ob = interval_bits(O, w, g.n);
+        if (!ob) continue;
+        const uint32_t xb = interval_bits(X, w, g.n);
+        const uint32_t ib = interval_bits(In, w, g.n) & ~xb;
+        ob &= ~xb;
+        uint32_t* wp = am + i * W + w;
+        uint32_t cur = *reinterpret_cast<volatile uint32_t*>(wp);
+        if (ib & ~cur) {
+            atomicOr(wp, ib);
+            cur |= ib;
+        }
+        uint32_t band = ob & ~ib & ~cur;
+        while (band) {
+            const int b = __ffs(band) - 1;
+            band &= band - 1u;
+            push_band(p, am, r.vidx, p.vox_main[r.vidx], i * g.n + (w << 5) + b, wp, 1u << b, cnt);
+        }
+    }
+}
+
+// a5-a7: one (voxel, phi-row) task per thread into a shared AM seeded from the
+// global AM (rows already full are skipped), then OR-ed into the global AM.
+template <bool COARSE>
+__global__ void __launch_bounds__(kThreads) row_kernel(const __grid_constant__ StreamParams p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ unsigned int sCnt[CT_COUNT];
-    // shared copy of the parameters for the out-of-line process_live_warp (a
-    // reference to the kernel parameter would make every call copy it)
-    __shared__ StreamParams sP;
-    if (threadIdx.x < (int)(sizeof(StreamParams) / 4))
-        reinterpret_cast<unsigned int*>(&sP)[threadIdx.x] = reinterpret_cast<const unsigned int*>(&p)[threadIdx.x];
     const int m = p.grid.m, W = p.grid.W, MW = m * W;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
     uint32_t* sRowFull = sAM + MW;
-    float* sCos = reinterpret_cast<float*>(sRowFull + ((m + 31) >> 5));
-    float* sSin = sCos + m;
-    const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
-    if ((unsigned long long)blockIdx.x * kThreads >= nlive) return;
-    for (int i = threadIdx.x; i < m; i += blockDim.x) {
-        sCos[i] = p.tab[i];
-        sSin[i] = p.tab[m + i];
-    }
+    const unsigned long long ntask = min(*p.task_count, p.task_cap);
+    if ((unsigned long long)blockIdx.x * kThreads >= ntask) return;
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
     if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
     __syncthreads();
@@ -324,26 +307,24 @@ __global__ void __launch_bounds__(kThreads) live_kernel(const __grid_constant__ 
     }
     __syncthreads();
     const Counters cnt{sCnt};
-    // warps stride over groups of 32 entries (the loop bound is warp-uniform)
-    for (unsigned long long e0 = (blockIdx.x * (unsigned long long)kThreads) + warp * 32ull; e0 < nlive;
-         e0 += (unsigned long long)gridDim.x * kThreads) {
-        const unsigned long long e = e0 + lane;
-        const bool valid = e < nlive;
-        unsigned int vidx = 0;
-        float4 q = make_float4(0.f, 0.f, 0.f, 1.f);
-        if (valid) {
-            vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
-            q = p.vox[vidx];
-        }
-        process_live_warp<COARSE>(sP, valid, vidx, q, sAM, sRowFull, sCos, sSin, cnt);
+    unsigned int rows = 0;
+    for (unsigned long long k = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; k < ntask;
+         k += (unsigned long long)gridDim.x * kThreads) {
+        const unsigned long long t = p.tasks[k];
+        const ConeRec r = p.recs[t >> 16];
+        if (r.i0 < 0) continue;
+        const int i = r.i0 + (int)(t & 0xffffu);
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        ++rows;
+        raster_row<COARSE>(p, r, i, sAM, cnt);
     }
+    if (rows) atomicAdd(sCnt + CT_ROWS, rows);
     __syncthreads();
     for (int w = threadIdx.x; w < MW; w += blockDim.x) {
         const uint32_t sv = sAM[w];
         if (sv & ~ld_cg(p.gam + w)) atomicOr(p.gam + w, sv);
     }
     if (threadIdx.x == 0) {
-        atomicAdd(p.stats + ST_LIVE, (unsigned long long)sCnt[CT_LIVE]);
         atomicAdd(p.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
         atomicAdd(p.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
         atomicAdd(p.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);

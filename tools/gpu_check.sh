@@ -26,7 +26,7 @@ for w in $WHAT; do
         --log-file $OUT/launches_$TAG.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/launches_$TAG.log 2>&1
       echo "launches rc=$?" ;;
     full)
-      timeout 1200 ncu --set full --clock-control none --import-source on -k regex:${KREGEX:-filter_kernel} -s 5 -c 1 \
+      timeout 1200 ncu --set full --clock-control none --import-source on -k regex:${KREGEX:-filter_kernel} -s ${KSKIP:-5} -c ${KCOUNT:-1} \
         -o $OUT/prof_$TAG -f python bench.py --steps 8 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/full_$TAG.log 2>&1
       echo "full rc=$?" ;;
   esac
