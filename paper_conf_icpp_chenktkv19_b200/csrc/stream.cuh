@@ -1,7 +1,7 @@
 // stream.cuh -- the voxel-streaming AICA kernels.
 //
-// The full stream is split in two launches so the part that touches every
-// voxel stays lean:
+// The full stream is split in three launches so the part that touches every
+// voxel stays lean and the rest stays balanced:
 //
 // filter_kernel (a1, a2, cheap cones; every voxel): coalesced 16-byte float4
 //   loads (4 independent LDG.128 per thread in flight, streaming cache hint),
@@ -183,55 +183,87 @@ template <bool COARSE>
 __global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
+    const int lane = threadIdx.x & 31;
     const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
-    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < nlive;
-         e += (unsigned long long)gridDim.x * blockDim.x) {
-        const unsigned int vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
-        const float4 q = p.vox[vidx];
-        const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
-        const float D = sqrtf(vx * vx + vy * vy + vz * vz);
-        if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
-            fill_all(p, p.gam);  // the pivot lies in the closed box: every orientation collides
-            continue;
-        }
-        atomicAdd(p.stats + ST_LIVE, 1ull);
-        Cones c;
-        if (COARSE) {
-            c.cin = c.cout = inner_cone(D, h, T);
-            c.clo = 2.f;
-        } else {
-            c = tool_cones(D, h, T);
-        }
-        if (c.cout > 1.f) continue;
-        // the exact outer cone against the clear-direction map: no clear cell
-        // within it means this voxel cannot change the map
-        if (__ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) continue;
-        const float rxy = sqrtf(vx * vx + vy * vy);
-        const float phv = atan2f(rxy, vz);
-        const float ao = acosf(fmaxf(c.cout, -1.f));
-        const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-        const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-        if (a0 > a1) continue;
-        const float invD = 1.f / D;
+    const unsigned long long wstride = (unsigned long long)gridDim.x * blockDim.x;
+    // warp-uniform loop: the slot reservations below are warp-aggregated
+    for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < nlive;
+         e0 += wstride) {
+        const unsigned long long e = e0 + lane;
+        int nrows = 0;
+        bool counted = false;
         ConeRec r;
-        r.cin = c.cin;
-        r.cout = c.cout;
-        r.clo = c.clo;
-        r.cphv = vz * invD;
-        r.sphv = rxy * invD;
-        r.gv = atan2f(vy, vx);
-        r.vidx = vidx;
-        r.i0 = a0;
-        const int nrows = a1 - a0 + 1;
-        const unsigned int slot = atomicAdd(p.rec_count, 1u);
-        const unsigned long long t0 = atomicAdd(p.task_count, (unsigned long long)nrows);
-        if (slot < p.rec_cap && t0 + nrows <= p.task_cap) {
-            p.recs[slot] = r;
-            for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
-        } else {
-            // buffers full: rasterise this voxel's rows here, straight into the global AM
-            for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, a0 + k, p.gam, Counters{nullptr});
-            if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
+        if (e < nlive) {
+            const unsigned int vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
+            const float4 q = p.vox[vidx];
+            const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
+            const float D = sqrtf(vx * vx + vy * vy + vz * vz);
+            if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
+                fill_all(p, p.gam);  // the pivot lies in the closed box: every orientation collides
+            } else {
+                counted = true;
+                Cones c;
+                if (COARSE) {
+                    c.cin = c.cout = inner_cone(D, h, T);
+                    c.clo = 2.f;
+                } else {
+                    c = tool_cones(D, h, T);
+                }
+                // the exact outer cone against the clear-direction map: no clear
+                // cell within it means this voxel cannot change the map
+                if (c.cout <= 1.f &&
+                    __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) >= c.cout * fabsf(c.cout)) {
+                    const float rxy = sqrtf(vx * vx + vy * vy);
+                    const float phv = atan2f(rxy, vz);
+                    const float ao = acosf(fmaxf(c.cout, -1.f));
+                    const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+                    const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+                    if (a0 <= a1) {
+                        const float invD = 1.f / D;
+                        r.cin = c.cin;
+                        r.cout = c.cout;
+                        r.clo = c.clo;
+                        r.cphv = vz * invD;
+                        r.sphv = rxy * invD;
+                        r.gv = atan2f(vy, vx);
+                        r.vidx = vidx;
+                        r.i0 = a0;
+                        nrows = a1 - a0 + 1;
+                    }
+                }
+            }
+        }
+        const unsigned int mcount = __ballot_sync(0xffffffffu, counted);
+        if (lane == 0 && mcount) atomicAdd(p.stats + ST_LIVE, (unsigned long long)__popc(mcount));
+        const unsigned int mrec = __ballot_sync(0xffffffffu, nrows > 0);
+        if (!mrec) continue;
+        // one record slot per surviving lane, nrows task slots each
+        int incl = nrows;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += t;
+        }
+        unsigned int sbase = 0;
+        unsigned long long tbase = 0;
+        const int total = __shfl_sync(0xffffffffu, incl, 31);
+        if (lane == 0) {
+            sbase = atomicAdd(p.rec_count, (unsigned int)__popc(mrec));
+            tbase = atomicAdd(p.task_count, (unsigned long long)total);
+        }
+        sbase = __shfl_sync(0xffffffffu, sbase, 0);
+        tbase = __shfl_sync(0xffffffffu, tbase, 0);
+        if (nrows > 0) {
+            const unsigned int slot = sbase + __popc(mrec & ((1u << lane) - 1u));
+            const unsigned long long t0 = tbase + (unsigned long long)(incl - nrows);
+            if (slot < p.rec_cap && t0 + nrows <= p.task_cap) {
+                p.recs[slot] = r;
+                for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+            } else {
+                // buffers full: rasterise this voxel's rows here, straight into the global AM
+                for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
+                if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
+            }
         }
     }
 }
