@@ -333,7 +333,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     }
     if (!(ctx->diag & 1)) {
         if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, cm, true, s))) return rc;
-        band_exact_kernel<<<(unsigned)(ctx->sms * 4), kThreads, 0, s>>>(p);
+        band_exact_kernel<<<(unsigned)ctx->sms, kThreads, 0, s>>>(p);
         CK(cudaGetLastError());
     }
     if (ctx->d_prev)  // allocated once diagnostics were enabled

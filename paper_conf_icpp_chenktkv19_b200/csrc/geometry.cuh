@@ -195,6 +195,22 @@ __device__ __forceinline__ float inner_cone(float D, float h, const ToolDev& T) 
     return (cm <= 1.f) ? cm + kCosGuard : 2.f;
 }
 
+// acos on [-1, 1] with |error| <= 2e-8 (Abramowitz & Stegun 4.4.46) plus fp32
+// rounding (~1e-7): far inside the kGamGuard the interval ends carry.
+__device__ __forceinline__ float fast_acos(float x) {
+    const float a = fabsf(x);
+    float p = -0.0012624911f;
+    p = fmaf(p, a, 0.0066700901f);
+    p = fmaf(p, a, -0.0170881256f);
+    p = fmaf(p, a, 0.0308918810f);
+    p = fmaf(p, a, -0.0501743046f);
+    p = fmaf(p, a, 0.0889789874f);
+    p = fmaf(p, a, -0.2145988016f);
+    p = fmaf(p, a, 1.5707963050f);
+    const float r = sqrtf(1.f - a) * p;
+    return x < 0.f ? kPi - r : r;
+}
+
 // Cells j of one phi-row with base + den * cos(gamma_j - gv) >= cthr, as the
 // cyclic range [lo, lo + len) (mod n).  grow = +1 widens the interval by the
 // guards (outer cone), grow = -1 narrows it (inner cone / ring exclusion).
@@ -215,7 +231,7 @@ __device__ __forceinline__ Interval gamma_interval(float cthr, float base, float
     const float x = (cthr - base) / den;
     if (x <= -1.f) { I.len = g.n; return I; }
     if (x > 1.f) return I;
-    dl = acosf(x) + (grow > 0 ? kGamGuard : -kGamGuard);
+    dl = fast_acos(x) + (grow > 0 ? kGamGuard : -kGamGuard);
     if (dl < 0.f) return I;
     if (dl >= kPi) { I.len = g.n; return I; }
     const float slack = grow > 0 ? kCellSlack : -kCellSlack;

@@ -217,6 +217,7 @@ __global__ void __launch_bounds__(256) clear_map_kernel(const float4* __restrict
 __global__ void __launch_bounds__(kThreads) band_exact_kernel(const StreamParams p) {
     const unsigned long long cnt = *p.qcount;
     const long long n = (long long)(cnt < (unsigned long long)p.qcap ? cnt : (unsigned long long)p.qcap);
+    if ((long long)blockIdx.x * blockDim.x >= n) return;  // (whole CTA: nothing queued for it)
     unsigned long long tests = 0, hits = 0;
     for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < n;
          k += (long long)gridDim.x * blockDim.x) {

@@ -288,6 +288,12 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
     }
     const Interval O = gamma_interval(r.cout, rb, rd, r.gv, +1, g);
     if (O.len == 0) return;
+    {  // nothing to do when every cell of the outer interval is already blocked
+        uint32_t fresh = 0u;
+        for (int w = 0; w < W; ++w)
+            fresh |= interval_bits(O, w, g.n) & ~*reinterpret_cast<volatile uint32_t*>(am + i * W + w);
+        if (!fresh) return;
+    }
     const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
     const Interval X = gamma_interval(r.clo, rb, rd, r.gv, -1, g);
     for (int w = 0; w < W; ++w) {
