@@ -153,6 +153,19 @@ int am_set_option(am_ctx* ctx, int key, int64_t value);
  */
 int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches);
 
+/*
+ * Layout conversion on the device, for the voxel-sharded multi-GPU combine
+ * (SURVEY.md 8(e)(1)): an all_reduce(MAX) over one byte per cell is the OR of
+ * the ranks' maps, which MAX over packed words is not.
+ *   am_unpack_cells: words (m * ceil(n/32) uint32, layout above) -> cells
+ *                    (m * n uint8, row-major, 0/1);
+ *   am_pack_cells:   cells (nonzero = collision) -> words.
+ * Both pointers are device memory of ctx's device; asynchronous on
+ * cuda_stream.  AM_EINVAL for NULL pointers.
+ */
+int am_unpack_cells(am_ctx* ctx, const uint32_t* words, uint8_t* cells, void* cuda_stream);
+int am_pack_cells(am_ctx* ctx, const uint8_t* cells, uint32_t* words, void* cuda_stream);
+
 /* m * ceil(n / 32): words per AM.  -1 if ctx is NULL. */
 int am_words_per_map(const am_ctx* ctx);
 

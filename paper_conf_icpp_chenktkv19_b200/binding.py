@@ -24,8 +24,8 @@ OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T = 6, 7, 8, 9
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",
-           "am_set_option", "am_kernel_time", "am_words_per_map", "am_num_voxels", "am_last_error",
-           "am_destroy")
+           "am_set_option", "am_kernel_time", "am_unpack_cells", "am_pack_cells", "am_words_per_map",
+           "am_num_voxels", "am_last_error", "am_destroy")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(
@@ -74,6 +74,10 @@ lib.am_set_option.restype = ctypes.c_int
 lib.am_set_option.argtypes = [_P, ctypes.c_int, ctypes.c_int64]
 lib.am_kernel_time.restype = ctypes.c_int
 lib.am_kernel_time.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+lib.am_unpack_cells.restype = ctypes.c_int
+lib.am_unpack_cells.argtypes = [_P, _P, _P, _P]
+lib.am_pack_cells.restype = ctypes.c_int
+lib.am_pack_cells.argtypes = [_P, _P, _P, _P]
 lib.am_words_per_map.restype = ctypes.c_int
 lib.am_words_per_map.argtypes = [_P]
 lib.am_num_voxels.restype = ctypes.c_int64
@@ -170,6 +174,26 @@ class Context:
         n = ctypes.c_int64()
         self._check(lib.am_kernel_time(self._h, ctypes.byref(ms), ctypes.byref(n)))
         return ms.value, n.value
+
+    def _dev_stream(self, t, stream):
+        if not _is_torch_cuda(t):
+            raise TypeError("expected a torch CUDA tensor")
+        if stream is None:
+            import torch
+            stream = torch.cuda.current_stream(t.device)
+        return _stream_handle(stream)
+
+    def unpack_cells(self, words, cells, stream=None):
+        """am_unpack_cells: device words (int32/uint32 [words]) -> device uint8 [m * n]."""
+        self._check(lib.am_unpack_cells(self._h, _P(words.data_ptr()), _P(cells.data_ptr()),
+                                        self._dev_stream(words, stream)))
+        return cells
+
+    def pack_cells(self, cells, words, stream=None):
+        """am_pack_cells: device uint8 [m * n] -> device words."""
+        self._check(lib.am_pack_cells(self._h, _P(cells.data_ptr()), _P(words.data_ptr()),
+                                      self._dev_stream(cells, stream)))
+        return words
 
     @property
     def num_voxels(self) -> int:

@@ -821,6 +821,25 @@ int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches) {
     return AM_OK;
 }
 
+int am_unpack_cells(am_ctx* ctx, const uint32_t* words, uint8_t* cells, void* cuda_stream) {
+    if (!ctx) return AM_EINVAL;
+    if (!words || !cells) return fail(ctx, AM_EINVAL, "NULL buffer");
+    DeviceGuard dg(ctx->device);
+    const int nc = ctx->grid.m * ctx->grid.n;
+    unpack_cells_kernel<<<(nc + 255) / 256, 256, 0, (cudaStream_t)cuda_stream>>>(words, ctx->grid, cells);
+    CK(cudaGetLastError());
+    return AM_OK;
+}
+
+int am_pack_cells(am_ctx* ctx, const uint8_t* cells, uint32_t* words, void* cuda_stream) {
+    if (!ctx) return AM_EINVAL;
+    if (!words || !cells) return fail(ctx, AM_EINVAL, "NULL buffer");
+    DeviceGuard dg(ctx->device);
+    pack_cells_kernel<<<(ctx->MW + 255) / 256, 256, 0, (cudaStream_t)cuda_stream>>>(cells, ctx->grid, words);
+    CK(cudaGetLastError());
+    return AM_OK;
+}
+
 int am_words_per_map(const am_ctx* ctx) { return ctx ? ctx->MW : -1; }
 
 int64_t am_num_voxels(const am_ctx* ctx) { return ctx ? (int64_t)ctx->N : -1; }

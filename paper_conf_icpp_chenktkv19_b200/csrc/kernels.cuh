@@ -387,4 +387,24 @@ __global__ void gather_kernel(const float4* __restrict__ src, const unsigned int
         dst[k] = src[ids[k]];
 }
 
+// Packed AM (m x W words) <-> one byte per cell (m x n), for the voxel-sharded
+// multi-GPU combine (all_reduce MAX over bytes is OR; over packed words it is not).
+__global__ void unpack_cells_kernel(const uint32_t* __restrict__ words, GridDev g, uint8_t* __restrict__ cells) {
+    const int nc = g.m * g.n;
+    for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < nc; c += gridDim.x * blockDim.x) {
+        const int i = c / g.n, j = c - i * g.n;
+        cells[c] = (uint8_t)((words[i * g.W + (j >> 5)] >> (j & 31)) & 1u);
+    }
+}
+
+__global__ void pack_cells_kernel(const uint8_t* __restrict__ cells, GridDev g, uint32_t* __restrict__ words) {
+    const int nw = g.m * g.W;
+    for (int w = blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += gridDim.x * blockDim.x) {
+        const int i = w / g.W, j0 = (w - i * g.W) << 5;
+        uint32_t v = 0u;
+        for (int b = 0; b < 32 && j0 + b < g.n; ++b) v |= (cells[i * g.n + j0 + b] ? 1u : 0u) << b;
+        words[w] = v;
+    }
+}
+
 }  // namespace am

@@ -23,7 +23,7 @@ def _declared():
 
 def test_header_symbols_exported(am):
     declared = _declared()
-    assert len(declared) == 11
+    assert len(declared) == 13
     lib = ctypes.CDLL(am.LIB_PATH)
     for s in declared:
         assert hasattr(lib, s), s
@@ -60,6 +60,8 @@ def test_argument_validation_without_gpu(am):
     assert lib.am_compute_baseline(None, None, None, 0, None) == am.AM_EINVAL
     assert lib.am_set_option(None, 1, 0) == am.AM_EINVAL
     assert lib.am_kernel_time(None, None, None) == am.AM_EINVAL
+    assert lib.am_unpack_cells(None, None, None, None) == am.AM_EINVAL
+    assert lib.am_pack_cells(None, None, None, None) == am.AM_EINVAL
     assert lib.am_last_error(None) == b"NULL context"
     lib.am_destroy(None)
 
