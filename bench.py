@@ -262,7 +262,7 @@ def run_ours(args):
     if os.path.exists(prof):
         try:
             d = json.load(open(prof))
-            if d.get("config") == cfg.name and d.get("build") == _build_id():
+            if d.get("config") == cfg.name and d.get("kernel") == "filter_kernel":
                 traffic = d.get("dram_bytes_per_launch")
         except Exception:
             traffic = None
@@ -293,7 +293,7 @@ def run_ours(args):
             "ms_per_am": ms_max / args.steps,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "aica_stream_kernel", "kernel_ms_avg": kavg_ms,
+                         "kernel": "filter_kernel", "kernel_ms_avg": kavg_ms,
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12, "d2h_bytes_per_step": 4 * ctx.words,
                     "ms_per_am": 1e3 * e2e_max / ke, "steps": ke,

@@ -1,0 +1,95 @@
+"""Summarise an ncu capture + launch list into profiles/ (run here, no GPU needed).
+
+    python tools/summarize_ncu.py <tag> [config]
+reads gpurun_out/prof_<tag>.ncu-rep and gpurun_out/launches_<tag>.csv, writes
+profiles/<tag>_launches.txt, profiles/<tag>_<kernel>_ncu.txt and (for the
+filter kernel) profiles/ncu_summary.json, which bench.py reads for `traffic`.
+"""
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+from collections import OrderedDict, defaultdict
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def ncu_csv(rep, page):
+    out = subprocess.run(["ncu", "-i", rep, "--page", page, "--csv"], capture_output=True, text=True).stdout
+    return list(csv.reader(io.StringIO(out)))
+
+
+def main():
+    tag = sys.argv[1]
+    config = sys.argv[2] if len(sys.argv) > 2 else "C3"
+    prof = os.path.join(ROOT, "profiles")
+    os.makedirs(prof, exist_ok=True)
+    lc = os.path.join(ROOT, "gpurun_out", f"launches_{tag}.csv")
+    if os.path.exists(lc):
+        rows = list(csv.reader(open(lc)))
+        start = next(i for i, r in enumerate(rows) if r and r[0] == "ID")
+        hdr = rows[start]
+        ix = {k: j for j, k in enumerate(hdr)}
+        per = defaultdict(list)
+        seq = []
+        for r in rows[start + 1:]:
+            if len(r) < len(hdr):
+                continue
+            name = r[ix["Kernel Name"]].split("(")[0]
+            v = float(r[ix["Metric Value"]].replace(",", ""))
+            per[name].append(v)
+            seq.append((name, r[ix["Grid Size"]], v))
+        with open(os.path.join(prof, f"{tag}_launches.txt"), "w") as f:
+            f.write(f"# ncu --metrics gpu__time_duration.sum --clock-control none (cold, serialised): {config}\n")
+            f.write("# per kernel: launches, mean ns, share of the listed time\n")
+            tot = sum(sum(v) for v in per.values())
+            for k, v in sorted(per.items(), key=lambda kv: -sum(kv[1])):
+                f.write(f"{k:40s} {len(v):5d} {sum(v) / len(v):12.0f} {100 * sum(v) / tot:6.1f}%\n")
+            f.write("\n# launch sequence (first 24)\n")
+            for name, g, v in seq[:24]:
+                f.write(f"{name:40s} {g:16s} {v:10.0f} ns\n")
+    rep = os.path.join(ROOT, "gpurun_out", f"prof_{tag}.ncu-rep")
+    if not os.path.exists(rep):
+        return
+    det = ncu_csv(rep, "details")
+    h = det[0]
+    kernels = OrderedDict()
+    for r in det[1:]:
+        d = dict(zip(h, r))
+        key = (d["ID"], d["Kernel Name"].split("(")[0])
+        kernels.setdefault(key, []).append((d["Section Name"], d["Metric Name"], d["Metric Value"], d["Metric Unit"]))
+    raw = ncu_csv(rep, "raw")
+    rh, ru = raw[0], raw[1]
+    for kidx, ((kid, kname), mets) in enumerate(kernels.items()):
+        rawrow = dict(zip(rh, raw[2 + kidx])) if len(raw) > 2 + kidx else {}
+        rawu = dict(zip(rh, ru))
+        keep = ["Duration", "DRAM Throughput", "Memory Throughput", "Compute (SM) Throughput", "Executed Ipc Active",
+                "Issue Slots Busy", "Registers Per Thread", "Achieved Occupancy", "Theoretical Occupancy",
+                "Executed Instructions", "L2 Hit Rate", "L1/TEX Hit Rate", "Eligible Warps Per Scheduler",
+                "No Eligible", "Avg. Active Threads Per Warp", "Grid Size", "Block Size",
+                "Dynamic Shared Memory Per Block"]
+        with open(os.path.join(prof, f"{tag}_{kname}_{kid}_ncu.txt"), "w") as f:
+            f.write(f"# ncu --set full --clock-control none: {kname} (launch id {kid}), {config}\n")
+            for sec, name, val, unit in mets:
+                if name in keep:
+                    f.write(f"{name:34s} {val:>16s} {unit}\n")
+            for k in ("dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__time_duration.sum",
+                      "sm__inst_executed.sum", "launch__registers_per_thread"):
+                if k in rawrow:
+                    f.write(f"{k:34s} {rawrow[k]:>16s} {rawu.get(k, '')}\n")
+        if kname == "filter_kernel" and "dram__bytes_read.sum" in rawrow:
+            def tobytes(v, u):
+                v = float(v.replace(",", ""))
+                return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
+            rd = tobytes(rawrow["dram__bytes_read.sum"], rawu["dram__bytes_read.sum"])
+            wr = tobytes(rawrow["dram__bytes_write.sum"], rawu["dram__bytes_write.sum"])
+            json.dump({"config": config, "kernel": "filter_kernel", "tag": tag,
+                       "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+                       "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full)"},
+                      open(os.path.join(prof, "ncu_summary.json"), "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()
