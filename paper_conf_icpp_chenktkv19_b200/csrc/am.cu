@@ -59,6 +59,9 @@ struct am_ctx {
     int diag = 0;
     int cmapT = 128;
     int phases = 2;
+    float4* d_bricks = nullptr;            // bounding spheres of 256-voxel bricks of d_vox
+    unsigned int nbricks = 0;
+    int bricks_on = 1;
     float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -268,7 +271,17 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
         }
         CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
     }
-    filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
+    if (!coarse && ctx->bricks_on && ctx->d_bricks) {
+        p.bricks = ctx->d_bricks;
+        p.nbricks = ctx->nbricks;
+        long long gb = ((long long)ctx->nbricks + kThreads - 1) / kThreads;
+        const long long gmax = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * 8;
+        if (gb > gmax) gb = gmax;
+        if (gb < 1) gb = 1;
+        brick_stream_kernel<<<(unsigned)gb, kThreads, 0, s>>>(p);
+    } else {
+        filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
+    }
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
     return launch_cones_rows(ctx, p, coarse, coarse ? 1 : 2, s);
@@ -594,6 +607,14 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     } else {
         UK(cudaMemcpy(ctx->d_vox, raw, (size_t)N * sizeof(float4), cudaMemcpyDeviceToDevice));
     }
+    // bricks of kThreads consecutive (Morton-ordered) voxels and their bounding spheres
+    cudaFree(ctx->d_bricks);
+    ctx->d_bricks = nullptr;
+    ctx->nbricks = (unsigned int)((N + kThreads - 1) / kThreads);
+    UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
+    brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
+                                                                                        ctx->nbricks);
+    UK(cudaGetLastError());
     // coarse levels for the clear-direction map: level 0 = the n0 largest
     // voxels, level 1 = the next ones up to n1 plus every 512th voxel
     cudaFree(ctx->d_coarse);
@@ -674,7 +695,6 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         static_assert(sizeof(am_stats) == ST_PASSED * sizeof(int64_t), "am_stats mirrors StatIdx");
         for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
         // every voxel goes through the filter once; the rest of it was dropped
-        o[ST_STREAMED] = (int64_t)ctx->N;
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
     } else if (!dst_is_device) {
         CK(cudaStreamSynchronize(s));
@@ -781,6 +801,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         }
         ctx->diag = (int)value;
         return AM_OK;
+    case AM_OPT_BRICKS:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "bricks must be 0 or 1");
+        ctx->bricks_on = (int)value;
+        return AM_OK;
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
         {
@@ -863,6 +887,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_live);
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);
+    cudaFree(ctx->d_bricks);
     cudaFree(ctx->d_texels);
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);

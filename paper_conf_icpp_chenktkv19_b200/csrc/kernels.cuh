@@ -66,6 +66,9 @@ struct StreamParams {
     unsigned long long* task_count;
     unsigned int rec_cap;
     unsigned long long task_cap;
+    // bricks of kThreads consecutive voxels of vox: bounding spheres (x, y, z, r)
+    const float4* __restrict__ bricks;
+    unsigned int nbricks;
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,

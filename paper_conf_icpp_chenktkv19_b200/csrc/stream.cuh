@@ -153,6 +153,128 @@ __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant_
     if (threadIdx.x == 0) {
         atomicAdd(p.stats + ST_CULLED, (unsigned long long)sCulled);
         atomicAdd(p.stats + ST_PASSED, (unsigned long long)sPassed);
+        if (blockIdx.x == 0) atomicAdd(p.stats + ST_STREAMED, (unsigned long long)p.N);  // every voxel is read
+    }
+}
+
+// The cheap outer cone of a sphere (centre p + v, radius r) against the
+// clear-direction map: true when the sphere -- hence every voxel inside it --
+// can no longer change the AM (all its possibly blocked directions are
+// blocked already) or lies beyond the tool's reach.
+__device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, float vy, float vz, float r) {
+    const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
+    if (D2 <= r * r * 1.0001f) return false;  // the pivot is (almost) inside: keep
+    const float invD = rsqrtf(D2);
+    const float D = D2 * invD;
+    if (p.may_cull && D - r > p.cull_dist) return true;
+    const float Reff = reach_radius(p.tool, (D + r) * (1.f + kRadRel));
+    const float s = fmaf((Reff + r) * invD, 1.f + 1.6e-5f, 1e-6f);
+    const float c = fmaf(r * invD, 1.f + 1.6e-5f, 1e-6f);
+    const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
+    return __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < thr;
+}
+
+// Full stream with brick culling (the paper's octree
+// pruning of Alg. 2 L218-219 turned into a bulk test): the voxels are grouped
+// into bricks of kThreads Morton-consecutive voxels, each with a bounding
+// sphere (upload).  A CTA tests 256 bricks at once (one per thread); the
+// bricks whose sphere still reaches a clear cell are streamed voxel by voxel
+// through fast_filter (one voxel per thread, kVPT bricks in flight); the
+// others are never read.  Exact-safe: a voxel's cone lies inside its brick's.
+__global__ void __launch_bounds__(kThreads) brick_stream_kernel(const __grid_constant__ StreamParams p) {
+    __shared__ unsigned int sList[kThreads];
+    __shared__ int sN;
+    __shared__ unsigned int sCulled, sPassed;
+    __shared__ unsigned long long sStreamed;
+    if (threadIdx.x == 0) {
+        sCulled = sPassed = 0u;
+        sStreamed = 0ull;
+    }
+    const int lane = threadIdx.x & 31;
+    unsigned int nculled = 0, npassed = 0;
+    unsigned long long streamed = 0;
+    const unsigned int nb = p.nbricks;
+    for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
+        __syncthreads();  // previous round done with sList / sN
+        if (threadIdx.x == 0) sN = 0;
+        __syncthreads();
+        const unsigned int b = b0 + threadIdx.x;
+        bool keep = false;
+        if (b < nb) {
+            const float4 s = __ldg(p.bricks + b);
+            keep = !sphere_dropped(p, s.x - p.px, s.y - p.py, s.z - p.pz, s.w);
+        }
+        const unsigned int mk = __ballot_sync(0xffffffffu, keep);
+        if (mk) {
+            int base = 0;
+            const int leader = __ffs(mk) - 1;
+            if (lane == leader) base = atomicAdd(&sN, __popc(mk));
+            base = __shfl_sync(0xffffffffu, base, leader);
+            if (keep) sList[base + __popc(mk & ((1u << lane) - 1u))] = b;
+        }
+        __syncthreads();
+        const int nk = sN;
+        for (int k0 = 0; k0 < nk; k0 += kVPT) {
+            float4 q[kVPT];
+            unsigned int idx[kVPT];
+            bool ok[kVPT];
+#pragma unroll
+            for (int k = 0; k < kVPT; ++k) {
+                ok[k] = k0 + k < nk;
+                idx[k] = ok[k] ? sList[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
+                ok[k] = ok[k] && idx[k] < (unsigned long long)p.N;
+                q[k] = ok[k] ? __ldcs(p.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
+            }
+#pragma unroll
+            for (int k = 0; k < kVPT; ++k) {
+                const int f = ok[k] ? fast_filter(p, q[k], p.gam) : F_DROP;
+                nculled += f >> 1;
+                append_live(p, f == F_LIVE, idx[k], npassed);
+                streamed += ok[k];
+            }
+        }
+    }
+    if (lane == 0) atomicAdd(&sPassed, npassed);
+    if (nculled) atomicAdd(&sCulled, nculled);
+    if (streamed) atomicAdd(&sStreamed, streamed);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        atomicAdd(p.stats + ST_CULLED, (unsigned long long)sCulled);
+        atomicAdd(p.stats + ST_PASSED, (unsigned long long)sPassed);
+        atomicAdd(p.stats + ST_STREAMED, sStreamed);
+    }
+}
+
+// Bounding spheres of the bricks of kThreads consecutive voxels (one warp per
+// brick): centre of the box enclosing the voxel cubes, radius its half
+// diagonal, grown for rounding.
+__global__ void brick_bounds_kernel(const float4* __restrict__ vox, long long N, float4* __restrict__ bricks,
+                                    unsigned int nb) {
+    const int lane = threadIdx.x & 31;
+    const unsigned int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (w >= nb) return;
+    float lo[3] = {3e38f, 3e38f, 3e38f}, hi[3] = {-3e38f, -3e38f, -3e38f};
+    for (int k = lane; k < kThreads; k += 32) {
+        const long long i = (long long)w * kThreads + k;
+        if (i >= N) break;
+        const float4 q = vox[i];
+        lo[0] = fminf(lo[0], q.x - q.w); hi[0] = fmaxf(hi[0], q.x + q.w);
+        lo[1] = fminf(lo[1], q.y - q.w); hi[1] = fmaxf(hi[1], q.y + q.w);
+        lo[2] = fminf(lo[2], q.z - q.w); hi[2] = fmaxf(hi[2], q.z + q.w);
+    }
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            lo[a] = fminf(lo[a], __shfl_xor_sync(0xffffffffu, lo[a], o));
+            hi[a] = fmaxf(hi[a], __shfl_xor_sync(0xffffffffu, hi[a], o));
+        }
+    }
+    if (lane == 0) {
+        const float cx = 0.5f * (lo[0] + hi[0]), cy = 0.5f * (lo[1] + hi[1]), cz = 0.5f * (lo[2] + hi[2]);
+        const float ex = hi[0] - lo[0], ey = hi[1] - lo[1], ez = hi[2] - lo[2];
+        const float r = 0.5f * sqrtf(ex * ex + ey * ey + ez * ez);
+        bricks[w] = make_float4(cx, cy, cz, r * (1.f + 1e-5f) + 1e-6f * (fabsf(cx) + fabsf(cy) + fabsf(cz)));
     }
 }
 

@@ -235,7 +235,12 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     ref = ctx.compute_batch(P)
     ctx.set_option(am.binding.OPT_PHASES, 0)
     assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_BRICKS, 0)
+    assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_PHASES, 1)
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_BRICKS, 1)
+    ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
     assert np.array_equal(ctx.compute_batch(P), ref)
