@@ -60,6 +60,7 @@ struct am_ctx {
     int cmapT = 128;
     int phases = 2;
     float4* d_bricks = nullptr;            // bounding spheres of 256-voxel bricks of d_vox
+    unsigned int* d_brick_list = nullptr;  // bricks kept per map (capacity nbricks)
     unsigned int nbricks = 0;
     int bricks_on = 1;
     float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
@@ -79,7 +80,8 @@ namespace {
 constexpr int kCtrTiles = 1 + ST_COUNT;      // live count: full stream (+0), level 1 (+4)
 constexpr int kCtrClear = kCtrTiles + 1;     // clear-cell counts of the (up to 3) maps of a call
 constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, task count at +2s+1
-constexpr int kCtrWords = kCtrRT + 6;
+constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
+constexpr int kCtrWords = kCtrBricks + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
 constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
 constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
@@ -274,11 +276,15 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     if (!coarse && ctx->bricks_on && ctx->d_bricks) {
         p.bricks = ctx->d_bricks;
         p.nbricks = ctx->nbricks;
+        p.brick_list = ctx->d_brick_list;
+        p.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
         long long gb = ((long long)ctx->nbricks + kThreads - 1) / kThreads;
         const long long gmax = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * 8;
         if (gb > gmax) gb = gmax;
         if (gb < 1) gb = 1;
-        brick_stream_kernel<<<(unsigned)gb, kThreads, 0, s>>>(p);
+        brick_test_kernel<<<(unsigned)gb, kThreads, 0, s>>>(p);
+        CK(cudaGetLastError());
+        brick_voxels_kernel<<<(unsigned)gmax, kThreads, 0, s>>>(p);
     } else {
         filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
     }
@@ -609,9 +615,12 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     }
     // bricks of kThreads consecutive (Morton-ordered) voxels and their bounding spheres
     cudaFree(ctx->d_bricks);
+    cudaFree(ctx->d_brick_list);
     ctx->d_bricks = nullptr;
+    ctx->d_brick_list = nullptr;
     ctx->nbricks = (unsigned int)((N + kThreads - 1) / kThreads);
     UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
+    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->nbricks * sizeof(unsigned int)));
     brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
                                                                                         ctx->nbricks);
     UK(cudaGetLastError());
@@ -888,6 +897,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);
     cudaFree(ctx->d_bricks);
+    cudaFree(ctx->d_brick_list);
     cudaFree(ctx->d_texels);
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);

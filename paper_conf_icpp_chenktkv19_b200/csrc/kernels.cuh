@@ -69,6 +69,8 @@ struct StreamParams {
     // bricks of kThreads consecutive voxels of vox: bounding spheres (x, y, z, r)
     const float4* __restrict__ bricks;
     unsigned int nbricks;
+    unsigned int* brick_list;      // bricks kept by brick_test_kernel (capacity nbricks)
+    unsigned int* brick_count;     // zeroed per map
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,

@@ -177,27 +177,15 @@ __device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, 
 // Full stream with brick culling (the paper's octree
 // pruning of Alg. 2 L218-219 turned into a bulk test): the voxels are grouped
 // into bricks of kThreads Morton-consecutive voxels, each with a bounding
-// sphere (upload).  A CTA tests 256 bricks at once (one per thread); the
-// bricks whose sphere still reaches a clear cell are streamed voxel by voxel
-// through fast_filter (one voxel per thread, kVPT bricks in flight); the
-// others are never read.  Exact-safe: a voxel's cone lies inside its brick's.
-__global__ void __launch_bounds__(kThreads) brick_stream_kernel(const __grid_constant__ StreamParams p) {
-    __shared__ unsigned int sList[kThreads];
-    __shared__ int sN;
-    __shared__ unsigned int sCulled, sPassed;
-    __shared__ unsigned long long sStreamed;
-    if (threadIdx.x == 0) {
-        sCulled = sPassed = 0u;
-        sStreamed = 0ull;
-    }
+// sphere (upload).  brick_test_kernel tests every brick (one per thread) and
+// lists the bricks whose sphere still reaches a clear cell; brick_voxels_kernel
+// streams only those, kVPT bricks per CTA step (one voxel per thread per
+// brick), through fast_filter.  Exact-safe: a voxel's cone lies inside its
+// brick's.
+__global__ void __launch_bounds__(kThreads) brick_test_kernel(const __grid_constant__ StreamParams p) {
     const int lane = threadIdx.x & 31;
-    unsigned int nculled = 0, npassed = 0;
-    unsigned long long streamed = 0;
     const unsigned int nb = p.nbricks;
     for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
-        __syncthreads();  // previous round done with sList / sN
-        if (threadIdx.x == 0) sN = 0;
-        __syncthreads();
         const unsigned int b = b0 + threadIdx.x;
         bool keep = false;
         if (b < nb) {
@@ -206,32 +194,44 @@ __global__ void __launch_bounds__(kThreads) brick_stream_kernel(const __grid_con
         }
         const unsigned int mk = __ballot_sync(0xffffffffu, keep);
         if (mk) {
-            int base = 0;
+            unsigned int base = 0;
             const int leader = __ffs(mk) - 1;
-            if (lane == leader) base = atomicAdd(&sN, __popc(mk));
+            if (lane == leader) base = atomicAdd(p.brick_count, (unsigned int)__popc(mk));
             base = __shfl_sync(0xffffffffu, base, leader);
-            if (keep) sList[base + __popc(mk & ((1u << lane) - 1u))] = b;
+            if (keep) p.brick_list[base + __popc(mk & ((1u << lane) - 1u))] = b;
         }
-        __syncthreads();
-        const int nk = sN;
-        for (int k0 = 0; k0 < nk; k0 += kVPT) {
-            float4 q[kVPT];
-            unsigned int idx[kVPT];
-            bool ok[kVPT];
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) brick_voxels_kernel(const __grid_constant__ StreamParams p) {
+    __shared__ unsigned int sCulled, sPassed;
+    __shared__ unsigned long long sStreamed;
+    if (threadIdx.x == 0) {
+        sCulled = sPassed = 0u;
+        sStreamed = 0ull;
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    unsigned int nculled = 0, npassed = 0;
+    unsigned long long streamed = 0;
+    const unsigned int nk = *p.brick_count;
+    for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
+        float4 q[kVPT];
+        unsigned int idx[kVPT];
+        bool ok[kVPT];
 #pragma unroll
-            for (int k = 0; k < kVPT; ++k) {
-                ok[k] = k0 + k < nk;
-                idx[k] = ok[k] ? sList[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
-                ok[k] = ok[k] && idx[k] < (unsigned long long)p.N;
-                q[k] = ok[k] ? __ldcs(p.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
-            }
+        for (int k = 0; k < kVPT; ++k) {
+            ok[k] = k0 + k < nk;
+            idx[k] = ok[k] ? p.brick_list[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
+            ok[k] = ok[k] && idx[k] < (unsigned long long)p.N;
+            q[k] = ok[k] ? __ldcs(p.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
+        }
 #pragma unroll
-            for (int k = 0; k < kVPT; ++k) {
-                const int f = ok[k] ? fast_filter(p, q[k], p.gam) : F_DROP;
-                nculled += f >> 1;
-                append_live(p, f == F_LIVE, idx[k], npassed);
-                streamed += ok[k];
-            }
+        for (int k = 0; k < kVPT; ++k) {
+            const int f = ok[k] ? fast_filter(p, q[k], p.gam) : F_DROP;
+            nculled += f >> 1;
+            append_live(p, f == F_LIVE, idx[k], npassed);
+            streamed += ok[k];
         }
     }
     if (lane == 0) atomicAdd(&sPassed, npassed);
