@@ -18,6 +18,7 @@
 #include "../../include/am.h"
 #include "kernels.cuh"
 #include "stream.cuh"
+#include "fused.cuh"
 
 using namespace am;
 
@@ -63,6 +64,9 @@ struct am_ctx {
     unsigned int* d_brick_list = nullptr;  // bricks kept per map (capacity nbricks)
     unsigned int nbricks = 0;
     int bricks_on = 1;
+    int fused = 1;                         // one cooperative launch per map (fused.cuh)
+    int fused_grid = 0;
+    size_t smem_fused = 0;
     float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -220,6 +224,19 @@ int configure_launch(am_ctx* ctx) {
                     ctx->grid.n, ctx->smem);
     }
     ctx->occ = occ;
+    // the fused pipeline: all CTAs co-resident (cooperative launch)
+    ctx->smem_fused = fused_smem_bytes(m, ctx->grid.W);
+    ctx->fused_grid = 0;
+    if (ctx->smem_fused <= 232448 &&
+        cudaFuncSetAttribute(am_pipeline_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused) ==
+            cudaSuccess) {
+        int occf = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occf, am_pipeline_kernel, kThreads, ctx->smem_fused) ==
+                cudaSuccess &&
+            occf > 0)
+            ctx->fused_grid = occf * ctx->sms;
+    }
+    cudaGetLastError();
     return AM_OK;
 }
 
@@ -331,6 +348,62 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
     const float* cm = ctx->d_cmap_ones;
+    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+    if (ctx->fused && ctx->fused_grid > 0 && !ctx->diag && ctx->phases == 2 && ctx->n_l0 > 0 && ctx->bricks_on &&
+        ctx->d_bricks && ntex <= 4 * ctx->fused_grid * kThreads) {
+        // the whole map in one cooperative launch (fused.cuh)
+        FusedParams F;
+        F.main = p;
+        F.main.vox = ctx->d_vox;
+        F.main.N = ctx->N;
+        F.main.cmap = ctx->d_cmap;
+        F.main.bricks = ctx->d_bricks;
+        F.main.nbricks = ctx->nbricks;
+        F.main.brick_list = ctx->d_brick_list;
+        F.main.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
+        F.main.recs = ctx->d_recs;
+        F.main.tasks = ctx->d_tasks;
+        F.main.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 4);
+        F.main.task_count = ctx->d_ctr + kCtrRT + 5;
+        F.main.rec_cap = kRecCap;
+        F.main.task_cap = kTaskCap;
+        F.lvl = F.main;
+        F.lvl.vox = ctx->d_coarse;
+        F.lvl.N = ctx->n_l0;
+        F.lvl.cmap = ctx->d_cmap_ones;
+        F.lvl.stats = ctx->d_ctr + kCtrWords;
+        F.lvl.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT);
+        F.lvl.task_count = ctx->d_ctr + kCtrRT + 1;
+        F.lvl.rec_cap = kRecCap / 2;
+        F.lvl.task_cap = kTaskCap / 2;
+        F.l1 = ctx->d_coarse + ctx->n_l0;
+        F.n0 = (unsigned int)ctx->n_l0;
+        F.n1 = (unsigned int)(ctx->n_l1 - ctx->n_l0);
+        F.rec1 = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2);
+        F.task1 = ctx->d_ctr + kCtrRT + 3;
+        F.live1 = nullptr;
+        F.texels = ctx->d_texels;
+        F.ntex = ntex;
+        F.use_l1 = 1;
+        const bool timed = ctx->timing != 0;
+        if (timed) {
+            if (ctx->ev_used == ctx->ev_start.size()) {
+                cudaEvent_t a, b;
+                CK(cudaEventCreate(&a));
+                CK(cudaEventCreate(&b));
+                ctx->ev_start.push_back(a);
+                ctx->ev_stop.push_back(b);
+            }
+            CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
+        }
+        void* args[] = {&F};
+        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel, dim3(ctx->fused_grid), dim3(kThreads), args,
+                                       ctx->smem_fused, s));
+        if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+        if (ctx->d_prev)
+            CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+        return AM_OK;
+    }
     if (ctx->diag & 2) {
         // diagnostic: clear map from the previous map computed on this context
         // (exact only when the previous call used the same pivot)
@@ -813,6 +886,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_BRICKS:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "bricks must be 0 or 1");
         ctx->bricks_on = (int)value;
+        return AM_OK;
+    case AM_OPT_FUSED:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "fused must be 0 or 1");
+        ctx->fused = (int)value;
         return AM_OK;
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");

@@ -1,0 +1,374 @@
+// fused.cuh -- the whole AICA map as ONE persistent cooperative kernel.
+//
+// The multi-kernel pipeline (stream.cuh) is a chain of ~15 dependent launches
+// whose work is small and latency-bound once the clear-direction map and the
+// brick culling have removed >98 % of the voxels; every launch boundary costs
+// a drain, a launch and a ramp.  am_pipeline_kernel runs the same phases in
+// one launch of SMs x occupancy CTAs (all co-resident: cooperative launch),
+// separated by grid-wide barriers:
+//
+//   1. level-0 cones   (largest voxels, inner cones)      -> records/tasks
+//   2. level-0 rows    (one task per thread, shared AM)    -> global AM
+//   3. clear-direction map from the global AM (every CTA compacts the clear
+//      cells into shared memory; one texel per thread)
+//   4. level-1 voxels  (filter + inner cones, optional)    -> records/tasks
+//   5. level-1 rows                                         -> global AM
+//   6. clear-direction map again
+//   7. brick test      (one brick per thread)               -> kept-brick list
+//   8. brick voxels    (filter; the few live voxels compute both cones at once)
+//   9. rows            (outer/inner/ring intervals, band pairs queued)
+//  10. band            (exact CHECKBOX where the bit is still clear)
+//
+// Every phase uses the same device functions as the multi-kernel path, so the
+// two produce the same map bit for bit (tests).
+#pragma once
+#include <cooperative_groups.h>
+
+#include "stream.cuh"
+
+namespace am {
+
+struct FusedParams {
+    StreamParams main;        // full stream: vox, bricks, cmap (written in phase 3/6), stage-2 counters
+    StreamParams lvl;         // clear-map levels: scratch stats, stage-0 counters, vox = level-0 array
+    const float4* l1;         // level-1 voxels (vox_coarse + n_l0) and their count
+    unsigned int n0, n1;
+    unsigned int* rec1;       // stage-1 counters
+    unsigned long long* task1;
+    unsigned int* live1;      // level-1 live count (unused: level 1 computes cones inline)
+    const float4* texels;     // clear-map texels
+    int ntex;
+    int use_l1;
+};
+
+// Dynamic shared memory: AM, row-full bits, a chunk of clear directions.
+constexpr int kFusedDirs = 1024;
+__host__ __device__ inline size_t fused_smem_bytes(int m, int W) {
+    return (size_t)(m * W + ((m + 31) >> 5) + 1) * sizeof(uint32_t) + 15 + (size_t)kFusedDirs * sizeof(float4);
+}
+
+__device__ __forceinline__ float4* fused_dirs(uint32_t* sAM, int MW, int m) {
+    uintptr_t a = reinterpret_cast<uintptr_t>(sAM + MW + ((m + 31) >> 5) + 1);
+    return reinterpret_cast<float4*>((a + 15) & ~uintptr_t(15));
+}
+
+// Seed the shared AM from the global AM and compute the row-full bits.
+__device__ void fused_seed(const StreamParams& p, uint32_t* sAM, uint32_t* sRowFull) {
+    const int m = p.grid.m, W = p.grid.W, MW = m * W;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int base = 0; base < m; base += blockDim.x) {
+        const int i = base + threadIdx.x;
+        bool full = false;
+        if (i < m) {
+            full = true;
+            for (int w = 0; w < W; ++w)
+                if (sAM[i * W + w] != row_word_mask(w, p.grid.n)) full = false;
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, full);
+        if (lane == 0 && base + warp * 32 < m) sRowFull[(base + warp * 32) >> 5] = bal;
+    }
+    __syncthreads();
+}
+
+// OR the shared AM into the global AM (words with new bits only).
+__device__ void fused_flush(const StreamParams& p, const uint32_t* sAM) {
+    __syncthreads();
+    const int MW = p.grid.m * p.grid.W;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        const uint32_t sv = sAM[w];
+        if (sv & ~ld_cg(p.gam + w)) atomicOr(p.gam + w, sv);
+    }
+}
+
+// Rasterise the tasks of one stage (grid-stride), into the shared AM.
+template <bool COARSE>
+__device__ void fused_rows(const StreamParams& p, const unsigned long long* task_count, uint32_t* sAM,
+                           const uint32_t* sRowFull, Counters cnt) {
+    const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(task_count), p.task_cap);
+    unsigned int rows = 0;
+    for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
+         k += (unsigned long long)gridDim.x * blockDim.x) {
+        const unsigned long long t = p.tasks[k];
+        const ConeRec r = p.recs[t >> 16];
+        if (r.i0 < 0) continue;
+        const int i = r.i0 + (int)(t & 0xffffu);
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        ++rows;
+        raster_row<COARSE>(p, r, i, sAM, cnt);
+    }
+    if (rows && cnt.c) atomicAdd(cnt.c + CT_ROWS, rows);
+}
+
+// Phases 3/6: the clear-direction map from the global AM.
+__device__ void fused_clear_map(const StreamParams& p, const float4* texels, int ntex, float* V, uint32_t* sAM,
+                                float4* sDirs, int* sN) {
+    const GridDev& g = p.grid;
+    const int MW = g.m * g.W;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
+    constexpr int kMaxT = 4;  // texels per thread (ntex <= 4 * grid * block, checked by the host)
+    float best[kMaxT];
+    float4 c[kMaxT];
+#pragma unroll
+    for (int j = 0; j < kMaxT; ++j) {
+        best[j] = -2.f;
+        const int t = (j * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
+        c[j] = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
+    }
+    int w0 = 0;
+    while (true) {
+        __syncthreads();
+        if (threadIdx.x == 0) *sN = 0;
+        __syncthreads();
+        // compact the clear cells of the next words (at most kFusedDirs per round)
+        const int wend = min(MW, w0 + kFusedDirs / 32);
+        for (int w = w0 + threadIdx.x; w < wend; w += blockDim.x) {
+            const int i = w / g.W, wj = w - i * g.W;
+            uint32_t clear = ~sAM[w] & row_word_mask(wj, g.n);
+            if (!clear) continue;
+            int pos = atomicAdd(sN, __popc(clear));
+            const float cph = __ldg(p.tab + i), sph = __ldg(p.tab + g.m + i);
+            while (clear) {
+                const int j = (wj << 5) + __ffs(clear) - 1;
+                clear &= clear - 1u;
+                sDirs[pos++] = make_float4(sph * __ldg(p.tab + 2 * g.m + j), sph * __ldg(p.tab + 2 * g.m + g.n + j),
+                                           cph, 0.f);
+            }
+        }
+        __syncthreads();
+        const int k = *sN;
+        for (int e = 0; e < k; ++e) {
+            const float4 d = sDirs[e];
+#pragma unroll
+            for (int j = 0; j < kMaxT; ++j)
+                best[j] = fmaxf(best[j], fmaf(c[j].x, d.x, fmaf(c[j].y, d.y, c[j].z * d.z)));
+        }
+        w0 = wend;
+        if (w0 >= MW) break;
+    }
+#pragma unroll
+    for (int j = 0; j < kMaxT; ++j) {
+        const int t = (j * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
+        if (t >= ntex) continue;
+        float u = -2.f;
+        if (best[j] >= -1.5f) {
+            const float th = acosf(fminf(best[j] + 2e-6f, 1.f));
+            const float r = c[j].w;
+            u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+        }
+        V[t] = u * fabsf(u);
+    }
+}
+
+__global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_constant__ FusedParams F) {
+    namespace cg = cooperative_groups;
+    cg::grid_group grid = cg::this_grid();
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ unsigned int sCnt[CT_COUNT];
+    __shared__ int sN;
+    __shared__ unsigned int sCulled, sPassed;
+    __shared__ unsigned long long sStreamed;
+    const StreamParams& P = F.main;
+    const StreamParams& L = F.lvl;
+    const int m = P.grid.m, MW = m * P.grid.W;
+    uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
+    uint32_t* sRowFull = sAM + MW;
+    float4* sDirs = fused_dirs(sAM, MW, m);
+    const int lane = threadIdx.x & 31;
+    const unsigned long long gstride = (unsigned long long)gridDim.x * blockDim.x;
+    if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
+    if (threadIdx.x == 0) {
+        sCulled = sPassed = 0u;
+        sStreamed = 0ull;
+    }
+    const Counters none{nullptr};
+
+    // 1. level-0 cones (inner), every voxel of the level is live
+    for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < F.n0;
+         e0 += gstride) {
+        const unsigned long long e = e0 + lane;
+        int nrows = 0;
+        bool counted = false;
+        ConeRec r;
+        if (e < F.n0) nrows = cone_of_voxel<true>(L, L.vox[e], (unsigned int)e, r, counted);
+        emit_cones<true>(L, nrows, r, counted);
+    }
+    grid.sync();
+    // 2. level-0 rows
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = 0u;
+    for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
+    __syncthreads();
+    fused_rows<true>(L, L.task_count, sAM, sRowFull, none);
+    fused_flush(L, sAM);
+    grid.sync();
+    // 3. clear-direction map
+    fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
+    grid.sync();
+    if (F.use_l1) {
+        // 4. level-1 voxels: filter against the map, inner cones inline (stage 1)
+        StreamParams& L1 = const_cast<StreamParams&>(L);  // only the counter pointers differ
+        (void)L1;
+        for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < F.n1;
+             e0 += gstride) {
+            const unsigned long long e = e0 + lane;
+            int nrows = 0;
+            bool counted = false;
+            ConeRec r;
+            if (e < F.n1) {
+                const float4 q = F.l1[e];
+                if (fast_filter(P, q, P.gam) == F_LIVE) {
+                    // the level-1 records index the level-1 array
+                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
+                }
+            }
+            // stage-1 record/task buffers live after stage 0's in the same arrays
+            const int lane_ = lane;
+            (void)lane_;
+            const unsigned int mrec = __ballot_sync(0xffffffffu, nrows > 0);
+            if (mrec) {
+                int incl = nrows;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int t = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += t;
+                }
+                unsigned int sbase = 0;
+                unsigned long long tbase = 0;
+                const int total = __shfl_sync(0xffffffffu, incl, 31);
+                if (lane == 0) {
+                    sbase = atomicAdd(F.rec1, (unsigned int)__popc(mrec));
+                    tbase = atomicAdd(F.task1, (unsigned long long)total);
+                }
+                sbase = __shfl_sync(0xffffffffu, sbase, 0);
+                tbase = __shfl_sync(0xffffffffu, tbase, 0);
+                if (nrows > 0) {
+                    // stage 1 uses the upper half of the record / task buffers
+                    const unsigned int slot = sbase + __popc(mrec & ((1u << lane) - 1u)) + P.rec_cap / 2;
+                    const unsigned long long t0 = tbase + (unsigned long long)(incl - nrows) + P.task_cap / 2;
+                    if (slot < P.rec_cap && t0 + nrows <= P.task_cap) {
+                        P.recs[slot] = r;
+                        for (int k = 0; k < nrows; ++k)
+                            P.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+                    } else {
+                        for (int k = 0; k < nrows; ++k) raster_row<true>(P, r, r.i0 + k, P.gam, none);
+                    }
+                }
+            }
+        }
+        grid.sync();
+        // 5. level-1 rows (tasks in the upper halves)
+        fused_seed(P, sAM, sRowFull);
+        {
+            const unsigned long long ntask =
+                min(*reinterpret_cast<const volatile unsigned long long*>(F.task1), P.task_cap / 2);
+            for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
+                 k += gstride) {
+                const unsigned long long t = P.tasks[P.task_cap / 2 + k];
+                const ConeRec r = P.recs[t >> 16];
+                if (r.i0 < 0) continue;
+                const int i = r.i0 + (int)(t & 0xffffu);
+                if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+                raster_row<true>(P, r, i, sAM, none);
+            }
+        }
+        fused_flush(P, sAM);
+        grid.sync();
+        // 6. clear-direction map again
+        fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
+        grid.sync();
+    }
+    // 7. brick test
+    {
+        const unsigned int nb = P.nbricks;
+        for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
+            const unsigned int b = b0 + threadIdx.x;
+            bool keep = false;
+            if (b < nb) {
+                const float4 s = __ldg(P.bricks + b);
+                keep = !sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
+            }
+            const unsigned int mk = __ballot_sync(0xffffffffu, keep);
+            if (mk) {
+                unsigned int base = 0;
+                const int leader = __ffs(mk) - 1;
+                if (lane == leader) base = atomicAdd(P.brick_count, (unsigned int)__popc(mk));
+                base = __shfl_sync(0xffffffffu, base, leader);
+                if (keep) P.brick_list[base + __popc(mk & ((1u << lane) - 1u))] = b;
+            }
+        }
+    }
+    grid.sync();
+    // 8. brick voxels: filter; live voxels compute both cones at once (stage 2)
+    {
+        unsigned int nculled = 0, npassed = 0;
+        unsigned long long streamed = 0;
+        const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
+        for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
+            float4 q[kVPT];
+            unsigned int idx[kVPT];
+            bool ok[kVPT];
+#pragma unroll
+            for (int k = 0; k < kVPT; ++k) {
+                ok[k] = k0 + k < nk;
+                idx[k] = ok[k] ? P.brick_list[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
+                ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
+                q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
+            }
+#pragma unroll 1
+            for (int k = 0; k < kVPT; ++k) {
+                const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
+                nculled += f >> 1;
+                npassed += f == F_LIVE;
+                streamed += ok[k];
+                int nrows = 0;
+                bool counted = false;
+                ConeRec r;
+                if (f == F_LIVE) nrows = cone_of_voxel<false>(P, q[k], idx[k], r, counted);
+                emit_cones<false>(P, nrows, r, counted);
+            }
+        }
+        if (npassed) atomicAdd(&sPassed, npassed);
+        if (nculled) atomicAdd(&sCulled, nculled);
+        if (streamed) atomicAdd(&sStreamed, streamed);
+    }
+    grid.sync();
+    // 9. rows of the full stream (both cones, band pairs queued)
+    fused_seed(P, sAM, sRowFull);
+    fused_rows<false>(P, P.task_count, sAM, sRowFull, Counters{sCnt});
+    fused_flush(P, sAM);
+    grid.sync();
+    // 10. band: exact test where the bit is still clear
+    {
+        const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
+        const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
+        unsigned long long tests = 0, hits = 0;
+        for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += gstride) {
+            const unsigned long long e = P.queue[k];
+            const unsigned int vidx = (unsigned int)(e >> 32);
+            const int cell = (int)(e & 0xffffffffu);
+            const int i = cell / P.grid.n, j = cell - i * P.grid.n;
+            uint32_t* wp = P.gam + i * P.grid.W + (j >> 5);
+            const uint32_t bit = 1u << (j & 31);
+            if (ld_cg(wp) & bit) continue;
+            ++tests;
+            if (exact_pair(P, P.vox_main[vidx], cell)) {
+                ++hits;
+                atomicOr(wp, bit);
+            }
+        }
+        if (tests) atomicAdd(P.stats + ST_EXACT, tests);
+        if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        atomicAdd(P.stats + ST_CULLED, (unsigned long long)sCulled);
+        atomicAdd(P.stats + ST_PASSED, (unsigned long long)sPassed);
+        atomicAdd(P.stats + ST_STREAMED, sStreamed);
+        atomicAdd(P.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
+        atomicAdd(P.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
+        atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+    }
+}
+
+}  // namespace am

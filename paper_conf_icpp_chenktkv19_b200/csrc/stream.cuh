@@ -296,19 +296,98 @@ struct ConeRec {
 template <bool COARSE>
 __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint32_t* am, Counters cnt);
 
-// a3-a4 for the live voxels (one per thread): the paper's two cones
-// (GETTOOLICA twice, Alg. 1; COARSE: the inner one only), the exact
-// outer cone checked against the clear-direction map, the phi-row range; one
-// record per surviving voxel and one task per (voxel, row).  With
-// p.live_idx == nullptr every voxel of vox[0, N) is live (clear-map level 0).
+// a3-a4 for one live voxel q (index vidx): the paper's two cones (GETTOOLICA
+// twice, Alg. 1; COARSE: the inner one only), the exact outer cone
+// checked against the clear-direction map, the phi-row range.  Returns the
+// number of phi-rows to rasterise (0: nothing to do) and fills r.  `counted`
+// tells whether the voxel reached the cone computation (am_stats voxels_live).
 template <bool COARSE>
-__global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
+__device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, unsigned int vidx, ConeRec& r,
+                                             bool& counted) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
+    counted = false;
+    const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
+    const float D = sqrtf(vx * vx + vy * vy + vz * vz);
+    if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
+        fill_all(p, p.gam);  // the pivot lies in the closed box: every orientation collides
+        return 0;
+    }
+    counted = true;
+    Cones c;
+    if (COARSE) {
+        c.cin = c.cout = inner_cone(D, h, T);
+        c.clo = 2.f;
+    } else {
+        c = tool_cones(D, h, T);
+    }
+    // the exact outer cone against the clear-direction map: no clear cell
+    // within it means this voxel cannot change the map
+    if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
+    const float rxy = sqrtf(vx * vx + vy * vy);
+    const float phv = atan2f(rxy, vz);
+    const float ao = acosf(fmaxf(c.cout, -1.f));
+    const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+    const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+    if (a0 > a1) return 0;
+    const float invD = 1.f / D;
+    r.cin = c.cin;
+    r.cout = c.cout;
+    r.clo = c.clo;
+    r.cphv = vz * invD;
+    r.sphv = rxy * invD;
+    r.gv = atan2f(vy, vx);
+    r.vidx = vidx;
+    r.i0 = a0;
+    return a1 - a0 + 1;
+}
+
+// Warp-uniform: store the records of the lanes with nrows > 0 and one task per
+// (voxel, row), with one pair of atomics per warp.  When the buffers are full
+// the lane rasterises its rows itself, straight into the global AM.
+template <bool COARSE>
+__device__ __forceinline__ void emit_cones(const StreamParams& p, int nrows, const ConeRec& r, bool counted) {
+    const int lane = threadIdx.x & 31;
+    const unsigned int mcount = __ballot_sync(0xffffffffu, counted);
+    if (lane == 0 && mcount) atomicAdd(p.stats + ST_LIVE, (unsigned long long)__popc(mcount));
+    const unsigned int mrec = __ballot_sync(0xffffffffu, nrows > 0);
+    if (!mrec) return;
+    int incl = nrows;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    unsigned int sbase = 0;
+    unsigned long long tbase = 0;
+    const int total = __shfl_sync(0xffffffffu, incl, 31);
+    if (lane == 0) {
+        sbase = atomicAdd(p.rec_count, (unsigned int)__popc(mrec));
+        tbase = atomicAdd(p.task_count, (unsigned long long)total);
+    }
+    sbase = __shfl_sync(0xffffffffu, sbase, 0);
+    tbase = __shfl_sync(0xffffffffu, tbase, 0);
+    if (nrows > 0) {
+        const unsigned int slot = sbase + __popc(mrec & ((1u << lane) - 1u));
+        const unsigned long long t0 = tbase + (unsigned long long)(incl - nrows);
+        if (slot < p.rec_cap && t0 + nrows <= p.task_cap) {
+            p.recs[slot] = r;
+            for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+        } else {
+            for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
+            if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
+        }
+    }
+}
+
+// a3-a4 over the live list (one voxel per thread): records and row tasks.
+// With p.live_idx == nullptr every voxel of vox[0, N) is live (clear-map level 0).
+template <bool COARSE>
+__global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
     const int lane = threadIdx.x & 31;
     const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
     const unsigned long long wstride = (unsigned long long)gridDim.x * blockDim.x;
-    // warp-uniform loop: the slot reservations below are warp-aggregated
+    // warp-uniform loop: the slot reservations are warp-aggregated
     for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < nlive;
          e0 += wstride) {
         const unsigned long long e = e0 + lane;
@@ -317,76 +396,9 @@ __global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ 
         ConeRec r;
         if (e < nlive) {
             const unsigned int vidx = p.live_idx ? p.live_idx[e] : (unsigned int)e;
-            const float4 q = p.vox[vidx];
-            const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
-            const float D = sqrtf(vx * vx + vy * vy + vz * vz);
-            if (D <= kSqrt3 * h && fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) {
-                fill_all(p, p.gam);  // the pivot lies in the closed box: every orientation collides
-            } else {
-                counted = true;
-                Cones c;
-                if (COARSE) {
-                    c.cin = c.cout = inner_cone(D, h, T);
-                    c.clo = 2.f;
-                } else {
-                    c = tool_cones(D, h, T);
-                }
-                // the exact outer cone against the clear-direction map: no clear
-                // cell within it means this voxel cannot change the map
-                if (c.cout <= 1.f &&
-                    __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) >= c.cout * fabsf(c.cout)) {
-                    const float rxy = sqrtf(vx * vx + vy * vy);
-                    const float phv = atan2f(rxy, vz);
-                    const float ao = acosf(fmaxf(c.cout, -1.f));
-                    const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-                    const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-                    if (a0 <= a1) {
-                        const float invD = 1.f / D;
-                        r.cin = c.cin;
-                        r.cout = c.cout;
-                        r.clo = c.clo;
-                        r.cphv = vz * invD;
-                        r.sphv = rxy * invD;
-                        r.gv = atan2f(vy, vx);
-                        r.vidx = vidx;
-                        r.i0 = a0;
-                        nrows = a1 - a0 + 1;
-                    }
-                }
-            }
+            nrows = cone_of_voxel<COARSE>(p, p.vox[vidx], vidx, r, counted);
         }
-        const unsigned int mcount = __ballot_sync(0xffffffffu, counted);
-        if (lane == 0 && mcount) atomicAdd(p.stats + ST_LIVE, (unsigned long long)__popc(mcount));
-        const unsigned int mrec = __ballot_sync(0xffffffffu, nrows > 0);
-        if (!mrec) continue;
-        // one record slot per surviving lane, nrows task slots each
-        int incl = nrows;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += t;
-        }
-        unsigned int sbase = 0;
-        unsigned long long tbase = 0;
-        const int total = __shfl_sync(0xffffffffu, incl, 31);
-        if (lane == 0) {
-            sbase = atomicAdd(p.rec_count, (unsigned int)__popc(mrec));
-            tbase = atomicAdd(p.task_count, (unsigned long long)total);
-        }
-        sbase = __shfl_sync(0xffffffffu, sbase, 0);
-        tbase = __shfl_sync(0xffffffffu, tbase, 0);
-        if (nrows > 0) {
-            const unsigned int slot = sbase + __popc(mrec & ((1u << lane) - 1u));
-            const unsigned long long t0 = tbase + (unsigned long long)(incl - nrows);
-            if (slot < p.rec_cap && t0 + nrows <= p.task_cap) {
-                p.recs[slot] = r;
-                for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
-            } else {
-                // buffers full: rasterise this voxel's rows here, straight into the global AM
-                for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
-                if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
-            }
-        }
+        emit_cones<COARSE>(p, nrows, r, counted);
     }
 }
 

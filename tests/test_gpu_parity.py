@@ -232,7 +232,10 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     C, H = cfg.leaves()
     P = cfg.pivots(3)
     ctx = _ctx(am, cfg, C, H)
-    ref = ctx.compute_batch(P)
+    ref = ctx.compute_batch(P)  # default: the fused cooperative pipeline
+    ctx.set_option(am.binding.OPT_FUSED, 0)
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_FUSED, 1)
     ctx.set_option(am.binding.OPT_PHASES, 0)
     assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_BRICKS, 0)
