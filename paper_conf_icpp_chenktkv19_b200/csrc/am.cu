@@ -57,7 +57,9 @@ struct am_ctx {
     float* d_cmap = nullptr;
     float* d_cmap_ones = nullptr;          // the all-clear map (no voxel can be dropped)
     uint32_t* d_prev = nullptr;            // diagnostics: copy of the last map
+    unsigned long long* d_ts = nullptr;    // diagnostics: fused-phase timestamps
     int diag = 0;
+    int diag_ts = 0;
     int cmapT = 128;
     int phases = 2;
     float4* d_bricks = nullptr;            // bounding spheres of 256-voxel bricks of d_vox
@@ -349,7 +351,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     int rc;
     const float* cm = ctx->d_cmap_ones;
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
-    if (ctx->fused && ctx->fused_grid > 0 && !ctx->diag && ctx->phases == 2 && ctx->n_l0 > 0 && ctx->bricks_on &&
+    if (ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases == 2 && ctx->n_l0 > 0 && ctx->bricks_on &&
         ctx->d_bricks && ntex <= 4 * ctx->fused_grid * kThreads) {
         // the whole map in one cooperative launch (fused.cuh)
         FusedParams F;
@@ -385,6 +387,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         F.texels = ctx->d_texels;
         F.ntex = ntex;
         F.use_l1 = 1;
+        F.ts = (ctx->diag_ts && ctx->d_ts) ? ctx->d_ts : nullptr;
         const bool timed = ctx->timing != 0;
         if (timed) {
             if (ctx->ev_used == ctx->ev_start.size()) {
@@ -778,6 +781,15 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
         // every voxel goes through the filter once; the rest of it was dropped
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
+        if (ctx->diag_ts && ctx->d_ts) {  // diagnostics: fused-phase durations (us) on stderr
+            unsigned long long t[16];
+            CK(cudaMemcpy(t, ctx->d_ts, sizeof t, cudaMemcpyDeviceToHost));
+            fprintf(stderr, "am fused phases (us):");
+            for (int k = 1; k < 16; ++k)
+                if (t[k] >= t[0] && t[k]) fprintf(stderr, " %d:%.1f", k, (t[k] - t[0]) * 1e-3);
+            fprintf(stderr, "\n");
+            CK(cudaMemset(ctx->d_ts, 0, sizeof t));
+        }
     } else if (!dst_is_device) {
         CK(cudaStreamSynchronize(s));
     }
@@ -876,12 +888,17 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
-        if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "diag must be in [0, 3]");
-        if (value && !ctx->d_prev) {
+        if (value < 0 || value > 7) return fail(ctx, AM_EINVAL, "diag must be in [0, 7]");
+        if ((value & 3) && !ctx->d_prev) {
             CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
         }
+        if ((value & 4) && !ctx->d_ts) {
+            CK(cudaMalloc(&ctx->d_ts, 16 * sizeof(unsigned long long)));
+            CK(cudaMemset(ctx->d_ts, 0, 16 * sizeof(unsigned long long)));
+        }
         ctx->diag = (int)value;
+        ctx->diag_ts = (value & 4) != 0;
         return AM_OK;
     case AM_OPT_BRICKS:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "bricks must be 0 or 1");
@@ -979,6 +996,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);
     cudaFree(ctx->d_prev);
+    cudaFree(ctx->d_ts);
     cudaFree(ctx->d_dirs);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);

@@ -39,7 +39,16 @@ struct FusedParams {
     const float4* texels;     // clear-map texels
     int ntex;
     int use_l1;
+    unsigned long long* ts;   // diagnostics: %globaltimer after each phase (CTA 0), or nullptr
 };
+
+__device__ __forceinline__ void fused_mark(const FusedParams& F, int k) {
+    if (F.ts && blockIdx.x == 0 && threadIdx.x == 0) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        F.ts[k] = t;
+    }
+}
 
 // Dynamic shared memory: AM, row-full bits, a chunk of clear directions.
 constexpr int kFusedDirs = 1024;
@@ -183,6 +192,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         sStreamed = 0ull;
     }
     const Counters none{nullptr};
+    fused_mark(F, 0);
 
     // 1. level-0 cones (inner), every voxel of the level is live
     for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < F.n0;
@@ -195,6 +205,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         emit_cones<true>(L, nrows, r, counted);
     }
     grid.sync();
+    fused_mark(F, 1);
     // 2. level-0 rows
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = 0u;
     for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
@@ -202,9 +213,11 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     fused_rows<true>(L, L.task_count, sAM, sRowFull, none);
     fused_flush(L, sAM);
     grid.sync();
+    fused_mark(F, 2);
     // 3. clear-direction map
     fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
     grid.sync();
+    fused_mark(F, 3);
     if (F.use_l1) {
         // 4. level-1 voxels: filter against the map, inner cones inline (stage 1)
         StreamParams& L1 = const_cast<StreamParams&>(L);  // only the counter pointers differ
@@ -257,6 +270,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
             }
         }
         grid.sync();
+    fused_mark(F, 4);
         // 5. level-1 rows (tasks in the upper halves)
         fused_seed(P, sAM, sRowFull);
         {
@@ -274,9 +288,11 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
         fused_flush(P, sAM);
         grid.sync();
+    fused_mark(F, 5);
         // 6. clear-direction map again
         fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
         grid.sync();
+    fused_mark(F, 6);
     }
     // 7. brick test
     {
@@ -299,6 +315,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
     }
     grid.sync();
+    fused_mark(F, 7);
     // 8. brick voxels: filter; live voxels compute both cones at once (stage 2)
     {
         unsigned int nculled = 0, npassed = 0;
@@ -333,11 +350,13 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         if (streamed) atomicAdd(&sStreamed, streamed);
     }
     grid.sync();
+    fused_mark(F, 8);
     // 9. rows of the full stream (both cones, band pairs queued)
     fused_seed(P, sAM, sRowFull);
     fused_rows<false>(P, P.task_count, sAM, sRowFull, Counters{sCnt});
     fused_flush(P, sAM);
     grid.sync();
+    fused_mark(F, 9);
     // 10. band: exact test where the bit is still clear
     {
         const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
@@ -361,6 +380,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
     }
     __syncthreads();
+    fused_mark(F, 15);
     if (threadIdx.x == 0) {
         atomicAdd(P.stats + ST_CULLED, (unsigned long long)sCulled);
         atomicAdd(P.stats + ST_PASSED, (unsigned long long)sPassed);
