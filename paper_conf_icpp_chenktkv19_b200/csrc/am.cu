@@ -369,6 +369,8 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         F.main.task_count = ctx->d_ctr + kCtrRT + 5;
         F.main.rec_cap = kRecCap;
         F.main.task_cap = kTaskCap;
+        F.main.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
+        F.main.live_idx = ctx->d_live;
         F.lvl = F.main;
         F.lvl.vox = ctx->d_coarse;
         F.lvl.N = ctx->n_l0;

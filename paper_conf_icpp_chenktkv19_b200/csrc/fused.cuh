@@ -332,22 +332,35 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
                 q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
             }
-#pragma unroll 1
+#pragma unroll
             for (int k = 0; k < kVPT; ++k) {
                 const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
                 nculled += f >> 1;
-                npassed += f == F_LIVE;
                 streamed += ok[k];
-                int nrows = 0;
-                bool counted = false;
-                ConeRec r;
-                if (f == F_LIVE) nrows = cone_of_voxel<false>(P, q[k], idx[k], r, counted);
-                emit_cones<false>(P, nrows, r, counted);
+                append_live(P, f == F_LIVE, idx[k], npassed);
             }
         }
-        if (npassed) atomicAdd(&sPassed, npassed);
+        if ((threadIdx.x & 31) == 0 && npassed) atomicAdd(&sPassed, npassed);
         if (nculled) atomicAdd(&sCulled, nculled);
         if (streamed) atomicAdd(&sStreamed, streamed);
+    }
+    grid.sync();
+    fused_mark(F, 10);
+    // 8b. cones of the live voxels, spread over every thread of the grid
+    {
+        const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
+        for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < nlive;
+             e0 += gstride) {
+            const unsigned long long e = e0 + lane;
+            int nrows = 0;
+            bool counted = false;
+            ConeRec r;
+            if (e < nlive) {
+                const unsigned int vidx = P.live_idx[e];
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+            }
+            emit_cones<false>(P, nrows, r, counted);
+        }
     }
     grid.sync();
     fused_mark(F, 8);
