@@ -170,6 +170,67 @@ __device__ void fused_clear_map(const StreamParams& p, const float4* texels, int
     }
 }
 
+// CTA-wide reservation (every thread of the CTA calls it): `cnt` slots for
+// this thread in an array filled through the global counter `g`, with ONE
+// atomic per CTA (many warps hitting one counter serialise in L2).  Returns
+// this thread's first slot.  sScan: kWarps + 1 words of shared memory.
+template <typename T>
+__device__ __forceinline__ T cta_reserve(T cnt, T* g, T* sScan) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const T t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    if (lane == 31) sScan[warp] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        T run = 0;
+        for (int w = 0; w < kWarps; ++w) {
+            const T t = sScan[w];
+            sScan[w] = run;
+            run += t;
+        }
+        sScan[kWarps] = run ? atomicAdd(g, run) : (T)0;
+    }
+    __syncthreads();
+    const T base = sScan[kWarps] + sScan[warp] + incl - cnt;
+    __syncthreads();
+    return base;
+}
+
+struct FusedScratch {
+    unsigned int r32[kWarps + 1];
+    unsigned long long r64[kWarps + 1];
+};
+
+// CTA-wide emit_cones: records at slot_off + [reserved], tasks at
+// task_off + [reserved]; rows rasterised inline when the buffers are full.
+template <bool COARSE>
+__device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned int* rec_count,
+                                               unsigned long long* task_count, unsigned int slot_off,
+                                               unsigned long long task_off, unsigned int slot_cap,
+                                               unsigned long long task_cap, int nrows, const ConeRec& r, bool counted,
+                                               FusedScratch* sc, unsigned long long* live_stat) {
+    if (live_stat) {
+        const unsigned int c = __popc(__ballot_sync(0xffffffffu, counted));
+        if ((threadIdx.x & 31) == 0 && c) atomicAdd(live_stat, (unsigned long long)c);
+    }
+    const unsigned int slot = cta_reserve<unsigned int>(nrows > 0 ? 1u : 0u, rec_count, sc->r32) + slot_off;
+    const unsigned long long t0 =
+        cta_reserve<unsigned long long>((unsigned long long)nrows, task_count, sc->r64) + task_off;
+    if (nrows > 0) {
+        if (slot < slot_cap && t0 + nrows <= task_cap) {
+            p.recs[slot] = r;
+            for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+        } else {
+            for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
+            if (slot < slot_cap) p.recs[slot].i0 = -1;
+        }
+    }
+}
+
 __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_constant__ FusedParams F) {
     namespace cg = cooperative_groups;
     cg::grid_group grid = cg::this_grid();
@@ -178,6 +239,8 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     __shared__ int sN;
     __shared__ unsigned int sCulled, sPassed;
     __shared__ unsigned long long sStreamed;
+    __shared__ FusedScratch sc;
+    __shared__ unsigned int sLive[kVPT * kThreads];
     const StreamParams& P = F.main;
     const StreamParams& L = F.lvl;
     const int m = P.grid.m, MW = m * P.grid.W;
@@ -194,15 +257,15 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     const Counters none{nullptr};
     fused_mark(F, 0);
 
-    // 1. level-0 cones (inner), every voxel of the level is live
-    for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < F.n0;
-         e0 += gstride) {
-        const unsigned long long e = e0 + lane;
+    // 1. level-0 cones (inner), every voxel of the level is live (CTA-uniform loop)
+    for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < F.n0; b0 += gstride) {
+        const unsigned long long e = b0 + threadIdx.x;
         int nrows = 0;
         bool counted = false;
         ConeRec r;
         if (e < F.n0) nrows = cone_of_voxel<true>(L, L.vox[e], (unsigned int)e, r, counted);
-        emit_cones<true>(L, nrows, r, counted);
+        emit_cones_cta<true>(L, L.rec_count, L.task_count, 0u, 0ull, L.rec_cap, L.task_cap, nrows, r, counted, &sc,
+                             nullptr);
     }
     grid.sync();
     fused_mark(F, 1);
@@ -219,58 +282,22 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     grid.sync();
     fused_mark(F, 3);
     if (F.use_l1) {
-        // 4. level-1 voxels: filter against the map, inner cones inline (stage 1)
-        StreamParams& L1 = const_cast<StreamParams&>(L);  // only the counter pointers differ
-        (void)L1;
-        for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < F.n1;
-             e0 += gstride) {
-            const unsigned long long e = e0 + lane;
+        // 4. level-1 voxels: filter against the map, inner cones (stage 1: upper
+        //    halves of the record / task buffers; the records index the level-1 array)
+        for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < F.n1; b0 += gstride) {
+            const unsigned long long e = b0 + threadIdx.x;
             int nrows = 0;
             bool counted = false;
             ConeRec r;
             if (e < F.n1) {
                 const float4 q = F.l1[e];
-                if (fast_filter(P, q, P.gam) == F_LIVE) {
-                    // the level-1 records index the level-1 array
-                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
-                }
+                if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
             }
-            // stage-1 record/task buffers live after stage 0's in the same arrays
-            const int lane_ = lane;
-            (void)lane_;
-            const unsigned int mrec = __ballot_sync(0xffffffffu, nrows > 0);
-            if (mrec) {
-                int incl = nrows;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const int t = __shfl_up_sync(0xffffffffu, incl, o);
-                    if (lane >= o) incl += t;
-                }
-                unsigned int sbase = 0;
-                unsigned long long tbase = 0;
-                const int total = __shfl_sync(0xffffffffu, incl, 31);
-                if (lane == 0) {
-                    sbase = atomicAdd(F.rec1, (unsigned int)__popc(mrec));
-                    tbase = atomicAdd(F.task1, (unsigned long long)total);
-                }
-                sbase = __shfl_sync(0xffffffffu, sbase, 0);
-                tbase = __shfl_sync(0xffffffffu, tbase, 0);
-                if (nrows > 0) {
-                    // stage 1 uses the upper half of the record / task buffers
-                    const unsigned int slot = sbase + __popc(mrec & ((1u << lane) - 1u)) + P.rec_cap / 2;
-                    const unsigned long long t0 = tbase + (unsigned long long)(incl - nrows) + P.task_cap / 2;
-                    if (slot < P.rec_cap && t0 + nrows <= P.task_cap) {
-                        P.recs[slot] = r;
-                        for (int k = 0; k < nrows; ++k)
-                            P.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
-                    } else {
-                        for (int k = 0; k < nrows; ++k) raster_row<true>(P, r, r.i0 + k, P.gam, none);
-                    }
-                }
-            }
+            emit_cones_cta<true>(P, F.rec1, F.task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
+                                 counted, &sc, nullptr);
         }
         grid.sync();
-    fused_mark(F, 4);
+        fused_mark(F, 4);
         // 5. level-1 rows (tasks in the upper halves)
         fused_seed(P, sAM, sRowFull);
         {
@@ -288,11 +315,11 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
         fused_flush(P, sAM);
         grid.sync();
-    fused_mark(F, 5);
+        fused_mark(F, 5);
         // 6. clear-direction map again
         fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
         grid.sync();
-    fused_mark(F, 6);
+        fused_mark(F, 6);
     }
     // 7. brick test
     {
@@ -304,24 +331,21 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 const float4 s = __ldg(P.bricks + b);
                 keep = !sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
             }
-            const unsigned int mk = __ballot_sync(0xffffffffu, keep);
-            if (mk) {
-                unsigned int base = 0;
-                const int leader = __ffs(mk) - 1;
-                if (lane == leader) base = atomicAdd(P.brick_count, (unsigned int)__popc(mk));
-                base = __shfl_sync(0xffffffffu, base, leader);
-                if (keep) P.brick_list[base + __popc(mk & ((1u << lane) - 1u))] = b;
-            }
+            const unsigned int pos = cta_reserve<unsigned int>(keep ? 1u : 0u, P.brick_count, sc.r32);
+            if (keep) P.brick_list[pos] = b;
         }
     }
     grid.sync();
     fused_mark(F, 7);
-    // 8. brick voxels: filter; live voxels compute both cones at once (stage 2)
+    // 8. kept bricks: filter (kVPT bricks per CTA step), compact the live voxels
+    //    in shared memory, then both cones for them with the whole CTA (stage 2)
     {
         unsigned int nculled = 0, npassed = 0;
         unsigned long long streamed = 0;
         const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
         for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
+            if (threadIdx.x == 0) sN = 0;
+            __syncthreads();
             float4 q[kVPT];
             unsigned int idx[kVPT];
             bool ok[kVPT];
@@ -337,30 +361,35 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
                 nculled += f >> 1;
                 streamed += ok[k];
-                append_live(P, f == F_LIVE, idx[k], npassed);
+                const unsigned int ml = __ballot_sync(0xffffffffu, f == F_LIVE);
+                if (ml) {
+                    int base = 0;
+                    const int leader = __ffs(ml) - 1;
+                    if (lane == leader) base = atomicAdd(&sN, __popc(ml));
+                    base = __shfl_sync(0xffffffffu, base, leader);
+                    if (f == F_LIVE) sLive[base + __popc(ml & ((1u << lane) - 1u))] = idx[k];
+                    if (lane == 0) npassed += __popc(ml);
+                }
             }
+            __syncthreads();
+            const int nl = sN;
+            for (int e0 = 0; e0 < nl; e0 += kThreads) {
+                const int e = e0 + threadIdx.x;
+                int nrows = 0;
+                bool counted = false;
+                ConeRec r;
+                if (e < nl) {
+                    const unsigned int vidx = sLive[e];
+                    nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+                }
+                emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
+                                      &sc, P.stats + ST_LIVE);
+            }
+            __syncthreads();
         }
-        if ((threadIdx.x & 31) == 0 && npassed) atomicAdd(&sPassed, npassed);
+        if (npassed) atomicAdd(&sPassed, npassed);
         if (nculled) atomicAdd(&sCulled, nculled);
         if (streamed) atomicAdd(&sStreamed, streamed);
-    }
-    grid.sync();
-    fused_mark(F, 10);
-    // 8b. cones of the live voxels, spread over every thread of the grid
-    {
-        const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
-        for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < nlive;
-             e0 += gstride) {
-            const unsigned long long e = e0 + lane;
-            int nrows = 0;
-            bool counted = false;
-            ConeRec r;
-            if (e < nlive) {
-                const unsigned int vidx = P.live_idx[e];
-                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
-            }
-            emit_cones<false>(P, nrows, r, counted);
-        }
     }
     grid.sync();
     fused_mark(F, 8);
