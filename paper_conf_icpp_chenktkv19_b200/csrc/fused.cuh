@@ -212,18 +212,29 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
                                                unsigned long long* task_count, unsigned int slot_off,
                                                unsigned long long task_off, unsigned int slot_cap,
                                                unsigned long long task_cap, int nrows, const ConeRec& r, bool counted,
-                                               FusedScratch* sc, unsigned long long* live_stat) {
+                                               FusedScratch* sc, unsigned long long* live_stat,
+                                               const uint32_t* rowfull) {
     if (live_stat) {
         const unsigned int c = __popc(__ballot_sync(0xffffffffu, counted));
         if ((threadIdx.x & 31) == 0 && c) atomicAdd(live_stat, (unsigned long long)c);
     }
-    const unsigned int slot = cta_reserve<unsigned int>(nrows > 0 ? 1u : 0u, rec_count, sc->r32) + slot_off;
+    // rows already full in the global AM need no task
+    int ntask = 0;
+    for (int k = 0; k < nrows; ++k) {
+        const int i = r.i0 + k;
+        ntask += !((rowfull[i >> 5] >> (i & 31)) & 1u);
+    }
+    const unsigned int slot = cta_reserve<unsigned int>(ntask > 0 ? 1u : 0u, rec_count, sc->r32) + slot_off;
     const unsigned long long t0 =
-        cta_reserve<unsigned long long>((unsigned long long)nrows, task_count, sc->r64) + task_off;
-    if (nrows > 0) {
-        if (slot < slot_cap && t0 + nrows <= task_cap) {
+        cta_reserve<unsigned long long>((unsigned long long)ntask, task_count, sc->r64) + task_off;
+    if (ntask > 0) {
+        if (slot < slot_cap && t0 + ntask <= task_cap) {
             p.recs[slot] = r;
-            for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
+            unsigned long long t = t0;
+            for (int k = 0; k < nrows; ++k) {
+                const int i = r.i0 + k;
+                if (!((rowfull[i >> 5] >> (i & 31)) & 1u)) p.tasks[t++] = ((unsigned long long)slot << 16) | (unsigned int)k;
+            }
         } else {
             for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
             if (slot < slot_cap) p.recs[slot].i0 = -1;
@@ -240,7 +251,6 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     __shared__ unsigned int sCulled, sPassed;
     __shared__ unsigned long long sStreamed;
     __shared__ FusedScratch sc;
-    __shared__ unsigned int sLive[kVPT * kThreads];
     const StreamParams& P = F.main;
     const StreamParams& L = F.lvl;
     const int m = P.grid.m, MW = m * P.grid.W;
@@ -255,6 +265,8 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         sStreamed = 0ull;
     }
     const Counters none{nullptr};
+    for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
+    __syncthreads();
     fused_mark(F, 0);
 
     // 1. level-0 cones (inner), every voxel of the level is live (CTA-uniform loop)
@@ -265,7 +277,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         ConeRec r;
         if (e < F.n0) nrows = cone_of_voxel<true>(L, L.vox[e], (unsigned int)e, r, counted);
         emit_cones_cta<true>(L, L.rec_count, L.task_count, 0u, 0ull, L.rec_cap, L.task_cap, nrows, r, counted, &sc,
-                             nullptr);
+                             nullptr, sRowFull);
     }
     grid.sync();
     fused_mark(F, 1);
@@ -284,6 +296,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     if (F.use_l1) {
         // 4. level-1 voxels: filter against the map, inner cones (stage 1: upper
         //    halves of the record / task buffers; the records index the level-1 array)
+        fused_seed(P, sAM, sRowFull);
         for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < F.n1; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
             int nrows = 0;
@@ -294,7 +307,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
             }
             emit_cones_cta<true>(P, F.rec1, F.task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
-                                 counted, &sc, nullptr);
+                                 counted, &sc, nullptr, sRowFull);
         }
         grid.sync();
         fused_mark(F, 4);
@@ -337,15 +350,13 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     }
     grid.sync();
     fused_mark(F, 7);
-    // 8. kept bricks: filter (kVPT bricks per CTA step), compact the live voxels
-    //    in shared memory, then both cones for them with the whole CTA (stage 2)
+    // 8a. kept bricks: filter (kVPT bricks per CTA step); live voxels go to the
+    //     global live list with one atomic per CTA step
     {
         unsigned int nculled = 0, npassed = 0;
         unsigned long long streamed = 0;
         const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
         for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
-            if (threadIdx.x == 0) sN = 0;
-            __syncthreads();
             float4 q[kVPT];
             unsigned int idx[kVPT];
             bool ok[kVPT];
@@ -356,40 +367,44 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
                 q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
             }
+            bool live[kVPT];
+            unsigned int nl = 0;
 #pragma unroll
             for (int k = 0; k < kVPT; ++k) {
                 const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
                 nculled += f >> 1;
                 streamed += ok[k];
-                const unsigned int ml = __ballot_sync(0xffffffffu, f == F_LIVE);
-                if (ml) {
-                    int base = 0;
-                    const int leader = __ffs(ml) - 1;
-                    if (lane == leader) base = atomicAdd(&sN, __popc(ml));
-                    base = __shfl_sync(0xffffffffu, base, leader);
-                    if (f == F_LIVE) sLive[base + __popc(ml & ((1u << lane) - 1u))] = idx[k];
-                    if (lane == 0) npassed += __popc(ml);
-                }
+                live[k] = f == F_LIVE;
+                nl += live[k];
             }
-            __syncthreads();
-            const int nl = sN;
-            for (int e0 = 0; e0 < nl; e0 += kThreads) {
-                const int e = e0 + threadIdx.x;
-                int nrows = 0;
-                bool counted = false;
-                ConeRec r;
-                if (e < nl) {
-                    const unsigned int vidx = sLive[e];
-                    nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
-                }
-                emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
-                                      &sc, P.stats + ST_LIVE);
-            }
-            __syncthreads();
+            npassed += nl;
+            unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
+#pragma unroll
+            for (int k = 0; k < kVPT; ++k)
+                if (live[k]) P.live_idx[pos++] = idx[k];
         }
         if (npassed) atomicAdd(&sPassed, npassed);
         if (nculled) atomicAdd(&sCulled, nculled);
         if (streamed) atomicAdd(&sStreamed, streamed);
+    }
+    fused_seed(P, sAM, sRowFull);  // row-full bits of the global AM (unchanged until phase 9)
+    grid.sync();
+    fused_mark(F, 10);
+    // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2)
+    {
+        const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
+        for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
+            const unsigned long long e = b0 + threadIdx.x;
+            int nrows = 0;
+            bool counted = false;
+            ConeRec r;
+            if (e < nlive) {
+                const unsigned int vidx = P.live_idx[e];
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+            }
+            emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
+                                  &sc, P.stats + ST_LIVE, sRowFull);
+        }
     }
     grid.sync();
     fused_mark(F, 8);
