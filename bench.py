@@ -178,12 +178,46 @@ def run_reference(args):
     return 0
 
 
-def _config_dict(cfg, N):
+def _config_dict(cfg, N, flushed=True):
     return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
                         f"pivots on the {cfg.offset:g} mm path",
             "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
-            "l2": f"inputs ({16 * N / 1e6:.0f} MB) {'exceed' if 16 * N > L2_BYTES else 'fit in'} L2 (126 MB); no flush",
+            "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
+                   f"every timed step, outside the per-step CUDA events") if flushed else
+                  f"inputs {16 * N / 1e6:.0f} MB; no flush",
             "parallelism": "pivot-sharded (weak)"}
+
+
+def _ncu_traffic(cfg_name, kernel):
+    """DRAM bytes per launch of `kernel` from the committed ncu --set full summary (or None)."""
+    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(prof))
+        k = d.get("kernels", {}).get(kernel)
+        if k and k.get("config") == cfg_name:
+            return k.get("dram_bytes_per_launch"), k.get("tag")
+    except Exception:
+        pass
+    return None, None
+
+
+def _timed_maps(ctx, piv, out, stream, steps, flush, torch):
+    """Per-step CUDA events around each am_compute on `stream`; L2 flushed (a write larger
+    than L2) before every step when `flush` is a tensor.  Returns (sum of step ms, wall ms)."""
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for k in range(steps):
+        if flush is not None:
+            with torch.cuda.stream(stream):
+                flush.fill_(k & 0xFF)
+        evs[k][0].record(stream)
+        ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
+        evs[k][1].record(stream)
+    t1.record(stream)
+    stream.synchronize()
+    return sum(a.elapsed_time(b) for a, b in evs), t0.elapsed_time(t1)
 
 
 def run_ours(args):
@@ -197,6 +231,7 @@ def run_ours(args):
     dev = torch.device("cuda", local if ws > 1 else 0)
     torch.cuda.set_device(dev)
     import paper_conf_icpp_chenktkv19_b200 as am
+    B = am.binding
 
     cfg, C, H, gen_s = _scene(args.config)
     N = len(H)
@@ -210,42 +245,61 @@ def run_ours(args):
     upload_s = time.time() - t0
     stream = torch.cuda.Stream(dev)
     out = torch.zeros((len(piv), ctx.words), dtype=torch.int32, device=dev)
+    flush = None if args.no_flush else torch.empty(2 * L2_BYTES, dtype=torch.uint8, device=dev)
     # warm-up
     for k in range(args.warmup):
         ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
     stream.synchronize()
-    # stats of one map (outside the timed region)
-    _, st = ctx.compute(piv[0], stats=True)
-    ctx.set_option(am.binding.OPT_KERNEL_TIMING, 1)
+    # per-pivot counters (outside the timed region)
+    stats = [ctx.compute(p, stats=True)[1] for p in piv]
+    mean = {k: float(np.mean([getattr(s_, k) for s_ in stats])) for k in stats[0].__dict__}
+
+    # ---- timed region: K maps, L2 flushed before each, CUDA events on the launching stream
+    ctx.set_option(B.OPT_KERNEL_TIMING, 1)
     ctx.kernel_time()
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
     with ClockSampler(dev.index) as clk:
-        ev0.record(stream)
-        for k in range(args.steps):
-            ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
-        ev1.record(stream)
-        stream.synchronize()
+        ms, wall_ms = _timed_maps(ctx, piv, out, stream, args.steps, flush, torch)
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
-    ms = ev0.elapsed_time(ev1)
     kms, klaunch = ctx.kernel_time()
-    ctx.set_option(am.binding.OPT_KERNEL_TIMING, 0)
-    # e2e: the public API with HOST buffers (pivot in, packed AM out), synchronous per step
+    # warm-L2 variant (back to back, no flush): detail only
+    ms_warm, _ = _timed_maps(ctx, piv, out, stream, min(args.steps, 200), None, torch)
+    ms_warm /= min(args.steps, 200)
+    ctx.kernel_time()
+    # ---- full-scan leg: every voxel read by filter_kernel (no brick skipping, one launch per stage)
+    full = None
+    if not args.no_full_scan:
+        ctx.set_option(B.OPT_FUSED, 0)
+        ctx.set_option(B.OPT_BRICKS, 0)
+        kf = max(1, min(args.steps, 50))
+        fms, _ = _timed_maps(ctx, piv, out, stream, kf, flush, torch)
+        fk, fl = ctx.kernel_time()
+        ctx.set_option(B.OPT_BRICKS, 1)
+        ctx.set_option(B.OPT_FUSED, 1)
+        full = {"ms_per_am": fms / kf, "kernel_ms_avg": fk / max(fl, 1), "steps": kf}
+    ctx.set_option(B.OPT_KERNEL_TIMING, 0)
+
+    # ---- e2e: the public API with HOST buffers (pivot in, packed AM out), synchronous per step
     host_out = np.zeros(ctx.words, dtype=np.uint32)
     for k in range(min(args.warmup, 3)):
         ctx.compute(piv[k % len(piv)], out=host_out)
     ke = max(1, min(args.steps, args.e2e_steps))
     if dist:
         dist.barrier()
-    t0 = time.perf_counter()
+    e2e_s = 0.0
+    # clocked per step so the flush stays outside
     for k in range(ke):
+        if flush is not None:
+            with torch.cuda.stream(stream):
+                flush.fill_(k & 0xFF)
+            stream.synchronize()
+        t1 = time.perf_counter()
         ctx.compute(piv[k % len(piv)], out=host_out)
-    e2e_s = time.perf_counter() - t0
+        e2e_s += time.perf_counter() - t1
     t = torch.tensor([ms, e2e_s, kms / max(klaunch, 1)], dtype=torch.float64, device=dev)
     if dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -255,20 +309,15 @@ def run_ours(args):
     value = tests_per_map * maps / (ms_max / 1e3)
     e2e_value = tests_per_map * ke * ws / e2e_max
     peak, peak_src = _peaks()
+    # algorithmic bytes per AM = 16 N (one read of every leaf) + m n / 8 (AM write)
     alg_bytes = 16.0 * N + cfg.m * cfg.n / 8.0
     achieved = alg_bytes / (kavg_ms / 1e3) / 1e9
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
-    if os.path.exists(prof):
-        try:
-            d = json.load(open(prof))
-            if d.get("config") == cfg.name and d.get("kernel") == "filter_kernel":
-                traffic = d.get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    # bytes the fused kernel actually needs: brick spheres, kept bricks' voxels, both map levels
+    touched = 16.0 * (ctx_nbricks(N) + mean["voxels_streamed"] + mean["level_voxels"]) + cfg.m * cfg.n / 8.0
+    traffic, traffic_tag = _ncu_traffic(cfg.name, "am_pipeline_kernel")
     baseline_ms = None
     if args.baseline and rank == 0:
-        ctx.set_option(am.binding.OPT_BASELINE_REJECT, 1)
+        ctx.set_option(B.OPT_BASELINE_REJECT, 1)
         bo = torch.zeros(ctx.words, dtype=torch.int32, device=dev)
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -284,27 +333,43 @@ def run_ours(args):
                "sample": f"{r['cells']} seeded cells of one {cfg.name} map (pivot 0), every voxel per cell, "
                          f"{r['seconds']:.1f} s"}
     if rank == 0:
-        ncpu = os.cpu_count()
+        full_roof = None
+        if full:
+            fa = 16.0 * N / (full["kernel_ms_avg"] / 1e3) / 1e9
+            ft, ftag = _ncu_traffic(cfg.name, "filter_kernel")
+            full_roof = {"kernel": "filter_kernel", "bound": "hbm", "achieved": fa, "peak": peak, "unit": "GB/s",
+                         "frac": fa / peak, "traffic": ft, "traffic_tag": ftag,
+                         "kernel_ms_avg": full["kernel_ms_avg"], "algorithmic_bytes_per_launch": 16.0 * N,
+                         "ms_per_am": full["ms_per_am"],
+                         "note": "AM_OPT_FUSED=0, AM_OPT_BRICKS=0: every voxel read once per map (no skipping)"}
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N),
+            "config": _config_dict(cfg, N, flush is not None),
             "ms_per_am": ms_max / args.steps,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "filter_kernel", "kernel_ms_avg": kavg_ms,
-                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
+                         "frac": achieved / peak, "traffic": traffic, "traffic_tag": traffic_tag,
+                         "kernel": "am_pipeline_kernel", "kernel_ms_avg": kavg_ms,
+                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+                         "touched_bytes_per_launch": touched,
+                         "touched_gbs": touched / (kavg_ms / 1e3) / 1e9,
+                         "note": "achieved = SURVEY 8(d) algorithmic bytes (16 N + m n / 8) / kernel time; "
+                                 "the kernel skips most of them (touched_bytes, traffic), so frac is the "
+                                 "speed relative to one full HBM pass, not bandwidth use"},
+            "full_scan_roofline": full_roof,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12, "d2h_bytes_per_step": 4 * ctx.words,
                     "ms_per_am": 1e3 * e2e_max / ke, "steps": ke,
                     "note": "am_compute with a host pivot (12 B, passed in the launch) and a host AM buffer; "
-                            "synchronous per step; voxels resident (upload excluded, PAPER.md L313)"},
-            "gpu_launches": 2 * args.steps,
+                            "synchronous per step; voxels resident (upload excluded, PAPER.md L313); "
+                            "L2 flushed before each step, outside the per-step clock"},
+            "gpu_launches": klaunch,
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
-            "detail": {"stats_pivot0": st.__dict__, "upload_s": upload_s, "scene_gen_s": gen_s,
+            "detail": {"stats_mean_over_pivots": mean, "upload_s": upload_s, "scene_gen_s": gen_s,
                        "pivots_per_rank": len(piv), "baseline_ms_per_am": baseline_ms,
-                       "host_cpus": ncpu,
+                       "warm_l2_ms_per_am": ms_warm, "timed_wall_ms_incl_flush": wall_ms,
+                       "host_cpus": os.cpu_count(), "build": _build_id(),
                        "paper_context": "PAPER.md L32/L75: <18 ms per AM, 27M octree nodes x 4096 orientations, "
                                         "GTX 1080(Ti); 'over 23x' vs PBox"},
         }
@@ -313,6 +378,10 @@ def run_ours(args):
     if dist:
         dist.destroy_process_group()
     return 0
+
+
+def ctx_nbricks(N):
+    return (N + 255) // 256
 
 
 def _build_id():
@@ -337,6 +406,8 @@ def main():
     ap.add_argument("--ref-seconds", type=float, default=60.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--baseline", action="store_true", help="also time am_compute_baseline once")
+    ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
+    ap.add_argument("--no-full-scan", action="store_true", help="skip the full-scan (filter_kernel) leg")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

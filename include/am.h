@@ -62,6 +62,8 @@ typedef struct {
     int64_t exact_hits;        /* of which collided                                             */
     int64_t queue_overflow;    /* band pairs resolved inline because the queue was full         */
     int64_t early_exit;        /* 1 if the AM filled up and the stream stopped early (a7)       */
+    int64_t bricks_kept;       /* 256-voxel bricks whose voxels were read (AM_OPT_BRICKS)       */
+    int64_t level_voxels;      /* voxels of the clear-map levels (read once more per map)       */
 } am_stats;
 
 enum {
@@ -150,9 +152,12 @@ int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int
 int am_set_option(am_ctx* ctx, int key, int64_t value);
 
 /*
- * Device time of the voxel-streaming kernel (steps a1-a5, the dominant kernel)
- * summed over its launches since the previous call, measured with CUDA events
- * recorded on the launching stream while AM_OPT_KERNEL_TIMING is 1.  Waits for
+ * Device time of the dominant kernel summed over its launches since the
+ * previous call: the fused pipeline kernel (am_pipeline_kernel, every step of
+ * the map in one launch) when AM_OPT_FUSED applies, otherwise the full-stream
+ * launch of steps a1-a3 (brick_test + brick_voxels, or filter_kernel when
+ * AM_OPT_BRICKS = 0).  Measured with CUDA events recorded on the launching
+ * stream while AM_OPT_KERNEL_TIMING is 1.  Waits for
  * the recorded events, then resets the accumulator.  *total_ms and *launches
  * must be non-NULL.
  */

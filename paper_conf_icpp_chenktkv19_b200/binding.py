@@ -40,7 +40,8 @@ class _Cyl(ctypes.Structure):
 class _Stats(ctypes.Structure):
     _fields_ = [(k, ctypes.c_int64) for k in (
         "voxels_streamed", "voxels_culled", "voxels_skipped", "voxels_live", "rows_rasterised",
-        "band_pairs", "exact_tests", "exact_hits", "queue_overflow", "early_exit")]
+        "band_pairs", "exact_tests", "exact_hits", "queue_overflow", "early_exit", "bricks_kept",
+        "level_voxels")]
 
 
 @dataclass
@@ -55,6 +56,8 @@ class Stats:
     exact_hits: int
     queue_overflow: int
     early_exit: int
+    bricks_kept: int
+    level_voxels: int
 
 
 lib = ctypes.CDLL(LIB_PATH)

@@ -779,10 +779,12 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         CK(cudaMemcpyAsync(h, ctx->d_ctr, sizeof h, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         int64_t* o = reinterpret_cast<int64_t*>(stats);
-        static_assert(sizeof(am_stats) == ST_PASSED * sizeof(int64_t), "am_stats mirrors StatIdx");
+        static_assert(sizeof(am_stats) == (ST_PASSED + 2) * sizeof(int64_t), "am_stats mirrors StatIdx");
         for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
         // every voxel goes through the filter once; the rest of it was dropped
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
+        stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks) ? (int64_t)h[kCtrBricks] : (int64_t)ctx->nbricks;
+        stats->level_voxels = ctx->phases == 0 ? 0 : ctx->phases == 1 ? ctx->n_l0 : ctx->n_l1;
         if (ctx->diag_ts && ctx->d_ts) {  // diagnostics: fused-phase durations (us) on stderr
             unsigned long long t[16];
             CK(cudaMemcpy(t, ctx->d_ts, sizeof t, cudaMemcpyDeviceToHost));

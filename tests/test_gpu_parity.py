@@ -182,6 +182,11 @@ def test_small_queue_overflow_is_exact(am):
     ctx.set_option(am.binding.OPT_BAND_QUEUE, 3)
     out, st2 = ctx.compute(p, stats=True)
     assert st2.queue_overflow > 0 or st.band_pairs <= 3
+    # counter consistency: every voxel is culled, skipped or passed; kept bricks within the model
+    assert st.voxels_culled + st.voxels_skipped <= len(H)
+    assert 0 <= st.bricks_kept <= (len(H) + 255) // 256
+    assert st.voxels_streamed <= min(len(H), 256 * st.bricks_kept)
+    assert 0 < st.level_voxels < len(H)
     S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n)
     assert _compare(am.unpack(out, cfg.m, cfg.n), S)[0] == 0
     ctx.close()

@@ -2,8 +2,8 @@
 
     python tools/summarize_ncu.py <tag> [config]
 reads gpurun_out/prof_<tag>.ncu-rep and gpurun_out/launches_<tag>.csv, writes
-profiles/<tag>_launches.txt, profiles/<tag>_<kernel>_ncu.txt and (for the
-filter kernel) profiles/ncu_summary.json, which bench.py reads for `traffic`.
+profiles/<tag>_launches.txt, profiles/<tag>_<kernel>_ncu.txt and merges each captured
+kernel's DRAM bytes into profiles/ncu_summary.json, which bench.py reads for `traffic`.
 """
 import csv
 import io
@@ -79,17 +79,21 @@ def main():
                       "sm__inst_executed.sum", "launch__registers_per_thread"):
                 if k in rawrow:
                     f.write(f"{k:34s} {rawrow[k]:>16s} {rawu.get(k, '')}\n")
-        if kname == "filter_kernel" and "dram__bytes_read.sum" in rawrow:
+        if "dram__bytes_read.sum" in rawrow:
             def tobytes(v, u):
                 v = float(v.replace(",", ""))
                 return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
             rd = tobytes(rawrow["dram__bytes_read.sum"], rawu["dram__bytes_read.sum"])
             wr = tobytes(rawrow["dram__bytes_write.sum"], rawu["dram__bytes_write.sum"])
-            json.dump({"config": config, "kernel": "filter_kernel", "tag": tag,
-                       "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
-                       "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full)"},
-                      open(os.path.join(prof, "ncu_summary.json"), "w"), indent=1)
-
+            sp = os.path.join(prof, "ncu_summary.json")
+            try:
+                summ = json.load(open(sp))
+            except Exception:
+                summ = {}
+            summ.setdefault("kernels", {})[kname] = {
+                "config": config, "tag": tag, "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+                "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full), launch id {kid}"}
+            json.dump({"kernels": summ["kernels"]}, open(sp, "w"), indent=1)
 
 if __name__ == "__main__":
     main()
