@@ -2,12 +2,14 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl ours|reference]
 
-A step is one accessibility map -- the whole hot path (a1-a8 of SURVEY.md 8(a))
-for one pivot of the seeded 1 mm path over the resident voxel model.  Default
-workload: C3 (head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096
-orientations), the configuration BASELINE.json's metric is quoted on.
-For N > 1 (torchrun), every rank computes its own pivots of the toolpath batch
-(pivot sharding): no data-path collective, weak scaling.
+A step is one am_compute_batch call: the whole hot path (a1-a8 of SURVEY.md
+8(a)) for --batch (default 8) consecutive pivots of the seeded 1 mm path over
+the resident voxel model, one fused launch (8(f) NEXT 2).  Default workload: C3
+(head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096 orientations),
+the configuration BASELINE.json's metric is quoted on.  The one-pivot latency
+(am_compute) is reported beside it.  For N > 1 (torchrun), every rank computes
+its own pivots of the toolpath (pivot sharding): no
+data-path collective, weak scaling.
 
 value = voxel.orientation tests / s = N_vox * m * n * maps / max-over-ranks time.
 """
@@ -168,7 +170,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": _config_dict(cfg, len(H)),
+        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                          "sample": f"{cells} cells of {args.steps} maps (seeded cells, pivots of the 1 mm path), "
                                    f"every voxel per cell, fp64 clip-project-hull test with exact-safe shortcuts"},
@@ -178,13 +180,14 @@ def run_reference(args):
     return 0
 
 
-def _config_dict(cfg, N, flushed=True):
+def _config_dict(cfg, N, flushed=True, batch=1):
     return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
                         f"pivots on the {cfg.offset:g} mm path",
             "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
             "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
                    f"every timed step, outside the per-step CUDA events") if flushed else
                   f"inputs {16 * N / 1e6:.0f} MB; no flush",
+            "pivots_per_step": batch,
             "parallelism": "pivot-sharded (weak)"}
 
 
@@ -201,19 +204,26 @@ def _ncu_traffic(cfg_name, kernel):
     return None, None
 
 
-def _timed_maps(ctx, piv, out, stream, steps, flush, torch):
-    """Per-step CUDA events around each am_compute on `stream`; L2 flushed (a write larger
-    than L2) before every step when `flush` is a tensor.  Returns (sum of step ms, wall ms)."""
+def _timed_maps(ctx, piv, out, stream, steps, flush, torch, batch=1):
+    """Per-step CUDA events around each call on `stream` (batch = 1: am_compute of one
+    pivot; else am_compute_batch of `batch` consecutive pivots); L2 flushed (a write
+    larger than L2) before every step when `flush` is a tensor.  Returns (sum of the
+    step times in ms, wall ms of the whole loop including the flushes)."""
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
+    nchunk = max(1, len(piv) // batch)
     t0.record(stream)
     for k in range(steps):
         if flush is not None:
             with torch.cuda.stream(stream):
                 flush.fill_(k & 0xFF)
         evs[k][0].record(stream)
-        ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
+        if batch == 1:
+            ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
+        else:
+            c = (k % nchunk) * batch
+            ctx.compute_batch(piv[c:c + batch], out=out[c:c + batch], stream=stream)
         evs[k][1].record(stream)
     t1.record(stream)
     stream.synchronize()
@@ -235,10 +245,12 @@ def run_ours(args):
 
     cfg, C, H, gen_s = _scene(args.config)
     N = len(H)
-    npiv = args.pivots
+    bsz = args.batch
+    npiv = max(args.pivots, bsz) // bsz * bsz
     piv_all = cfg.pivots(npiv * ws)
     piv = piv_all[rank::ws]  # pivot sharding: rank r takes pivots r, r + G, ...
     ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
+    ctx.set_option(B.OPT_BATCH, bsz)
     t0 = time.time()
     ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
     torch.cuda.synchronize(dev)
@@ -246,29 +258,33 @@ def run_ours(args):
     stream = torch.cuda.Stream(dev)
     out = torch.zeros((len(piv), ctx.words), dtype=torch.int32, device=dev)
     flush = None if args.no_flush else torch.empty(2 * L2_BYTES, dtype=torch.uint8, device=dev)
-    # warm-up
-    for k in range(args.warmup):
-        ctx.compute(piv[k % len(piv)], out=out[k % len(piv)], stream=stream)
-    stream.synchronize()
+    # warm-up (both launch shapes)
+    _timed_maps(ctx, piv, out, stream, args.warmup, None, torch, bsz)
+    _timed_maps(ctx, piv, out, stream, 3, None, torch, 1)
     # per-pivot counters (outside the timed region)
     stats = [ctx.compute(p, stats=True)[1] for p in piv]
     mean = {k: float(np.mean([getattr(s_, k) for s_ in stats])) for k in stats[0].__dict__}
 
-    # ---- timed region: K maps, L2 flushed before each, CUDA events on the launching stream
+    # ---- timed region: K steps of `bsz` pivots each (one am_compute_batch call, one fused
+    #      launch), L2 flushed before each step, CUDA events on the launching stream
     ctx.set_option(B.OPT_KERNEL_TIMING, 1)
     ctx.kernel_time()
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
     with ClockSampler(dev.index) as clk:
-        ms, wall_ms = _timed_maps(ctx, piv, out, stream, args.steps, flush, torch)
+        ms, wall_ms = _timed_maps(ctx, piv, out, stream, args.steps, flush, torch, bsz)
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
     kms, klaunch = ctx.kernel_time()
-    # warm-L2 variant (back to back, no flush): detail only
-    ms_warm, _ = _timed_maps(ctx, piv, out, stream, min(args.steps, 200), None, torch)
-    ms_warm /= min(args.steps, 200)
+    # single-pivot latency (am_compute, one fused launch per map), flushed: detail
+    ks = max(1, min(args.steps, 100))
+    ms_single, _ = _timed_maps(ctx, piv, out, stream, ks, flush, torch, 1)
+    ks_k, ks_l = ctx.kernel_time()
+    # warm-L2 variant of the timed loop (no flush): detail
+    kw = max(1, min(args.steps, 200))
+    ms_warm, _ = _timed_maps(ctx, piv, out, stream, kw, None, torch, bsz)
     ctx.kernel_time()
     # ---- full-scan leg: every voxel read by filter_kernel (no brick skipping, one launch per stage)
     full = None
@@ -276,44 +292,47 @@ def run_ours(args):
         ctx.set_option(B.OPT_FUSED, 0)
         ctx.set_option(B.OPT_BRICKS, 0)
         kf = max(1, min(args.steps, 50))
-        fms, _ = _timed_maps(ctx, piv, out, stream, kf, flush, torch)
+        fms, _ = _timed_maps(ctx, piv, out, stream, kf, flush, torch, 1)
         fk, fl = ctx.kernel_time()
         ctx.set_option(B.OPT_BRICKS, 1)
         ctx.set_option(B.OPT_FUSED, 1)
         full = {"ms_per_am": fms / kf, "kernel_ms_avg": fk / max(fl, 1), "steps": kf}
     ctx.set_option(B.OPT_KERNEL_TIMING, 0)
 
-    # ---- e2e: the public API with HOST buffers (pivot in, packed AM out), synchronous per step
-    host_out = np.zeros(ctx.words, dtype=np.uint32)
+    # ---- e2e: the public API with HOST buffers (pivots in, packed AMs out), synchronous per step
+    host_piv = np.ascontiguousarray(piv, dtype=np.float32)
+    host_out = np.zeros((bsz, ctx.words), dtype=np.uint32)
+    nchunk = len(piv) // bsz
     for k in range(min(args.warmup, 3)):
-        ctx.compute(piv[k % len(piv)], out=host_out)
+        ctx.compute_batch(host_piv[(k % nchunk) * bsz:(k % nchunk + 1) * bsz], out=host_out)
     ke = max(1, min(args.steps, args.e2e_steps))
     if dist:
         dist.barrier()
     e2e_s = 0.0
-    # clocked per step so the flush stays outside
-    for k in range(ke):
+    for k in range(ke):  # clocked per step so the flush stays outside
         if flush is not None:
             with torch.cuda.stream(stream):
                 flush.fill_(k & 0xFF)
             stream.synchronize()
+        c = (k % nchunk) * bsz
         t1 = time.perf_counter()
-        ctx.compute(piv[k % len(piv)], out=host_out)
+        ctx.compute_batch(host_piv[c:c + bsz], out=host_out)
         e2e_s += time.perf_counter() - t1
     t = torch.tensor([ms, e2e_s, kms / max(klaunch, 1)], dtype=torch.float64, device=dev)
     if dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max, e2e_max, kavg_ms = t.tolist()
-    maps = args.steps * ws
+    maps = args.steps * bsz * ws
     tests_per_map = float(N) * cfg.m * cfg.n
     value = tests_per_map * maps / (ms_max / 1e3)
-    e2e_value = tests_per_map * ke * ws / e2e_max
+    e2e_value = tests_per_map * ke * bsz * ws / e2e_max
     peak, peak_src = _peaks()
-    # algorithmic bytes per AM = 16 N (one read of every leaf) + m n / 8 (AM write)
-    alg_bytes = 16.0 * N + cfg.m * cfg.n / 8.0
+    # algorithmic bytes per AM = 16 N (one read of every leaf) + m n / 8
+    # (AM write); one launch computes bsz maps
+    alg_bytes = bsz * (16.0 * N + cfg.m * cfg.n / 8.0)
     achieved = alg_bytes / (kavg_ms / 1e3) / 1e9
     # bytes the fused kernel actually needs: brick spheres, kept bricks' voxels, both map levels
-    touched = 16.0 * (ctx_nbricks(N) + mean["voxels_streamed"] + mean["level_voxels"]) + cfg.m * cfg.n / 8.0
+    touched = bsz * (16.0 * (ctx_nbricks(N) + mean["voxels_streamed"] + mean["level_voxels"]) + cfg.m * cfg.n / 8.0)
     traffic, traffic_tag = _ncu_traffic(cfg.name, "am_pipeline_kernel")
     baseline_ms = None
     if args.baseline and rank == 0:
@@ -346,29 +365,32 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N, flush is not None),
-            "ms_per_am": ms_max / args.steps,
+            "config": _config_dict(cfg, N, flush is not None, bsz),
+            "ms_per_am": ms_max / args.steps / bsz,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_tag": traffic_tag,
-                         "kernel": "am_pipeline_kernel", "kernel_ms_avg": kavg_ms,
+                         "kernel": "am_pipeline_kernel", "kernel_ms_avg": kavg_ms, "maps_per_launch": bsz,
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
                          "touched_bytes_per_launch": touched,
                          "touched_gbs": touched / (kavg_ms / 1e3) / 1e9,
-                         "note": "achieved = SURVEY 8(d) algorithmic bytes (16 N + m n / 8) / kernel time; "
-                                 "the kernel skips most of them (touched_bytes, traffic), so frac is the "
-                                 "speed relative to one full HBM pass, not bandwidth use"},
+                         "note": "achieved = SURVEY 8(d) algorithmic bytes (16 N + m n / 8 per map, maps_per_launch "
+                                 "maps) / kernel time; the kernel skips most of them (touched_bytes, traffic), so "
+                                 "frac is the speed relative to one full HBM pass per map, not bandwidth use"},
             "full_scan_roofline": full_roof,
-            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12, "d2h_bytes_per_step": 4 * ctx.words,
-                    "ms_per_am": 1e3 * e2e_max / ke, "steps": ke,
-                    "note": "am_compute with a host pivot (12 B, passed in the launch) and a host AM buffer; "
-                            "synchronous per step; voxels resident (upload excluded, PAPER.md L313); "
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12 * bsz,
+                    "d2h_bytes_per_step": 4 * ctx.words * bsz,
+                    "ms_per_am": 1e3 * e2e_max / ke / bsz, "steps": ke,
+                    "note": f"am_compute_batch with {bsz} host pivots (12 B each, copied into the launch) and a "
+                            "host AM buffer; synchronous per step; voxels resident (upload excluded, PAPER.md L313); "
                             "L2 flushed before each step, outside the per-step clock"},
             "gpu_launches": klaunch,
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
             "detail": {"stats_mean_over_pivots": mean, "upload_s": upload_s, "scene_gen_s": gen_s,
                        "pivots_per_rank": len(piv), "baseline_ms_per_am": baseline_ms,
-                       "warm_l2_ms_per_am": ms_warm, "timed_wall_ms_incl_flush": wall_ms,
+                       "single_pivot_ms_per_am": ms_single / ks,
+                       "single_pivot_kernel_ms": ks_k / max(ks_l, 1),
+                       "warm_l2_ms_per_am": ms_warm / kw / bsz, "timed_wall_ms_incl_flush": wall_ms,
                        "host_cpus": os.cpu_count(), "build": _build_id(),
                        "paper_context": "PAPER.md L32/L75: <18 ms per AM, 27M octree nodes x 4096 orientations, "
                                         "GTX 1080(Ti); 'over 23x' vs PBox"},
@@ -396,11 +418,12 @@ def _build_id():
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--config", default="C3")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--pivots", type=int, default=64, help="pivots per rank (cycled over the steps)")
+    ap.add_argument("--batch", type=int, default=8, help="pivots per step (one am_compute_batch call)")
     ap.add_argument("--e2e-steps", type=int, default=100)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--ref-seconds", type=float, default=60.0)

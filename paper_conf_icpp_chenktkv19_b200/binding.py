@@ -20,7 +20,7 @@ LIB_PATH = os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
-OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED = 6, 7, 8, 9, 10, 11
+OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

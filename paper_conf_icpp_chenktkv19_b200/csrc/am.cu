@@ -67,6 +67,8 @@ struct am_ctx {
     unsigned int nbricks = 0;
     int bricks_on = 1;
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
+    int batch = 8;                         // pivots per batched fused launch (AM_OPT_BATCH)
+    int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     int fused_grid = 0;
     size_t smem_fused = 0;
     float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
@@ -89,6 +91,8 @@ constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, ta
 constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
 constexpr int kCtrWords = kCtrBricks + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
+constexpr int kCtrBar = kCtrAll;             // group barrier of a batched launch (2 words)
+constexpr int kCtrStride = kCtrAll + 2;      // 64-bit words per slot
 constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
 constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
 
@@ -204,8 +208,39 @@ int ensure_queue(am_ctx* ctx, long long cap) {
     if (ctx->d_queue) cudaFree(ctx->d_queue);
     ctx->d_queue = nullptr;
     ctx->qcap = 0;
-    CK(cudaMalloc(&ctx->d_queue, (size_t)cap * sizeof(unsigned long long)));
+    CK(cudaMalloc(&ctx->d_queue, (size_t)ctx->slots * cap * sizeof(unsigned long long)));
     ctx->qcap = cap;
+    return AM_OK;
+}
+
+// Per-map buffers for K slots (slot s of each = the buffer of pivot s of a
+// batched launch; the single-map paths use slot 0).
+int ensure_slots(am_ctx* ctx, int K) {
+    if (ctx->slots >= K) return AM_OK;
+    const size_t ntex = (size_t)6 * ctx->cmapT * ctx->cmapT;
+    cudaFree(ctx->d_ctr);
+    cudaFree(ctx->d_queue);
+    cudaFree(ctx->d_recs);
+    cudaFree(ctx->d_tasks);
+    cudaFree(ctx->d_cmap);
+    cudaFree(ctx->d_live);
+    cudaFree(ctx->d_brick_list);
+    ctx->d_ctr = nullptr;
+    ctx->d_queue = nullptr;
+    ctx->d_recs = nullptr;
+    ctx->d_tasks = nullptr;
+    ctx->d_cmap = nullptr;
+    ctx->d_live = nullptr;
+    ctx->d_brick_list = nullptr;
+    ctx->slots = K;
+    CK(cudaMalloc(&ctx->d_ctr, (size_t)K * kCtrStride * sizeof(unsigned long long)));
+    CK(cudaMemset(ctx->d_ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long)));
+    CK(cudaMalloc(&ctx->d_queue, (size_t)K * ctx->qcap * sizeof(unsigned long long)));
+    CK(cudaMalloc(&ctx->d_recs, (size_t)K * kRecCap * sizeof(ConeRec)));
+    CK(cudaMalloc(&ctx->d_tasks, (size_t)K * kTaskCap * sizeof(unsigned long long)));
+    CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float)));
+    if (ctx->vox_cap > 0) CK(cudaMalloc(&ctx->d_live, (size_t)K * ctx->vox_cap * sizeof(unsigned int)));
+    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * ctx->nbricks * sizeof(unsigned int)));
     return AM_OK;
 }
 
@@ -230,13 +265,17 @@ int configure_launch(am_ctx* ctx) {
     ctx->smem_fused = fused_smem_bytes(m, ctx->grid.W);
     ctx->fused_grid = 0;
     if (ctx->smem_fused <= 232448 &&
-        cudaFuncSetAttribute(am_pipeline_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused) ==
-            cudaSuccess) {
-        int occf = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occf, am_pipeline_kernel, kThreads, ctx->smem_fused) ==
-                cudaSuccess &&
-            occf > 0)
-            ctx->fused_grid = occf * ctx->sms;
+        cudaFuncSetAttribute(am_pipeline_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ctx->smem_fused) == cudaSuccess &&
+        cudaFuncSetAttribute(am_pipeline_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ctx->smem_fused) == cudaSuccess) {
+        int occf = 0, occb = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occf, am_pipeline_kernel<false>, kThreads,
+                                                          ctx->smem_fused) == cudaSuccess &&
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occb, am_pipeline_kernel<true>, kThreads,
+                                                          ctx->smem_fused) == cudaSuccess &&
+            occf > 0 && occb > 0)
+            ctx->fused_grid = std::min(occf, occb) * ctx->sms;
     }
     cudaGetLastError();
     return AM_OK;
@@ -343,72 +382,101 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, int slot, cudaStream_t s)
 //   deferred band.  The coarse levels only make the filter effective; they are
 //   subsets of the model, so the map is the same with any number of them
 //   (AM_OPT_PHASES = 0, 1 or 2 levels).
+// Can the whole map run as one fused cooperative launch?
+bool fused_ok(const am_ctx* ctx) {
+    return ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases == 2 && ctx->n_l0 > 0 &&
+           ctx->bricks_on && ctx->d_bricks && ctx->N > 0;
+}
+
+// K maps (pivots[3K], K <= ctx->slots) into gam0 + k * MW with one fused
+// launch: am_pipeline_kernel<false> for K = 1, <true> (one CTA group per
+// pivot) otherwise.  Zeroes the maps and the K counter slots first.
+int launch_fused(am_ctx* ctx, const float* pivots, int K, uint32_t* gam0, cudaStream_t s) {
+    CK(cudaMemsetAsync(gam0, 0, (size_t)K * ctx->MW * sizeof(uint32_t), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long), s));
+    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+    FusedParams F{};
+    F.main = make_params(ctx, pivots, gam0);
+    F.main.vox = ctx->d_vox;
+    F.main.N = ctx->N;
+    F.main.cmap = ctx->d_cmap;
+    F.main.bricks = ctx->d_bricks;
+    F.main.nbricks = ctx->nbricks;
+    F.main.brick_list = ctx->d_brick_list;
+    F.main.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
+    F.main.recs = ctx->d_recs;
+    F.main.tasks = ctx->d_tasks;
+    F.main.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 4);
+    F.main.task_count = ctx->d_ctr + kCtrRT + 5;
+    F.main.rec_cap = kRecCap;
+    F.main.task_cap = kTaskCap;
+    F.main.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
+    F.main.live_idx = ctx->d_live;
+    F.lvl = F.main;
+    F.lvl.vox = ctx->d_coarse;
+    F.lvl.N = ctx->n_l0;
+    F.lvl.cmap = ctx->d_cmap_ones;
+    F.lvl.stats = ctx->d_ctr + kCtrWords;
+    F.lvl.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT);
+    F.lvl.task_count = ctx->d_ctr + kCtrRT + 1;
+    F.lvl.rec_cap = kRecCap / 2;
+    F.lvl.task_cap = kTaskCap / 2;
+    F.l1 = ctx->d_coarse + ctx->n_l0;
+    F.n0 = (unsigned int)ctx->n_l0;
+    F.n1 = (unsigned int)(ctx->n_l1 - ctx->n_l0);
+    F.rec1 = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2);
+    F.task1 = ctx->d_ctr + kCtrRT + 3;
+    F.live1 = nullptr;
+    F.texels = ctx->d_texels;
+    F.ntex = ntex;
+    F.use_l1 = 1;
+    F.ts = (ctx->diag_ts && ctx->d_ts && K == 1) ? ctx->d_ts : nullptr;
+    F.nslot = K;
+    for (int k = 0; k < K; ++k) {
+        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
+        F.piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    }
+    F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
+    F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
+    F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
+    F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
+    F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
+    F.cmap_stride = (unsigned long long)ntex * sizeof(float);
+    F.blist_stride = (unsigned long long)ctx->nbricks * sizeof(unsigned int);
+    F.gam_stride = (unsigned long long)ctx->MW * sizeof(uint32_t);
+    F.bar = ctx->d_ctr + kCtrBar;
+    const bool timed = ctx->timing != 0;
+    if (timed) {
+        if (ctx->ev_used == ctx->ev_start.size()) {
+            cudaEvent_t a, b;
+            CK(cudaEventCreate(&a));
+            CK(cudaEventCreate(&b));
+            ctx->ev_start.push_back(a);
+            ctx->ev_stop.push_back(b);
+        }
+        CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
+    }
+    void* args[] = {&F};
+    if (K == 1)
+        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads),
+                                       args, ctx->smem_fused, s));
+    else
+        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<true>, dim3(ctx->fused_grid), dim3(kThreads),
+                                       args, ctx->smem_fused, s));
+    if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    if (ctx->d_prev && K == 1)
+        CK(cudaMemcpyAsync(ctx->d_prev, gam0, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    return AM_OK;
+}
+
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
+    if (fused_ok(ctx)) return launch_fused(ctx, pivot, 1, gam, s);
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
-    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrAll * sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrStride * sizeof(unsigned long long), s));
     if (ctx->N == 0) return AM_OK;
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
     const float* cm = ctx->d_cmap_ones;
-    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
-    if (ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases == 2 && ctx->n_l0 > 0 && ctx->bricks_on &&
-        ctx->d_bricks && ntex <= 4 * ctx->fused_grid * kThreads) {
-        // the whole map in one cooperative launch (fused.cuh)
-        FusedParams F;
-        F.main = p;
-        F.main.vox = ctx->d_vox;
-        F.main.N = ctx->N;
-        F.main.cmap = ctx->d_cmap;
-        F.main.bricks = ctx->d_bricks;
-        F.main.nbricks = ctx->nbricks;
-        F.main.brick_list = ctx->d_brick_list;
-        F.main.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
-        F.main.recs = ctx->d_recs;
-        F.main.tasks = ctx->d_tasks;
-        F.main.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 4);
-        F.main.task_count = ctx->d_ctr + kCtrRT + 5;
-        F.main.rec_cap = kRecCap;
-        F.main.task_cap = kTaskCap;
-        F.main.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
-        F.main.live_idx = ctx->d_live;
-        F.lvl = F.main;
-        F.lvl.vox = ctx->d_coarse;
-        F.lvl.N = ctx->n_l0;
-        F.lvl.cmap = ctx->d_cmap_ones;
-        F.lvl.stats = ctx->d_ctr + kCtrWords;
-        F.lvl.rec_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT);
-        F.lvl.task_count = ctx->d_ctr + kCtrRT + 1;
-        F.lvl.rec_cap = kRecCap / 2;
-        F.lvl.task_cap = kTaskCap / 2;
-        F.l1 = ctx->d_coarse + ctx->n_l0;
-        F.n0 = (unsigned int)ctx->n_l0;
-        F.n1 = (unsigned int)(ctx->n_l1 - ctx->n_l0);
-        F.rec1 = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2);
-        F.task1 = ctx->d_ctr + kCtrRT + 3;
-        F.live1 = nullptr;
-        F.texels = ctx->d_texels;
-        F.ntex = ntex;
-        F.use_l1 = 1;
-        F.ts = (ctx->diag_ts && ctx->d_ts) ? ctx->d_ts : nullptr;
-        const bool timed = ctx->timing != 0;
-        if (timed) {
-            if (ctx->ev_used == ctx->ev_start.size()) {
-                cudaEvent_t a, b;
-                CK(cudaEventCreate(&a));
-                CK(cudaEventCreate(&b));
-                ctx->ev_start.push_back(a);
-                ctx->ev_stop.push_back(b);
-            }
-            CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
-        }
-        void* args[] = {&F};
-        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel, dim3(ctx->fused_grid), dim3(kThreads), args,
-                                       ctx->smem_fused, s));
-        if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
-        if (ctx->d_prev)
-            CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
-        return AM_OK;
-    }
     if (ctx->diag & 2) {
         // diagnostic: clear map from the previous map computed on this context
         // (exact only when the previous call used the same pivot)
@@ -547,7 +615,7 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
     };
     if (cudaMalloc(&ctx->d_tab, tab.size() * sizeof(float)) != cudaSuccess ||
         cudaMemcpy(ctx->d_tab, tab.data(), tab.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMalloc(&ctx->d_ctr, kCtrAll * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMalloc(&ctx->d_ctr, kCtrStride * sizeof(unsigned long long)) != cudaSuccess ||
         cudaMalloc(&ctx->d_am, (size_t)ctx->MW * sizeof(uint32_t)) != cudaSuccess) {
         cudaGetLastError();
         return bail(AM_ENOMEM);
@@ -647,7 +715,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
         ctx->d_live = nullptr;
         ctx->vox_cap = 0;
         UK(cudaMalloc(&ctx->d_vox, (size_t)N * sizeof(float4)));
-        UK(cudaMalloc(&ctx->d_live, (size_t)N * sizeof(unsigned int)));
+        UK(cudaMalloc(&ctx->d_live, (size_t)ctx->slots * N * sizeof(unsigned int)));
         ctx->vox_cap = N;
     }
     UK(cudaMalloc(&raw, (size_t)N * sizeof(float4)));
@@ -698,7 +766,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     ctx->d_brick_list = nullptr;
     ctx->nbricks = (unsigned int)((N + kThreads - 1) / kThreads);
     UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
-    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->nbricks * sizeof(unsigned int)));
+    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * ctx->nbricks * sizeof(unsigned int)));
     brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
                                                                                         ctx->nbricks);
     UK(cudaGetLastError());
@@ -824,8 +892,18 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
         dst = ctx->d_am;
     }
     int rc;
-    for (int64_t k = 0; k < P; ++k)
-        if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
+    const int K = (int)std::min<int64_t>(P, ctx->batch);
+    if (K > 1 && fused_ok(ctx)) {
+        // batched fused launches of up to K pivots each (8(f) NEXT 2)
+        if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
+        for (int64_t k = 0; k < P; k += K) {
+            const int kk = (int)std::min<int64_t>(K, P - k);
+            if ((rc = launch_fused(ctx, pivots + 3 * k, kk, dst + k * ctx->MW, s)) != AM_OK) return rc;
+        }
+    } else {
+        for (int64_t k = 0; k < P; ++k)
+            if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
+    }
     if (!dst_is_device) {
         CK(cudaMemcpyAsync(am_out, dst, (size_t)P * ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
@@ -912,6 +990,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "fused must be 0 or 1");
         ctx->fused = (int)value;
         return AM_OK;
+    case AM_OPT_BATCH:
+        if (value < 1 || value > kMaxSlots) return fail(ctx, AM_EINVAL, "batch must be in [1, %d]", kMaxSlots);
+        ctx->batch = (int)value;
+        return AM_OK;
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
         {
@@ -924,7 +1006,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
             ctx->d_cmap = ctx->d_cmap_ones = nullptr;
             CK(cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)));
             CK(cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
-            CK(cudaMalloc(&ctx->d_cmap, ones.size() * sizeof(float)));
+            CK(cudaMalloc(&ctx->d_cmap, (size_t)ctx->slots * ones.size() * sizeof(float)));
             CK(cudaMalloc(&ctx->d_cmap_ones, ones.size() * sizeof(float)));
             CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice));
             ctx->cmapT = (int)value;

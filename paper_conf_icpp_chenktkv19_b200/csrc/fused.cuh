@@ -21,12 +21,23 @@
 //
 // Every phase uses the same device functions as the multi-kernel path, so the
 // two produce the same map bit for bit (tests).
+//
+// Batched pivots: one map is a chain of ~10 short,
+// latency-bound phases, so a single map leaves most of the GPU idle between
+// barriers.  am_pipeline_kernel<true> splits the co-resident CTAs into one
+// group per pivot; each group runs the same phases for its pivot, with its own
+// barrier and its own slot of every per-map buffer, so K maps share the GPU
+// and the barrier latency of one.
 #pragma once
 #include <cooperative_groups.h>
+
+#include <type_traits>
 
 #include "stream.cuh"
 
 namespace am {
+
+constexpr int kMaxSlots = 16;  // pivots per batched launch
 
 struct FusedParams {
     StreamParams main;        // full stream: vox, bricks, cmap (written in phase 3/6), stage-2 counters
@@ -40,7 +51,64 @@ struct FusedParams {
     int ntex;
     int use_l1;
     unsigned long long* ts;   // diagnostics: %globaltimer after each phase (CTA 0), or nullptr
+    // batched launch (am_pipeline_kernel<true>): the CTAs form nslot groups; group s
+    // computes the map of pivot s with slot s of every per-map buffer, i.e. the
+    // slot-0 pointers above advanced by s strides (bytes).
+    int nslot;
+    float4 piv[kMaxSlots];    // pivot xyz, w = may_cull
+    unsigned long long ctr_stride, q_stride, rec_stride, task_stride, live_stride, cmap_stride, blist_stride,
+        gam_stride;
+    unsigned long long* bar;  // slot 0's group barrier: [arrivals, generation] (zeroed with the counters)
 };
+
+template <typename T>
+__device__ __forceinline__ T* shift_bytes(T* p, unsigned long long b) {
+    return p ? reinterpret_cast<T*>(reinterpret_cast<char*>(const_cast<typename std::remove_const<T>::type*>(p)) + b)
+             : p;
+}
+
+// The slot-s copy of a StreamParams (pivot and per-map buffers of slot s).
+__device__ void slot_params(StreamParams& p, const FusedParams& F, int s, bool own_cmap) {
+    const unsigned long long c = s * F.ctr_stride;
+    p.px = F.piv[s].x;
+    p.py = F.piv[s].y;
+    p.pz = F.piv[s].z;
+    p.may_cull = F.piv[s].w != 0.f;
+    p.gam = shift_bytes(p.gam, s * F.gam_stride);
+    p.qcount = shift_bytes(p.qcount, c);
+    p.stats = shift_bytes(p.stats, c);
+    p.live_count = shift_bytes(p.live_count, c);
+    p.rec_count = shift_bytes(p.rec_count, c);
+    p.task_count = shift_bytes(p.task_count, c);
+    p.brick_count = shift_bytes(p.brick_count, c);
+    p.queue = shift_bytes(p.queue, s * F.q_stride);
+    p.live_idx = shift_bytes(p.live_idx, s * F.live_stride);
+    p.recs = shift_bytes(p.recs, s * F.rec_stride);
+    p.tasks = shift_bytes(p.tasks, s * F.task_stride);
+    p.brick_list = shift_bytes(p.brick_list, s * F.blist_stride);
+    if (own_cmap) p.cmap = shift_bytes(p.cmap, s * F.cmap_stride);
+}
+
+// Barrier over the nb CTAs of one group (all co-resident: cooperative launch).
+// bar[0] counts arrivals, bar[1] is the generation; the last arrival resets the
+// count and advances the generation.
+__device__ __forceinline__ void group_sync(unsigned long long* bar, unsigned int nb) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        volatile unsigned long long* gen = bar + 1;
+        const unsigned long long g0 = *gen;
+        __threadfence();
+        if (atomicAdd(bar, 1ull) == nb - 1) {
+            atomicExch(bar, 0ull);
+            __threadfence();
+            atomicAdd(bar + 1, 1ull);
+        } else {
+            while (*gen == g0) __nanosleep(20);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
 
 __device__ __forceinline__ void fused_mark(const FusedParams& F, int k) {
     if (F.ts && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -94,11 +162,11 @@ __device__ void fused_flush(const StreamParams& p, const uint32_t* sAM) {
 // Rasterise the tasks of one stage (grid-stride), into the shared AM.
 template <bool COARSE>
 __device__ void fused_rows(const StreamParams& p, const unsigned long long* task_count, uint32_t* sAM,
-                           const uint32_t* sRowFull, Counters cnt) {
+                           const uint32_t* sRowFull, Counters cnt, unsigned int gb, unsigned int gn) {
     const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(task_count), p.task_cap);
     unsigned int rows = 0;
-    for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
-         k += (unsigned long long)gridDim.x * blockDim.x) {
+    for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
+         k += (unsigned long long)gn * blockDim.x) {
         const unsigned long long t = p.tasks[k];
         const ConeRec r = p.recs[t >> 16];
         if (r.i0 < 0) continue;
@@ -110,63 +178,67 @@ __device__ void fused_rows(const StreamParams& p, const unsigned long long* task
     if (rows && cnt.c) atomicAdd(cnt.c + CT_ROWS, rows);
 }
 
-// Phases 3/6: the clear-direction map from the global AM.
+// Phases 3/6: the clear-direction map from the global AM.  The gn CTAs of the
+// group cover the texels kMaxT per thread per pass.
 __device__ void fused_clear_map(const StreamParams& p, const float4* texels, int ntex, float* V, uint32_t* sAM,
-                                float4* sDirs, int* sN) {
+                                float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
     const GridDev& g = p.grid;
     const int MW = g.m * g.W;
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
-    constexpr int kMaxT = 4;  // texels per thread (ntex <= 4 * grid * block, checked by the host)
-    float best[kMaxT];
-    float4 c[kMaxT];
+    constexpr int kMaxT = 4;  // texels per thread per pass
+    const int per_pass = kMaxT * gn * blockDim.x;
+    for (int t0 = 0; t0 < ntex; t0 += per_pass) {
+        float best[kMaxT];
+        float4 c[kMaxT];
 #pragma unroll
-    for (int j = 0; j < kMaxT; ++j) {
-        best[j] = -2.f;
-        const int t = (j * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
-        c[j] = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
-    }
-    int w0 = 0;
-    while (true) {
-        __syncthreads();
-        if (threadIdx.x == 0) *sN = 0;
-        __syncthreads();
-        // compact the clear cells of the next words (at most kFusedDirs per round)
-        const int wend = min(MW, w0 + kFusedDirs / 32);
-        for (int w = w0 + threadIdx.x; w < wend; w += blockDim.x) {
-            const int i = w / g.W, wj = w - i * g.W;
-            uint32_t clear = ~sAM[w] & row_word_mask(wj, g.n);
-            if (!clear) continue;
-            int pos = atomicAdd(sN, __popc(clear));
-            const float cph = __ldg(p.tab + i), sph = __ldg(p.tab + g.m + i);
-            while (clear) {
-                const int j = (wj << 5) + __ffs(clear) - 1;
-                clear &= clear - 1u;
-                sDirs[pos++] = make_float4(sph * __ldg(p.tab + 2 * g.m + j), sph * __ldg(p.tab + 2 * g.m + g.n + j),
-                                           cph, 0.f);
+        for (int j = 0; j < kMaxT; ++j) {
+            best[j] = -2.f;
+            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
+            c[j] = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
+        }
+        int w0 = 0;
+        while (true) {
+            __syncthreads();
+            if (threadIdx.x == 0) *sN = 0;
+            __syncthreads();
+            // compact the clear cells of the next words (at most kFusedDirs per round)
+            const int wend = min(MW, w0 + kFusedDirs / 32);
+            for (int w = w0 + threadIdx.x; w < wend; w += blockDim.x) {
+                const int i = w / g.W, wj = w - i * g.W;
+                uint32_t clear = ~sAM[w] & row_word_mask(wj, g.n);
+                if (!clear) continue;
+                int pos = atomicAdd(sN, __popc(clear));
+                const float cph = __ldg(p.tab + i), sph = __ldg(p.tab + g.m + i);
+                while (clear) {
+                    const int j = (wj << 5) + __ffs(clear) - 1;
+                    clear &= clear - 1u;
+                    sDirs[pos++] = make_float4(sph * __ldg(p.tab + 2 * g.m + j),
+                                               sph * __ldg(p.tab + 2 * g.m + g.n + j), cph, 0.f);
+                }
             }
-        }
-        __syncthreads();
-        const int k = *sN;
-        for (int e = 0; e < k; ++e) {
-            const float4 d = sDirs[e];
+            __syncthreads();
+            const int k = *sN;
+            for (int e = 0; e < k; ++e) {
+                const float4 d = sDirs[e];
 #pragma unroll
-            for (int j = 0; j < kMaxT; ++j)
-                best[j] = fmaxf(best[j], fmaf(c[j].x, d.x, fmaf(c[j].y, d.y, c[j].z * d.z)));
+                for (int j = 0; j < kMaxT; ++j)
+                    best[j] = fmaxf(best[j], fmaf(c[j].x, d.x, fmaf(c[j].y, d.y, c[j].z * d.z)));
+            }
+            w0 = wend;
+            if (w0 >= MW) break;
         }
-        w0 = wend;
-        if (w0 >= MW) break;
-    }
 #pragma unroll
-    for (int j = 0; j < kMaxT; ++j) {
-        const int t = (j * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
-        if (t >= ntex) continue;
-        float u = -2.f;
-        if (best[j] >= -1.5f) {
-            const float th = acosf(fminf(best[j] + 2e-6f, 1.f));
-            const float r = c[j].w;
-            u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+        for (int j = 0; j < kMaxT; ++j) {
+            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
+            if (t >= ntex) continue;
+            float u = -2.f;
+            if (best[j] >= -1.5f) {
+                const float th = acosf(fminf(best[j] + 2e-6f, 1.f));
+                const float r = c[j].w;
+                u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+            }
+            V[t] = u * fabsf(u);
         }
-        V[t] = u * fabsf(u);
     }
 }
 
@@ -242,23 +314,55 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
     }
 }
 
+// BATCH = false: one map, the whole grid, cooperative-groups grid barriers.
+// BATCH = true: F.nslot maps at once; contiguous CTA ranges form one group per
+// pivot, each with its own slot of the per-map buffers and its own barrier.
+template <bool BATCH>
 __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_constant__ FusedParams F) {
     namespace cg = cooperative_groups;
-    cg::grid_group grid = cg::this_grid();
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ unsigned int sCnt[CT_COUNT];
     __shared__ int sN;
     __shared__ unsigned int sCulled, sPassed;
     __shared__ unsigned long long sStreamed;
     __shared__ FusedScratch sc;
-    const StreamParams& P = F.main;
-    const StreamParams& L = F.lvl;
+    __shared__ StreamParams sP, sL;
+    __shared__ unsigned int* sRec1;
+    __shared__ unsigned long long* sTask1;
+    // group of this CTA: CTAs [start(s), start(s + 1)), start(s) = s * G / nslot
+    const unsigned int G = gridDim.x;
+    const unsigned int K = BATCH ? (unsigned int)F.nslot : 1u;
+    const unsigned int slot = BATCH ? (unsigned int)(((blockIdx.x + 1ull) * K - 1ull) / G) : 0u;
+    const unsigned int gstart = BATCH ? (unsigned int)((unsigned long long)slot * G / K) : 0u;
+    const unsigned int gb = blockIdx.x - gstart;
+    const unsigned int gn = BATCH ? (unsigned int)((unsigned long long)(slot + 1) * G / K) - gstart : G;
+    unsigned long long* bar = BATCH ? shift_bytes(F.bar, slot * F.ctr_stride) : nullptr;
+    if (BATCH) {
+        if (threadIdx.x == 0) {
+            sP = F.main;
+            sL = F.lvl;
+            slot_params(sP, F, (int)slot, true);
+            slot_params(sL, F, (int)slot, false);
+            sRec1 = shift_bytes(F.rec1, slot * F.ctr_stride);
+            sTask1 = shift_bytes(F.task1, slot * F.ctr_stride);
+        }
+        __syncthreads();
+    }
+    auto gsync = [&]() {
+        if (BATCH)
+            group_sync(bar, gn);
+        else
+            cg::this_grid().sync();
+    };
+    const StreamParams& P = *(BATCH ? &sP : &F.main);
+    const StreamParams& L = *(BATCH ? &sL : &F.lvl);
+    unsigned int* const rec1 = BATCH ? sRec1 : F.rec1;
+    unsigned long long* const task1 = BATCH ? sTask1 : F.task1;
     const int m = P.grid.m, MW = m * P.grid.W;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
     uint32_t* sRowFull = sAM + MW;
     float4* sDirs = fused_dirs(sAM, MW, m);
-    const int lane = threadIdx.x & 31;
-    const unsigned long long gstride = (unsigned long long)gridDim.x * blockDim.x;
+    const unsigned long long gstride = (unsigned long long)gn * blockDim.x;
     if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
     if (threadIdx.x == 0) {
         sCulled = sPassed = 0u;
@@ -270,7 +374,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     fused_mark(F, 0);
 
     // 1. level-0 cones (inner), every voxel of the level is live (CTA-uniform loop)
-    for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < F.n0; b0 += gstride) {
+    for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < F.n0; b0 += gstride) {
         const unsigned long long e = b0 + threadIdx.x;
         int nrows = 0;
         bool counted = false;
@@ -279,25 +383,25 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         emit_cones_cta<true>(L, L.rec_count, L.task_count, 0u, 0ull, L.rec_cap, L.task_cap, nrows, r, counted, &sc,
                              nullptr, sRowFull);
     }
-    grid.sync();
+    gsync();
     fused_mark(F, 1);
     // 2. level-0 rows
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = 0u;
     for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
     __syncthreads();
-    fused_rows<true>(L, L.task_count, sAM, sRowFull, none);
+    fused_rows<true>(L, L.task_count, sAM, sRowFull, none, gb, gn);
     fused_flush(L, sAM);
-    grid.sync();
+    gsync();
     fused_mark(F, 2);
     // 3. clear-direction map
-    fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
-    grid.sync();
+    fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN, gb, gn);
+    gsync();
     fused_mark(F, 3);
     if (F.use_l1) {
         // 4. level-1 voxels: filter against the map, inner cones (stage 1: upper
         //    halves of the record / task buffers; the records index the level-1 array)
         fused_seed(P, sAM, sRowFull);
-        for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < F.n1; b0 += gstride) {
+        for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < F.n1; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
             int nrows = 0;
             bool counted = false;
@@ -306,17 +410,17 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                 const float4 q = F.l1[e];
                 if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
             }
-            emit_cones_cta<true>(P, F.rec1, F.task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
+            emit_cones_cta<true>(P, rec1, task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
                                  counted, &sc, nullptr, sRowFull);
         }
-        grid.sync();
+        gsync();
         fused_mark(F, 4);
         // 5. level-1 rows (tasks in the upper halves)
         fused_seed(P, sAM, sRowFull);
         {
             const unsigned long long ntask =
-                min(*reinterpret_cast<const volatile unsigned long long*>(F.task1), P.task_cap / 2);
-            for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
+                min(*reinterpret_cast<const volatile unsigned long long*>(task1), P.task_cap / 2);
+            for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
                  k += gstride) {
                 const unsigned long long t = P.tasks[P.task_cap / 2 + k];
                 const ConeRec r = P.recs[t >> 16];
@@ -327,17 +431,17 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
             }
         }
         fused_flush(P, sAM);
-        grid.sync();
+        gsync();
         fused_mark(F, 5);
         // 6. clear-direction map again
-        fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN);
-        grid.sync();
+        fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN, gb, gn);
+        gsync();
         fused_mark(F, 6);
     }
     // 7. brick test
     {
         const unsigned int nb = P.nbricks;
-        for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
+        for (unsigned int b0 = gb * kThreads; b0 < nb; b0 += gn * kThreads) {
             const unsigned int b = b0 + threadIdx.x;
             bool keep = false;
             if (b < nb) {
@@ -348,7 +452,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
             if (keep) P.brick_list[pos] = b;
         }
     }
-    grid.sync();
+    gsync();
     fused_mark(F, 7);
     // 8a. kept bricks: filter (kVPT bricks per CTA step); live voxels go to the
     //     global live list with one atomic per CTA step
@@ -356,7 +460,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         unsigned int nculled = 0, npassed = 0;
         unsigned long long streamed = 0;
         const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
-        for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
+        for (unsigned int k0 = gb * kVPT; k0 < nk; k0 += gn * kVPT) {
             float4 q[kVPT];
             unsigned int idx[kVPT];
             bool ok[kVPT];
@@ -388,12 +492,12 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         if (streamed) atomicAdd(&sStreamed, streamed);
     }
     fused_seed(P, sAM, sRowFull);  // row-full bits of the global AM (unchanged until phase 9)
-    grid.sync();
+    gsync();
     fused_mark(F, 10);
     // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2)
     {
         const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
-        for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
+        for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
             int nrows = 0;
             bool counted = false;
@@ -406,20 +510,20 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                                   &sc, P.stats + ST_LIVE, sRowFull);
         }
     }
-    grid.sync();
+    gsync();
     fused_mark(F, 8);
     // 9. rows of the full stream (both cones, band pairs queued)
     fused_seed(P, sAM, sRowFull);
-    fused_rows<false>(P, P.task_count, sAM, sRowFull, Counters{sCnt});
+    fused_rows<false>(P, P.task_count, sAM, sRowFull, Counters{sCnt}, gb, gn);
     fused_flush(P, sAM);
-    grid.sync();
+    gsync();
     fused_mark(F, 9);
     // 10. band: exact test where the bit is still clear
     {
         const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
         const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
         unsigned long long tests = 0, hits = 0;
-        for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += gstride) {
+        for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += gstride) {
             const unsigned long long e = P.queue[k];
             const unsigned int vidx = (unsigned int)(e >> 32);
             const int cell = (int)(e & 0xffffffffu);

@@ -248,6 +248,10 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     ctx.set_option(am.binding.OPT_PHASES, 1)
     assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_BRICKS, 1)
+    ctx.set_option(am.binding.OPT_BATCH, 1)  # one fused launch per pivot
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_BATCH, 2)  # groups of 2 + a single
+    assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
@@ -255,22 +259,51 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     ctx.close()
 
 
+@pytest.mark.parametrize("batch", [16, 5, 3])
+def test_batched_launch_matches_single_maps(am, batch):
+    """Batched fused launches (one CTA group per pivot, per-slot buffers, group
+    barriers) give the maps of one-pivot launches bit for bit, including a ragged
+    last group and more pivots than groups."""
+    cfg = scenes.CONFIGS["C2"]
+    C, H = cfg.leaves()
+    P = cfg.pivots(11)
+    ctx = _ctx(am, cfg, C, H)
+    single = np.stack([ctx.compute(p)[0] for p in P])
+    ctx.set_option(am.binding.OPT_BATCH, batch)
+    assert np.array_equal(ctx.compute_batch(P), single)
+    assert np.array_equal(ctx.compute_batch(P[::-1]), single[::-1])  # slots see other pivots
+    ctx.close()
+
+
+def _check_sampled(cfg, C, H, p, g, rng, nclear=64, nblocked=32):
+    clear = np.nonzero(g == 0)[0]
+    blocked = np.nonzero(g == 1)[0]
+    assert len(clear) > 0 and len(blocked) > 0
+    cells = np.concatenate([rng.choice(clear, size=min(nclear, len(clear)), replace=False),
+                            rng.choice(blocked, size=min(nblocked, len(blocked)), replace=False)])
+    S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n, cells=cells)
+    robust = S != 1
+    assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
+
+
 def test_c3_bench_config_sampled(am):
-    """C3 (~27M leaves) in the launch configuration bench.py times: every
-    GPU-clear cell (up to 64) and a seeded sample of blocked cells against the
-    oracle, one by one."""
+    """C3 (~27M leaves) in the launch configuration bench.py times (a batch of
+    8 pivots in one fused launch): every batched map equals its one-pivot map,
+    and every GPU-clear cell (up to 64) plus a seeded sample of blocked cells of
+    two of them match the oracle, one by one."""
+    import torch
     cfg = scenes.CONFIGS["C3"]
     C, H = cfg.leaves()
     ctx = _ctx(am, cfg, C, H)
     rng = np.random.default_rng(3)
-    p = cfg.pivots(1)[0]
-    g = ctx.am(p).reshape(-1)
-    clear = np.nonzero(g == 0)[0]
-    blocked = np.nonzero(g == 1)[0]
-    assert len(clear) > 0 and len(blocked) > 0
-    cells = np.concatenate([rng.choice(clear, size=min(64, len(clear)), replace=False),
-                            rng.choice(blocked, size=min(32, len(blocked)), replace=False)])
-    S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n, cells=cells)
-    robust = S != 1
-    assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
+    P = cfg.pivots(8)
+    out = torch.zeros((8, ctx.words), dtype=torch.int32, device="cuda:0")
+    ctx.compute_batch(P, out=out)
+    torch.cuda.synchronize()
+    batch = out.cpu().numpy().view(np.uint32)
+    for k in range(8):
+        assert np.array_equal(batch[k], ctx.compute(P[k])[0]), k
+    for k in (0, 5):
+        g = am.unpack(batch[k], cfg.m, cfg.n).reshape(-1)
+        _check_sampled(cfg, C, H, P[k], g, rng)
     ctx.close()
