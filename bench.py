@@ -3,8 +3,9 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl ours|reference]
 
 A step is one am_compute_batch call: the whole hot path (a1-a8 of SURVEY.md
-8(a)) for --batch (default 8) consecutive pivots of the seeded 1 mm path over
-the resident voxel model, one fused launch (8(f) NEXT 2).  Default workload: C3
+8(a)) for --batch (default 64) consecutive pivots of the seeded 1 mm path over
+the resident voxel model, in one fused launch whose --groups (default 16) CTA
+groups take the pivots from a device queue (8(f) NEXT 2).  Default workload: C3
 (head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096 orientations),
 the configuration BASELINE.json's metric is quoted on.  The one-pivot latency
 (am_compute) is reported beside it.  For N > 1 (torchrun), every rank computes
@@ -170,7 +171,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch),
+        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch, args.groups),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                          "sample": f"{cells} cells of {args.steps} maps (seeded cells, pivots of the 1 mm path), "
                                    f"every voxel per cell, fp64 clip-project-hull test with exact-safe shortcuts"},
@@ -180,14 +181,14 @@ def run_reference(args):
     return 0
 
 
-def _config_dict(cfg, N, flushed=True, batch=1):
+def _config_dict(cfg, N, flushed=True, batch=1, groups=1):
     return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
                         f"pivots on the {cfg.offset:g} mm path",
             "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
             "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
                    f"every timed step, outside the per-step CUDA events") if flushed else
                   f"inputs {16 * N / 1e6:.0f} MB; no flush",
-            "pivots_per_step": batch,
+            "pivots_per_step": batch, "concurrent_maps": groups,
             "parallelism": "pivot-sharded (weak)"}
 
 
@@ -250,7 +251,7 @@ def run_ours(args):
     piv_all = cfg.pivots(npiv * ws)
     piv = piv_all[rank::ws]  # pivot sharding: rank r takes pivots r, r + G, ...
     ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
-    ctx.set_option(B.OPT_BATCH, bsz)
+    ctx.set_option(B.OPT_BATCH, args.groups)
     t0 = time.time()
     ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
     torch.cuda.synchronize(dev)
@@ -365,7 +366,7 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N, flush is not None, bsz),
+            "config": _config_dict(cfg, N, flush is not None, bsz, args.groups),
             "ms_per_am": ms_max / args.steps / bsz,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_tag": traffic_tag,
@@ -423,7 +424,9 @@ def main():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--pivots", type=int, default=64, help="pivots per rank (cycled over the steps)")
-    ap.add_argument("--batch", type=int, default=8, help="pivots per step (one am_compute_batch call)")
+    ap.add_argument("--batch", type=int, default=64, help="pivots per step (one am_compute_batch call)")
+    ap.add_argument("--groups", type=int, default=16,
+                    help="AM_OPT_BATCH: maps computed concurrently by the batched launch (CTA groups)")
     ap.add_argument("--e2e-steps", type=int, default=100)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--ref-seconds", type=float, default=60.0)

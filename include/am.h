@@ -94,7 +94,7 @@ enum {
     AM_OPT_BRICKS = 10,          /* 1 = skip whole 256-voxel bricks whose bounding sphere reaches
                                     no clear cell (default); 0 = read every voxel.  Same map     */
     AM_OPT_FUSED = 11,           /* 1 = the whole map in one persistent cooperative launch when
-                                    phases = 2 and bricks = 1 (default); 0 = one launch per
+                                    phases >= 1 and bricks = 1 (default); 0 = one launch per
                                     stage.  Same map                                            */
     AM_OPT_BATCH = 12            /* am_compute_batch: pivots computed concurrently by one fused
                                     launch (1..16, default 8; each needs its own set of per-map

@@ -45,7 +45,7 @@ struct am_ctx {
     int refresh_tiles = 8;
     int morton = 1;
     int baseline_reject = 0;
-    size_t smem = 0, smem_coarse = 0;
+    size_t smem = 0, smem_coarse = 0, smem_cmap = 0;
     int occ = 0;
     // coarse levels (largest voxels + a strided sample) and the clear-direction map
     float4* d_coarse = nullptr;
@@ -69,9 +69,12 @@ struct am_ctx {
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
     int batch = 8;                         // pivots per batched fused launch (AM_OPT_BATCH)
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
+    float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
+    long long piv_cap = 0;
+    std::vector<float4> h_piv;
+    unsigned long long* d_bctl = nullptr;  // batched launch: group barriers, pivot queue
     int fused_grid = 0;
     size_t smem_fused = 0;
-    float4* d_dirs = nullptr;              // clear-cell directions (m * n), clear_list_kernel
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
     int timing = 0;
@@ -91,8 +94,8 @@ constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, ta
 constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
 constexpr int kCtrWords = kCtrBricks + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
-constexpr int kCtrBar = kCtrAll;             // group barrier of a batched launch (2 words)
-constexpr int kCtrStride = kCtrAll + 2;      // 64-bit words per slot
+constexpr int kCtrStride = kCtrAll;          // 64-bit words per slot
+constexpr int kBctlWords = 2 * kMaxSlots + 1 + kMaxSlots / 2;  // bars, then queue head + per-group pivot (u32)
 constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
 constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
 
@@ -253,6 +256,8 @@ int configure_launch(am_ctx* ctx) {
                     ctx->grid.n, ctx->smem);
     CK(cudaFuncSetAttribute(row_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
     CK(cudaFuncSetAttribute(row_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem));
+    ctx->smem_cmap = clear_map_smem_bytes(ctx->MW);
+    CK(cudaFuncSetAttribute(clear_map_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_cmap));
     int occ = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, filter_kernel, kThreads, 0);
     if (e != cudaSuccess || occ < 1) {
@@ -364,13 +369,12 @@ int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     return launch_cones_rows(ctx, p, true, stage, s);
 }
 
-// Clear-direction map from `gam`; `slot` picks a zeroed counter of d_ctr.
-int launch_clear_map(am_ctx* ctx, const uint32_t* gam, int slot, cudaStream_t s) {
+// Clear-direction map from `gam` into d_cmap (slot 0).
+int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
-    unsigned int* n = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrClear + slot);
-    clear_list_kernel<<<1, 1024, 0, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_dirs, n);
-    CK(cudaGetLastError());
-    clear_map_kernel<<<(ntex + 255) / 256, 256, 0, s>>>(ctx->d_dirs, n, ctx->d_texels, ntex, ctx->d_cmap);
+    const int gcm = std::max(1, std::min(ctx->sms * 4, (ntex / 16 + 7) / 8));
+    clear_map_kernel<<<gcm, 256, ctx->smem_cmap, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_texels, ctx->cmapT,
+                                                      ctx->d_cmap);
     CK(cudaGetLastError());
     return AM_OK;
 }
@@ -384,19 +388,14 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, int slot, cudaStream_t s)
 //   (AM_OPT_PHASES = 0, 1 or 2 levels).
 // Can the whole map run as one fused cooperative launch?
 bool fused_ok(const am_ctx* ctx) {
-    return ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases == 2 && ctx->n_l0 > 0 &&
+    return ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases >= 1 && ctx->n_l0 > 0 &&
            ctx->bricks_on && ctx->d_bricks && ctx->N > 0;
 }
 
-// K maps (pivots[3K], K <= ctx->slots) into gam0 + k * MW with one fused
-// launch: am_pipeline_kernel<false> for K = 1, <true> (one CTA group per
-// pivot) otherwise.  Zeroes the maps and the K counter slots first.
-int launch_fused(am_ctx* ctx, const float* pivots, int K, uint32_t* gam0, cudaStream_t s) {
-    CK(cudaMemsetAsync(gam0, 0, (size_t)K * ctx->MW * sizeof(uint32_t), s));
-    CK(cudaMemsetAsync(ctx->d_ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long), s));
-    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+// The fused launch parameters for slot 0 and the map gam.
+FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     FusedParams F{};
-    F.main = make_params(ctx, pivots, gam0);
+    F.main = make_params(ctx, pivot, gam);
     F.main.vox = ctx->d_vox;
     F.main.N = ctx->N;
     F.main.cmap = ctx->d_cmap;
@@ -428,14 +427,67 @@ int launch_fused(am_ctx* ctx, const float* pivots, int K, uint32_t* gam0, cudaSt
     F.task1 = ctx->d_ctr + kCtrRT + 3;
     F.live1 = nullptr;
     F.texels = ctx->d_texels;
-    F.ntex = ntex;
-    F.use_l1 = 1;
-    F.ts = (ctx->diag_ts && ctx->d_ts && K == 1) ? ctx->d_ts : nullptr;
-    F.nslot = K;
-    for (int k = 0; k < K; ++k) {
-        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
-        F.piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    F.ntex = 6 * ctx->cmapT * ctx->cmapT;
+    F.use_l1 = ctx->phases == 2;
+    F.ts = (ctx->diag_ts && ctx->d_ts) ? ctx->d_ts : nullptr;  // batched: group 0
+    return F;
+}
+
+int timed_begin(am_ctx* ctx, cudaStream_t s) {
+    if (!ctx->timing) return AM_OK;
+    if (ctx->ev_used == ctx->ev_start.size()) {
+        cudaEvent_t a, b;
+        CK(cudaEventCreate(&a));
+        CK(cudaEventCreate(&b));
+        ctx->ev_start.push_back(a);
+        ctx->ev_stop.push_back(b);
     }
+    CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
+    return AM_OK;
+}
+
+int timed_end(am_ctx* ctx, cudaStream_t s) {
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
+    return AM_OK;
+}
+
+// One map (pivot) into gam with one fused cooperative launch over the whole grid.
+int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s) {
+    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
+    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrStride * sizeof(unsigned long long), s));
+    FusedParams F = fused_params(ctx, pivot, gam);
+    int rc;
+    if ((rc = timed_begin(ctx, s))) return rc;
+    void* args[] = {&F};
+    CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads), args,
+                                   ctx->smem_fused, s));
+    if ((rc = timed_end(ctx, s))) return rc;
+    if (ctx->d_prev)
+        CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    return AM_OK;
+}
+
+// P maps (pivots[3P]) into gam0 + k * MW with ONE fused launch: K groups of
+// CTAs (K <= ctx->slots) take pivots from a device queue (fused.cuh).
+int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint32_t* gam0, cudaStream_t s) {
+    if (ctx->piv_cap < P) {
+        cudaFree(ctx->d_piv);
+        ctx->d_piv = nullptr;
+        ctx->piv_cap = 0;
+        CK(cudaMalloc(&ctx->d_piv, (size_t)P * sizeof(float4)));
+        ctx->piv_cap = P;
+    }
+    if (!ctx->d_bctl) CK(cudaMalloc(&ctx->d_bctl, kBctlWords * sizeof(unsigned long long)));
+    ctx->h_piv.resize((size_t)P);
+    for (int64_t k = 0; k < P; ++k) {
+        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
+        ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    }
+    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv.data(), (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(ctx->d_bctl, 0, kBctlWords * sizeof(unsigned long long), s));
+    FusedParams F = fused_params(ctx, pivots, gam0);
+    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+    F.nslot = K;
     F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
     F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
     F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
@@ -443,34 +495,24 @@ int launch_fused(am_ctx* ctx, const float* pivots, int K, uint32_t* gam0, cudaSt
     F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
     F.cmap_stride = (unsigned long long)ntex * sizeof(float);
     F.blist_stride = (unsigned long long)ctx->nbricks * sizeof(unsigned int);
-    F.gam_stride = (unsigned long long)ctx->MW * sizeof(uint32_t);
-    F.bar = ctx->d_ctr + kCtrBar;
-    const bool timed = ctx->timing != 0;
-    if (timed) {
-        if (ctx->ev_used == ctx->ev_start.size()) {
-            cudaEvent_t a, b;
-            CK(cudaEventCreate(&a));
-            CK(cudaEventCreate(&b));
-            ctx->ev_start.push_back(a);
-            ctx->ev_stop.push_back(b);
-        }
-        CK(cudaEventRecord(ctx->ev_start[ctx->ev_used], s));
-    }
+    F.piv = ctx->d_piv;
+    F.npiv = (unsigned int)P;
+    F.gam0 = gam0;
+    F.ctr0 = ctx->d_ctr;
+    F.ctr_words = kCtrStride;
+    F.bar = ctx->d_bctl;                                             // 2 words per group
+    F.qnext = reinterpret_cast<unsigned int*>(ctx->d_bctl + 2 * kMaxSlots);
+    F.cur = F.qnext + 1;                                             // kMaxSlots words
+    int rc;
+    if ((rc = timed_begin(ctx, s))) return rc;
     void* args[] = {&F};
-    if (K == 1)
-        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads),
-                                       args, ctx->smem_fused, s));
-    else
-        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<true>, dim3(ctx->fused_grid), dim3(kThreads),
-                                       args, ctx->smem_fused, s));
-    if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
-    if (ctx->d_prev && K == 1)
-        CK(cudaMemcpyAsync(ctx->d_prev, gam0, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
-    return AM_OK;
+    CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<true>, dim3(ctx->fused_grid), dim3(kThreads), args,
+                                   ctx->smem_fused, s));
+    return timed_end(ctx, s);
 }
 
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
-    if (fused_ok(ctx)) return launch_fused(ctx, pivot, 1, gam, s);
+    if (fused_ok(ctx)) return launch_fused(ctx, pivot, gam, s);
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrStride * sizeof(unsigned long long), s));
     if (ctx->N == 0) return AM_OK;
@@ -481,18 +523,18 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
         // diagnostic: clear map from the previous map computed on this context
         // (exact only when the previous call used the same pivot)
         CK(cudaMemcpyAsync(gam, ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
-        if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
+        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         cm = ctx->d_cmap;
     } else if (ctx->phases > 0 && ctx->n_l0 > 0) {
         if ((rc = launch_coarse(ctx, p, ctx->d_coarse, ctx->n_l0, ctx->d_cmap_ones, 0, s))) return rc;
-        if ((rc = launch_clear_map(ctx, gam, 0, s))) return rc;
+        if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         if (ctx->phases > 1) {
             // level 1 through the same filter + live pipeline as the full stream
             // (inner cones only, no band)
             if ((rc = launch_stream(ctx, p, ctx->d_coarse + ctx->n_l0, ctx->n_l1 - ctx->n_l0, ctx->d_cmap, false, s,
                                     true)))
                 return rc;
-            if ((rc = launch_clear_map(ctx, gam, 1, s))) return rc;
+            if ((rc = launch_clear_map(ctx, gam, s))) return rc;
         }
         cm = ctx->d_cmap;
     }
@@ -503,6 +545,20 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     }
     if (ctx->d_prev)  // allocated once diagnostics were enabled
         CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    return AM_OK;
+}
+
+// Diagnostics (AM_OPT_DIAG bit 2): fused-phase end times (us) of the last
+// launch on stderr (batched launches: group 0).
+int print_phase_times(am_ctx* ctx) {
+    if (!ctx->diag_ts || !ctx->d_ts) return AM_OK;
+    unsigned long long t[16];
+    CK(cudaMemcpy(t, ctx->d_ts, sizeof t, cudaMemcpyDeviceToHost));
+    fprintf(stderr, "am fused phases (us):");
+    for (int k = 1; k < 16; ++k)
+        if (t[k] >= t[0] && t[k]) fprintf(stderr, " %d:%.1f", k, (t[k] - t[0]) * 1e-3);
+    fprintf(stderr, "\n");
+    CK(cudaMemset(ctx->d_ts, 0, sizeof t));
     return AM_OK;
 }
 
@@ -639,8 +695,7 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
             return bail(AM_ECUDA);
         }
     }
-    if (cudaMalloc(&ctx->d_dirs, (size_t)m * n * sizeof(float4)) != cudaSuccess ||
-        cudaMalloc(&ctx->d_recs, (size_t)kRecCap * sizeof(ConeRec)) != cudaSuccess ||
+    if (cudaMalloc(&ctx->d_recs, (size_t)kRecCap * sizeof(ConeRec)) != cudaSuccess ||
         cudaMalloc(&ctx->d_tasks, (size_t)kTaskCap * sizeof(unsigned long long)) != cudaSuccess) {
         cudaGetLastError();
         return bail(AM_ENOMEM);
@@ -853,15 +908,7 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
         stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks) ? (int64_t)h[kCtrBricks] : (int64_t)ctx->nbricks;
         stats->level_voxels = ctx->phases == 0 ? 0 : ctx->phases == 1 ? ctx->n_l0 : ctx->n_l1;
-        if (ctx->diag_ts && ctx->d_ts) {  // diagnostics: fused-phase durations (us) on stderr
-            unsigned long long t[16];
-            CK(cudaMemcpy(t, ctx->d_ts, sizeof t, cudaMemcpyDeviceToHost));
-            fprintf(stderr, "am fused phases (us):");
-            for (int k = 1; k < 16; ++k)
-                if (t[k] >= t[0] && t[k]) fprintf(stderr, " %d:%.1f", k, (t[k] - t[0]) * 1e-3);
-            fprintf(stderr, "\n");
-            CK(cudaMemset(ctx->d_ts, 0, sizeof t));
-        }
+        if ((rc = print_phase_times(ctx)) != AM_OK) return rc;
     } else if (!dst_is_device) {
         CK(cudaStreamSynchronize(s));
     }
@@ -896,10 +943,7 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
     if (K > 1 && fused_ok(ctx)) {
         // batched fused launches of up to K pivots each (8(f) NEXT 2)
         if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
-        for (int64_t k = 0; k < P; k += K) {
-            const int kk = (int)std::min<int64_t>(K, P - k);
-            if ((rc = launch_fused(ctx, pivots + 3 * k, kk, dst + k * ctx->MW, s)) != AM_OK) return rc;
-        }
+        if ((rc = launch_fused_batch(ctx, pivots, P, K, dst, s)) != AM_OK) return rc;
     } else {
         for (int64_t k = 0; k < P; ++k)
             if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
@@ -907,6 +951,10 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
     if (!dst_is_device) {
         CK(cudaMemcpyAsync(am_out, dst, (size_t)P * ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
+    }
+    if (ctx->diag_ts) {
+        CK(cudaStreamSynchronize(s));
+        if ((rc = print_phase_times(ctx)) != AM_OK) return rc;
     }
     return AM_OK;
 }
@@ -1083,7 +1131,8 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_cmap_ones);
     cudaFree(ctx->d_prev);
     cudaFree(ctx->d_ts);
-    cudaFree(ctx->d_dirs);
+    cudaFree(ctx->d_piv);
+    cudaFree(ctx->d_bctl);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

@@ -52,13 +52,18 @@ struct FusedParams {
     int use_l1;
     unsigned long long* ts;   // diagnostics: %globaltimer after each phase (CTA 0), or nullptr
     // batched launch (am_pipeline_kernel<true>): the CTAs form nslot groups; group s
-    // computes the map of pivot s with slot s of every per-map buffer, i.e. the
-    // slot-0 pointers above advanced by s strides (bytes).
+    // owns slot s of every per-map buffer (the slot-0 pointers above advanced by
+    // s strides, in bytes) and takes pivots from a queue until it is empty.
     int nslot;
-    float4 piv[kMaxSlots];    // pivot xyz, w = may_cull
-    unsigned long long ctr_stride, q_stride, rec_stride, task_stride, live_stride, cmap_stride, blist_stride,
-        gam_stride;
-    unsigned long long* bar;  // slot 0's group barrier: [arrivals, generation] (zeroed with the counters)
+    unsigned long long ctr_stride, q_stride, rec_stride, task_stride, live_stride, cmap_stride, blist_stride;
+    const float4* piv;        // npiv pivots: xyz, w = may_cull
+    unsigned int npiv;
+    uint32_t* gam0;           // map of pivot k at gam0 + k * m * W
+    unsigned long long* ctr0; // slot s's counters: ctr0 + s * ctr_stride bytes, ctr_words 64-bit words
+    int ctr_words;
+    unsigned int* qnext;      // pivot queue head (zeroed)
+    unsigned int* cur;        // per group: its current pivot
+    unsigned long long* bar;  // per group: [arrivals, generation] (zeroed)
 };
 
 template <typename T>
@@ -67,14 +72,10 @@ __device__ __forceinline__ T* shift_bytes(T* p, unsigned long long b) {
              : p;
 }
 
-// The slot-s copy of a StreamParams (pivot and per-map buffers of slot s).
+// The slot-s copy of a StreamParams: per-map buffers of slot s (the pivot and
+// its map are set per pivot).
 __device__ void slot_params(StreamParams& p, const FusedParams& F, int s, bool own_cmap) {
     const unsigned long long c = s * F.ctr_stride;
-    p.px = F.piv[s].x;
-    p.py = F.piv[s].y;
-    p.pz = F.piv[s].z;
-    p.may_cull = F.piv[s].w != 0.f;
-    p.gam = shift_bytes(p.gam, s * F.gam_stride);
     p.qcount = shift_bytes(p.qcount, c);
     p.stats = shift_bytes(p.stats, c);
     p.live_count = shift_bytes(p.live_count, c);
@@ -87,6 +88,14 @@ __device__ void slot_params(StreamParams& p, const FusedParams& F, int s, bool o
     p.tasks = shift_bytes(p.tasks, s * F.task_stride);
     p.brick_list = shift_bytes(p.brick_list, s * F.blist_stride);
     if (own_cmap) p.cmap = shift_bytes(p.cmap, s * F.cmap_stride);
+}
+
+__device__ __forceinline__ void set_pivot(StreamParams& p, float4 v, uint32_t* gam) {
+    p.px = v.x;
+    p.py = v.y;
+    p.pz = v.z;
+    p.may_cull = v.w != 0.f;
+    p.gam = gam;
 }
 
 // Barrier over the nb CTAs of one group (all co-resident: cooperative launch).
@@ -118,15 +127,13 @@ __device__ __forceinline__ void fused_mark(const FusedParams& F, int k) {
     }
 }
 
-// Dynamic shared memory: AM, row-full bits, a chunk of clear directions.
-constexpr int kFusedDirs = 1024;
-__host__ __device__ inline size_t fused_smem_bytes(int m, int W) {
-    return (size_t)(m * W + ((m + 31) >> 5) + 1) * sizeof(uint32_t) + 15 + (size_t)kFusedDirs * sizeof(float4);
+// Dynamic shared memory: AM, row-full bits, then (16-byte aligned) the
+// clear directions of the clear-direction map phases.
+__host__ __device__ inline size_t fused_dirs_offset(int m, int W) {
+    return ((size_t)(m * W + ((m + 31) >> 5) + 1) * sizeof(uint32_t) + 15) & ~(size_t)15;
 }
-
-__device__ __forceinline__ float4* fused_dirs(uint32_t* sAM, int MW, int m) {
-    uintptr_t a = reinterpret_cast<uintptr_t>(sAM + MW + ((m + 31) >> 5) + 1);
-    return reinterpret_cast<float4*>((a + 15) & ~uintptr_t(15));
+__host__ __device__ inline size_t fused_smem_bytes(int m, int W) {
+    return fused_dirs_offset(m, W) + (size_t)kMapDirs * sizeof(float4);
 }
 
 // Seed the shared AM from the global AM and compute the row-full bits.
@@ -176,70 +183,6 @@ __device__ void fused_rows(const StreamParams& p, const unsigned long long* task
         raster_row<COARSE>(p, r, i, sAM, cnt);
     }
     if (rows && cnt.c) atomicAdd(cnt.c + CT_ROWS, rows);
-}
-
-// Phases 3/6: the clear-direction map from the global AM.  The gn CTAs of the
-// group cover the texels kMaxT per thread per pass.
-__device__ void fused_clear_map(const StreamParams& p, const float4* texels, int ntex, float* V, uint32_t* sAM,
-                                float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
-    const GridDev& g = p.grid;
-    const int MW = g.m * g.W;
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
-    constexpr int kMaxT = 4;  // texels per thread per pass
-    const int per_pass = kMaxT * gn * blockDim.x;
-    for (int t0 = 0; t0 < ntex; t0 += per_pass) {
-        float best[kMaxT];
-        float4 c[kMaxT];
-#pragma unroll
-        for (int j = 0; j < kMaxT; ++j) {
-            best[j] = -2.f;
-            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
-            c[j] = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
-        }
-        int w0 = 0;
-        while (true) {
-            __syncthreads();
-            if (threadIdx.x == 0) *sN = 0;
-            __syncthreads();
-            // compact the clear cells of the next words (at most kFusedDirs per round)
-            const int wend = min(MW, w0 + kFusedDirs / 32);
-            for (int w = w0 + threadIdx.x; w < wend; w += blockDim.x) {
-                const int i = w / g.W, wj = w - i * g.W;
-                uint32_t clear = ~sAM[w] & row_word_mask(wj, g.n);
-                if (!clear) continue;
-                int pos = atomicAdd(sN, __popc(clear));
-                const float cph = __ldg(p.tab + i), sph = __ldg(p.tab + g.m + i);
-                while (clear) {
-                    const int j = (wj << 5) + __ffs(clear) - 1;
-                    clear &= clear - 1u;
-                    sDirs[pos++] = make_float4(sph * __ldg(p.tab + 2 * g.m + j),
-                                               sph * __ldg(p.tab + 2 * g.m + g.n + j), cph, 0.f);
-                }
-            }
-            __syncthreads();
-            const int k = *sN;
-            for (int e = 0; e < k; ++e) {
-                const float4 d = sDirs[e];
-#pragma unroll
-                for (int j = 0; j < kMaxT; ++j)
-                    best[j] = fmaxf(best[j], fmaf(c[j].x, d.x, fmaf(c[j].y, d.y, c[j].z * d.z)));
-            }
-            w0 = wend;
-            if (w0 >= MW) break;
-        }
-#pragma unroll
-        for (int j = 0; j < kMaxT; ++j) {
-            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
-            if (t >= ntex) continue;
-            float u = -2.f;
-            if (best[j] >= -1.5f) {
-                const float th = acosf(fminf(best[j] + 2e-6f, 1.f));
-                const float r = c[j].w;
-                u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
-            }
-            V[t] = u * fabsf(u);
-        }
-    }
 }
 
 // CTA-wide reservation (every thread of the CTA calls it): `cnt` slots for
@@ -314,64 +257,34 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
     }
 }
 
-// BATCH = false: one map, the whole grid, cooperative-groups grid barriers.
-// BATCH = true: F.nslot maps at once; contiguous CTA ranges form one group per
-// pivot, each with its own slot of the per-map buffers and its own barrier.
-template <bool BATCH>
-__global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_constant__ FusedParams F) {
-    namespace cg = cooperative_groups;
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    __shared__ unsigned int sCnt[CT_COUNT];
-    __shared__ int sN;
-    __shared__ unsigned int sCulled, sPassed;
-    __shared__ unsigned long long sStreamed;
-    __shared__ FusedScratch sc;
-    __shared__ StreamParams sP, sL;
-    __shared__ unsigned int* sRec1;
-    __shared__ unsigned long long* sTask1;
-    // group of this CTA: CTAs [start(s), start(s + 1)), start(s) = s * G / nslot
-    const unsigned int G = gridDim.x;
-    const unsigned int K = BATCH ? (unsigned int)F.nslot : 1u;
-    const unsigned int slot = BATCH ? (unsigned int)(((blockIdx.x + 1ull) * K - 1ull) / G) : 0u;
-    const unsigned int gstart = BATCH ? (unsigned int)((unsigned long long)slot * G / K) : 0u;
-    const unsigned int gb = blockIdx.x - gstart;
-    const unsigned int gn = BATCH ? (unsigned int)((unsigned long long)(slot + 1) * G / K) - gstart : G;
-    unsigned long long* bar = BATCH ? shift_bytes(F.bar, slot * F.ctr_stride) : nullptr;
-    if (BATCH) {
-        if (threadIdx.x == 0) {
-            sP = F.main;
-            sL = F.lvl;
-            slot_params(sP, F, (int)slot, true);
-            slot_params(sL, F, (int)slot, false);
-            sRec1 = shift_bytes(F.rec1, slot * F.ctr_stride);
-            sTask1 = shift_bytes(F.task1, slot * F.ctr_stride);
-        }
-        __syncthreads();
-    }
-    auto gsync = [&]() {
-        if (BATCH)
-            group_sync(bar, gn);
-        else
-            cg::this_grid().sync();
-    };
-    const StreamParams& P = *(BATCH ? &sP : &F.main);
-    const StreamParams& L = *(BATCH ? &sL : &F.lvl);
-    unsigned int* const rec1 = BATCH ? sRec1 : F.rec1;
-    unsigned long long* const task1 = BATCH ? sTask1 : F.task1;
+struct FusedShared {
+    unsigned int cnt[CT_COUNT];
+    unsigned int culled, passed, streamed;
+    FusedScratch sc;
+    int n;
+};
+
+// The phases of one map (P: main stream, L: clear-map levels) by the CTAs
+// gb = 0..gn-1 of a group; gsync() = the group's barrier.
+template <bool BATCH, typename Sync>
+__device__ __forceinline__ void map_phases(const FusedParams& F, const StreamParams& P, const StreamParams& L,
+                                           unsigned int* rec1, unsigned long long* task1, unsigned int gb,
+                                           unsigned int gn, Sync gsync, FusedShared& S, unsigned char* smem_raw) {
+    auto& sCnt = S.cnt;
+    auto& sc = S.sc;
     const int m = P.grid.m, MW = m * P.grid.W;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
     uint32_t* sRowFull = sAM + MW;
-    float4* sDirs = fused_dirs(sAM, MW, m);
+    float4* sDirs = reinterpret_cast<float4*>(smem_raw + fused_dirs_offset(m, P.grid.W));
     const unsigned long long gstride = (unsigned long long)gn * blockDim.x;
     if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
     if (threadIdx.x == 0) {
-        sCulled = sPassed = 0u;
-        sStreamed = 0ull;
+        S.culled = S.passed = 0u;
+        S.streamed = 0u;
     }
     const Counters none{nullptr};
     for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
     __syncthreads();
-    fused_mark(F, 0);
 
     // 1. level-0 cones (inner), every voxel of the level is live (CTA-uniform loop)
     for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < F.n0; b0 += gstride) {
@@ -384,7 +297,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                              nullptr, sRowFull);
     }
     gsync();
-    fused_mark(F, 1);
+    if (!BATCH || gb == 0) fused_mark(F, 1);
     // 2. level-0 rows
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = 0u;
     for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
@@ -392,11 +305,11 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
     fused_rows<true>(L, L.task_count, sAM, sRowFull, none, gb, gn);
     fused_flush(L, sAM);
     gsync();
-    fused_mark(F, 2);
+    if (!BATCH || gb == 0) fused_mark(F, 2);
     // 3. clear-direction map
-    fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN, gb, gn);
+    clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
     gsync();
-    fused_mark(F, 3);
+    if (!BATCH || gb == 0) fused_mark(F, 3);
     if (F.use_l1) {
         // 4. level-1 voxels: filter against the map, inner cones (stage 1: upper
         //    halves of the record / task buffers; the records index the level-1 array)
@@ -414,7 +327,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
                                  counted, &sc, nullptr, sRowFull);
         }
         gsync();
-        fused_mark(F, 4);
+        if (!BATCH || gb == 0) fused_mark(F, 4);
         // 5. level-1 rows (tasks in the upper halves)
         fused_seed(P, sAM, sRowFull);
         {
@@ -432,11 +345,11 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
         fused_flush(P, sAM);
         gsync();
-        fused_mark(F, 5);
+        if (!BATCH || gb == 0) fused_mark(F, 5);
         // 6. clear-direction map again
-        fused_clear_map(P, F.texels, F.ntex, const_cast<float*>(P.cmap), sAM, sDirs, &sN, gb, gn);
+        clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
         gsync();
-        fused_mark(F, 6);
+        if (!BATCH || gb == 0) fused_mark(F, 6);
     }
     // 7. brick test
     {
@@ -453,7 +366,7 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
     }
     gsync();
-    fused_mark(F, 7);
+    if (!BATCH || gb == 0) fused_mark(F, 7);
     // 8a. kept bricks: filter (kVPT bricks per CTA step); live voxels go to the
     //     global live list with one atomic per CTA step
     {
@@ -487,13 +400,19 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
             for (int k = 0; k < kVPT; ++k)
                 if (live[k]) P.live_idx[pos++] = idx[k];
         }
-        if (npassed) atomicAdd(&sPassed, npassed);
-        if (nculled) atomicAdd(&sCulled, nculled);
-        if (streamed) atomicAdd(&sStreamed, streamed);
+        // warp sums, one shared atomic per warp (a 64-bit shared atomic would be a CAS loop)
+        npassed = __reduce_add_sync(0xffffffffu, npassed);
+        nculled = __reduce_add_sync(0xffffffffu, nculled);
+        const unsigned int nstream = __reduce_add_sync(0xffffffffu, (unsigned int)streamed);
+        if ((threadIdx.x & 31) == 0) {
+            if (npassed) atomicAdd(&S.passed, npassed);
+            if (nculled) atomicAdd(&S.culled, nculled);
+            if (nstream) atomicAdd(&S.streamed, nstream);
+        }
     }
     fused_seed(P, sAM, sRowFull);  // row-full bits of the global AM (unchanged until phase 9)
     gsync();
-    fused_mark(F, 10);
+    if (!BATCH || gb == 0) fused_mark(F, 10);
     // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2)
     {
         const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
@@ -511,13 +430,13 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         }
     }
     gsync();
-    fused_mark(F, 8);
+    if (!BATCH || gb == 0) fused_mark(F, 8);
     // 9. rows of the full stream (both cones, band pairs queued)
     fused_seed(P, sAM, sRowFull);
     fused_rows<false>(P, P.task_count, sAM, sRowFull, Counters{sCnt}, gb, gn);
     fused_flush(P, sAM);
     gsync();
-    fused_mark(F, 9);
+    if (!BATCH || gb == 0) fused_mark(F, 9);
     // 10. band: exact test where the bit is still clear
     {
         const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
@@ -541,14 +460,74 @@ __global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_c
         if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
     }
     __syncthreads();
-    fused_mark(F, 15);
+    if (!BATCH) fused_mark(F, 15);
     if (threadIdx.x == 0) {
-        atomicAdd(P.stats + ST_CULLED, (unsigned long long)sCulled);
-        atomicAdd(P.stats + ST_PASSED, (unsigned long long)sPassed);
-        atomicAdd(P.stats + ST_STREAMED, sStreamed);
+        atomicAdd(P.stats + ST_CULLED, (unsigned long long)S.culled);
+        atomicAdd(P.stats + ST_PASSED, (unsigned long long)S.passed);
+        atomicAdd(P.stats + ST_STREAMED, (unsigned long long)S.streamed);
         atomicAdd(P.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
         atomicAdd(P.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
         atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+    }
+}
+
+
+// BATCH = false: one map, the whole grid, cooperative-groups grid barriers.
+// BATCH = true: F.nslot groups of contiguous CTAs; each group takes pivots from
+// the queue F.qnext until it is empty and computes their maps with its own
+// slot of the per-map buffers and its own barrier (a slow pivot delays only
+// its group).
+template <bool BATCH>
+__global__ void __launch_bounds__(kThreads, 2) am_pipeline_kernel(const __grid_constant__ FusedParams F) {
+    namespace cg = cooperative_groups;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ FusedShared S;
+    if (!BATCH) {
+        fused_mark(F, 0);
+        map_phases<false>(F, F.main, F.lvl, F.rec1, F.task1, blockIdx.x, gridDim.x,
+                          []() { cg::this_grid().sync(); }, S, smem_raw);
+        return;
+    }
+    __shared__ StreamParams sP, sL;
+    __shared__ unsigned int* sRec1;
+    __shared__ unsigned long long* sTask1;
+    // group of this CTA: CTAs [start(s), start(s + 1)), start(s) = s * G / nslot
+    const unsigned int G = gridDim.x;
+    const unsigned int K = (unsigned int)F.nslot;
+    const unsigned int slot = (unsigned int)(((blockIdx.x + 1ull) * K - 1ull) / G);
+    const unsigned int gstart = (unsigned int)((unsigned long long)slot * G / K);
+    const unsigned int gb = blockIdx.x - gstart;
+    const unsigned int gn = (unsigned int)((unsigned long long)(slot + 1) * G / K) - gstart;
+    unsigned long long* bar = F.bar + 2 * slot;
+    unsigned long long* ctr = shift_bytes(F.ctr0, slot * F.ctr_stride);
+    fused_mark(F, 0);
+    if (threadIdx.x == 0) {
+        sP = F.main;
+        sL = F.lvl;
+        slot_params(sP, F, (int)slot, true);
+        slot_params(sL, F, (int)slot, false);
+        sRec1 = shift_bytes(F.rec1, slot * F.ctr_stride);
+        sTask1 = shift_bytes(F.task1, slot * F.ctr_stride);
+    }
+    auto gsync = [bar, gn]() { group_sync(bar, gn); };
+    const int MW = F.main.grid.m * F.main.grid.W;
+    while (true) {
+        if (gb == 0 && threadIdx.x == 0) F.cur[slot] = atomicAdd(F.qnext, 1u);
+        group_sync(bar, gn);
+        const unsigned int k = *reinterpret_cast<volatile unsigned int*>(F.cur + slot);
+        if (k >= F.npiv) break;
+        uint32_t* gam = F.gam0 + (size_t)k * MW;
+        if (threadIdx.x == 0) {
+            const float4 v = F.piv[k];
+            set_pivot(sP, v, gam);
+            set_pivot(sL, v, gam);
+        }
+        if (gb == 0) {  // this pivot's map and the slot's counters start at zero
+            for (int w = threadIdx.x; w < MW; w += blockDim.x) gam[w] = 0u;
+            for (int w = threadIdx.x; w < F.ctr_words; w += blockDim.x) ctr[w] = 0ull;
+        }
+        group_sync(bar, gn);
+        map_phases<true>(F, sP, sL, sRec1, sTask1, gb, gn, gsync, S, smem_raw);
     }
 }
 

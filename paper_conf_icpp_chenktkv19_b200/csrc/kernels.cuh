@@ -164,58 +164,170 @@ __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, 
 // Cells only ever get blocked, so a map built from a partial AM stays valid
 // for the final one.
 //
-// Step 1 (one CTA): the directions of the cells still clear, counted in *n.
-__global__ void __launch_bounds__(1024) clear_list_kernel(const uint32_t* __restrict__ gam, GridDev g,
-                                                          const float* __restrict__ tab,
-                                                          float4* __restrict__ dirs, unsigned int* n) {
-    const int MW = g.m * g.W;
-    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+//
+// Texels are processed in 4 x 4 blocks ("coarse texels", one warp each): the
+// warp first finds the coarse centre's nearest clear angle theta_C over every
+// clear direction, then only directions within theta_C + 2 rho of the coarse
+// centre (rho = the block's angular radius) can be nearest to any of its 16
+// texels (triangle inequality), and only those are tried per texel.  With few
+// clear cells (the common case once the coarse levels are in: ~100 of 4096 at
+// C3), more than fit in shared memory, or T not a multiple of 4, every texel
+// tries every clear direction (in chunks), 4 texels per thread.
+
+constexpr int kMapDirs = 2048;  // clear directions staged in shared memory per chunk
+constexpr int kMapBrute = 512;  // up to this many clear cells, every texel tries every one
+
+__device__ __forceinline__ float dot3(float4 a, float4 b) { return fmaf(a.x, b.x, fmaf(a.y, b.y, a.z * b.z)); }
+
+// V_t from the best cosine of texel (c, r): the nearest-cell angle rounded
+// down and the bound rounded up (fp32 guards).
+__device__ __forceinline__ float clear_map_value(float best, float r) {
+    float u = -2.f;
+    if (best >= -1.5f) {
+        const float th = acosf(fminf(best + 2e-6f, 1.f));
+        u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+    }
+    return u * fabsf(u);
+}
+
+// Compact the directions of the clear cells of words [w0, w1) of sAM into
+// sDirs (at most kMapDirs: the caller sizes the range); count in *sN.
+__device__ void compact_clear_dirs(const uint32_t* sAM, const GridDev& g, const float* __restrict__ tab, int w0,
+                                   int w1, float4* sDirs, int* sN) {
+    __syncthreads();
+    if (threadIdx.x == 0) *sN = 0;
+    __syncthreads();
+    for (int w = w0 + threadIdx.x; w < w1; w += blockDim.x) {
         const int i = w / g.W, wj = w - i * g.W;
-        uint32_t clear = ~ld_cg(gam + w) & row_word_mask(wj, g.n);
+        uint32_t clear = ~sAM[w] & row_word_mask(wj, g.n);
         if (!clear) continue;
-        unsigned int pos = atomicAdd(n, (unsigned int)__popc(clear));
+        int pos = atomicAdd(sN, __popc(clear));
         const float cph = __ldg(tab + i), sph = __ldg(tab + g.m + i);
         while (clear) {
             const int j = (wj << 5) + __ffs(clear) - 1;
             clear &= clear - 1u;
-            dirs[pos++] = make_float4(sph * __ldg(tab + 2 * g.m + j), sph * __ldg(tab + 2 * g.m + g.n + j), cph,
-                                      0.f);
+            sDirs[pos++] = make_float4(sph * __ldg(tab + 2 * g.m + j), sph * __ldg(tab + 2 * g.m + g.n + j), cph, 0.f);
+        }
+    }
+    __syncthreads();
+}
+
+// The clear-direction map of `gam` into V (6 T^2 texels), computed by the CTAs
+// gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
+// (kMapDirs), sN.
+__device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
+                              const float4* __restrict__ texels, int T, float* __restrict__ V, uint32_t* sAM,
+                              float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
+    const int MW = g.m * g.W;
+    const int ntex = 6 * T * T;
+    __syncthreads();
+    if (threadIdx.x == 0) *sN = 0;
+    __syncthreads();
+    int cnt = 0;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+        const uint32_t a = ld_cg(gam + w);
+        sAM[w] = a;
+        cnt += __popc(~a & row_word_mask(w % g.W, g.n));
+    }
+    if (cnt) atomicAdd(sN, cnt);
+    __syncthreads();
+    const int total = *sN;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    if (total > kMapBrute && total <= kMapDirs && (T & 3) == 0) {
+        compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
+        const int Tc = T >> 2, nct = 6 * Tc * Tc;
+        const int half = lane >> 4, sub = lane & 15;
+        for (int ct = gb * nwarps + warp; ct < nct; ct += gn * nwarps) {
+            const int face = ct / (Tc * Tc), rem = ct - face * Tc * Tc, cw = rem / Tc, cu = rem - cw * Tc;
+            const int t = (face * T + 4 * cw + (sub >> 2)) * T + 4 * cu + (sub & 3);
+            const float4 cf = texels[t];
+            // coarse centre: the normalised sum of the 16 texel centres (each half-warp)
+            float sx = cf.x, sy = cf.y, sz = cf.z;
+#pragma unroll
+            for (int o = 1; o < 16; o <<= 1) {
+                sx += __shfl_xor_sync(0xffffffffu, sx, o);
+                sy += __shfl_xor_sync(0xffffffffu, sy, o);
+                sz += __shfl_xor_sync(0xffffffffu, sz, o);
+            }
+            const float inv = rsqrtf(fmaf(sx, sx, fmaf(sy, sy, sz * sz)));
+            const float4 c = make_float4(sx * inv, sy * inv, sz * inv, 0.f);
+            // rho: block radius (angles rounded up)
+            float rho = acosf(fmaxf(dot3(cf, c) - 1e-6f, -1.f));
+#pragma unroll
+            for (int o = 1; o < 16; o <<= 1) rho = fmaxf(rho, __shfl_xor_sync(0xffffffffu, rho, o));
+            // theta_C over every clear direction
+            float bc = -2.f;
+            for (int e = lane; e < total; e += 32) bc = fmaxf(bc, dot3(c, sDirs[e]));
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) bc = fmaxf(bc, __shfl_xor_sync(0xffffffffu, bc, o));
+            // candidates: angle(c, d) <= theta_C + 2 rho (rounded up, + slack)
+            const float th = acosf(fmaxf(bc - 1e-6f, -1.f)) + 2.f * rho + 1e-4f;
+            const float thr = th >= 3.14159f ? -2.f : cosf(th) - 1e-6f;
+            float bf = -2.f;
+            for (int base = 0; base < total; base += 32) {
+                const int e = base + lane;
+                unsigned int mask = __ballot_sync(0xffffffffu, e < total && dot3(c, sDirs[e]) >= thr);
+                while (mask) {  // half-warps take alternate candidates
+                    const int k0 = __ffs(mask) - 1;
+                    mask &= mask - 1u;
+                    int k = half ? -1 : k0;
+                    if (mask) {
+                        if (half) k = __ffs(mask) - 1;
+                        mask &= mask - 1u;
+                    }
+                    if (k >= 0) bf = fmaxf(bf, dot3(cf, sDirs[base + k]));
+                }
+            }
+            bf = fmaxf(bf, __shfl_xor_sync(0xffffffffu, bf, 16));
+            if (!half) V[t] = clear_map_value(bf, cf.w);
+        }
+        return;
+    }
+    // every texel against every clear direction, kMaxT texels per thread per
+    // pass, the directions in chunks of whole words
+    constexpr int kMaxT = 4;
+    const int per_pass = kMaxT * gn * blockDim.x;
+    for (int t0 = 0; t0 < ntex; t0 += per_pass) {
+        float best[kMaxT];
+        float4 c[kMaxT];
+#pragma unroll
+        for (int j = 0; j < kMaxT; ++j) {
+            best[j] = -2.f;
+            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
+            c[j] = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
+        }
+        for (int w0 = 0; w0 < MW; w0 += kMapDirs / 32) {
+            compact_clear_dirs(sAM, g, tab, w0, min(MW, w0 + kMapDirs / 32), sDirs, sN);
+            const int k = *sN;
+            for (int e = 0; e < k; ++e) {
+                const float4 d = sDirs[e];
+#pragma unroll
+                for (int j = 0; j < kMaxT; ++j) best[j] = fmaxf(best[j], dot3(c[j], d));
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kMaxT; ++j) {
+            const int t = t0 + (j * gn + gb) * blockDim.x + threadIdx.x;
+            if (t < ntex) V[t] = clear_map_value(best[j], c[j].w);
         }
     }
 }
 
-// Step 2: one thread per texel, the clear directions staged through shared
-// memory in chunks.
-__global__ void __launch_bounds__(256) clear_map_kernel(const float4* __restrict__ dirs,
-                                                        const unsigned int* n,
-                                                        const float4* __restrict__ texels, int ntex,
+// Stand-alone launch of clear_map_cta (multi-kernel path); dynamic shared
+// memory: m * W words, then kMapDirs float4 (16-byte aligned).
+__host__ __device__ inline size_t clear_map_smem_bytes(int MW) {
+    return (((size_t)MW * sizeof(uint32_t) + 15) & ~(size_t)15) + (size_t)kMapDirs * sizeof(float4);
+}
+
+__global__ void __launch_bounds__(256) clear_map_kernel(const uint32_t* __restrict__ gam, GridDev g,
+                                                        const float* __restrict__ tab,
+                                                        const float4* __restrict__ texels, int T,
                                                         float* __restrict__ V) {
-    constexpr int kChunkDirs = 1024;
-    __shared__ float4 sd[kChunkDirs];
-    const unsigned int cnt = *n;
-    const int t = blockIdx.x * blockDim.x + threadIdx.x;
-    const float4 c = t < ntex ? texels[t] : make_float4(0.f, 0.f, 1.f, 0.f);
-    float best = -2.f;
-    for (unsigned int base = 0; base < cnt; base += kChunkDirs) {
-        const unsigned int k = min((unsigned int)kChunkDirs, cnt - base);
-        __syncthreads();
-        for (unsigned int e = threadIdx.x; e < k; e += blockDim.x) sd[e] = dirs[base + e];
-        __syncthreads();
-        for (unsigned int e = 0; e < k; ++e) {
-            const float4 d = sd[e];
-            best = fmaxf(best, fmaf(c.x, d.x, fmaf(c.y, d.y, c.z * d.z)));
-        }
-    }
-    if (t < ntex) {
-        float u = -2.f;
-        if (best >= -1.5f) {
-            // round the nearest-cell angle down and the bound up (fp32 guards)
-            const float th = acosf(fminf(best + 2e-6f, 1.f));
-            const float r = c.w;
-            u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
-        }
-        V[t] = u * fabsf(u);
-    }
+    extern __shared__ __align__(16) unsigned char smem_cm[];
+    __shared__ int sN;
+    uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_cm);
+    float4* sDirs = reinterpret_cast<float4*>(smem_cm + (((size_t)g.m * g.W * sizeof(uint32_t) + 15) & ~(size_t)15));
+    clear_map_cta(gam, g, tab, texels, T, V, sAM, sDirs, &sN, blockIdx.x, gridDim.x);
 }
 
 // a6: exact test for queued band pairs whose AM bit is still clear.

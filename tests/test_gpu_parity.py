@@ -252,6 +252,8 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_BATCH, 2)  # groups of 2 + a single
     assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_CMAP_T, 18)  # not a multiple of 4: per-texel search over all cells
+    assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
