@@ -252,6 +252,8 @@ def run_ours(args):
     piv = piv_all[rank::ws]  # pivot sharding: rank r takes pivots r, r + G, ...
     ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
     ctx.set_option(B.OPT_BATCH, args.groups)
+    if args.cmap_t:
+        ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
     t0 = time.time()
     ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
     torch.cuda.synchronize(dev)
@@ -433,6 +435,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--baseline", action="store_true", help="also time am_compute_baseline once")
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
+    ap.add_argument("--cmap-t", type=int, default=0, help="AM_OPT_CMAP_T (0 = library default)")
     ap.add_argument("--no-full-scan", action="store_true", help="skip the full-scan (filter_kernel) leg")
     args = ap.parse_args()
     if args.warmup < 3:

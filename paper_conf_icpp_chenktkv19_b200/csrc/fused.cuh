@@ -220,8 +220,58 @@ struct FusedScratch {
     unsigned long long r64[kWarps + 1];
 };
 
+// Rows i0 .. i0 + nrows - 1 that are not yet full, word w of the row-full bits.
+__device__ __forceinline__ uint32_t open_rows_word(const uint32_t* rowfull, int i0, int i1, int w) {
+    uint32_t b = ~rowfull[w];
+    if (w == (i0 >> 5)) b &= 0xffffffffu << (i0 & 31);
+    if (w == (i1 >> 5)) b &= 0xffffffffu >> (31 - (i1 & 31));
+    return b;
+}
+
+// cta_reserve of two counters at once (one scan, one barrier sequence).
+__device__ __forceinline__ void cta_reserve2(unsigned int ca, unsigned int* ga, unsigned long long cb,
+                                             unsigned long long* gb_, FusedScratch* sc, unsigned int& ba,
+                                             unsigned long long& bb) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    unsigned int ia = ca;
+    unsigned long long ib = cb;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned int ta = __shfl_up_sync(0xffffffffu, ia, o);
+        const unsigned long long tb = __shfl_up_sync(0xffffffffu, ib, o);
+        if (lane >= o) {
+            ia += ta;
+            ib += tb;
+        }
+    }
+    if (lane == 31) {
+        sc->r32[warp] = ia;
+        sc->r64[warp] = ib;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned int ra = 0;
+        unsigned long long rb = 0;
+        for (int w = 0; w < kWarps; ++w) {
+            const unsigned int ta = sc->r32[w];
+            const unsigned long long tb = sc->r64[w];
+            sc->r32[w] = ra;
+            sc->r64[w] = rb;
+            ra += ta;
+            rb += tb;
+        }
+        sc->r32[kWarps] = ra ? atomicAdd(ga, ra) : 0u;
+        sc->r64[kWarps] = rb ? atomicAdd(gb_, rb) : 0ull;
+    }
+    __syncthreads();
+    ba = sc->r32[kWarps] + sc->r32[warp] + ia - ca;
+    bb = sc->r64[kWarps] + sc->r64[warp] + ib - cb;
+    __syncthreads();
+}
+
 // CTA-wide emit_cones: records at slot_off + [reserved], tasks at
-// task_off + [reserved]; rows rasterised inline when the buffers are full.
+// task_off + [reserved] for the rows of the cone not yet full; rows
+// rasterised inline when the buffers are full.
 template <bool COARSE>
 __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned int* rec_count,
                                                unsigned long long* task_count, unsigned int slot_off,
@@ -233,22 +283,26 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
         const unsigned int c = __popc(__ballot_sync(0xffffffffu, counted));
         if ((threadIdx.x & 31) == 0 && c) atomicAdd(live_stat, (unsigned long long)c);
     }
-    // rows already full in the global AM need no task
+    const int i0 = r.i0, i1 = r.i0 + nrows - 1;
     int ntask = 0;
-    for (int k = 0; k < nrows; ++k) {
-        const int i = r.i0 + k;
-        ntask += !((rowfull[i >> 5] >> (i & 31)) & 1u);
-    }
-    const unsigned int slot = cta_reserve<unsigned int>(ntask > 0 ? 1u : 0u, rec_count, sc->r32) + slot_off;
-    const unsigned long long t0 =
-        cta_reserve<unsigned long long>((unsigned long long)ntask, task_count, sc->r64) + task_off;
+    if (nrows > 0)
+        for (int w = i0 >> 5; w <= (i1 >> 5); ++w) ntask += __popc(open_rows_word(rowfull, i0, i1, w));
+    unsigned int slot;
+    unsigned long long t0;
+    cta_reserve2(ntask > 0 ? 1u : 0u, rec_count, (unsigned long long)ntask, task_count, sc, slot, t0);
+    slot += slot_off;
+    t0 += task_off;
     if (ntask > 0) {
         if (slot < slot_cap && t0 + ntask <= task_cap) {
             p.recs[slot] = r;
             unsigned long long t = t0;
-            for (int k = 0; k < nrows; ++k) {
-                const int i = r.i0 + k;
-                if (!((rowfull[i >> 5] >> (i & 31)) & 1u)) p.tasks[t++] = ((unsigned long long)slot << 16) | (unsigned int)k;
+            for (int w = i0 >> 5; w <= (i1 >> 5); ++w) {
+                uint32_t b = open_rows_word(rowfull, i0, i1, w);
+                while (b) {
+                    const int i = (w << 5) + __ffs(b) - 1;
+                    b &= b - 1u;
+                    p.tasks[t++] = ((unsigned long long)slot << 16) | (unsigned int)(i - i0);
+                }
             }
         } else {
             for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
