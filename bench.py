@@ -4,8 +4,8 @@
 
 A step is one am_compute_batch call: the whole hot path (a1-a8 of SURVEY.md
 8(a)) for --batch (default 64) consecutive pivots of the seeded 1 mm path over
-the resident voxel model, in one fused launch whose --groups (default 16) CTA
-groups take the pivots from a device queue (8(f) NEXT 2).  Default workload: C3
+the resident voxel model, computed phase by phase with --slots (default 64)
+pivots per launch (8(f) NEXT 2, csrc/batch.cuh).  Default workload: C3
 (head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096 orientations),
 the configuration BASELINE.json's metric is quoted on.  The one-pivot latency
 (am_compute) is reported beside it.  For N > 1 (torchrun), every rank computes
@@ -171,7 +171,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch, args.groups),
+        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch, args.slots),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                          "sample": f"{cells} cells of {args.steps} maps (seeded cells, pivots of the 1 mm path), "
                                    f"every voxel per cell, fp64 clip-project-hull test with exact-safe shortcuts"},
@@ -181,25 +181,26 @@ def run_reference(args):
     return 0
 
 
-def _config_dict(cfg, N, flushed=True, batch=1, groups=1):
+def _config_dict(cfg, N, flushed=True, batch=1, slots=1):
     return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
                         f"pivots on the {cfg.offset:g} mm path",
             "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
             "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
                    f"every timed step, outside the per-step CUDA events") if flushed else
                   f"inputs {16 * N / 1e6:.0f} MB; no flush",
-            "pivots_per_step": batch, "concurrent_maps": groups,
+            "pivots_per_step": batch, "pivots_per_launch": slots,
             "parallelism": "pivot-sharded (weak)"}
 
 
-def _ncu_traffic(cfg_name, kernel):
-    """DRAM bytes per launch of `kernel` from the committed ncu --set full summary (or None)."""
+def _ncu_traffic(cfg_name, kernel, maps=1):
+    """DRAM bytes per launch of `kernel` from the committed ncu --set full summary, for a
+    launch computing `maps` AMs (scaled from the captured launch's AM count), or None."""
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         d = json.load(open(prof))
         k = d.get("kernels", {}).get(kernel)
         if k and k.get("config") == cfg_name:
-            return k.get("dram_bytes_per_launch"), k.get("tag")
+            return k.get("dram_bytes_per_launch") * maps / k.get("maps_per_launch", 1), k.get("tag")
     except Exception:
         pass
     return None, None
@@ -251,7 +252,7 @@ def run_ours(args):
     piv_all = cfg.pivots(npiv * ws)
     piv = piv_all[rank::ws]  # pivot sharding: rank r takes pivots r, r + G, ...
     ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
-    ctx.set_option(B.OPT_BATCH, args.groups)
+    ctx.set_option(B.OPT_BATCH, args.slots)
     if args.cmap_t:
         ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
     t0 = time.time()
@@ -336,7 +337,7 @@ def run_ours(args):
     achieved = alg_bytes / (kavg_ms / 1e3) / 1e9
     # bytes the fused kernel actually needs: brick spheres, kept bricks' voxels, both map levels
     touched = bsz * (16.0 * (ctx_nbricks(N) + mean["voxels_streamed"] + mean["level_voxels"]) + cfg.m * cfg.n / 8.0)
-    traffic, traffic_tag = _ncu_traffic(cfg.name, "am_pipeline_kernel")
+    traffic, traffic_tag = _ncu_traffic(cfg.name, "am_pipeline_kernel", bsz)
     baseline_ms = None
     if args.baseline and rank == 0:
         ctx.set_option(B.OPT_BASELINE_REJECT, 1)
@@ -368,7 +369,7 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N, flush is not None, bsz, args.groups),
+            "config": _config_dict(cfg, N, flush is not None, bsz, args.slots),
             "ms_per_am": ms_max / args.steps / bsz,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_tag": traffic_tag,
@@ -427,8 +428,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--pivots", type=int, default=64, help="pivots per rank (cycled over the steps)")
     ap.add_argument("--batch", type=int, default=64, help="pivots per step (one am_compute_batch call)")
-    ap.add_argument("--groups", type=int, default=16,
-                    help="AM_OPT_BATCH: maps computed concurrently by the batched launch (CTA groups)")
+    ap.add_argument("--slots", type=int, default=64,
+                    help="AM_OPT_BATCH: pivots computed together, phase by phase (one launch per phase)")
     ap.add_argument("--e2e-steps", type=int, default=100)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--ref-seconds", type=float, default=60.0)

@@ -96,9 +96,9 @@ enum {
     AM_OPT_FUSED = 11,           /* 1 = the whole map in one persistent cooperative launch when
                                     phases >= 1 and bricks = 1 (default); 0 = one launch per
                                     stage.  Same map                                            */
-    AM_OPT_BATCH = 12            /* am_compute_batch: pivots computed concurrently by one fused
-                                    launch (1..16, default 8; each needs its own set of per-map
-                                    buffers, ~4 N + 100 MB of device memory).  Same maps        */
+    AM_OPT_BATCH = 12            /* am_compute_batch: pivots computed together, phase by phase,
+                                    one launch per phase (1..64, default 32; each needs its own
+                                    per-map buffers, ~4 N + 100 MB of device memory).  Same maps */
 };
 
 /*
@@ -136,8 +136,8 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
 /*
  * AMs of P pivots (host array pivots[3*P]); am_out receives P consecutive maps
  * of am_words_per_map(ctx) words each (host or device as above).  Same maps as
- * P calls of am_compute (the toolpath batch of SURVEY.md 8(e)(2)); with the
- * fused path, up to AM_OPT_BATCH pivots share one launch (8(f) NEXT 2).
+ * P calls of am_compute (the toolpath batch of SURVEY.md 8(e)(2)); up to
+ * AM_OPT_BATCH pivots run together, one launch per phase (8(f) NEXT 2).
  */
 int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_out,
                      int dst_is_device, void* cuda_stream);

@@ -19,6 +19,7 @@
 #include "kernels.cuh"
 #include "stream.cuh"
 #include "fused.cuh"
+#include "batch.cuh"
 
 using namespace am;
 
@@ -67,7 +68,8 @@ struct am_ctx {
     unsigned int nbricks = 0;
     int bricks_on = 1;
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
-    int batch = 8;                         // pivots per batched fused launch (AM_OPT_BATCH)
+    int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
+    int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
     long long piv_cap = 0;
@@ -95,6 +97,7 @@ constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
 constexpr int kCtrWords = kCtrBricks + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
 constexpr int kCtrStride = kCtrAll;          // 64-bit words per slot
+constexpr int kMaxBatch = 64;                // pivots per layered batch launch (slots)
 constexpr int kBctlWords = 2 * kMaxSlots + 1 + kMaxSlots / 2;  // bars, then queue head + per-group pivot (u32)
 constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
 constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
@@ -283,6 +286,15 @@ int configure_launch(am_ctx* ctx) {
             ctx->fused_grid = std::min(occf, occb) * ctx->sms;
     }
     cudaGetLastError();
+    // batched phases (batch.cuh)
+    const int sm_rows = (int)((ctx->MW + ((m + 31) >> 5) + 1) * sizeof(uint32_t));
+    CK(cudaFuncSetAttribute(bk_cones<BK_L0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_cones<BK_L1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_cones<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_rows<BK_L0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_rows<BK_L1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_rows<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_map, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     return AM_OK;
 }
 
@@ -509,6 +521,72 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<true>, dim3(ctx->fused_grid), dim3(kThreads), args,
                                    ctx->smem_fused, s));
     return timed_end(ctx, s);
+}
+
+// P maps (pivots[3P]) into gam0 + k * MW, phase by phase over chunks of up to
+// ctx->batch pivots (batch.cuh): each phase is one launch with blockIdx.y =
+// pivot of the chunk.
+int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* gam0, cudaStream_t s) {
+    const int K = (int)std::min<int64_t>(P, ctx->batch);
+    int rc;
+    if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
+    if (ctx->piv_cap < P) {
+        cudaFree(ctx->d_piv);
+        ctx->d_piv = nullptr;
+        ctx->piv_cap = 0;
+        CK(cudaMalloc(&ctx->d_piv, (size_t)P * sizeof(float4)));
+        ctx->piv_cap = P;
+    }
+    ctx->h_piv.resize((size_t)P);
+    for (int64_t k = 0; k < P; ++k) {
+        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
+        ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    }
+    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv.data(), (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
+    const int ntex = 6 * ctx->cmapT * ctx->cmapT;
+    const size_t sm_rows = (size_t)(ctx->MW + ((ctx->grid.m + 31) >> 5) + 1) * sizeof(uint32_t);
+    for (int64_t c0 = 0; c0 < P; c0 += K) {
+        const int kk = (int)std::min<int64_t>(K, P - c0);
+        uint32_t* g = gam0 + c0 * ctx->MW;
+        CK(cudaMemsetAsync(g, 0, (size_t)kk * ctx->MW * sizeof(uint32_t), s));
+        CK(cudaMemsetAsync(ctx->d_ctr, 0, (size_t)kk * kCtrStride * sizeof(unsigned long long), s));
+        FusedParams F = fused_params(ctx, pivots + 3 * c0, g);
+        F.nslot = kk;
+        F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
+        F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
+        F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
+        F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
+        F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
+        F.cmap_stride = (unsigned long long)ntex * sizeof(float);
+        F.blist_stride = (unsigned long long)ctx->nbricks * sizeof(unsigned int);
+        F.piv = ctx->d_piv + c0;
+        F.npiv = (unsigned int)kk;
+        F.gam0 = g;
+        F.ctr0 = ctx->d_ctr;
+        F.ctr_words = kCtrStride;
+        if ((rc = timed_begin(ctx, s))) return rc;
+        auto grid = [&](long long items, long long per_cta, int cap) {
+            long long gx = (items + per_cta - 1) / per_cta;
+            return dim3((unsigned)std::max<long long>(1, std::min<long long>(gx, cap)), (unsigned)kk);
+        };
+        const dim3 b(kThreads);
+        bk_cones<BK_L0><<<grid(ctx->n_l0, kThreads, 1 << 16), b, sm_rows, s>>>(F);
+        bk_rows<BK_L0><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        if (F.use_l1) {
+            bk_cones<BK_L1><<<grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), b, sm_rows, s>>>(F);
+            bk_rows<BK_L1><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+            bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        }
+        bk_bricks<<<grid(ctx->nbricks, 4 * kThreads, 1 << 16), b, 0, s>>>(F);
+        bk_voxels<<<grid(1 << 30, 1, ctx->bk_voxel_ctas), b, 0, s>>>(F);
+        bk_cones<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_cone_ctas), b, sm_rows, s>>>(F);
+        bk_rows<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        bk_band<<<grid(1 << 30, 1, 8), b, 0, s>>>(F);
+        CK(cudaGetLastError());
+        if ((rc = timed_end(ctx, s))) return rc;
+    }
+    return AM_OK;
 }
 
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
@@ -940,10 +1018,14 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
     }
     int rc;
     const int K = (int)std::min<int64_t>(P, ctx->batch);
-    if (K > 1 && fused_ok(ctx)) {
-        // batched fused launches of up to K pivots each (8(f) NEXT 2)
-        if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
-        if ((rc = launch_fused_batch(ctx, pivots, P, K, dst, s)) != AM_OK) return rc;
+    if (K > 1 && fused_ok(ctx) && (ctx->diag & 8)) {
+        // diagnostic: one cooperative launch, K CTA groups taking pivots from a queue
+        const int Kg = std::min(K, (int)kMaxSlots);
+        if ((rc = ensure_slots(ctx, Kg)) != AM_OK) return rc;
+        if ((rc = launch_fused_batch(ctx, pivots, P, Kg, dst, s)) != AM_OK) return rc;
+    } else if (K > 1 && fused_ok(ctx)) {
+        // the batch phase by phase, up to ctx->batch pivots per launch (8(f) NEXT 2)
+        if ((rc = launch_batch_layers(ctx, pivots, P, dst, s)) != AM_OK) return rc;
     } else {
         for (int64_t k = 0; k < P; ++k)
             if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
@@ -1018,7 +1100,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
-        if (value < 0 || value > 7) return fail(ctx, AM_EINVAL, "diag must be in [0, 7]");
+        if (value < 0 || value > 15) return fail(ctx, AM_EINVAL, "diag must be in [0, 15]");
         if ((value & 3) && !ctx->d_prev) {
             CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
@@ -1039,7 +1121,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->fused = (int)value;
         return AM_OK;
     case AM_OPT_BATCH:
-        if (value < 1 || value > kMaxSlots) return fail(ctx, AM_EINVAL, "batch must be in [1, %d]", kMaxSlots);
+        if (value < 1 || value > kMaxBatch) return fail(ctx, AM_EINVAL, "batch must be in [1, %d]", kMaxBatch);
         ctx->batch = (int)value;
         return AM_OK;
     case AM_OPT_CMAP_T:

@@ -1,0 +1,267 @@
+// batch.cuh -- the AICA maps of a batch of pivots, one launch per phase.
+//
+// The fused kernel (fused.cuh) minimises the latency of ONE map, but a map is
+// a chain of ~10 short phases whose work is a few hundred thousand voxels: one
+// map keeps the GPU busy only in bursts, and the fused kernel's register
+// budget (the heaviest phase sets it for all) caps occupancy at 16 warps/SM.
+// For a toolpath batch the same phases run here as
+// separate kernels over ALL pivots of the batch at once: blockIdx.y is the
+// pivot, each pivot owns slot blockIdx.y of every per-map buffer (the slot-0
+// pointers of FusedParams advanced by the slot strides), and each kernel gets
+// the registers -- and so the occupancy -- its own phase needs.  Kernel
+// boundaries replace the grid barriers, and the block scheduler balances
+// pivots of different cost.
+//
+// Phases (same device functions as fused.cuh, so the maps are bit-identical):
+//   bk_cones<L0>  level-0 inner cones        -> stage-0 records/tasks
+//   bk_rows<0>    their rows                 -> map
+//   bk_map        clear-direction map
+//   bk_cones<L1>  level-1 filter + cones     -> stage-1 records/tasks
+//   bk_rows<1>, bk_map
+//   bk_bricks     brick test                 -> kept bricks
+//   bk_voxels     kept bricks' voxels filter -> live list
+//   bk_cones<LIVE> both cones of live voxels -> stage-2 records/tasks
+//   bk_rows<2>    rows + band queue
+//   bk_band       exact test of queued band pairs still clear
+#pragma once
+#include "fused.cuh"
+
+namespace am {
+
+// StreamParams of pivot p (slot p) into shared memory (thread 0; the kernel
+// parameter is read by plain member access: a dynamically indexed pointer into
+// a __grid_constant__ parameter is not a global address); `lvl` selects the
+// clear-map-level copy.  Ends with a barrier.
+__device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParams& F, int p, bool lvl) {
+    if (threadIdx.x == 0) {
+        if (lvl)
+            out = F.lvl;
+        else
+            out = F.main;
+        slot_params(out, F, p, !lvl);
+        set_pivot(out, F.piv[p], F.gam0 + (size_t)p * F.main.grid.m * F.main.grid.W);
+    }
+    __syncthreads();
+}
+
+enum { BK_L0 = 0, BK_L1 = 1, BK_LIVE = 2 };
+
+// Cones of one stage: level 0 (every voxel of the level, inner cones), level 1
+// (filtered against the map, inner cones), or the live voxels (both cones).
+template <int STAGE>
+__global__ void __launch_bounds__(kThreads) bk_cones(const __grid_constant__ FusedParams F) {
+    extern __shared__ __align__(16) uint32_t smem_bk[];
+    __shared__ StreamParams sP;
+    __shared__ FusedScratch sc;
+    const int p = blockIdx.y;
+    pivot_params(sP, F, p, STAGE == BK_L0);
+    const StreamParams& P = sP;
+    const int m = P.grid.m, MW = m * P.grid.W;
+    uint32_t* sAM = smem_bk;
+    uint32_t* sRowFull = sAM + MW;
+    unsigned long long n;
+    if (STAGE == BK_L0) {
+        n = F.n0;
+        for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
+        __syncthreads();
+    } else {
+        // (two statements: a conditional between a parameter and a volatile load
+        // can be lowered to ONE load through a selected pointer, which is not
+        // valid for a parameter address)
+        if (STAGE == BK_L1)
+            n = F.n1;
+        else
+            n = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
+        if ((unsigned long long)blockIdx.x * blockDim.x >= n) return;  // CTA-uniform
+        fused_seed(P, sAM, sRowFull);
+    }
+    unsigned int* rc = STAGE == BK_L1 ? shift_bytes(F.rec1, p * F.ctr_stride) : P.rec_count;
+    unsigned long long* tc = STAGE == BK_L1 ? shift_bytes(F.task1, p * F.ctr_stride) : P.task_count;
+    const unsigned int roff = STAGE == BK_L1 ? P.rec_cap / 2 : 0u;
+    const unsigned long long toff = STAGE == BK_L1 ? P.task_cap / 2 : 0ull;
+    const unsigned int rcap = P.rec_cap;  // (level 0: the level copy's caps are the lower halves)
+    const unsigned long long tcap = P.task_cap;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long b0 = blockIdx.x * (unsigned long long)blockDim.x; b0 < n; b0 += stride) {
+        const unsigned long long e = b0 + threadIdx.x;
+        int nrows = 0;
+        bool counted = false;
+        ConeRec r;
+        if (e < n) {
+            if (STAGE == BK_L0) {
+                nrows = cone_of_voxel<true>(P, P.vox[e], (unsigned int)e, r, counted);
+            } else if (STAGE == BK_L1) {
+                const float4 q = F.l1[e];
+                if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
+            } else {
+                const unsigned int vidx = P.live_idx[e];
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+            }
+        }
+        emit_cones_cta<STAGE != BK_LIVE>(P, rc, tc, roff, toff, rcap, tcap, nrows, r, counted, &sc,
+                                         STAGE == BK_LIVE ? P.stats + ST_LIVE : nullptr, sRowFull);
+    }
+}
+
+// Rows of one stage into the CTA's shared AM (seeded from the map, so rows
+// already full are skipped), then OR-ed into the map.
+template <int STAGE>
+__global__ void __launch_bounds__(kThreads) bk_rows(const __grid_constant__ FusedParams F) {
+    extern __shared__ __align__(16) uint32_t smem_bk[];
+    __shared__ StreamParams sP;
+    __shared__ unsigned int sCnt[CT_COUNT];
+    const int p = blockIdx.y;
+    if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
+    pivot_params(sP, F, p, STAGE == BK_L0);
+    const StreamParams& P = sP;
+    const unsigned long long* tc =
+        STAGE == BK_L1 ? shift_bytes(F.task1, p * F.ctr_stride) : P.task_count;
+    const unsigned long long cap = STAGE == BK_L1 ? P.task_cap / 2 : P.task_cap;
+    const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(tc), cap);
+    if ((unsigned long long)blockIdx.x * blockDim.x >= ntask) return;  // CTA-uniform
+    uint32_t* sAM = smem_bk;
+    uint32_t* sRowFull = sAM + P.grid.m * P.grid.W;
+    fused_seed(P, sAM, sRowFull);
+    const unsigned long long toff = STAGE == BK_L1 ? P.task_cap / 2 : 0ull;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned int rows = 0;
+    for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask; k += stride) {
+        const unsigned long long t = P.tasks[toff + k];
+        const ConeRec r = P.recs[t >> 16];
+        if (r.i0 < 0) continue;
+        const int i = r.i0 + (int)(t & 0xffffu);
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        ++rows;
+        raster_row<STAGE != BK_LIVE>(P, r, i, sAM, Counters{STAGE == BK_LIVE ? sCnt : nullptr});
+    }
+    fused_flush(P, sAM);
+    if (STAGE == BK_LIVE) {
+        rows = __reduce_add_sync(0xffffffffu, rows);
+        if ((threadIdx.x & 31) == 0 && rows) atomicAdd(&sCnt[CT_ROWS], rows);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (sCnt[CT_ROWS]) atomicAdd(P.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
+            if (sCnt[CT_BAND]) atomicAdd(P.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
+            if (sCnt[CT_OVERFLOW]) atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+        }
+    }
+}
+
+// Clear-direction map of pivot p's map (kernels.cuh clear_map_cta).
+__global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ FusedParams F) {
+    extern __shared__ __align__(16) unsigned char smem_bm[];
+    __shared__ StreamParams sP;
+    __shared__ int sN;
+    const int p = blockIdx.y;
+    pivot_params(sP, F, p, false);
+    const StreamParams& P = sP;
+    uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
+    float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
+    clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float*>(P.cmap), sAM, sDirs, &sN, blockIdx.x,
+                  gridDim.x);
+}
+
+// Brick test: bricks whose bounding sphere may still reach a clear cell.
+__global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ FusedParams F) {
+    __shared__ StreamParams sP;
+    __shared__ FusedScratch sc;
+    const int p = blockIdx.y;
+    pivot_params(sP, F, p, false);
+    const StreamParams& P = sP;
+    const unsigned int nb = P.nbricks;
+    for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
+        const unsigned int b = b0 + threadIdx.x;
+        bool keep = false;
+        if (b < nb) {
+            const float4 s = __ldg(P.bricks + b);
+            keep = !sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
+        }
+        const unsigned int pos = cta_reserve<unsigned int>(keep ? 1u : 0u, P.brick_count, sc.r32);
+        if (keep) P.brick_list[pos] = b;
+    }
+}
+
+// Kept bricks' voxels through the filter; live voxels to the live list.
+__global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ FusedParams F) {
+    __shared__ StreamParams sP;
+    __shared__ FusedScratch sc;
+    __shared__ unsigned int sStat[3];
+    const int p = blockIdx.y;
+    if (threadIdx.x < 3) sStat[threadIdx.x] = 0u;
+    pivot_params(sP, F, p, false);
+    const StreamParams& P = sP;
+    const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
+    if (blockIdx.x * kVPT >= nk) return;  // CTA-uniform
+    unsigned int nculled = 0, npassed = 0, streamed = 0;
+    for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
+        float4 q[kVPT];
+        unsigned int idx[kVPT];
+        bool ok[kVPT];
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) {
+            ok[k] = k0 + k < nk;
+            idx[k] = ok[k] ? P.brick_list[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
+            ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
+            q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
+        }
+        bool live[kVPT];
+        unsigned int nl = 0;
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k) {
+            const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
+            nculled += f >> 1;
+            streamed += ok[k];
+            live[k] = f == F_LIVE;
+            nl += live[k];
+        }
+        npassed += nl;
+        unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
+#pragma unroll
+        for (int k = 0; k < kVPT; ++k)
+            if (live[k]) P.live_idx[pos++] = idx[k];
+    }
+    npassed = __reduce_add_sync(0xffffffffu, npassed);
+    nculled = __reduce_add_sync(0xffffffffu, nculled);
+    streamed = __reduce_add_sync(0xffffffffu, streamed);
+    if ((threadIdx.x & 31) == 0) {
+        if (npassed) atomicAdd(&sStat[0], npassed);
+        if (nculled) atomicAdd(&sStat[1], nculled);
+        if (streamed) atomicAdd(&sStat[2], streamed);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (sStat[0]) atomicAdd(P.stats + ST_PASSED, (unsigned long long)sStat[0]);
+        if (sStat[1]) atomicAdd(P.stats + ST_CULLED, (unsigned long long)sStat[1]);
+        if (sStat[2]) atomicAdd(P.stats + ST_STREAMED, (unsigned long long)sStat[2]);
+    }
+}
+
+// Band: exact test of the queued pairs whose bit is still clear.
+__global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ FusedParams F) {
+    __shared__ StreamParams sP;
+    const int p = blockIdx.y;
+    pivot_params(sP, F, p, false);
+    const StreamParams& P = sP;
+    const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
+    const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
+    unsigned long long tests = 0, hits = 0;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += stride) {
+        const unsigned long long e = P.queue[k];
+        const unsigned int vidx = (unsigned int)(e >> 32);
+        const int cell = (int)(e & 0xffffffffu);
+        const int i = cell / P.grid.n, j = cell - i * P.grid.n;
+        uint32_t* wp = P.gam + i * P.grid.W + (j >> 5);
+        const uint32_t bit = 1u << (j & 31);
+        if (ld_cg(wp) & bit) continue;
+        ++tests;
+        if (exact_pair(P, P.vox_main[vidx], cell)) {
+            ++hits;
+            atomicOr(wp, bit);
+        }
+    }
+    if (tests) atomicAdd(P.stats + ST_EXACT, tests);
+    if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
+}
+
+}  // namespace am

@@ -261,16 +261,18 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     ctx.close()
 
 
-@pytest.mark.parametrize("batch", [16, 5, 3])
-def test_batched_launch_matches_single_maps(am, batch):
-    """Batched fused launches (one CTA group per pivot, per-slot buffers, group
-    barriers) give the maps of one-pivot launches bit for bit, including a ragged
-    last group and more pivots than groups."""
+@pytest.mark.parametrize("batch,diag", [(16, 0), (5, 0), (3, 0), (64, 0), (16, 8), (3, 8)])
+def test_batched_launch_matches_single_maps(am, batch, diag):
+    """Batched launches give the maps of one-pivot launches bit for bit: the
+    phase-by-phase path (blockIdx.y = pivot, per-slot buffers; chunks of
+    `batch` pivots with a ragged last chunk) and, with AM_OPT_DIAG bit 3, the
+    single cooperative launch whose CTA groups take pivots from a queue."""
     cfg = scenes.CONFIGS["C2"]
     C, H = cfg.leaves()
     P = cfg.pivots(11)
     ctx = _ctx(am, cfg, C, H)
     single = np.stack([ctx.compute(p)[0] for p in P])
+    ctx.set_option(am.binding.OPT_DIAG, diag)
     ctx.set_option(am.binding.OPT_BATCH, batch)
     assert np.array_equal(ctx.compute_batch(P), single)
     assert np.array_equal(ctx.compute_batch(P[::-1]), single[::-1])  # slots see other pivots

@@ -22,7 +22,7 @@ for w in $WHAT; do
     bench2)
       timeout 900 python bench.py --config C2 --baseline --no-cpu-baseline > $OUT/bench_c2_$TAG.log 2>&1; echo "bench2 rc=$?"; tail -c 2500 $OUT/bench_c2_$TAG.log ;;
     launches)
-      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -s 40 -c 60 --csv \
+      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -s 70 -c 40 --csv \
         --log-file $OUT/launches_$TAG.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/launches_$TAG.log 2>&1
       echo "launches rc=$?" ;;
     full)

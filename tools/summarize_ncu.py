@@ -1,6 +1,6 @@
 """Summarise an ncu capture + launch list into profiles/ (run here, no GPU needed).
 
-    python tools/summarize_ncu.py <tag> [config]
+    python tools/summarize_ncu.py <tag> [config] [maps per captured launch]
 reads gpurun_out/prof_<tag>.ncu-rep and gpurun_out/launches_<tag>.csv, writes
 profiles/<tag>_launches.txt, profiles/<tag>_<kernel>_ncu.txt and merges each captured
 kernel's DRAM bytes into profiles/ncu_summary.json, which bench.py reads for `traffic`.
@@ -10,10 +10,17 @@ import io
 import json
 import os
 import subprocess
+import re
 import sys
 from collections import OrderedDict, defaultdict
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def base_name(k):
+    """'void am::am_pipeline_kernel<(bool)1>(am::FusedParams)' -> 'am_pipeline_kernel'."""
+    k = re.sub(r"<.*>", "", k.split("(")[0] if "<" not in k.split("(")[0] else k[:k.index("<")])
+    return k.replace("void ", "").split("::")[-1].strip()
 
 
 def ncu_csv(rep, page):
@@ -24,6 +31,7 @@ def ncu_csv(rep, page):
 def main():
     tag = sys.argv[1]
     config = sys.argv[2] if len(sys.argv) > 2 else "C3"
+    maps = int(sys.argv[3]) if len(sys.argv) > 3 else 1  # AMs computed by the captured launch
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
     lc = os.path.join(ROOT, "gpurun_out", f"launches_{tag}.csv")
@@ -37,7 +45,7 @@ def main():
         for r in rows[start + 1:]:
             if len(r) < len(hdr):
                 continue
-            name = r[ix["Kernel Name"]].split("(")[0]
+            name = base_name(r[ix["Kernel Name"]])
             v = float(r[ix["Metric Value"]].replace(",", ""))
             per[name].append(v)
             seq.append((name, r[ix["Grid Size"]], v))
@@ -58,7 +66,7 @@ def main():
     kernels = OrderedDict()
     for r in det[1:]:
         d = dict(zip(h, r))
-        key = (d["ID"], d["Kernel Name"].split("(")[0])
+        key = (d["ID"], base_name(d["Kernel Name"]))
         kernels.setdefault(key, []).append((d["Section Name"], d["Metric Name"], d["Metric Value"], d["Metric Unit"]))
     raw = ncu_csv(rep, "raw")
     rh, ru = raw[0], raw[1]
@@ -91,7 +99,8 @@ def main():
             except Exception:
                 summ = {}
             summ.setdefault("kernels", {})[kname] = {
-                "config": config, "tag": tag, "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+                "config": config, "tag": tag, "maps_per_launch": maps,
+                "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
                 "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full), launch id {kid}"}
             json.dump({"kernels": summ["kernels"]}, open(sp, "w"), indent=1)
 
