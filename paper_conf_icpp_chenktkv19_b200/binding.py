@@ -16,7 +16,8 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libam.so")
+# AM_LIBRARY: an alternative build of the same library (A/B experiments only)
+LIB_PATH = os.environ.get("AM_LIBRARY") or os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5

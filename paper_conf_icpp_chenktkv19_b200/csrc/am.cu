@@ -290,7 +290,7 @@ int configure_launch(am_ctx* ctx) {
     const int sm_rows = (int)((ctx->MW + ((m + 31) >> 5) + 1) * sizeof(uint32_t));
     CK(cudaFuncSetAttribute(bk_cones<BK_L0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_cones<BK_L1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
-    CK(cudaFuncSetAttribute(bk_cones<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_cones<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     CK(cudaFuncSetAttribute(bk_rows<BK_L0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_rows<BK_L1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_rows<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
@@ -580,7 +580,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         bk_bricks<<<grid(ctx->nbricks, 4 * kThreads, 1 << 16), b, 0, s>>>(F);
         bk_voxels<<<grid(1 << 30, 1, ctx->bk_voxel_ctas), b, 0, s>>>(F);
-        bk_cones<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_cone_ctas), b, sm_rows, s>>>(F);
+        bk_cones<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_cone_ctas), b, ctx->smem_fused, s>>>(F);
         bk_rows<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
         bk_band<<<grid(1 << 30, 1, 8), b, 0, s>>>(F);
         CK(cudaGetLastError());

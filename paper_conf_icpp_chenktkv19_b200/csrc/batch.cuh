@@ -26,6 +26,10 @@
 #pragma once
 #include "fused.cuh"
 
+#ifndef AM_LIVE_MIN_BLOCKS
+#define AM_LIVE_MIN_BLOCKS 4  // CTAs per SM the live-voxel stages are compiled for
+#endif
+
 namespace am {
 
 // StreamParams of pivot p (slot p) into shared memory (thread 0; the kernel
@@ -49,16 +53,19 @@ enum { BK_L0 = 0, BK_L1 = 1, BK_LIVE = 2 };
 // Cones of one stage: level 0 (every voxel of the level, inner cones), level 1
 // (filtered against the map, inner cones), or the live voxels (both cones).
 template <int STAGE>
-__global__ void __launch_bounds__(kThreads) bk_cones(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : 1) bk_cones(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) uint32_t smem_bk[];
     __shared__ StreamParams sP;
     __shared__ FusedScratch sc;
     const int p = blockIdx.y;
     pivot_params(sP, F, p, STAGE == BK_L0);
+    __shared__ int sN;
     const StreamParams& P = sP;
     const int m = P.grid.m, MW = m * P.grid.W;
     uint32_t* sAM = smem_bk;
     uint32_t* sRowFull = sAM + MW;
+    float4* sDirs = reinterpret_cast<float4*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_dirs_offset(m, P.grid.W));
+    int nclear = -1;
     unsigned long long n;
     if (STAGE == BK_L0) {
         n = F.n0;
@@ -74,6 +81,7 @@ __global__ void __launch_bounds__(kThreads) bk_cones(const __grid_constant__ Fus
             n = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
         if ((unsigned long long)blockIdx.x * blockDim.x >= n) return;  // CTA-uniform
         fused_seed(P, sAM, sRowFull);
+        if (STAGE == BK_LIVE) nclear = clear_list_cta(sAM, P.grid, P.tab, sDirs, &sN);
     }
     unsigned int* rc = STAGE == BK_L1 ? shift_bytes(F.rec1, p * F.ctr_stride) : P.rec_count;
     unsigned long long* tc = STAGE == BK_L1 ? shift_bytes(F.task1, p * F.ctr_stride) : P.task_count;
@@ -95,7 +103,7 @@ __global__ void __launch_bounds__(kThreads) bk_cones(const __grid_constant__ Fus
                 if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
             } else {
                 const unsigned int vidx = P.live_idx[e];
-                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear);
             }
         }
         emit_cones_cta<STAGE != BK_LIVE>(P, rc, tc, roff, toff, rcap, tcap, nrows, r, counted, &sc,
@@ -106,7 +114,7 @@ __global__ void __launch_bounds__(kThreads) bk_cones(const __grid_constant__ Fus
 // Rows of one stage into the CTA's shared AM (seeded from the map, so rows
 // already full are skipped), then OR-ed into the map.
 template <int STAGE>
-__global__ void __launch_bounds__(kThreads) bk_rows(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : 1) bk_rows(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) uint32_t smem_bk[];
     __shared__ StreamParams sP;
     __shared__ unsigned int sCnt[CT_COUNT];

@@ -467,8 +467,10 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     fused_seed(P, sAM, sRowFull);  // row-full bits of the global AM (unchanged until phase 9)
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 10);
-    // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2)
+    // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2),
+    //     checked against the list of cells still clear
     {
+        const int nclear = clear_list_cta(sAM, P.grid, P.tab, sDirs, &S.n);
         const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
         for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
@@ -477,7 +479,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             ConeRec r;
             if (e < nlive) {
                 const unsigned int vidx = P.live_idx[e];
-                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted);
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear);
             }
             emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
                                   &sc, P.stats + ST_LIVE, sRowFull);

@@ -66,6 +66,7 @@ constexpr float kRadRel = 4e-6f;       // relative sphere-radius guard (x (D + r
 constexpr float kGamGuard = 4e-6f;     // gamma-domain interval guard (rad)
 constexpr float kCellSlack = 1e-4f;    // interval ends, in cells
 constexpr float kRowSlack = 1e-4f;     // phi-row range slack (rad); loop bound only
+constexpr float kClearSlack = 1e-4f;   // cosine slack of the live voxels' clear-cell check (stream.cuh)
 
 // Blocked-angle candidates of a sphere of radius r whose centre is at distance D
 // from the pivot, against ONE cylinder's meridian rectangle [z0, z1] x [0, R]

@@ -212,6 +212,24 @@ __device__ void compact_clear_dirs(const uint32_t* sAM, const GridDev& g, const 
     __syncthreads();
 }
 
+// The cells still clear in sAM as directions in sDirs, by the whole CTA; returns
+// their count, or -1 (and no list) when there are more than kMapDirs.
+__device__ int clear_list_cta(const uint32_t* sAM, const GridDev& g, const float* __restrict__ tab, float4* sDirs,
+                              int* sN) {
+    const int MW = g.m * g.W;
+    __syncthreads();
+    if (threadIdx.x == 0) *sN = 0;
+    __syncthreads();
+    int cnt = 0;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) cnt += __popc(~sAM[w] & row_word_mask(w % g.W, g.n));
+    if (cnt) atomicAdd(sN, cnt);
+    __syncthreads();
+    const int total = *sN;
+    if (total > kMapDirs) return -1;
+    compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
+    return total;
+}
+
 // The clear-direction map of `gam` into V (6 T^2 texels), computed by the CTAs
 // gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
 // (kMapDirs), sN.

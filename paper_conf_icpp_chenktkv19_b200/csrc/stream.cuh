@@ -301,9 +301,17 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
 // checked against the clear-direction map, the phi-row range.  Returns the
 // number of phi-rows to rasterise (0: nothing to do) and fills r.  `counted`
 // tells whether the voxel reached the cone computation (am_stats voxels_live).
+//
+// With a list of the cells still clear (clear[0, nclear), nclear >= 0) the
+// exact cones are also checked against it: a voxel none of whose relevant
+// cells (outer cone, minus the inside of a ring) is still clear cannot change
+// the map -- its inner cone lies in blocked cells and its band cells are
+// blocked -- so it is dropped before any row is emitted.  The slack covers the
+// raster's own interval slack, so the check never drops a voxel the raster
+// would use.
 template <bool COARSE>
 __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, unsigned int vidx, ConeRec& r,
-                                             bool& counted) {
+                                             bool& counted, const float4* clear = nullptr, int nclear = -1) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
     counted = false;
@@ -324,6 +332,21 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
     if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
+    if (nclear >= 0) {
+        const float inv = 1.f / D;
+        const float ux = vx * inv, uy = vy * inv, uz = vz * inv;
+        const float lo = c.cout - kClearSlack, hi = c.clo + kClearSlack;
+        bool any = false;
+        for (int e = 0; e < nclear; ++e) {
+            const float4 d = clear[e];
+            const float cd = fmaf(ux, d.x, fmaf(uy, d.y, uz * d.z));
+            if (cd >= lo && cd <= hi) {
+                any = true;
+                break;
+            }
+        }
+        if (!any) return 0;
+    }
     const float rxy = sqrtf(vx * vx + vy * vy);
     const float phv = atan2f(rxy, vz);
     const float ao = acosf(fmaxf(c.cout, -1.f));
