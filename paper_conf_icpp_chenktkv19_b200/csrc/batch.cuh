@@ -26,8 +26,15 @@
 #pragma once
 #include "fused.cuh"
 
+// CTAs per SM each stage is compiled for (register budget vs occupancy)
 #ifndef AM_LIVE_MIN_BLOCKS
-#define AM_LIVE_MIN_BLOCKS 4  // CTAs per SM the live-voxel stages are compiled for
+#define AM_LIVE_MIN_BLOCKS 6
+#endif
+#ifndef AM_LEVEL_ROWS_MIN_BLOCKS
+#define AM_LEVEL_ROWS_MIN_BLOCKS 8
+#endif
+#ifndef AM_LEVEL_CONES_MIN_BLOCKS
+#define AM_LEVEL_CONES_MIN_BLOCKS 8
 #endif
 
 namespace am {
@@ -53,7 +60,7 @@ enum { BK_L0 = 0, BK_L1 = 1, BK_LIVE = 2 };
 // Cones of one stage: level 0 (every voxel of the level, inner cones), level 1
 // (filtered against the map, inner cones), or the live voxels (both cones).
 template <int STAGE>
-__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : 1) bk_cones(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM_LEVEL_CONES_MIN_BLOCKS) bk_cones(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) uint32_t smem_bk[];
     __shared__ StreamParams sP;
     __shared__ FusedScratch sc;
@@ -114,7 +121,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : 1)
 // Rows of one stage into the CTA's shared AM (seeded from the map, so rows
 // already full are skipped), then OR-ed into the map.
 template <int STAGE>
-__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : 1) bk_rows(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM_LEVEL_ROWS_MIN_BLOCKS) bk_rows(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) uint32_t smem_bk[];
     __shared__ StreamParams sP;
     __shared__ unsigned int sCnt[CT_COUNT];
