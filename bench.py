@@ -271,8 +271,9 @@ def run_ours(args):
 
     # ---- timed region: K steps of `bsz` pivots each (one am_compute_batch call, one fused
     #      launch), L2 flushed before each step, CUDA events on the launching stream
-    ctx.set_option(B.OPT_KERNEL_TIMING, 1)
+    ctx.set_option(B.OPT_KERNEL_TIMING, 2)  # events around the batch AND after every kernel launch
     ctx.kernel_time()
+    ctx.kernel_stats()
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
@@ -282,6 +283,8 @@ def run_ours(args):
         dist.barrier()
     torch.cuda.synchronize(dev)
     kms, klaunch = ctx.kernel_time()
+    kstats = {k: v for k, v in ctx.kernel_stats().items() if v[1] > 0}
+    ctx.set_option(B.OPT_KERNEL_TIMING, 1)
     # single-pivot latency (am_compute, one fused launch per map), flushed: detail
     ks = max(1, min(args.steps, 100))
     ms_single, _ = _timed_maps(ctx, piv, out, stream, ks, flush, torch, 1)
@@ -327,6 +330,7 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max, e2e_max, kavg_ms = t.tolist()
     maps = args.steps * bsz * ws
+    maps_rank = args.steps * bsz
     tests_per_map = float(N) * cfg.m * cfg.n
     value = tests_per_map * maps / (ms_max / 1e3)
     e2e_value = tests_per_map * ke * bsz * ws / e2e_max
@@ -337,7 +341,8 @@ def run_ours(args):
     achieved = alg_bytes / (kavg_ms / 1e3) / 1e9
     # bytes the fused kernel actually needs: brick spheres, kept bricks' voxels, both map levels
     touched = bsz * (16.0 * (ctx_nbricks(N) + mean["voxels_streamed"] + mean["level_voxels"]) + cfg.m * cfg.n / 8.0)
-    traffic, traffic_tag = _ncu_traffic(cfg.name, "am_pipeline_kernel", bsz)
+    dom_roof = _dominant_roofline(kstats, mean, cfg, N, bsz, peak, peak_src,
+                                  clk.summary().get("sm_max_mhz"))
     baseline_ms = None
     if args.baseline and rank == 0:
         ctx.set_option(B.OPT_BASELINE_REJECT, 1)
@@ -359,7 +364,7 @@ def run_ours(args):
         full_roof = None
         if full:
             fa = 16.0 * N / (full["kernel_ms_avg"] / 1e3) / 1e9
-            ft, ftag = _ncu_traffic(cfg.name, "filter_kernel")
+            ft, ftag = _ncu_traffic(cfg.name, "filter")
             full_roof = {"kernel": "filter_kernel", "bound": "hbm", "achieved": fa, "peak": peak, "unit": "GB/s",
                          "frac": fa / peak, "traffic": ft, "traffic_tag": ftag,
                          "kernel_ms_avg": full["kernel_ms_avg"], "algorithmic_bytes_per_launch": 16.0 * N,
@@ -371,15 +376,16 @@ def run_ours(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": _config_dict(cfg, N, flush is not None, bsz, args.slots),
             "ms_per_am": ms_max / args.steps / bsz,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "traffic_tag": traffic_tag,
-                         "kernel": "am_pipeline_kernel", "kernel_ms_avg": kavg_ms, "maps_per_launch": bsz,
-                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
-                         "touched_bytes_per_launch": touched,
-                         "touched_gbs": touched / (kavg_ms / 1e3) / 1e9,
-                         "note": "achieved = SURVEY 8(d) algorithmic bytes (16 N + m n / 8 per map, maps_per_launch "
-                                 "maps) / kernel time; the kernel skips most of them (touched_bytes, traffic), so "
-                                 "frac is the speed relative to one full HBM pass per map, not bandwidth use"},
+            "roofline": dom_roof,
+            "step_roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                              "frac": achieved / peak, "kernel": "the whole batch (all launches of one step)",
+                              "ms_per_launch_chain": kavg_ms, "maps_per_launch": bsz,
+                              "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+                              "touched_bytes_per_launch": touched,
+                              "touched_gbs": touched / (kavg_ms / 1e3) / 1e9,
+                              "note": "SURVEY 8(d): algorithmic bytes 16 N + m n / 8 per map over the step's "
+                                      "device time; the method skips most of them (touched_bytes), so frac is "
+                                      "the speed relative to one full HBM pass per map, not bandwidth use"},
             "full_scan_roofline": full_roof,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 12 * bsz,
                     "d2h_bytes_per_step": 4 * ctx.words * bsz,
@@ -387,7 +393,10 @@ def run_ours(args):
                     "note": f"am_compute_batch with {bsz} host pivots (12 B each, copied into the launch) and a "
                             "host AM buffer; synchronous per step; voxels resident (upload excluded, PAPER.md L313); "
                             "L2 flushed before each step, outside the per-step clock"},
-            "gpu_launches": klaunch,
+            "gpu_launches": int(sum(v[1] for v in kstats.values())),
+            "kernels": {k: {"ms_per_am": v[0] / maps_rank, "launches": v[1],
+                            "share": v[0] / max(sum(x[0] for x in kstats.values()), 1e-12)}
+                        for k, v in sorted(kstats.items(), key=lambda kv: -kv[1][0])},
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
             "detail": {"stats_mean_over_pivots": mean, "upload_s": upload_s, "scene_gen_s": gen_s,
@@ -404,6 +413,53 @@ def run_ours(args):
     if dist:
         dist.destroy_process_group()
     return 0
+
+
+# Kernels whose work is a read of voxel records (16 B per voxel):
+# units per map from the per-pivot stats.  Every other kernel is an ALU/issue-bound
+# search over cones, rows, texels or band pairs.
+def _hbm_units(name, mean, N, n_levels):
+    return {"voxels": mean["voxels_streamed"], "bricks": float(ctx_nbricks(N)),
+            "filter": float(N)}.get(name)
+
+
+def _dominant_roofline(kstats, mean, cfg, N, bsz, peak_gbs, peak_src, sm_max_mhz):
+    """Roofline of the kernel with the largest share of the live per-kernel device time
+    (CUDA events after every launch on the launching stream, AM_OPT_KERNEL_TIMING = 2)."""
+    tot = sum(v[0] for v in kstats.values())
+    if not kstats or tot <= 0:
+        return None
+    name, (ms, launches) = max(kstats.items(), key=lambda kv: kv[1][0])
+    t_launch = ms / launches / 1e3  # s per launch (one launch = bsz maps in the batched path)
+    maps = bsz if name not in ("fused_pipeline", "filter") else 1
+    traffic, tag = _ncu_traffic(cfg.name, name, maps)
+    u = _hbm_units(name, mean, N, 0)
+    base = {"kernel": name, "share_of_step": ms / tot, "launches": launches,
+            "ms_per_launch": t_launch * 1e3, "maps_per_launch": maps, "traffic": traffic, "traffic_tag": tag}
+    if u is not None:
+        by = 16.0 * u * maps
+        a = by / t_launch / 1e9
+        base.update({"bound": "hbm", "achieved": a, "peak": peak_gbs, "unit": "GB/s", "frac": a / peak_gbs,
+                     "algorithmic_bytes_per_launch": by, "peak_source": peak_src,
+                     "note": "16 B per voxel record the launch reads (SURVEY 8(d)) / live launch time"})
+        return base
+    # ALU/issue roofline: 148 SMs x 4 schedulers x 1 warp-instruction per clock (DESIGN.md 6)
+    mhz = sm_max_mhz or 1965
+    pk = 148 * 4 * mhz * 1e6 / 1e9
+    inst = None
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))["kernels"].get(name)
+        if d and d.get("config") == cfg.name and d.get("warp_inst_per_launch"):
+            inst = d["warp_inst_per_launch"] * maps / d.get("maps_per_launch", 1)
+    except Exception:
+        pass
+    a = inst / t_launch / 1e9 if inst else None
+    base.update({"bound": "alu", "achieved": a, "peak": pk, "unit": "Gwarp-inst/s",
+                 "frac": (a / pk) if a else None, "warp_inst_per_launch": inst,
+                 "peak_source": f"derived: 148 SM x 4 schedulers x {mhz} MHz (B200_PROFILING.md unit counts)",
+                 "note": "data-dependent search (no dense contraction, no per-voxel HBM stream): achieved = "
+                         "warp instructions per launch (ncu --set full, committed profile) / live launch time"})
+    return base
 
 
 def ctx_nbricks(N):

@@ -81,7 +81,9 @@ enum {
     AM_OPT_MORTON_SORT = 3,      /* 1 = Morton-sort voxels at upload (default), 0 = keep order   */
     AM_OPT_BASELINE_REJECT = 4,  /* 1 = baseline uses an exact-safe bounding-sphere reject        */
     AM_OPT_BAND_QUEUE = 5,       /* capacity of the deferred band queue, in (voxel, cell) pairs  */
-    AM_OPT_KERNEL_TIMING = 6,    /* 1 = bracket every full-stream kernel launch with CUDA events */
+    AM_OPT_KERNEL_TIMING = 6,    /* 1 = bracket every full-stream kernel launch with CUDA events;
+                                    2 = also one event after every kernel launch (per-kernel
+                                    device times, am_kernel_stats)                              */
     AM_OPT_PHASES = 7,           /* 1 = coarse levels + clear-direction map before the full
                                     stream (default); 0 = one plain stream.  Same map either way */
     AM_OPT_DIAG = 8,             /* diagnostics, 0 in production: bit 0 = stop after the coarse
@@ -99,6 +101,25 @@ enum {
     AM_OPT_BATCH = 12            /* am_compute_batch: pivots computed together, phase by phase,
                                     one launch per phase (1..64, default 32; each needs its own
                                     per-map buffers, ~4 N + 100 MB of device memory).  Same maps */
+};
+
+/* Kernels of the library, for am_kernel_stats. */
+enum {
+    AM_K_L0_CONES = 0,  /* level-0 (largest voxels) inner cones, a3-a4                        */
+    AM_K_L0_ROWS,       /* their phi-rows, a5                                                  */
+    AM_K_CLEAR_MAP,     /* clear-direction map of the partial AM                 */
+    AM_K_L1_CONES,      /* level-1 filter + inner cones                                        */
+    AM_K_L1_ROWS,       /* their rows                                                          */
+    AM_K_BRICKS,        /* brick bounding-sphere test, a1-a2 (8(f) NEXT 1)                     */
+    AM_K_VOXELS,        /* kept bricks' voxels through the filter -> live list, a1-a3          */
+    AM_K_LIVE_CONES,    /* live voxels' inner + outer cones, a3-a4                             */
+    AM_K_LIVE_ROWS,     /* their rows + band queue, a5-a7                                      */
+    AM_K_BAND,          /* exact CHECKBOX of queued band pairs still clear, a6                 */
+    AM_K_FUSED,         /* am_pipeline_kernel: every step of a map in one cooperative launch   */
+    AM_K_FILTER,        /* full-stream filter of every voxel (AM_OPT_BRICKS = 0)               */
+    AM_K_BASELINE,      /* all-pairs CHECKBOX baseline, a9                                     */
+    AM_K_LAYOUT,        /* am_unpack_cells / am_pack_cells                                     */
+    AM_K_COUNT
 };
 
 /*
@@ -166,6 +187,20 @@ int am_set_option(am_ctx* ctx, int key, int64_t value);
  * must be non-NULL.
  */
 int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches);
+
+/*
+ * Per-kernel accounting since the previous call, indexed by AM_K_*: ms[k] =
+ * device time of kernel k's launches (only while AM_OPT_KERNEL_TIMING = 2,
+ * else 0: consecutive CUDA events on the launching stream, one after every
+ * launch, so a launch's interval also holds the gap before it), launches[k] =
+ * how many times kernel k was launched by any call (counted always).  Both
+ * arrays hold AM_K_COUNT entries, caller-owned.  Waits for the recorded
+ * events, then resets.  AM_EINVAL for NULL outputs.
+ */
+int am_kernel_stats(am_ctx* ctx, double* ms, int64_t* launches);
+
+/* Name of kernel k (static string), NULL if k is not an AM_K_* value. */
+const char* am_kernel_name(int k);
 
 /*
  * Layout conversion on the device, for the voxel-sharded multi-GPU combine

@@ -21,11 +21,12 @@ LIB_PATH = os.environ.get("AM_LIBRARY") or os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
+K_COUNT = 14  # AM_K_COUNT (include/am.h)
 OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",
-           "am_set_option", "am_kernel_time", "am_unpack_cells", "am_pack_cells", "am_words_per_map",
+           "am_set_option", "am_kernel_time", "am_kernel_stats", "am_kernel_name", "am_unpack_cells", "am_pack_cells", "am_words_per_map",
            "am_num_voxels", "am_last_error", "am_destroy")
 
 if not os.path.exists(LIB_PATH):
@@ -78,6 +79,10 @@ lib.am_set_option.restype = ctypes.c_int
 lib.am_set_option.argtypes = [_P, ctypes.c_int, ctypes.c_int64]
 lib.am_kernel_time.restype = ctypes.c_int
 lib.am_kernel_time.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+lib.am_kernel_stats.restype = ctypes.c_int
+lib.am_kernel_stats.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+lib.am_kernel_name.restype = ctypes.c_char_p
+lib.am_kernel_name.argtypes = [ctypes.c_int]
 lib.am_unpack_cells.restype = ctypes.c_int
 lib.am_unpack_cells.argtypes = [_P, _P, _P, _P]
 lib.am_pack_cells.restype = ctypes.c_int
@@ -90,6 +95,9 @@ lib.am_last_error.restype = ctypes.c_char_p
 lib.am_last_error.argtypes = [_P]
 lib.am_destroy.restype = None
 lib.am_destroy.argtypes = [_P]
+
+
+KERNEL_NAMES = tuple(lib.am_kernel_name(k).decode() for k in range(K_COUNT))
 
 
 def exported_symbols():
@@ -178,6 +186,14 @@ class Context:
         n = ctypes.c_int64()
         self._check(lib.am_kernel_time(self._h, ctypes.byref(ms), ctypes.byref(n)))
         return ms.value, n.value
+
+    def kernel_stats(self):
+        """am_kernel_stats: {kernel name: (device ms, launches)} since the last call
+        (ms only while OPT_KERNEL_TIMING = 2)."""
+        ms = (ctypes.c_double * K_COUNT)()
+        n = (ctypes.c_int64 * K_COUNT)()
+        self._check(lib.am_kernel_stats(self._h, ms, n))
+        return {KERNEL_NAMES[k]: (ms[k], n[k]) for k in range(K_COUNT)}
 
     def _dev_stream(self, t, stream):
         if not _is_torch_cuda(t):

@@ -82,6 +82,14 @@ struct am_ctx {
     int timing = 0;
     std::vector<cudaEvent_t> ev_start, ev_stop;
     size_t ev_used = 0;
+    // per-kernel accounting (am_kernel_stats): launches always, device time
+    // while AM_OPT_KERNEL_TIMING = 2 (an event after every launch, chained)
+    long long k_launches[AM_K_COUNT] = {};
+    std::vector<cudaEvent_t> kev;          // event pool
+    size_t kev_used = 0;
+    long long kev_prev = -1;               // chain: event recorded before the next launch
+    std::vector<std::pair<int, size_t>> kmarks;  // (kernel, index of its end event)
+    std::vector<size_t> kmark_begin;
     std::string err;
 };
 
@@ -123,6 +131,9 @@ int fail(am_ctx* c, int code, const char* fmt, ...) {
                         #call, cudaGetErrorString(e_), __FILE__, __LINE__);                  \
         }                                                                                     \
     } while (0)
+
+int kchain(am_ctx* ctx, cudaStream_t s);
+int kmark(am_ctx* ctx, cudaStream_t s, int k);
 
 // Restores the caller's current device on scope exit.
 struct DeviceGuard {
@@ -308,16 +319,18 @@ int launch_cones_rows(am_ctx* ctx, StreamParams p, bool coarse, int stage, cudaS
     p.task_cap = kTaskCap;
     const unsigned int gc = (unsigned int)(ctx->sms * 8);
     const unsigned int gr = (unsigned int)(ctx->sms * kLiveBlocksPerSM);
+    int rc;
     if (coarse) {
         cone_kernel<true><<<gc, kThreads, 0, s>>>(p);
-        CK(cudaGetLastError());
+        if ((rc = kmark(ctx, s, stage == 0 ? AM_K_L0_CONES : AM_K_L1_CONES))) return rc;
         row_kernel<true><<<gr, kThreads, ctx->smem, s>>>(p);
+        if ((rc = kmark(ctx, s, stage == 0 ? AM_K_L0_ROWS : AM_K_L1_ROWS))) return rc;
     } else {
         cone_kernel<false><<<gc, kThreads, 0, s>>>(p);
-        CK(cudaGetLastError());
+        if ((rc = kmark(ctx, s, AM_K_LIVE_CONES))) return rc;
         row_kernel<false><<<gr, kThreads, ctx->smem, s>>>(p);
+        if ((rc = kmark(ctx, s, AM_K_LIVE_ROWS))) return rc;
     }
-    CK(cudaGetLastError());
     return AM_OK;
 }
 
@@ -358,12 +371,15 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
         if (gb > gmax) gb = gmax;
         if (gb < 1) gb = 1;
         brick_test_kernel<<<(unsigned)gb, kThreads, 0, s>>>(p);
-        CK(cudaGetLastError());
+        int rc;
+        if ((rc = kmark(ctx, s, AM_K_BRICKS))) return rc;
         brick_voxels_kernel<<<(unsigned)gmax, kThreads, 0, s>>>(p);
+        if ((rc = kmark(ctx, s, AM_K_VOXELS))) return rc;
     } else {
         filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
+        int rc;
+        if ((rc = kmark(ctx, s, AM_K_FILTER))) return rc;
     }
-    CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(ctx->ev_stop[ctx->ev_used++], s));
     return launch_cones_rows(ctx, p, coarse, coarse ? 1 : 2, s);
 }
@@ -387,8 +403,7 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
     const int gcm = std::max(1, std::min(ctx->sms * 4, (ntex / 16 + 7) / 8));
     clear_map_kernel<<<gcm, 256, ctx->smem_cmap, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_texels, ctx->cmapT,
                                                       ctx->d_cmap);
-    CK(cudaGetLastError());
-    return AM_OK;
+    return kmark(ctx, s, AM_K_CLEAR_MAP);
 }
 
 // One AICA map into device buffer gam (asynchronous on s):
@@ -463,6 +478,46 @@ int timed_end(am_ctx* ctx, cudaStream_t s) {
     return AM_OK;
 }
 
+// Per-kernel accounting.  kchain(): start a chain of launches on s (records an
+// event when timing per kernel).  kmark(k): one launch of kernel k just went
+// onto s -- counts it and, when timing per kernel, records the event that ends
+// it (the previous event of the chain starts it; launches on one stream run in
+// order, so the interval is that kernel's device time plus the gap between).
+int kpool_event(am_ctx* ctx, size_t* idx) {
+    if (ctx->kev_used == ctx->kev.size()) {
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e));
+        ctx->kev.push_back(e);
+    }
+    *idx = ctx->kev_used++;
+    return AM_OK;
+}
+
+int kchain(am_ctx* ctx, cudaStream_t s) {
+    ctx->kev_prev = -1;
+    if (ctx->timing != 2) return AM_OK;
+    size_t i;
+    int rc = kpool_event(ctx, &i);
+    if (rc) return rc;
+    CK(cudaEventRecord(ctx->kev[i], s));
+    ctx->kev_prev = (long long)i;
+    return AM_OK;
+}
+
+int kmark(am_ctx* ctx, cudaStream_t s, int k) {
+    CK(cudaGetLastError());
+    ctx->k_launches[k] += 1;
+    if (ctx->timing != 2 || ctx->kev_prev < 0) return AM_OK;
+    size_t i;
+    int rc = kpool_event(ctx, &i);
+    if (rc) return rc;
+    CK(cudaEventRecord(ctx->kev[i], s));
+    ctx->kmarks.emplace_back(k, i);
+    ctx->kmark_begin.push_back((size_t)ctx->kev_prev);
+    ctx->kev_prev = (long long)i;
+    return AM_OK;
+}
+
 // One map (pivot) into gam with one fused cooperative launch over the whole grid.
 int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s) {
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
@@ -470,9 +525,11 @@ int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s)
     FusedParams F = fused_params(ctx, pivot, gam);
     int rc;
     if ((rc = timed_begin(ctx, s))) return rc;
+    if ((rc = kchain(ctx, s))) return rc;
     void* args[] = {&F};
     CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads), args,
                                    ctx->smem_fused, s));
+    if ((rc = kmark(ctx, s, AM_K_FUSED))) return rc;
     if ((rc = timed_end(ctx, s))) return rc;
     if (ctx->d_prev)
         CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
@@ -517,9 +574,11 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     F.cur = F.qnext + 1;                                             // kMaxSlots words
     int rc;
     if ((rc = timed_begin(ctx, s))) return rc;
+    if ((rc = kchain(ctx, s))) return rc;
     void* args[] = {&F};
     CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<true>, dim3(ctx->fused_grid), dim3(kThreads), args,
                                    ctx->smem_fused, s));
+    if ((rc = kmark(ctx, s, AM_K_FUSED))) return rc;
     return timed_end(ctx, s);
 }
 
@@ -565,25 +624,38 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.ctr0 = ctx->d_ctr;
         F.ctr_words = kCtrStride;
         if ((rc = timed_begin(ctx, s))) return rc;
+        if ((rc = kchain(ctx, s))) return rc;
         auto grid = [&](long long items, long long per_cta, int cap) {
             long long gx = (items + per_cta - 1) / per_cta;
             return dim3((unsigned)std::max<long long>(1, std::min<long long>(gx, cap)), (unsigned)kk);
         };
         const dim3 b(kThreads);
+#define AM_KM(k) if ((rc = kmark(ctx, s, k))) return rc
         bk_cones<BK_L0><<<grid(ctx->n_l0, kThreads, 1 << 16), b, sm_rows, s>>>(F);
+        AM_KM(AM_K_L0_CONES);
         bk_rows<BK_L0><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        AM_KM(AM_K_L0_ROWS);
         bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
             bk_cones<BK_L1><<<grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), b, sm_rows, s>>>(F);
+            AM_KM(AM_K_L1_CONES);
             bk_rows<BK_L1><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+            AM_KM(AM_K_L1_ROWS);
             bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+            AM_KM(AM_K_CLEAR_MAP);
         }
         bk_bricks<<<grid(ctx->nbricks, 4 * kThreads, 1 << 16), b, 0, s>>>(F);
+        AM_KM(AM_K_BRICKS);
         bk_voxels<<<grid(1 << 30, 1, ctx->bk_voxel_ctas), b, 0, s>>>(F);
+        AM_KM(AM_K_VOXELS);
         bk_cones<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_cone_ctas), b, ctx->smem_fused, s>>>(F);
+        AM_KM(AM_K_LIVE_CONES);
         bk_rows<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        AM_KM(AM_K_LIVE_ROWS);
         bk_band<<<grid(1 << 30, 1, 8), b, 0, s>>>(F);
-        CK(cudaGetLastError());
+        AM_KM(AM_K_BAND);
+#undef AM_KM
         if ((rc = timed_end(ctx, s))) return rc;
     }
     return AM_OK;
@@ -596,6 +668,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     if (ctx->N == 0) return AM_OK;
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
+    if ((rc = kchain(ctx, s))) return rc;
     const float* cm = ctx->d_cmap_ones;
     if (ctx->diag & 2) {
         // diagnostic: clear map from the previous map computed on this context
@@ -619,7 +692,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     if (!(ctx->diag & 1)) {
         if ((rc = launch_stream(ctx, p, ctx->d_vox, ctx->N, cm, true, s))) return rc;
         band_exact_kernel<<<(unsigned)ctx->sms, kThreads, 0, s>>>(p);
-        CK(cudaGetLastError());
+        if ((rc = kmark(ctx, s, AM_K_BAND))) return rc;
     }
     if (ctx->d_prev)  // allocated once diagnostics were enabled
         CK(cudaMemcpyAsync(ctx->d_prev, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
@@ -1058,8 +1131,10 @@ int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int
         const int ncell = ctx->grid.m * ctx->grid.n;
         int g = ctx->sms * 8;
         if (g > ncell) g = ncell;
+        int rc;
+        if ((rc = kchain(ctx, s))) return rc;
         baseline_kernel<<<g, kThreads, 0, s>>>(p, ctx->baseline_reject);
-        CK(cudaGetLastError());
+        if ((rc = kmark(ctx, s, AM_K_BASELINE))) return rc;
     }
     if (!dst_is_device) {
         CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
@@ -1092,7 +1167,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value < 1 || value > (1LL << 28)) return fail(ctx, AM_EINVAL, "band queue out of range");
         return ensure_queue(ctx, value);
     case AM_OPT_KERNEL_TIMING:
-        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "kernel_timing must be 0 or 1");
+        if (value < 0 || value > 2) return fail(ctx, AM_EINVAL, "kernel_timing must be 0, 1 or 2");
         ctx->timing = (int)value;
         return AM_OK;
     case AM_OPT_PHASES:
@@ -1164,12 +1239,43 @@ int am_kernel_time(am_ctx* ctx, double* total_ms, int64_t* launches) {
     return AM_OK;
 }
 
+int am_kernel_stats(am_ctx* ctx, double* ms, int64_t* launches) {
+    if (!ctx) return AM_EINVAL;
+    if (!ms || !launches) return fail(ctx, AM_EINVAL, "NULL output");
+    DeviceGuard dg(ctx->device);
+    for (int k = 0; k < AM_K_COUNT; ++k) {
+        ms[k] = 0.0;
+        launches[k] = (int64_t)ctx->k_launches[k];
+        ctx->k_launches[k] = 0;
+    }
+    for (size_t j = 0; j < ctx->kmarks.size(); ++j) {
+        float t = 0.f;
+        CK(cudaEventSynchronize(ctx->kev[ctx->kmarks[j].second]));
+        CK(cudaEventElapsedTime(&t, ctx->kev[ctx->kmark_begin[j]], ctx->kev[ctx->kmarks[j].second]));
+        ms[ctx->kmarks[j].first] += t;
+    }
+    ctx->kmarks.clear();
+    ctx->kmark_begin.clear();
+    ctx->kev_used = 0;
+    ctx->kev_prev = -1;
+    return AM_OK;
+}
+
+const char* am_kernel_name(int k) {
+    static const char* names[AM_K_COUNT] = {
+        "l0_cones", "l0_rows", "clear_map", "l1_cones", "l1_rows", "bricks", "voxels",
+        "live_cones", "live_rows", "band", "fused_pipeline", "filter", "baseline", "layout"};
+    return (k >= 0 && k < AM_K_COUNT) ? names[k] : nullptr;
+}
+
 int am_unpack_cells(am_ctx* ctx, const uint32_t* words, uint8_t* cells, void* cuda_stream) {
     if (!ctx) return AM_EINVAL;
     if (!words || !cells) return fail(ctx, AM_EINVAL, "NULL buffer");
     DeviceGuard dg(ctx->device);
     const int nc = ctx->grid.m * ctx->grid.n;
+    if (kchain(ctx, (cudaStream_t)cuda_stream)) return AM_ECUDA;
     unpack_cells_kernel<<<(nc + 255) / 256, 256, 0, (cudaStream_t)cuda_stream>>>(words, ctx->grid, cells);
+    if (kmark(ctx, (cudaStream_t)cuda_stream, AM_K_LAYOUT)) return AM_ECUDA;
     CK(cudaGetLastError());
     return AM_OK;
 }
@@ -1178,7 +1284,9 @@ int am_pack_cells(am_ctx* ctx, const uint8_t* cells, uint32_t* words, void* cuda
     if (!ctx) return AM_EINVAL;
     if (!words || !cells) return fail(ctx, AM_EINVAL, "NULL buffer");
     DeviceGuard dg(ctx->device);
+    if (kchain(ctx, (cudaStream_t)cuda_stream)) return AM_ECUDA;
     pack_cells_kernel<<<(ctx->MW + 255) / 256, 256, 0, (cudaStream_t)cuda_stream>>>(cells, ctx->grid, words);
+    if (kmark(ctx, (cudaStream_t)cuda_stream, AM_K_LAYOUT)) return AM_ECUDA;
     CK(cudaGetLastError());
     return AM_OK;
 }
@@ -1215,6 +1323,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_ts);
     cudaFree(ctx->d_piv);
     cudaFree(ctx->d_bctl);
+    for (auto e : ctx->kev) cudaEventDestroy(e);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
     cudaGetLastError();

@@ -23,7 +23,7 @@ def _declared():
 
 def test_header_symbols_exported(am):
     declared = _declared()
-    assert len(declared) == 13
+    assert len(declared) == 15
     lib = ctypes.CDLL(am.LIB_PATH)
     for s in declared:
         assert hasattr(lib, s), s
@@ -60,6 +60,7 @@ def test_argument_validation_without_gpu(am):
     assert lib.am_compute_baseline(None, None, None, 0, None) == am.AM_EINVAL
     assert lib.am_set_option(None, 1, 0) == am.AM_EINVAL
     assert lib.am_kernel_time(None, None, None) == am.AM_EINVAL
+    assert lib.am_kernel_stats(None, None, None) == am.AM_EINVAL
     assert lib.am_unpack_cells(None, None, None, None) == am.AM_EINVAL
     assert lib.am_pack_cells(None, None, None, None) == am.AM_EINVAL
     assert lib.am_last_error(None) == b"NULL context"
@@ -73,3 +74,14 @@ def test_unpack_layout(am):
     assert u[0, 0] == 1 and u[0, 1] == 0 and u[0, 2] == 1 and u[0, 31] == 0
     assert u[0, 32] == 1  # row 0, word 1, bit 0
     assert u[1, 31] == 1 and u.sum() == 4
+
+
+def test_kernel_names_match_header(am):
+    """binding.K_COUNT / KERNEL_NAMES mirror the AM_K_* enum of include/am.h."""
+    src = open(os.path.join(ROOT, "include", "am.h")).read()
+    body = src[src.index("AM_K_L0_CONES"):src.index("AM_K_COUNT")]
+    names = re.findall(r"\b(AM_K_[A-Z0-9_]+)\b", body)
+    assert len(names) == am.binding.K_COUNT
+    assert len(set(am.binding.KERNEL_NAMES)) == am.binding.K_COUNT
+    assert am.lib.am_kernel_name(am.binding.K_COUNT) is None
+    assert am.lib.am_kernel_name(-1) is None

@@ -282,32 +282,37 @@ def test_batched_launch_matches_single_maps(am, batch, diag):
 def _check_sampled(cfg, C, H, p, g, rng, nclear=64, nblocked=32):
     clear = np.nonzero(g == 0)[0]
     blocked = np.nonzero(g == 1)[0]
-    assert len(clear) > 0 and len(blocked) > 0
+    assert len(clear) + len(blocked) > 0
     cells = np.concatenate([rng.choice(clear, size=min(nclear, len(clear)), replace=False),
-                            rng.choice(blocked, size=min(nblocked, len(blocked)), replace=False)])
+                            rng.choice(blocked, size=min(nblocked, len(blocked)), replace=False)]).astype(np.int64)
     S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n, cells=cells)
     robust = S != 1
     assert (((g[cells] == 1) != (S == 2))[robust]).sum() == 0
 
 
-def test_c3_bench_config_sampled(am):
-    """C3 (~27M leaves) in the launch configuration bench.py times (a batch of
-    8 pivots in one fused launch): every batched map equals its one-pivot map,
-    and every GPU-clear cell (up to 64) plus a seeded sample of blocked cells of
-    two of them match the oracle, one by one."""
+@pytest.mark.parametrize("name,npiv", [("C3", 64), ("C4", 16), ("C5", 64)])
+def test_full_size_bench_launch_config_sampled(am, name, npiv):
+    """Full-size configs in the launch configuration bench.py times (C3: a step of
+    64 pivots with AM_OPT_BATCH = 64, one launch per phase over all of them; C4
+    at 128x128; C5, the impeller of the toolpath-batch config): every batched map
+    equals its one-pivot map bit for bit, and every GPU-clear cell (up to 64)
+    plus a seeded sample of blocked cells of two maps match the fp64 oracle."""
     import torch
-    cfg = scenes.CONFIGS["C3"]
+    cfg = scenes.CONFIGS[name]
     C, H = cfg.leaves()
     ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_BATCH, 64)
     rng = np.random.default_rng(3)
-    P = cfg.pivots(8)
-    out = torch.zeros((8, ctx.words), dtype=torch.int32, device="cuda:0")
+    P = cfg.pivots(npiv)
+    out = torch.zeros((npiv, ctx.words), dtype=torch.int32, device="cuda:0")
     ctx.compute_batch(P, out=out)
     torch.cuda.synchronize()
     batch = out.cpu().numpy().view(np.uint32)
-    for k in range(8):
+    for k in range(npiv):
         assert np.array_equal(batch[k], ctx.compute(P[k])[0]), k
-    for k in (0, 5):
-        g = am.unpack(batch[k], cfg.m, cfg.n).reshape(-1)
-        _check_sampled(cfg, C, H, P[k], g, rng)
+    maps = [am.unpack(b, cfg.m, cfg.n).reshape(-1) for b in batch]
+    nclear = [int((g == 0).sum()) for g in maps]
+    assert max(nclear) > 0  # the path's pivots are not all enclosed
+    for k in (0, int(np.argmax(nclear))):  # the first map and the one with the most clear cells
+        _check_sampled(cfg, C, H, P[k], maps[k], rng)
     ctx.close()

@@ -22,8 +22,9 @@ for w in $WHAT; do
     bench2)
       timeout 900 python bench.py --config C2 --baseline --no-cpu-baseline > $OUT/bench_c2_$TAG.log 2>&1; echo "bench2 rc=$?"; tail -c 2500 $OUT/bench_c2_$TAG.log ;;
     launches)
-      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -s 70 -c 40 --csv \
-        --log-file $OUT/launches_$TAG.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/launches_$TAG.log 2>&1
+      # the default bench command, every launch (the driver's bench line comes from the same command)
+      timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+        --log-file $OUT/launches_$TAG.csv python bench.py > $OUT/launches_$TAG.log 2>&1
       echo "launches rc=$?" ;;
     full)
       timeout 1200 ncu --set full --clock-control none --import-source on -k regex:${KREGEX:-filter_kernel} -s ${KSKIP:-5} -c ${KCOUNT:-1} \

@@ -23,6 +23,23 @@ def base_name(k):
     return k.replace("void ", "").split("::")[-1].strip()
 
 
+_STAGES = {"bk_cones": ("l0_cones", "l1_cones", "live_cones"), "bk_rows": ("l0_rows", "l1_rows", "live_rows")}
+_PLAIN = {"bk_map": "clear_map", "bk_bricks": "bricks", "bk_voxels": "voxels", "bk_band": "band",
+          "am_pipeline_kernel": "fused_pipeline", "filter_kernel": "filter", "baseline_kernel": "baseline",
+          "clear_map_kernel": "clear_map", "band_exact_kernel": "band", "brick_test_kernel": "bricks",
+          "brick_voxels_kernel": "voxels"}
+
+
+def stage_name(full):
+    """Kernel name as am_kernel_name() reports it (AM_K_* of include/am.h), or the base name."""
+    b = base_name(full)
+    if b in _STAGES:
+        m = re.search(r"<\(int\)(\d)>|<(\d)>", full)
+        if m:
+            return _STAGES[b][int(m.group(1) or m.group(2))]
+    return _PLAIN.get(b, b)
+
+
 def ncu_csv(rep, page):
     out = subprocess.run(["ncu", "-i", rep, "--page", page, "--csv"], capture_output=True, text=True).stdout
     return list(csv.reader(io.StringIO(out)))
@@ -45,7 +62,7 @@ def main():
         for r in rows[start + 1:]:
             if len(r) < len(hdr):
                 continue
-            name = base_name(r[ix["Kernel Name"]])
+            name = stage_name(r[ix["Kernel Name"]])
             v = float(r[ix["Metric Value"]].replace(",", ""))
             per[name].append(v)
             seq.append((name, r[ix["Grid Size"]], v))
@@ -66,7 +83,7 @@ def main():
     kernels = OrderedDict()
     for r in det[1:]:
         d = dict(zip(h, r))
-        key = (d["ID"], base_name(d["Kernel Name"]))
+        key = (d["ID"], stage_name(d["Kernel Name"]))
         kernels.setdefault(key, []).append((d["Section Name"], d["Metric Name"], d["Metric Value"], d["Metric Unit"]))
     raw = ncu_csv(rep, "raw")
     rh, ru = raw[0], raw[1]
@@ -98,10 +115,24 @@ def main():
                 summ = json.load(open(sp))
             except Exception:
                 summ = {}
-            summ.setdefault("kernels", {})[kname] = {
-                "config": config, "tag": tag, "maps_per_launch": maps,
-                "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
-                "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full), launch id {kid}"}
+            ent = {"config": config, "tag": tag, "maps_per_launch": maps,
+                   "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+                   "source": f"gpurun_out/prof_{tag}.ncu-rep (ncu --set full), launch id {kid}"}
+            for sec, name, val, unit in mets:
+                if name == "Executed Instructions" and unit == "inst":
+                    ent["warp_inst_per_launch"] = float(val.replace(",", ""))
+            if "gpu__time_duration.sum" in rawrow:
+                ent["ncu_duration_us"] = tobytes(rawrow["gpu__time_duration.sum"], "") / (
+                    1e3 if rawu.get("gpu__time_duration.sum") == "nsecond" else 1)
+            old = summ.get("kernels", {}).get(kname)
+            if old and old.get("tag") == tag:  # same stage captured twice (clear_map): average
+                for k2 in ("dram_bytes_per_launch", "dram_read", "dram_write", "warp_inst_per_launch",
+                           "ncu_duration_us"):
+                    if k2 in ent and k2 in old:
+                        n_ = old.get("launches_averaged", 1)
+                        ent[k2] = (old[k2] * n_ + ent[k2]) / (n_ + 1)
+                ent["launches_averaged"] = old.get("launches_averaged", 1) + 1
+            summ.setdefault("kernels", {})[kname] = ent
             json.dump({"kernels": summ["kernels"]}, open(sp, "w"), indent=1)
 
 if __name__ == "__main__":
