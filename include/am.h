@@ -119,6 +119,8 @@ enum {
     AM_K_FILTER,        /* full-stream filter of every voxel (AM_OPT_BRICKS = 0)               */
     AM_K_BASELINE,      /* all-pairs CHECKBOX baseline, a9                                     */
     AM_K_LAYOUT,        /* am_unpack_cells / am_pack_cells                                     */
+    AM_K_ICA_MEMO,      /* am_compute_octree: parallel ICA calculation of the top S levels     */
+    AM_K_OCTREE,        /* am_compute_octree: one thread per orientation, Alg. 2               */
     AM_K_COUNT
 };
 
@@ -201,6 +203,47 @@ int am_kernel_stats(am_ctx* ctx, double* ms, int64_t* launches);
 
 /* Name of kernel k (static string), NULL if k is not an AM_K_* value. */
 const char* am_kernel_name(int k);
+
+/*
+ * The paper's own GPU schemes (§4),
+ * for comparison with am_compute: one thread per orientation traverses the
+ * octree with Alg. 2 CHECKOCTREE (L198-221) using the scheme's elementary test.
+ * All give the same map as am_compute outside the 1e-5 rad band (each falls
+ * back to the exact test); they differ in work.
+ */
+enum {
+    AM_SCHEME_PBOX = 0,       /* CHECKBOX on every visited node (the baseline, L269)          */
+    AM_SCHEME_PBOX_AABB = 1,  /* optimized PBox: rotated-box AABB reject first (L268)         */
+    AM_SCHEME_PICA = 2,       /* CHECKICA computed on the fly, CHECKBOX for corner cases      */
+    AM_SCHEME_MICA = 3,       /* + cones of the top S levels memoised in parallel (§4.2)      */
+    AM_SCHEME_AICA = 4        /* + corner cases expanded into children (§4.3)        */
+};
+
+/*
+ * Build the octree (root + interior + leaves) of the resident
+ * model.  The uploaded voxels must be the leaves of an adaptive octree whose
+ * root cube is [root_lo, root_lo + root_size]^3: every half size is
+ * root_size / 2^(l+1) for a level 0 <= l <= 20 and every centre the centre of
+ * a level-l cell; the cells must be disjoint.  AM_EINVAL otherwise (and for a
+ * non-finite or non-positive root), AM_ESTATE before am_upload_voxels.
+ * Interior nodes are the cells that contain leaves; children are stored
+ * contiguously, nodes in level (BFS) order.  *n_nodes (nullable) receives the
+ * node count.  Synchronous; a new upload discards the octree.
+ */
+int am_build_octree(am_ctx* ctx, const float root_lo[3], float root_size, int64_t* n_nodes);
+
+/*
+ * AM of one pivot with scheme AM_SCHEME_* over the octree (same output
+ * contract as am_compute).  S = levels whose cones are memoised by the
+ * parallel ICA calculation (MICA / AICA; 0..64, levels 0..S-1), vdepth =
+ * AICA's virtual expansion depth of band leaves before CHECKBOX (0..3).
+ * stats (nullable, 4 entries): nodes popped, CHECKBOX calls, on-the-fly ICA
+ * evaluations, max nodes popped by one thread (the critical thread of Fig. 13
+ * L323); filling it synchronises the stream.  AM_EINVAL for a bad scheme, S or
+ * vdepth; AM_ESTATE before am_build_octree.
+ */
+int am_compute_octree(am_ctx* ctx, const float pivot[3], int scheme, int S, int vdepth, uint32_t* am_out,
+                      int dst_is_device, void* cuda_stream, int64_t* stats);
 
 /*
  * Layout conversion on the device, for the voxel-sharded multi-GPU combine

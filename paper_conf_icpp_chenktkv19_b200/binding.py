@@ -21,12 +21,14 @@ LIB_PATH = os.environ.get("AM_LIBRARY") or os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
-K_COUNT = 14  # AM_K_COUNT (include/am.h)
+K_COUNT = 16  # AM_K_COUNT (include/am.h)
+SCHEME_PBOX, SCHEME_PBOX_AABB, SCHEME_PICA, SCHEME_MICA, SCHEME_AICA = 0, 1, 2, 3, 4  # AM_SCHEME_*
+SCHEMES = {"pbox": 0, "pbox_aabb": 1, "pica": 2, "mica": 3, "aica": 4}
 OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",
-           "am_set_option", "am_kernel_time", "am_kernel_stats", "am_kernel_name", "am_unpack_cells", "am_pack_cells", "am_words_per_map",
+           "am_set_option", "am_kernel_time", "am_kernel_stats", "am_kernel_name", "am_build_octree", "am_compute_octree", "am_unpack_cells", "am_pack_cells", "am_words_per_map",
            "am_num_voxels", "am_last_error", "am_destroy")
 
 if not os.path.exists(LIB_PATH):
@@ -81,6 +83,11 @@ lib.am_kernel_time.restype = ctypes.c_int
 lib.am_kernel_time.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
 lib.am_kernel_stats.restype = ctypes.c_int
 lib.am_kernel_stats.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+lib.am_build_octree.restype = ctypes.c_int
+lib.am_build_octree.argtypes = [_P, ctypes.POINTER(ctypes.c_float), ctypes.c_float, ctypes.POINTER(ctypes.c_int64)]
+lib.am_compute_octree.restype = ctypes.c_int
+lib.am_compute_octree.argtypes = [_P, ctypes.POINTER(ctypes.c_float), ctypes.c_int, ctypes.c_int, ctypes.c_int, _P,
+                                  ctypes.c_int, _P, ctypes.POINTER(ctypes.c_int64)]
 lib.am_kernel_name.restype = ctypes.c_char_p
 lib.am_kernel_name.argtypes = [ctypes.c_int]
 lib.am_unpack_cells.restype = ctypes.c_int
@@ -284,6 +291,35 @@ class Context:
                 out = np.zeros(self.words, dtype=np.uint32)
             self._check(lib.am_compute_baseline(self._h, pp, _P(out.ctypes.data), 0, _stream_handle(stream)))
         return out
+
+    def build_octree(self, root_lo, root_size) -> int:
+        """am_build_octree: the octree of the resident leaves in the root cube; returns the node count."""
+        _, lo = _f3(root_lo)
+        n = ctypes.c_int64()
+        self._check(lib.am_build_octree(self._h, lo, float(root_size), ctypes.byref(n)))
+        return n.value
+
+    def compute_octree(self, pivot, scheme, S=0, vdepth=0, out=None, stream=None, stats: bool = False):
+        """am_compute_octree: the paper's orientation-per-thread scheme (SCHEMES name or
+        AM_SCHEME_* value).  Returns (out, stats dict | None)."""
+        sc = SCHEMES[scheme] if isinstance(scheme, str) else int(scheme)
+        _, pp = _f3(pivot)
+        st = (ctypes.c_int64 * 4)() if stats else None
+        if out is not None and _is_torch_cuda(out):
+            if stream is None:
+                import torch
+                stream = torch.cuda.current_stream(out.device)
+            self._check(lib.am_compute_octree(self._h, pp, sc, int(S), int(vdepth), _P(out.data_ptr()), 1,
+                                              _stream_handle(stream), st))
+        else:
+            if out is None:
+                out = np.zeros(self.words, dtype=np.uint32)
+            self._check(lib.am_compute_octree(self._h, pp, sc, int(S), int(vdepth), _P(out.ctypes.data), 0,
+                                              _stream_handle(stream), st))
+        sd = None
+        if st is not None:
+            sd = {"nodes_popped": st[0], "box_tests": st[1], "ica_evals": st[2], "max_popped_per_thread": st[3]}
+        return out, sd
 
     def am(self, pivot) -> np.ndarray:
         """Convenience: uint8[m, n] AICA map of one pivot (host)."""

@@ -20,6 +20,10 @@
 #include "stream.cuh"
 #include "fused.cuh"
 #include "batch.cuh"
+#include "octree.cuh"
+
+#include <algorithm>
+#include <cstdint>
 
 using namespace am;
 
@@ -90,6 +94,14 @@ struct am_ctx {
     long long kev_prev = -1;               // chain: event recorded before the next launch
     std::vector<std::pair<int, size_t>> kmarks;  // (kernel, index of its end event)
     std::vector<size_t> kmark_begin;
+    // octree of the resident model (am_build_octree; paper-faithful schemes)
+    float4* d_onode = nullptr;             // node cubes, BFS order
+    int2* d_olink = nullptr;               // (first child, child count)
+    float4* d_omemo = nullptr;             // memoised cones of the top levels
+    unsigned long long* d_ostats = nullptr;
+    long long o_n = 0;
+    bool o_built = false;
+    std::vector<long long> o_level_end;    // nodes of levels <= L: [0, o_level_end[L])
     std::string err;
 };
 
@@ -869,6 +881,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     if (N == 0) {
         ctx->N = 0;
         ctx->uploaded = true;
+        ctx->o_built = false;
         return AM_OK;
     }
     const float* dc = centers_xyz;
@@ -1031,6 +1044,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     cleanup();
     ctx->N = N;
     ctx->uploaded = true;
+    ctx->o_built = false;  // the octree belongs to the previous model
     return rc;
 }
 
@@ -1264,8 +1278,215 @@ int am_kernel_stats(am_ctx* ctx, double* ms, int64_t* launches) {
 const char* am_kernel_name(int k) {
     static const char* names[AM_K_COUNT] = {
         "l0_cones", "l0_rows", "clear_map", "l1_cones", "l1_rows", "bricks", "voxels",
-        "live_cones", "live_rows", "band", "fused_pipeline", "filter", "baseline", "layout"};
+        "live_cones", "live_rows", "band", "fused_pipeline", "filter", "baseline", "layout",
+        "ica_memo", "octree"};
     return (k >= 0 && k < AM_K_COUNT) ? names[k] : nullptr;
+}
+
+// ---------------------------------------------------------------------------
+// Octree of the resident model for the paper's orientation-per-thread schemes
+// (octree.cuh).  Host-side build: every leaf's level and cell in the declared
+// root frame, a sort by the Morton code of its first finest-level cell, then
+// the nodes level by level (BFS), children of a node contiguous.
+// ---------------------------------------------------------------------------
+namespace {
+
+uint64_t spread3(uint64_t x) {  // 21 bits -> every third bit
+    x &= 0x1fffffull;
+    x = (x | x << 32) & 0x1f00000000ffffull;
+    x = (x | x << 16) & 0x1f0000ff0000ffull;
+    x = (x | x << 8) & 0x100f00f00f00f00full;
+    x = (x | x << 4) & 0x10c30c30c30c30c3ull;
+    x = (x | x << 2) & 0x1249249249249249ull;
+    return x;
+}
+
+}  // namespace
+
+int am_build_octree(am_ctx* ctx, const float root_lo[3], float root_size, int64_t* n_nodes) {
+    if (!ctx) return AM_EINVAL;
+    if (!root_lo || !(root_size > 0.f) || !is_finite_f(root_size)) return fail(ctx, AM_EINVAL, "bad root cube");
+    for (int k = 0; k < 3; ++k)
+        if (!is_finite_f(root_lo[k])) return fail(ctx, AM_EINVAL, "root_lo[%d] is not finite", k);
+    if (!ctx->uploaded) return fail(ctx, AM_ESTATE, "am_build_octree before am_upload_voxels");
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    const long long N = ctx->N;
+    std::vector<float4> leaf((size_t)N);
+    if (N > 0) CK(cudaMemcpy(leaf.data(), ctx->d_vox, (size_t)N * sizeof(float4), cudaMemcpyDeviceToHost));
+    // level and cell of every leaf
+    std::vector<int> lev((size_t)N);
+    std::vector<uint32_t> cx((size_t)N * 3);
+    int Lmax = 0;
+    for (long long i = 0; i < N; ++i) {
+        const double s = (double)root_size / (2.0 * leaf[i].w);
+        const int l = (int)std::lround(std::log2(s));
+        if (l < 0 || l > 20 || std::fabs(s - std::ldexp(1.0, l)) > 1e-3 * std::ldexp(1.0, l))
+            return fail(ctx, AM_EINVAL, "voxel %lld: half size %g is not root_size / 2^(l+1)", i, leaf[i].w);
+        lev[i] = l;
+        Lmax = std::max(Lmax, l);
+        const double cell = (double)root_size / std::ldexp(1.0, l);
+        const float c3[3] = {leaf[i].x, leaf[i].y, leaf[i].z};
+        for (int a = 0; a < 3; ++a) {
+            const double f = (c3[a] - (double)root_lo[a]) / cell - 0.5;
+            const long long q = std::llround(f);
+            if (q < 0 || q >= (1ll << l) || std::fabs(f - (double)q) > 1e-2)
+                return fail(ctx, AM_EINVAL, "voxel %lld is not a cell of the root cube's level %d", i, l);
+            cx[3 * i + a] = (uint32_t)q;
+        }
+    }
+    // sort by the Morton code of each leaf's first finest-level cell
+    std::vector<uint64_t> key((size_t)N);
+    for (long long i = 0; i < N; ++i) {
+        const int sh = Lmax - lev[i];
+        key[i] = spread3((uint64_t)cx[3 * i] << sh) | spread3((uint64_t)cx[3 * i + 1] << sh) << 1 |
+                 spread3((uint64_t)cx[3 * i + 2] << sh) << 2;
+    }
+    std::vector<long long> ord((size_t)N);
+    for (long long i = 0; i < N; ++i) ord[i] = i;
+    std::sort(ord.begin(), ord.end(), [&](long long a, long long b) { return key[a] < key[b]; });
+    for (long long t = 0; t + 1 < N; ++t) {  // leaves are disjoint cells
+        const long long a = ord[t], b = ord[t + 1];
+        const uint64_t span = 1ull << (3 * (Lmax - lev[a]));
+        if (key[b] < key[a] + span) return fail(ctx, AM_EINVAL, "voxels %lld and %lld overlap", a, b);
+    }
+    std::vector<uint64_t> skey((size_t)N);
+    for (long long t = 0; t < N; ++t) skey[t] = key[ord[t]];
+    // BFS: node = (level, first finest code, leaf range [a, b))
+    struct Pend { int L; uint64_t base; long long a, b; };
+    std::vector<Pend> q;
+    std::vector<float4> box;
+    std::vector<int2> link;
+    std::vector<long long> level_end;
+    if (N > 0) q.push_back({0, 0ull, 0, N});
+    size_t head = 0;
+    while (head < q.size()) {
+        const Pend nd = q[head];
+        const size_t self = head++;
+        (void)self;
+        while ((int)level_end.size() <= nd.L) level_end.push_back(0);
+        level_end[nd.L] = (long long)head;
+        const long long first = ord[nd.a];
+        if (nd.b - nd.a == 1 && lev[first] == nd.L) {  // a leaf: the uploaded voxel itself
+            box.push_back(leaf[first]);
+            link.push_back(make_int2(0, 0));
+            continue;
+        }
+        for (long long t = nd.a; t < nd.b; ++t)
+            if (lev[ord[t]] <= nd.L) return fail(ctx, AM_EINVAL, "voxel %lld overlaps a finer voxel", ord[t]);
+        if (nd.L >= Lmax) return fail(ctx, AM_EINVAL, "octree build: inconsistent levels");
+        const double cell = (double)root_size / std::ldexp(1.0, nd.L);
+        // the node cube from its first finest cell
+        uint32_t c3[3] = {0, 0, 0};
+        for (int bit = 0; bit < 21; ++bit)
+            for (int a = 0; a < 3; ++a) c3[a] |= (uint32_t)((nd.base >> (3 * bit + a)) & 1ull) << bit;
+        float4 bx;
+        bx.x = (float)(root_lo[0] + ((c3[0] >> (Lmax - nd.L)) + 0.5) * cell);
+        bx.y = (float)(root_lo[1] + ((c3[1] >> (Lmax - nd.L)) + 0.5) * cell);
+        bx.z = (float)(root_lo[2] + ((c3[2] >> (Lmax - nd.L)) + 0.5) * cell);
+        bx.w = (float)(0.5 * cell);
+        box.push_back(bx);
+        const int firstc = (int)q.size();
+        int nc = 0;
+        const uint64_t span = 1ull << (3 * (Lmax - nd.L - 1));
+        long long a = nd.a;
+        for (int c = 0; c < 8 && a < nd.b; ++c) {
+            const uint64_t hi = nd.base + (uint64_t)(c + 1) * span;
+            const long long b = std::lower_bound(skey.begin() + a, skey.begin() + nd.b, hi) - skey.begin();
+            if (b > a) {
+                q.push_back({nd.L + 1, nd.base + (uint64_t)c * span, a, b});
+                ++nc;
+            }
+            a = b;
+        }
+        if ((long long)q.size() > (1ll << 31) - 8) return fail(ctx, AM_ENOMEM, "octree too large");
+        link.push_back(make_int2(firstc, nc));
+    }
+    for (size_t L = 1; L < level_end.size(); ++L) level_end[L] = std::max(level_end[L], level_end[L - 1]);
+    cudaFree(ctx->d_onode);
+    cudaFree(ctx->d_olink);
+    cudaFree(ctx->d_omemo);
+    ctx->d_onode = nullptr;
+    ctx->d_olink = nullptr;
+    ctx->d_omemo = nullptr;
+    ctx->o_n = (long long)box.size();
+    ctx->o_level_end = level_end;
+    if (ctx->o_n > 0) {
+        CK(cudaMalloc(&ctx->d_onode, box.size() * sizeof(float4)));
+        CK(cudaMalloc(&ctx->d_olink, link.size() * sizeof(int2)));
+        CK(cudaMalloc(&ctx->d_omemo, box.size() * sizeof(float4)));
+        CK(cudaMemcpy(ctx->d_onode, box.data(), box.size() * sizeof(float4), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(ctx->d_olink, link.data(), link.size() * sizeof(int2), cudaMemcpyHostToDevice));
+    }
+    if (!ctx->d_ostats) CK(cudaMalloc(&ctx->d_ostats, 4 * sizeof(unsigned long long)));
+    ctx->o_built = true;
+    if (n_nodes) *n_nodes = ctx->o_n;
+    return AM_OK;
+}
+
+int am_compute_octree(am_ctx* ctx, const float pivot[3], int scheme, int S, int vdepth, uint32_t* am_out,
+                      int dst_is_device, void* cuda_stream, int64_t* stats) {
+    if (!ctx) return AM_EINVAL;
+    int rc = check_pivot(ctx, pivot);
+    if (rc) return rc;
+    if (!am_out) return fail(ctx, AM_EINVAL, "am_out is NULL");
+    if (scheme < AM_SCHEME_PBOX || scheme > AM_SCHEME_AICA) return fail(ctx, AM_EINVAL, "unknown scheme %d", scheme);
+    if (S < 0 || S > 64) return fail(ctx, AM_EINVAL, "S must be in [0, 64]");
+    if (vdepth < 0 || vdepth > 3) return fail(ctx, AM_EINVAL, "vdepth must be in [0, 3]");
+    if (!ctx->uploaded) return fail(ctx, AM_ESTATE, "am_compute_octree before am_upload_voxels");
+    if (!ctx->o_built) return fail(ctx, AM_ESTATE, "am_compute_octree before am_build_octree");
+    DeviceGuard dg(ctx->device);
+    if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
+    CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
+    CK(cudaMemsetAsync(ctx->d_ostats, 0, 4 * sizeof(unsigned long long), s));
+    if (ctx->o_n > 0) {
+        if ((rc = kchain(ctx, s))) return rc;
+        OctParams P{};
+        P.box = ctx->d_onode;
+        P.link = ctx->d_olink;
+        P.memo = ctx->d_omemo;
+        P.nmemo = 0;
+        P.px = pivot[0];
+        P.py = pivot[1];
+        P.pz = pivot[2];
+        P.tool = ctx->tool;
+        P.grid = ctx->grid;
+        P.tab = ctx->d_tab;
+        P.gam = gam;
+        P.vdepth = vdepth;
+        P.stats = ctx->d_ostats;
+        if ((scheme == AM_SCHEME_MICA || scheme == AM_SCHEME_AICA) && S > 0) {
+            // the parallel ICA calculation of the top S levels (levels 0 .. S-1)
+            const int L = std::min<int>(S, (int)ctx->o_level_end.size()) - 1;
+            P.nmemo = ctx->o_level_end[L];
+            const unsigned g = (unsigned)std::max<long long>(1, std::min<long long>((P.nmemo + 255) / 256, ctx->sms * 8));
+            ica_memo_kernel<<<g, 256, 0, s>>>(ctx->d_onode, P.nmemo, P.px, P.py, P.pz, ctx->tool, ctx->d_omemo);
+            if ((rc = kmark(ctx, s, AM_K_ICA_MEMO))) return rc;
+        }
+        const unsigned ncell = (unsigned)(ctx->grid.m * ctx->grid.n);
+        const unsigned g = (ncell + 31) / 32;
+        switch (scheme) {
+        case AM_SCHEME_PBOX: octree_kernel<SCHEME_PBOX><<<g, 32, 0, s>>>(P); break;
+        case AM_SCHEME_PBOX_AABB: octree_kernel<SCHEME_PBOX_AABB><<<g, 32, 0, s>>>(P); break;
+        case AM_SCHEME_PICA: octree_kernel<SCHEME_PICA><<<g, 32, 0, s>>>(P); break;
+        case AM_SCHEME_MICA: octree_kernel<SCHEME_MICA><<<g, 32, 0, s>>>(P); break;
+        default: octree_kernel<SCHEME_AICA><<<g, 32, 0, s>>>(P); break;
+        }
+        if ((rc = kmark(ctx, s, AM_K_OCTREE))) return rc;
+    }
+    if (!dst_is_device)
+        CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if (stats) {
+        unsigned long long h[4];
+        CK(cudaMemcpyAsync(h, ctx->d_ostats, sizeof h, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        for (int k = 0; k < 4; ++k) stats[k] = (int64_t)h[k];
+    } else if (!dst_is_device) {
+        CK(cudaStreamSynchronize(s));
+    }
+    return AM_OK;
 }
 
 int am_unpack_cells(am_ctx* ctx, const uint32_t* words, uint8_t* cells, void* cuda_stream) {
@@ -1323,6 +1544,10 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_ts);
     cudaFree(ctx->d_piv);
     cudaFree(ctx->d_bctl);
+    cudaFree(ctx->d_onode);
+    cudaFree(ctx->d_olink);
+    cudaFree(ctx->d_omemo);
+    cudaFree(ctx->d_ostats);
     for (auto e : ctx->kev) cudaEventDestroy(e);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);
