@@ -255,6 +255,8 @@ def run_ours(args):
     ctx.set_option(B.OPT_BATCH, args.slots)
     if args.cmap_t:
         ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
+    if args.band_subdiv:
+        ctx.set_option(B.OPT_BAND_SUBDIV, args.band_subdiv)
     t0 = time.time()
     ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
     torch.cuda.synchronize(dev)
@@ -493,6 +495,8 @@ def main():
     ap.add_argument("--baseline", action="store_true", help="also time am_compute_baseline once")
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
     ap.add_argument("--cmap-t", type=int, default=0, help="AM_OPT_CMAP_T (0 = library default)")
+    ap.add_argument("--band-subdiv", type=int, default=0,
+                    help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")
     ap.add_argument("--no-full-scan", action="store_true", help="skip the full-scan (filter_kernel) leg")
     args = ap.parse_args()
     if args.warmup < 3:

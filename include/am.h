@@ -98,9 +98,12 @@ enum {
     AM_OPT_FUSED = 11,           /* 1 = the whole map in one persistent cooperative launch when
                                     phases >= 1 and bricks = 1 (default); 0 = one launch per
                                     stage.  Same map                                            */
-    AM_OPT_BATCH = 12            /* am_compute_batch: pivots computed together, phase by phase,
+    AM_OPT_BATCH = 12,           /* am_compute_batch: pivots computed together, phase by phase,
                                     one launch per phase (1..64, default 32; each needs its own
                                     per-map buffers, ~4 N + 100 MB of device memory).  Same maps */
+    AM_OPT_BAND_SUBDIV = 13      /* band pairs: levels of virtual 2x2x2 sub-cubes decided by
+                                    CHECKICA before CHECKBOX (§4.3; 0..3,
+                                    default 0 = CHECKBOX directly).  Same map outside the band  */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

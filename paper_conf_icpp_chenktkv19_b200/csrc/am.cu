@@ -73,6 +73,7 @@ struct am_ctx {
     int bricks_on = 1;
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
+    int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
     int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
@@ -181,6 +182,7 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.vox_coarse = c->d_coarse;
     p.cmapT = c->cmapT;
     p.cull_dist = c->tool.rho_max * (1.f + 1e-5f) + 1e-6f;
+    p.band_vdepth = c->band_vdepth;
     // the reach cull can only fire when some voxel centre lies farther than
     // cull_dist from the pivot: compare with the farthest corner of the bbox
     double far2 = 0.0;
@@ -1212,6 +1214,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_BATCH:
         if (value < 1 || value > kMaxBatch) return fail(ctx, AM_EINVAL, "batch must be in [1, %d]", kMaxBatch);
         ctx->batch = (int)value;
+        return AM_OK;
+    case AM_OPT_BAND_SUBDIV:
+        if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "band_subdiv must be in [0, 3]");
+        ctx->band_vdepth = (int)value;
         return AM_OK;
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");

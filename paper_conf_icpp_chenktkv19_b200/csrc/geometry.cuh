@@ -417,4 +417,61 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
     return false;
 }
 
+// ---------------------------------------------------------------------------
+// CHECKICA on whole cubes and the corner-case expansion (Alg. 1, §4.3)
+// ---------------------------------------------------------------------------
+
+// Cones of a cube whose centre is v (relative to the pivot) at distance D;
+// (cin, cout, clo, 1/D) with 1/D = 0 and cin = -2 ("always meets") when the
+// pivot lies in the closed cube (the tool contains the pivot).
+__device__ __forceinline__ float4 node_cones(float vx, float vy, float vz, float h, const ToolDev& T) {
+    if (fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) return make_float4(-2.f, -2.f, 2.f, 0.f);
+    const float D = sqrtf(vx * vx + vy * vy + vz * vz);
+    const Cones c = tool_cones(D, h, T);
+    return make_float4(c.cin, c.cout, c.clo, 1.f / D);
+}
+
+// CHECKICA decision from the cones: 1 = certainly meets (angle <= ica1),
+// 0 = certainly misses (angle >= ica2, or inside the ring's hole), 2 = corner case.
+__device__ __forceinline__ int ica_decide(float4 c, float vx, float vy, float vz, float dx, float dy, float dz) {
+    const float ct = (vx * dx + vy * dy + vz * dz) * c.w;
+    if (ct >= c.x) return 1;
+    if (c.y > 1.f || ct < c.y || ct > c.z) return 0;
+    return 2;
+}
+
+// The corner-case optimisation of PAPER.md §4.3 (L248-256) on a leaf: the leaf (solid cube) meets the tool iff one
+// of its virtual 2x2x2 sub-cubes does; each is decided by CHECKICA, recursing
+// `depth` levels, CHECKBOX at the bottom.
+__device__ bool leaf_expand(float vx, float vy, float vz, float h, float dx, float dy, float dz, int depth,
+                            const ToolDev& T, unsigned int& nbox, unsigned int& nica) {
+    float4 st[8 * 4];
+    int lv[8 * 4];
+    int sp = 0;
+    st[sp] = make_float4(vx, vy, vz, h);
+    lv[sp++] = 0;
+    while (sp > 0) {
+        --sp;
+        const float4 c = st[sp];
+        const int l = lv[sp];
+        if (l > 0) {  // the root of this expansion is already known to be in the band
+            ++nica;
+            const int dcs = ica_decide(node_cones(c.x, c.y, c.z, c.w, T), c.x, c.y, c.z, dx, dy, dz);
+            if (dcs == 1) return true;
+            if (dcs == 0) continue;
+        }
+        if (l >= depth) {
+            ++nbox;
+            if (exact_hit(c.x, c.y, c.z, c.w, dx, dy, dz, T)) return true;
+            continue;
+        }
+        const float q = 0.5f * c.w;
+        for (int k = 0; k < 8; ++k) {
+            st[sp] = make_float4(c.x + ((k & 1) ? q : -q), c.y + ((k & 2) ? q : -q), c.z + ((k & 4) ? q : -q), q);
+            lv[sp++] = l + 1;
+        }
+    }
+    return false;
+}
+
 }  // namespace am

@@ -71,6 +71,7 @@ struct StreamParams {
     unsigned int nbricks;
     unsigned int* brick_list;      // bricks kept by brick_test_kernel (capacity nbricks)
     unsigned int* brick_count;     // zeroed per map
+    int band_vdepth;               // band pairs: virtual sub-cube levels before CHECKBOX (§4.3)
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,
@@ -113,6 +114,11 @@ __device__ __forceinline__ bool exact_pair(const StreamParams& p, float4 q, int 
     const float* t = p.tab;
     const float cph = __ldg(t + i), sph = __ldg(t + p.grid.m + i);
     const float cg = __ldg(t + 2 * p.grid.m + j), sg = __ldg(t + 2 * p.grid.m + p.grid.n + j);
+    if (p.band_vdepth > 0) {  // PAPER.md §4.3: virtual children by CHECKICA first
+        unsigned int nb = 0, ni = 0;
+        return leaf_expand(q.x - p.px, q.y - p.py, q.z - p.pz, q.w, sph * cg, sph * sg, cph, p.band_vdepth, p.tool,
+                           nb, ni);
+    }
     return exact_hit(q.x - p.px, q.y - p.py, q.z - p.pz, q.w, sph * cg, sph * sg, cph, p.tool);
 }
 

@@ -27,7 +27,8 @@
 // same map as am_compute; they differ only in work -- which is what the
 // paper's Table 3 / Fig. 13-18 comparisons measure.
 //
-// The cone tests use geometry.cuh's tool_cones (reading G8: inner cone on the
+// The cone tests (node_cones, ica_decide, leaf_expand) live in geometry.cuh
+// beside tool_cones (reading G8: inner cone on the
 // monotone-shrunk tool, outer on the true tool, ring voxels beyond the tool
 // end) -- the same device functions as the streaming path.
 #pragma once
@@ -53,25 +54,6 @@ struct OctParams {
 
 constexpr int kOctStack = 8 * 24;     // 8 children x (max depth 21 + slack)
 
-// Cones of a cube whose centre is v (relative to the pivot) at distance D;
-// (cin, cout, clo, 1/D) with 1/D = 0 and cin = -2 ("always meets") when the
-// pivot lies in the closed cube (the tool contains the pivot).
-__device__ __forceinline__ float4 node_cones(float vx, float vy, float vz, float h, const ToolDev& T) {
-    if (fabsf(vx) <= h && fabsf(vy) <= h && fabsf(vz) <= h) return make_float4(-2.f, -2.f, 2.f, 0.f);
-    const float D = sqrtf(vx * vx + vy * vy + vz * vz);
-    const Cones c = tool_cones(D, h, T);
-    return make_float4(c.cin, c.cout, c.clo, 1.f / D);
-}
-
-// CHECKICA decision from the cones: 1 = certainly meets (angle <= ica1),
-// 0 = certainly misses (angle >= ica2, or inside the ring's hole), 2 = corner case.
-__device__ __forceinline__ int ica_decide(float4 c, float vx, float vy, float vz, float dx, float dy, float dz) {
-    const float ct = (vx * dx + vy * dy + vz * dz) * c.w;
-    if (ct >= c.x) return 1;
-    if (c.y > 1.f || ct < c.y || ct > c.z) return 0;
-    return 2;
-}
-
 // The optimized PBox's reject: the rotated cube's axis-aligned box in the
 // tool frame (e1, e2, d) against every cylinder's box [-R, R]^2 x [z0, z1].
 __device__ __forceinline__ bool aabb_overlaps(float vx, float vy, float vz, float h, float dx, float dy, float dz,
@@ -94,40 +76,6 @@ __device__ __forceinline__ bool aabb_overlaps(float vx, float vy, float vz, floa
     for (int k = 0; k < T.ncyl; ++k) {
         const float R = T.R[k];
         if (fabsf(cX) <= R + hX && fabsf(cY) <= R + hY && cZ + hZ >= T.z0[k] && cZ - hZ <= T.z1[k]) return true;
-    }
-    return false;
-}
-
-// AICA's corner case on a leaf: the leaf (solid cube) meets the tool iff one
-// of its virtual 2x2x2 sub-cubes does; each is decided by CHECKICA, recursing
-// `depth` levels, CHECKBOX at the bottom.
-__device__ bool leaf_expand(float vx, float vy, float vz, float h, float dx, float dy, float dz, int depth,
-                            const ToolDev& T, unsigned int& nbox, unsigned int& nica) {
-    float4 st[8 * 4];
-    int lv[8 * 4];
-    int sp = 0;
-    st[sp] = make_float4(vx, vy, vz, h);
-    lv[sp++] = 0;
-    while (sp > 0) {
-        --sp;
-        const float4 c = st[sp];
-        const int l = lv[sp];
-        if (l > 0) {  // the root of this expansion is already known to be in the band
-            ++nica;
-            const int dcs = ica_decide(node_cones(c.x, c.y, c.z, c.w, T), c.x, c.y, c.z, dx, dy, dz);
-            if (dcs == 1) return true;
-            if (dcs == 0) continue;
-        }
-        if (l >= depth) {
-            ++nbox;
-            if (exact_hit(c.x, c.y, c.z, c.w, dx, dy, dz, T)) return true;
-            continue;
-        }
-        const float q = 0.5f * c.w;
-        for (int k = 0; k < 8; ++k) {
-            st[sp] = make_float4(c.x + ((k & 1) ? q : -q), c.y + ((k & 2) ? q : -q), c.z + ((k & 4) ? q : -q), q);
-            lv[sp++] = l + 1;
-        }
     }
     return false;
 }

@@ -316,3 +316,28 @@ def test_full_size_bench_launch_config_sampled(am, name, npiv):
     for k in (0, int(np.argmax(nclear))):  # the first map and the one with the most clear cells
         _check_sampled(cfg, C, H, P[k], maps[k], rng)
     ctx.close()
+
+
+@pytest.mark.parametrize("subdiv", [1, 2, 3])
+@pytest.mark.parametrize("name", ["T_head", "T_imp"])
+def test_band_subdivision_matches_oracle(am, name, subdiv):
+    """AM_OPT_BAND_SUBDIV (§4.3): band pairs are first
+    split into virtual 2x2x2 sub-cubes decided by CHECKICA, CHECKBOX only at the
+    bottom.  Exact: same map as CHECKBOX-direct outside the band, and every robust
+    cell equals the oracle's, for single and batched launches."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    P = cfg.pivots(3)
+    ref = ctx.compute_batch(P)
+    ctx.set_option(am.binding.OPT_BAND_SUBDIV, subdiv)
+    got = ctx.compute_batch(P)
+    single = np.stack([ctx.compute(p)[0] for p in P])
+    assert np.array_equal(got, single)
+    for k, p in enumerate(P):
+        S = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n)
+        g = am.unpack(got[k], cfg.m, cfg.n)
+        mism, _ = _compare(g, S)
+        assert mism == 0
+        assert int((g != am.unpack(ref[k], cfg.m, cfg.n))[S != 1].sum()) == 0
+    ctx.close()
