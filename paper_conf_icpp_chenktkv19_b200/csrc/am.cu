@@ -27,6 +27,18 @@
 
 using namespace am;
 
+// coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
+// level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_L0_DIV
+#define AM_L0_DIV 2048
+#endif
+#ifndef AM_L1_DIV
+#define AM_L1_DIV 256
+#endif
+#ifndef AM_L1_STRIDE
+#define AM_L1_STRIDE 512
+#endif
+
 struct am_ctx {
     int device = 0;
     int sms = 0;
@@ -997,9 +1009,9 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     ctx->d_coarse = nullptr;
     ctx->n_l0 = ctx->n_l1 = 0;
     if (N >= 2048) {
-        const long long n0 = std::min<long long>(N, std::max<long long>(1024, N / 2048));
-        const long long n1 = std::min<long long>(N, std::max<long long>(8192, N / 256));
-        const long long stride = 512, ns = N / stride;
+        const long long n0 = std::min<long long>(N, std::max<long long>(1024, N / AM_L0_DIV));
+        const long long n1 = std::min<long long>(N, std::max<long long>(8192, N / AM_L1_DIV));
+        const long long stride = AM_L1_STRIDE, ns = N / stride;
         unsigned int *sk = nullptr, *sk2 = nullptr, *si = nullptr, *si2 = nullptr, *cid = nullptr;
         void* ct = nullptr;
         auto cfree = [&]() {

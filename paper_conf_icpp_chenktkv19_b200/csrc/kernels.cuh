@@ -181,7 +181,10 @@ __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, 
 // tries every clear direction (in chunks), 4 texels per thread.
 
 constexpr int kMapDirs = 2048;  // clear directions staged in shared memory per chunk
-constexpr int kMapBrute = 512;  // up to this many clear cells, every texel tries every one
+#ifndef AM_MAP_BRUTE
+#define AM_MAP_BRUTE 512
+#endif
+constexpr int kMapBrute = AM_MAP_BRUTE;  // up to this many clear cells, every texel tries every one
 
 __device__ __forceinline__ float dot3(float4 a, float4 b) { return fmaf(a.x, b.x, fmaf(a.y, b.y, a.z * b.z)); }
 
