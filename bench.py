@@ -255,6 +255,8 @@ def run_ours(args):
     ctx.set_option(B.OPT_BATCH, args.slots)
     if args.cmap_t:
         ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
+    if args.cmap_t1:
+        ctx.set_option(B.OPT_CMAP_T1, args.cmap_t1)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
     if args.band_subdiv:
@@ -497,6 +499,7 @@ def main():
     ap.add_argument("--baseline", action="store_true", help="also time am_compute_baseline once")
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
     ap.add_argument("--cmap-t", type=int, default=0, help="AM_OPT_CMAP_T (0 = library default)")
+    ap.add_argument("--cmap-t1", type=int, default=0, help="AM_OPT_CMAP_T1 (0 = library default)")
     ap.add_argument("--phases", type=int, default=None, help="AM_OPT_PHASES (coarse levels, 1 or 2)")
     ap.add_argument("--band-subdiv", type=int, default=0,
                     help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")

@@ -101,9 +101,12 @@ enum {
     AM_OPT_BATCH = 12,           /* am_compute_batch: pivots computed together, phase by phase,
                                     one launch per phase (1..64, default 32; each needs its own
                                     per-map buffers, ~4 N + 100 MB of device memory).  Same maps */
-    AM_OPT_BAND_SUBDIV = 13      /* band pairs: levels of virtual 2x2x2 sub-cubes decided by
+    AM_OPT_BAND_SUBDIV = 13,     /* band pairs: levels of virtual 2x2x2 sub-cubes decided by
                                     CHECKICA before CHECKBOX (§4.3; 0..3,
                                     default 0 = CHECKBOX directly).  Same map outside the band  */
+    AM_OPT_CMAP_T1 = 14          /* resolution of the clear-direction map built after level 0,
+                                    which only filters level 1 (4..AM_OPT_CMAP_T, default 32).
+                                    Same map                                                    */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

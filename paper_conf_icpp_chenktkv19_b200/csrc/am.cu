@@ -29,8 +29,11 @@ using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
 // level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_CMAP_T1
+#define AM_CMAP_T1 32
+#endif
 #ifndef AM_L0_DIV
-#define AM_L0_DIV 2048
+#define AM_L0_DIV 8192
 #endif
 #ifndef AM_L1_DIV
 #define AM_L1_DIV 256
@@ -78,6 +81,8 @@ struct am_ctx {
     int diag = 0;
     int diag_ts = 0;
     int cmapT = 128;
+    int cmapT1 = AM_CMAP_T1;               // map after level 0 (AM_OPT_CMAP_T1, <= cmapT)
+    float4* d_texels1 = nullptr;
     int phases = 2;
     float4* d_bricks = nullptr;            // bounding spheres of 256-voxel bricks of d_vox
     unsigned int* d_brick_list = nullptr;  // bricks kept per map (capacity nbricks)
@@ -256,6 +261,18 @@ int ensure_queue(am_ctx* ctx, long long cap) {
     return AM_OK;
 }
 
+// Texels of the map after level 0 (T1 texels per face, T1 <= cmapT: the map
+// lives in the first 6 T1^2 floats of the slot's cmap).
+int set_texels1(am_ctx* ctx, int T1) {
+    const std::vector<float> tex = make_texels(T1);
+    cudaFree(ctx->d_texels1);
+    ctx->d_texels1 = nullptr;
+    CK(cudaMalloc(&ctx->d_texels1, tex.size() * sizeof(float)));
+    CK(cudaMemcpy(ctx->d_texels1, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
+    ctx->cmapT1 = T1;
+    return AM_OK;
+}
+
 // Per-map buffers for K slots (slot s of each = the buffer of pivot s of a
 // batched launch; the single-map paths use slot 0).
 int ensure_slots(am_ctx* ctx, int K) {
@@ -331,7 +348,8 @@ int configure_launch(am_ctx* ctx) {
     CK(cudaFuncSetAttribute(bk_rows<BK_L0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_rows<BK_L1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_rows<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
-    CK(cudaFuncSetAttribute(bk_map, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_map<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_map<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     return AM_OK;
 }
 
@@ -481,6 +499,8 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.live1 = nullptr;
     F.texels = ctx->d_texels;
     F.ntex = 6 * ctx->cmapT * ctx->cmapT;
+    F.texels1 = ctx->d_texels1;
+    F.cmapT1 = ctx->cmapT1;
     F.use_l1 = ctx->phases == 2;
     F.ts = (ctx->diag_ts && ctx->d_ts) ? ctx->d_ts : nullptr;  // batched: group 0
     return F;
@@ -661,14 +681,18 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         AM_KM(AM_K_L0_CONES);
         bk_rows<BK_L0><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
         AM_KM(AM_K_L0_ROWS);
-        bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        if (F.use_l1) {
+            bk_map<true><<<grid(6 * ctx->cmapT1 * ctx->cmapT1, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        } else {
+            bk_map<false><<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+        }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
             bk_cones<BK_L1><<<grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), b, sm_rows, s>>>(F);
             AM_KM(AM_K_L1_CONES);
             bk_rows<BK_L1><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
             AM_KM(AM_K_L1_ROWS);
-            bk_map<<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+            bk_map<false><<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
             AM_KM(AM_K_CLEAR_MAP);
         }
         bk_bricks<<<grid(ctx->nbricks, 4 * kThreads, 1 << 16), b, 0, s>>>(F);
@@ -864,6 +888,7 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
             return bail(AM_ENOMEM);
         }
     }
+    if (set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT)) != AM_OK) return bail(AM_ENOMEM);
     {
         const std::vector<float> ones((size_t)6 * ctx->cmapT * ctx->cmapT, 1.0f);
         if (cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice) !=
@@ -1001,7 +1026,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
     UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * ctx->nbricks * sizeof(unsigned int)));
     brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
-                                                                                        ctx->nbricks);
+                                                                                        ctx->nbricks, kThreads);
     UK(cudaGetLastError());
     // coarse levels for the clear-direction map: level 0 = the n0 largest
     // voxels, level 1 = the next ones up to n1 plus every 512th voxel
@@ -1231,6 +1256,9 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "band_subdiv must be in [0, 3]");
         ctx->band_vdepth = (int)value;
         return AM_OK;
+    case AM_OPT_CMAP_T1:
+        if (value < 4 || value > ctx->cmapT) return fail(ctx, AM_EINVAL, "cmap_T1 must be in [4, cmap_T]");
+        return set_texels1(ctx, (int)value);
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
         {
@@ -1248,7 +1276,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
             CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice));
             ctx->cmapT = (int)value;
         }
-        return AM_OK;
+        return set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT));
     default:
         return fail(ctx, AM_EINVAL, "unknown option %d", key);
     }
@@ -1556,6 +1584,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_bricks);
     cudaFree(ctx->d_brick_list);
     cudaFree(ctx->d_texels);
+    cudaFree(ctx->d_texels1);
     cudaFree(ctx->d_cmap);
     cudaFree(ctx->d_cmap_ones);
     cudaFree(ctx->d_prev);

@@ -48,6 +48,8 @@ struct FusedParams {
     unsigned long long* task1;
     unsigned int* live1;      // level-1 live count (unused: level 1 computes cones inline)
     const float4* texels;     // clear-map texels
+    const float4* texels1;    // texels of the map after level 0 when level 1 follows (cmapT1 <= main.cmapT)
+    int cmapT1;
     int ntex;
     int use_l1;
     unsigned long long* ts;   // diagnostics: %globaltimer after each phase (CTA 0), or nullptr
@@ -360,8 +362,9 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     fused_flush(L, sAM);
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 2);
-    // 3. clear-direction map
-    clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
+    // 3. clear-direction map (at cmapT1 texels per face when level 1 follows: it only filters level 1)
+    clear_map_cta(P.gam, P.grid, P.tab, F.use_l1 ? F.texels1 : F.texels, F.use_l1 ? F.cmapT1 : P.cmapT,
+                  const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 3);
     if (F.use_l1) {
@@ -375,7 +378,8 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             ConeRec r;
             if (e < F.n1) {
                 const float4 q = F.l1[e];
-                if (fast_filter(P, q, P.gam) == F_LIVE) nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted);
+                if (fast_filter(P, q, P.gam, F.cmapT1) == F_LIVE)
+                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1);
             }
             emit_cones_cta<true>(P, rec1, task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
                                  counted, &sc, nullptr, sRowFull);

@@ -54,7 +54,8 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T);
 // F_LIVE when the voxel may still change the AM, F_CULLED beyond reach,
 // F_DROP otherwise.  A voxel holding the pivot blocks every orientation: it
 // fills `am` (shared or global) directly.
-__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am) {
+// T: texels per face of the clear-direction map in p.cmap (0 = p.cmapT).
+__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am, int T = 0) {
     const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
     const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
     const float r2 = kSqrt3 * h;
@@ -76,7 +77,7 @@ __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint
     const float s = fmaf((Reff + r2) * invD, 1.f + 1.6e-5f, 1e-6f);
     const float c = fmaf(r2 * invD, 1.f + 1.6e-5f, 1e-6f);
     const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
-    return __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < thr ? F_DROP : F_LIVE;
+    return __ldg(p.cmap + texel_of(vx, vy, vz, T ? T : p.cmapT)) < thr ? F_DROP : F_LIVE;
 }
 
 // Cube-map texel of v (cube_texel of kernels.cuh with an approximate
@@ -245,17 +246,17 @@ __global__ void __launch_bounds__(kThreads) brick_voxels_kernel(const __grid_con
     }
 }
 
-// Bounding spheres of the bricks of kThreads consecutive voxels (one warp per
+// Bounding spheres of the bricks of bs consecutive voxels (one warp per
 // brick): centre of the box enclosing the voxel cubes, radius its half
 // diagonal, grown for rounding.
 __global__ void brick_bounds_kernel(const float4* __restrict__ vox, long long N, float4* __restrict__ bricks,
-                                    unsigned int nb) {
+                                    unsigned int nb, int bs) {
     const int lane = threadIdx.x & 31;
     const unsigned int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (w >= nb) return;
     float lo[3] = {3e38f, 3e38f, 3e38f}, hi[3] = {-3e38f, -3e38f, -3e38f};
-    for (int k = lane; k < kThreads; k += 32) {
-        const long long i = (long long)w * kThreads + k;
+    for (int k = lane; k < bs; k += 32) {
+        const long long i = (long long)w * bs + k;
         if (i >= N) break;
         const float4 q = vox[i];
         lo[0] = fminf(lo[0], q.x - q.w); hi[0] = fmaxf(hi[0], q.x + q.w);
@@ -311,7 +312,8 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
 // would use.
 template <bool COARSE>
 __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, unsigned int vidx, ConeRec& r,
-                                             bool& counted, const float4* clear = nullptr, int nclear = -1) {
+                                             bool& counted, const float4* clear = nullptr, int nclear = -1,
+                                             int cmT = 0) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
     counted = false;
@@ -331,7 +333,7 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
     }
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
-    if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
+    if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, cmT ? cmT : p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
     if (nclear >= 0) {
         const float inv = 1.f / D;
         const float ux = vx * inv, uy = vy * inv, uz = vz * inv;

@@ -254,6 +254,13 @@ def test_phases_and_tunables_give_identical_maps(am, name):
     assert np.array_equal(ctx.compute_batch(P), ref)
     ctx.set_option(am.binding.OPT_CMAP_T, 18)  # not a multiple of 4: per-texel search over all cells
     assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_CMAP_T, 128)
+    for t1 in (64, 37, 128):  # the map after level 0 at its own resolution (<= cmap_T)
+        ctx.set_option(am.binding.OPT_CMAP_T1, t1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+    with pytest.raises(am.AMError):
+        ctx.set_option(am.binding.OPT_CMAP_T1, 129)  # larger than cmap_T
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
