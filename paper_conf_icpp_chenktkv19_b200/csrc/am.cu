@@ -32,6 +32,9 @@ using namespace am;
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 32
 #endif
+#ifndef AM_MAP1_WARP_BLOCKS
+#define AM_MAP1_WARP_BLOCKS 4
+#endif
 #ifndef AM_L0_DIV
 #define AM_L0_DIV 8192
 #endif
@@ -682,7 +685,12 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         bk_rows<BK_L0><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
         AM_KM(AM_K_L0_ROWS);
         if (F.use_l1) {
-            bk_map<true><<<grid(6 * ctx->cmapT1 * ctx->cmapT1, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+            // (few texels, many clear cells after level 0: spread them over more CTAs -- one
+            // warp per 4 x 4 coarse texel on the coarse-block path)
+            const long long nt1 = 6ll * ctx->cmapT1 * ctx->cmapT1;
+            bk_map<true><<<grid(std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32))), 1,
+                                1 << 16),
+                           b, ctx->smem_fused, s>>>(F);
         } else {
             bk_map<false><<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
         }
