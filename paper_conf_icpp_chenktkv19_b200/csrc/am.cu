@@ -132,7 +132,6 @@ namespace {
 // [1, 1 + ST_COUNT) am_stats of the full stream, then the per-stage counters,
 // then scratch stats for the clear-map levels.
 constexpr int kCtrTiles = 1 + ST_COUNT;      // live count: full stream (+0), level 1 (+4)
-constexpr int kCtrClear = kCtrTiles + 1;     // clear-cell counts of the (up to 3) maps of a call
 constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, task count at +2s+1
 constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
 constexpr int kCtrWords = kCtrBricks + 1;

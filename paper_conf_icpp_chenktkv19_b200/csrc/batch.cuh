@@ -66,12 +66,12 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     __shared__ FusedScratch sc;
     const int p = blockIdx.y;
     pivot_params(sP, F, p, STAGE == BK_L0);
-    __shared__ int sN;
     const StreamParams& P = sP;
     const int m = P.grid.m, MW = m * P.grid.W;
     uint32_t* sAM = smem_bk;
     uint32_t* sRowFull = sAM + MW;
     float4* sDirs = reinterpret_cast<float4*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_dirs_offset(m, P.grid.W));
+    int* sRowStart = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_rows_offset(m, P.grid.W));
     int nclear = -1;
     unsigned long long n;
     if (STAGE == BK_L0) {
@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
             n = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
         if ((unsigned long long)blockIdx.x * blockDim.x >= n) return;  // CTA-uniform
         fused_seed(P, sAM, sRowFull);
-        if (STAGE == BK_LIVE) nclear = clear_list_cta(sAM, P.grid, P.tab, sDirs, &sN);
+        if (STAGE == BK_LIVE) nclear = clear_list_rows_cta(sAM, P.grid, P.tab, sDirs, sRowStart);
     }
     unsigned int* rc = STAGE == BK_L1 ? shift_bytes(F.rec1, p * F.ctr_stride) : P.rec_count;
     unsigned long long* tc = STAGE == BK_L1 ? shift_bytes(F.task1, p * F.ctr_stride) : P.task_count;
@@ -111,7 +111,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
                     nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1);
             } else {
                 const unsigned int vidx = P.live_idx[e];
-                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear);
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear, 0, sRowStart);
             }
         }
         emit_cones_cta<STAGE != BK_LIVE>(P, rc, tc, roff, toff, rcap, tcap, nrows, r, counted, &sc,

@@ -134,8 +134,12 @@ __device__ __forceinline__ void fused_mark(const FusedParams& F, int k) {
 __host__ __device__ inline size_t fused_dirs_offset(int m, int W) {
     return ((size_t)(m * W + ((m + 31) >> 5) + 1) * sizeof(uint32_t) + 15) & ~(size_t)15;
 }
-__host__ __device__ inline size_t fused_smem_bytes(int m, int W) {
+// then the row starts of the live phase's clear list (m + 1 ints)
+__host__ __device__ inline size_t fused_rows_offset(int m, int W) {
     return fused_dirs_offset(m, W) + (size_t)kMapDirs * sizeof(float4);
+}
+__host__ __device__ inline size_t fused_smem_bytes(int m, int W) {
+    return fused_rows_offset(m, W) + (size_t)(m + 1) * sizeof(int);
 }
 
 // Seed the shared AM from the global AM and compute the row-full bits.
@@ -474,7 +478,8 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     // 8b. both cones of the live voxels, spread over every thread of the grid (stage 2),
     //     checked against the list of cells still clear
     {
-        const int nclear = clear_list_cta(sAM, P.grid, P.tab, sDirs, &S.n);
+        int* sRowStart = reinterpret_cast<int*>(smem_raw + fused_rows_offset(m, P.grid.W));
+        const int nclear = clear_list_rows_cta(sAM, P.grid, P.tab, sDirs, sRowStart);
         const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
         for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
@@ -483,7 +488,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             ConeRec r;
             if (e < nlive) {
                 const unsigned int vidx = P.live_idx[e];
-                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear);
+                nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear, 0, sRowStart);
             }
             emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
                                   &sc, P.stats + ST_LIVE, sRowFull);

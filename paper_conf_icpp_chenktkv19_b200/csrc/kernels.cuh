@@ -239,6 +239,57 @@ __device__ int clear_list_cta(const uint32_t* sAM, const GridDev& g, const float
     return total;
 }
 
+// The cells still clear in sAM as directions in sDirs in row-major order, with
+// sRowStart[i] = index of row i's first (sRowStart[m] = the count), by the
+// whole CTA; returns the count, or -1 (no list) when there are more than
+// kMapDirs.  A cone that spans rows a0..a1 only needs [sRowStart[a0], sRowStart[a1 + 1]).
+__device__ int clear_list_rows_cta(const uint32_t* sAM, const GridDev& g, const float* __restrict__ tab,
+                                   float4* sDirs, int* sRowStart) {
+    const int m = g.m, W = g.W;
+    __syncthreads();
+    for (int i = threadIdx.x; i < m; i += blockDim.x) {
+        int c = 0;
+        for (int w = 0; w < W; ++w) c += __popc(~sAM[i * W + w] & row_word_mask(w, g.n));
+        sRowStart[i + 1] = c;
+    }
+    if (threadIdx.x == 0) sRowStart[0] = 0;
+    __syncthreads();
+    if (threadIdx.x < 32) {  // prefix sums: each lane a chunk of rows, then a warp scan of the chunk sums
+        const int lane = threadIdx.x, per = (m + 31) >> 5;
+        const int b = 1 + lane * per, e = min(m + 1, b + per);
+        int sum = 0;
+        for (int k = b; k < e; ++k) sum += sRowStart[k];
+        int incl = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += t;
+        }
+        int run = incl - sum;
+        for (int k = b; k < e; ++k) {
+            run += sRowStart[k];
+            sRowStart[k] = run;
+        }
+    }
+    __syncthreads();
+    const int total = sRowStart[m];
+    if (total > kMapDirs) return -1;
+    for (int i = threadIdx.x; i < m; i += blockDim.x) {
+        int pos = sRowStart[i];
+        const float cph = __ldg(tab + i), sph = __ldg(tab + m + i);
+        for (int w = 0; w < W; ++w) {
+            uint32_t clear = ~sAM[i * W + w] & row_word_mask(w, g.n);
+            while (clear) {
+                const int j = (w << 5) + __ffs(clear) - 1;
+                clear &= clear - 1u;
+                sDirs[pos++] = make_float4(sph * __ldg(tab + 2 * m + j), sph * __ldg(tab + 2 * m + g.n + j), cph, 0.f);
+            }
+        }
+    }
+    __syncthreads();
+    return total;
+}
+
 // The clear-direction map of `gam` into V (6 T^2 texels), computed by the CTAs
 // gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
 // (kMapDirs), sN.

@@ -313,7 +313,7 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
 template <bool COARSE>
 __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, unsigned int vidx, ConeRec& r,
                                              bool& counted, const float4* clear = nullptr, int nclear = -1,
-                                             int cmT = 0) {
+                                             int cmT = 0, const int* rowStart = nullptr) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
     counted = false;
@@ -334,12 +334,20 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
     if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, cmT ? cmT : p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
+    const float rxy = sqrtf(vx * vx + vy * vy);
+    const float phv = atan2f(rxy, vz);
+    const float ao = acosf(fmaxf(c.cout, -1.f));
+    const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
+    const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
+    if (a0 > a1) return 0;
     if (nclear >= 0) {
+        // only cells of the rows a0..a1 the raster would visit can be changed by this voxel
         const float inv = 1.f / D;
         const float ux = vx * inv, uy = vy * inv, uz = vz * inv;
         const float lo = c.cout - kClearSlack, hi = c.clo + kClearSlack;
         bool any = false;
-        for (int e = 0; e < nclear; ++e) {
+        const int e0 = rowStart ? rowStart[a0] : 0, e1 = rowStart ? rowStart[a1 + 1] : nclear;
+        for (int e = e0; e < e1; ++e) {
             const float4 d = clear[e];
             const float cd = fmaf(ux, d.x, fmaf(uy, d.y, uz * d.z));
             if (cd >= lo && cd <= hi) {
@@ -349,12 +357,6 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
         }
         if (!any) return 0;
     }
-    const float rxy = sqrtf(vx * vx + vy * vy);
-    const float phv = atan2f(rxy, vz);
-    const float ao = acosf(fmaxf(c.cout, -1.f));
-    const int a0 = max(0, (int)ceilf((phv - ao - kRowSlack) * g.inv_dphi - 0.5f));
-    const int a1 = min(g.m - 1, (int)floorf((phv + ao + kRowSlack) * g.inv_dphi - 0.5f));
-    if (a0 > a1) return 0;
     const float invD = 1.f / D;
     r.cin = c.cin;
     r.cout = c.cout;

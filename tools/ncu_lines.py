@@ -1,6 +1,6 @@
 """Attribute an ncu capture's per-SASS-instruction counts to CUDA source lines.
 
-    python tools/ncu_lines.py <report.ncu-rep> <mangled kernel name> [libam.so] [top]
+    python tools/ncu_lines.py <report.ncu-rep> <mangled kernel name> [libam.so] [top] [block index]
 
 Needs the .so that was profiled (line info from -lineinfo): its SASS offsets
 are matched with the report's SASS page.  Prints instructions executed and
@@ -68,6 +68,8 @@ def main():
             cur["rows"].append(r)
     lines = sass_lines(so, func)
     srcs = {}
+    if len(sys.argv) > 5:  # only the kernel block(s) of this index in the report (the one `func` names)
+        blocks = [blocks[int(i)] for i in sys.argv[5].split(",")]
     for b in blocks:
         hdr = b["rows"][0]
         ix = {k: i for i, k in enumerate(hdr)}
