@@ -275,9 +275,12 @@ def run_ours(args):
     stats = [ctx.compute(p, stats=True)[1] for p in piv]
     mean = {k: float(np.mean([getattr(s_, k) for s_ in stats])) for k in stats[0].__dict__}
 
-    # ---- timed region: K steps of `bsz` pivots each (one am_compute_batch call, one fused
-    #      launch), L2 flushed before each step, CUDA events on the launching stream
-    ctx.set_option(B.OPT_KERNEL_TIMING, 2)  # events around the batch AND after every kernel launch
+    # ---- timed region: K steps of `bsz` pivots each (one am_compute_batch call: one
+    #      launch per phase over all pivots), L2 flushed before each step, CUDA events on
+    #      the launching stream around each step (AM_OPT_KERNEL_TIMING = 1: no event
+    #      between the phase launches, which would serialise their programmatic
+    #      dependent launches)
+    ctx.set_option(B.OPT_KERNEL_TIMING, 1)
     ctx.kernel_time()
     ctx.kernel_stats()
     if dist:
@@ -289,6 +292,12 @@ def run_ours(args):
         dist.barrier()
     torch.cuda.synchronize(dev)
     kms, klaunch = ctx.kernel_time()
+    kstats_timed = {k: v for k, v in ctx.kernel_stats().items() if v[1] > 0}  # launch counts of the timed region
+    # ---- the same K steps again with a CUDA event after every kernel launch
+    #      (AM_OPT_KERNEL_TIMING = 2): per-kernel device times for `kernels` / `roofline`
+    ctx.set_option(B.OPT_KERNEL_TIMING, 2)
+    ms_kev, _ = _timed_maps(ctx, piv, out, stream, args.steps, flush, torch, bsz)
+    ctx.kernel_time()
     kstats = {k: v for k, v in ctx.kernel_stats().items() if v[1] > 0}
     ctx.set_option(B.OPT_KERNEL_TIMING, 1)
     # single-pivot latency (am_compute, one fused launch per map), flushed: detail
@@ -399,7 +408,10 @@ def run_ours(args):
                     "note": f"am_compute_batch with {bsz} host pivots (12 B each, copied into the launch) and a "
                             "host AM buffer; synchronous per step; voxels resident (upload excluded, PAPER.md L313); "
                             "L2 flushed before each step, outside the per-step clock"},
-            "gpu_launches": int(sum(v[1] for v in kstats.values())),
+            "gpu_launches": int(sum(v[1] for v in kstats_timed.values())),
+            "kernels_note": "per-kernel device times from a second pass of the same K steps with a CUDA event "
+                            "after every launch (serialises the phase launches: ms_per_am_with_kernel_events)",
+            "ms_per_am_with_kernel_events": ms_kev / args.steps / bsz,
             "kernels": {k: {"ms_per_am": v[0] / maps_rank, "launches": v[1],
                             "share": v[0] / max(sum(x[0] for x in kstats.values()), 1e-12)}
                         for k, v in sorted(kstats.items(), key=lambda kv: -kv[1][0])},

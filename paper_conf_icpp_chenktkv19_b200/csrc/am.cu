@@ -35,6 +35,9 @@ using namespace am;
 #ifndef AM_MAP1_WARP_BLOCKS
 #define AM_MAP1_WARP_BLOCKS 4
 #endif
+#ifndef AM_BAND_CTAS
+#define AM_BAND_CTAS 8
+#endif
 #ifndef AM_L0_DIV
 #define AM_L0_DIV 8192
 #endif
@@ -679,38 +682,44 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         };
         const dim3 b(kThreads);
 #define AM_KM(k) if ((rc = kmark(ctx, s, k))) return rc
+        auto L = [&](auto kern, dim3 g, size_t smem) -> int {
+            kern<<<g, b, smem, s>>>(F);
+            return AM_OK;
+        };
         bk_cones<BK_L0><<<grid(ctx->n_l0, kThreads, 1 << 16), b, sm_rows, s>>>(F);
         AM_KM(AM_K_L0_CONES);
-        bk_rows<BK_L0><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
         AM_KM(AM_K_L0_ROWS);
         if (F.use_l1) {
             // (few texels, many clear cells after level 0: spread them over more CTAs -- one
             // warp per 4 x 4 coarse texel on the coarse-block path)
             const long long nt1 = 6ll * ctx->cmapT1 * ctx->cmapT1;
-            bk_map<true><<<grid(std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32))), 1,
-                                1 << 16),
-                           b, ctx->smem_fused, s>>>(F);
+            if ((rc = L(bk_map<true>,
+                        grid(std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32))), 1,
+                             1 << 16),
+                        ctx->smem_fused)))
+                return rc;
         } else {
-            bk_map<false><<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, 1 << 16), ctx->smem_fused))) return rc;
         }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
-            bk_cones<BK_L1><<<grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), b, sm_rows, s>>>(F);
+            if ((rc = L(bk_cones<BK_L1>, grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), sm_rows))) return rc;
             AM_KM(AM_K_L1_CONES);
-            bk_rows<BK_L1><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+            if ((rc = L(bk_rows<BK_L1>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
             AM_KM(AM_K_L1_ROWS);
-            bk_map<false><<<grid(ntex, 4 * kThreads, 1 << 16), b, ctx->smem_fused, s>>>(F);
+            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, 1 << 16), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
         }
-        bk_bricks<<<grid(ctx->nbricks, 4 * kThreads, 1 << 16), b, 0, s>>>(F);
+        if ((rc = L(bk_bricks, grid(ctx->nbricks, 4 * kThreads, 1 << 16), 0))) return rc;
         AM_KM(AM_K_BRICKS);
-        bk_voxels<<<grid(1 << 30, 1, ctx->bk_voxel_ctas), b, 0, s>>>(F);
+        if ((rc = L(bk_voxels, grid(1 << 30, 1, ctx->bk_voxel_ctas), 0))) return rc;
         AM_KM(AM_K_VOXELS);
-        bk_cones<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_cone_ctas), b, ctx->smem_fused, s>>>(F);
+        if ((rc = L(bk_cones<BK_LIVE>, grid(1 << 30, 1, ctx->bk_cone_ctas), ctx->smem_fused))) return rc;
         AM_KM(AM_K_LIVE_CONES);
-        bk_rows<BK_LIVE><<<grid(1 << 30, 1, ctx->bk_rows_ctas), b, sm_rows, s>>>(F);
+        if ((rc = L(bk_rows<BK_LIVE>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
         AM_KM(AM_K_LIVE_ROWS);
-        bk_band<<<grid(1 << 30, 1, 8), b, 0, s>>>(F);
+        if ((rc = L(bk_band, grid(1 << 30, 1, AM_BAND_CTAS), 0))) return rc;
         AM_KM(AM_K_BAND);
 #undef AM_KM
         if ((rc = timed_end(ctx, s))) return rc;

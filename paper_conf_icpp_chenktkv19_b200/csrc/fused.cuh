@@ -241,13 +241,26 @@ __device__ __forceinline__ void cta_reserve2(unsigned int ca, unsigned int* ga, 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     unsigned int ia = ca;
     unsigned long long ib = cb;
+    if (__all_sync(0xffffffffu, ca <= 1u && cb < (1ull << 20))) {
+        // the common case (a record flag and a row count per thread): one 32-bit scan of
+        // (ca << 25) | cb -- over 32 lanes the sums stay below 2^6 and 2^25
+        unsigned int v = (ca << 25) | (unsigned int)cb;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const unsigned int ta = __shfl_up_sync(0xffffffffu, ia, o);
-        const unsigned long long tb = __shfl_up_sync(0xffffffffu, ib, o);
-        if (lane >= o) {
-            ia += ta;
-            ib += tb;
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned int t = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += t;
+        }
+        ia = v >> 25;
+        ib = v & ((1u << 25) - 1u);
+    } else {
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned int ta = __shfl_up_sync(0xffffffffu, ia, o);
+            const unsigned long long tb = __shfl_up_sync(0xffffffffu, ib, o);
+            if (lane >= o) {
+                ia += ta;
+                ib += tb;
+            }
         }
     }
     if (lane == 31) {
@@ -293,6 +306,7 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
     int ntask = 0;
     if (nrows > 0)
         for (int w = i0 >> 5; w <= (i1 >> 5); ++w) ntask += __popc(open_rows_word(rowfull, i0, i1, w));
+    if (!__syncthreads_or(ntask > 0)) return;  // nothing to emit in the whole CTA (CTA-uniform)
     unsigned int slot;
     unsigned long long t0;
     cta_reserve2(ntask > 0 ? 1u : 0u, rec_count, (unsigned long long)ntask, task_count, sc, slot, t0);
