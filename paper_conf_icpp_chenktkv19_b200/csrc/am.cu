@@ -36,7 +36,10 @@ using namespace am;
 #define AM_MAP1_WARP_BLOCKS 4
 #endif
 #ifndef AM_BAND_CTAS
-#define AM_BAND_CTAS 8
+#define AM_BAND_CTAS 24
+#endif
+#ifndef AM_BAND_THREADS
+#define AM_BAND_THREADS 256
 #endif
 #ifndef AM_L0_DIV
 #define AM_L0_DIV 8192
@@ -682,8 +685,8 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         };
         const dim3 b(kThreads);
 #define AM_KM(k) if ((rc = kmark(ctx, s, k))) return rc
-        auto L = [&](auto kern, dim3 g, size_t smem) -> int {
-            kern<<<g, b, smem, s>>>(F);
+        auto L = [&](auto kern, dim3 g, size_t smem, dim3 bd = dim3(kThreads)) -> int {
+            kern<<<g, bd, smem, s>>>(F);
             return AM_OK;
         };
         bk_cones<BK_L0><<<grid(ctx->n_l0, kThreads, 1 << 16), b, sm_rows, s>>>(F);
@@ -719,7 +722,8 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         AM_KM(AM_K_LIVE_CONES);
         if ((rc = L(bk_rows<BK_LIVE>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
         AM_KM(AM_K_LIVE_ROWS);
-        if ((rc = L(bk_band, grid(1 << 30, 1, AM_BAND_CTAS), 0))) return rc;
+        // (few pairs, each a long exact test: small CTAs spread them over the SMs)
+        if ((rc = L(bk_band, grid(1 << 30, 1, AM_BAND_CTAS), 0, dim3(AM_BAND_THREADS)))) return rc;
         AM_KM(AM_K_BAND);
 #undef AM_KM
         if ((rc = timed_end(ctx, s))) return rc;
