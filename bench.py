@@ -257,6 +257,14 @@ def run_ours(args):
         ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
     if args.cmap_t1:
         ctx.set_option(B.OPT_CMAP_T1, args.cmap_t1)
+    if args.cmap_rowscan >= 0:
+        ctx.set_option(B.OPT_CMAP_ROWSCAN, args.cmap_rowscan)
+    if args.cmap_brute >= 0:
+        ctx.set_option(B.OPT_CMAP_BRUTE, args.cmap_brute)
+    if args.cmap_block:
+        ctx.set_option(B.OPT_CMAP_BLOCK, args.cmap_block)
+    if args.map_ctas >= 0:
+        ctx.set_option(B.OPT_MAP_CTAS, args.map_ctas)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
     if args.band_subdiv:
@@ -512,6 +520,10 @@ def main():
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
     ap.add_argument("--cmap-t", type=int, default=0, help="AM_OPT_CMAP_T (0 = library default)")
     ap.add_argument("--cmap-t1", type=int, default=0, help="AM_OPT_CMAP_T1 (0 = library default)")
+    ap.add_argument("--cmap-rowscan", type=int, default=-1, help="AM_OPT_CMAP_ROWSCAN (-1 = library default)")
+    ap.add_argument("--cmap-brute", type=int, default=-1, help="AM_OPT_CMAP_BRUTE (-1 = library default)")
+    ap.add_argument("--cmap-block", type=int, default=0, help="AM_OPT_CMAP_BLOCK (0 = library default)")
+    ap.add_argument("--map-ctas", type=int, default=-1, help="AM_OPT_MAP_CTAS (-1 = library default)")
     ap.add_argument("--phases", type=int, default=None, help="AM_OPT_PHASES (coarse levels, 1 or 2)")
     ap.add_argument("--band-subdiv", type=int, default=0,
                     help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")

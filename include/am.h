@@ -104,8 +104,24 @@ enum {
     AM_OPT_BAND_SUBDIV = 13,     /* band pairs: levels of virtual 2x2x2 sub-cubes decided by
                                     CHECKICA before CHECKBOX (§4.3; 0..3,
                                     default 0 = CHECKBOX directly).  Same map outside the band  */
-    AM_OPT_CMAP_T1 = 14          /* resolution of the clear-direction map built after level 0,
+    AM_OPT_CMAP_T1 = 14,         /* resolution of the clear-direction map built after level 0,
                                     which only filters level 1 (4..AM_OPT_CMAP_T, default 32).
+                                    Same map                                                    */
+    AM_OPT_CMAP_ROWSCAN = 15,    /* clear-direction map: with more clear cells than this, each
+                                    texel finds its nearest clear cell row by row (nearest clear
+                                    gamma per phi-row, rows outward from the texel's phi, early
+                                    stop); otherwise every texel tries every clear cell
+                                    (0..2^21, default 2^21: off).                               */
+    AM_OPT_CMAP_BRUTE = 16,      /* clear-direction map: with at most this many clear cells every
+                                    texel tries every one; above, texel blocks first bound   
+                                    the candidates from the block centre (0..2^21, default
+                                    0).  Same map                                               */
+    AM_OPT_CMAP_BLOCK = 17,      /* clear-direction map: side of the texel blocks (one warp each)
+                                    whose centre bounds the candidate cells on that path: 4 or 8
+                                    (default 8; a map resolution that is not a multiple falls
+                                    back to 4, then to every texel x every cell).  Same map      */
+    AM_OPT_MAP_CTAS = 18         /* batched path: CTAs per pivot of the (final) clear-direction
+                                    map launch, 0..4096 (0 = one per 1024 texels; default 48).
                                     Same map                                                    */
 };
 

@@ -29,6 +29,18 @@ using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
 // level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_MAP_CTAS
+#define AM_MAP_CTAS 48
+#endif
+#ifndef AM_CMAP_BLOCK
+#define AM_CMAP_BLOCK 8
+#endif
+#ifndef AM_CMAP_BRUTE
+#define AM_CMAP_BRUTE 0
+#endif
+#ifndef AM_CMAP_ROWSCAN
+#define AM_CMAP_ROWSCAN 2097152
+#endif
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 32
 #endif
@@ -101,6 +113,7 @@ struct am_ctx {
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
     int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
+    int bk_map_ctas = AM_MAP_CTAS;         // per pivot, batched clear map (AM_OPT_MAP_CTAS; 0 = texels / 1024)
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
     long long piv_cap = 0;
@@ -684,6 +697,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             return dim3((unsigned)std::max<long long>(1, std::min<long long>(gx, cap)), (unsigned)kk);
         };
         const dim3 b(kThreads);
+        const int map_cap = ctx->bk_map_ctas > 0 ? ctx->bk_map_ctas : (1 << 16);
 #define AM_KM(k) if ((rc = kmark(ctx, s, k))) return rc
         auto L = [&](auto kern, dim3 g, size_t smem, dim3 bd = dim3(kThreads)) -> int {
             kern<<<g, bd, smem, s>>>(F);
@@ -703,7 +717,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
                         ctx->smem_fused)))
                 return rc;
         } else {
-            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, 1 << 16), ctx->smem_fused))) return rc;
+            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
         }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
@@ -711,7 +725,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             AM_KM(AM_K_L1_CONES);
             if ((rc = L(bk_rows<BK_L1>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
             AM_KM(AM_K_L1_ROWS);
-            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, 1 << 16), ctx->smem_fused))) return rc;
+            if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
         }
         if ((rc = L(bk_bricks, grid(ctx->nbricks, 4 * kThreads, 1 << 16), 0))) return rc;
@@ -866,6 +880,9 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
     G.inv_dphi = (float)(m / PI);
     G.dgam = (float)(2.0 * PI / n);
     G.inv_dgam = (float)(n / (2.0 * PI));
+    G.rowscan = AM_CMAP_ROWSCAN;
+    G.brute = AM_CMAP_BRUTE;
+    G.cblock = AM_CMAP_BLOCK;
     ctx->MW = m * G.W;
     int rc;
     cudaDeviceProp prop;
@@ -1275,6 +1292,22 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_BAND_SUBDIV:
         if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "band_subdiv must be in [0, 3]");
         ctx->band_vdepth = (int)value;
+        return AM_OK;
+    case AM_OPT_CMAP_ROWSCAN:
+        if (value < 0 || value > (1 << 21)) return fail(ctx, AM_EINVAL, "cmap_rowscan must be in [0, 2^21]");
+        ctx->grid.rowscan = (int)value;
+        return AM_OK;
+    case AM_OPT_CMAP_BRUTE:
+        if (value < 0 || value > (1 << 21)) return fail(ctx, AM_EINVAL, "cmap_brute must be in [0, 2^21]");
+        ctx->grid.brute = (int)value;
+        return AM_OK;
+    case AM_OPT_CMAP_BLOCK:
+        if (value != 4 && value != 8) return fail(ctx, AM_EINVAL, "cmap_block must be 4 or 8");
+        ctx->grid.cblock = (int)value;
+        return AM_OK;
+    case AM_OPT_MAP_CTAS:
+        if (value < 0 || value > 4096) return fail(ctx, AM_EINVAL, "map_ctas must be in [0, 4096]");
+        ctx->bk_map_ctas = (int)value;
         return AM_OK;
     case AM_OPT_CMAP_T1:
         if (value < 4 || value > ctx->cmapT) return fail(ctx, AM_EINVAL, "cmap_T1 must be in [4, cmap_T]");

@@ -55,6 +55,9 @@ struct GridDev {
     int m, n, W;            // rows (phi), columns (gamma), words per row
     float dphi, inv_dphi;   // pi / m
     float dgam, inv_dgam;   // 2 pi / n
+    int rowscan;            // clear map: above this many clear cells, the row-ordered search (AM_OPT_CMAP_ROWSCAN)
+    int brute;              // clear map: up to this many, every texel tries every clear cell (AM_OPT_CMAP_BRUTE)
+    int cblock;             // clear map: texel block side of the candidate-bounded path (AM_OPT_CMAP_BLOCK)
 };
 
 // Guards: the inner cone is shrunk and the outer cone

@@ -181,10 +181,6 @@ __device__ __forceinline__ void push_band(const StreamParams& p, uint32_t* sAM, 
 // tries every clear direction (in chunks), 4 texels per thread.
 
 constexpr int kMapDirs = 2048;  // clear directions staged in shared memory per chunk
-#ifndef AM_MAP_BRUTE
-#define AM_MAP_BRUTE 512
-#endif
-constexpr int kMapBrute = AM_MAP_BRUTE;  // up to this many clear cells, every texel tries every one
 
 __device__ __forceinline__ float dot3(float4 a, float4 b) { return fmaf(a.x, b.x, fmaf(a.y, b.y, a.z * b.z)); }
 
@@ -193,8 +189,17 @@ __device__ __forceinline__ float dot3(float4 a, float4 b) { return fmaf(a.x, b.x
 __device__ __forceinline__ float clear_map_value(float best, float r) {
     float u = -2.f;
     if (best >= -1.5f) {
-        const float th = acosf(fminf(best + 2e-6f, 1.f));
-        u = (th <= r) ? 1.f : fminf(cosf(th - r) + 4e-6f, 1.f);
+        // cos(max(0, th - r)) with cos th = b, without acos/cos: b cos r + sin th sin r
+        // (sin th = sqrt((1 - b)(1 + b)) >= 0); the error of the fast sin/cos and of
+        // the square root (< 1e-6 here: sin th is multiplied by sin r) is inside the guard
+        const float b = fminf(best + 2e-6f, 1.f);
+        const float cr = __cosf(r), sr = __sinf(r);
+        if (b >= cr) {
+            u = 1.f;
+        } else {
+            const float st = sqrtf(fmaxf((1.f - b) * (1.f + b), 0.f));
+            u = fminf(fmaf(b, cr, st * sr) + 4e-6f, 1.f);
+        }
     }
     return u * fabsf(u);
 }
@@ -219,6 +224,102 @@ __device__ void compact_clear_dirs(const uint32_t* sAM, const GridDev& g, const 
         }
     }
     __syncthreads();
+}
+
+// Row-ordered nearest-clear search (the clear map's large-count path).  For a
+// direction c = (sin phi_c cos g_c, sin phi_c sin g_c, cos phi_c) and a cell of
+// row i, cos angle = cos phi_i cos phi_c + sin phi_i sin phi_c cos(g_j - g_c):
+// both sines are >= 0 (phi in (0, pi)), so within a row the best cell is the
+// clear cell nearest to g_c in circular gamma -- the first clear cell at or
+// after g_c or the last one before it -- and no cell of row i can beat
+// ub_i = cos(phi_i - phi_c).  Rows are visited from phi_c outward (ub
+// decreasing in each direction, larger ub first) and the search stops once both
+// directions' ub fall below the best cosine found.  Result: the maximum of
+// c . d over the clear cells, as the all-pairs loop computes it, up to fp32
+// rounding of the same dot products (absorbed by clear_map_value's guards).
+// clr: per-row clear masks (W words per row, padding bits 0); rows: one bit per
+// row with a clear cell.
+__device__ __forceinline__ int next_row_at_or_after(const uint32_t* rows, int i, int m) {
+    if (i >= m) return m;
+    int w = i >> 5;
+    uint32_t x = rows[w] & (0xffffffffu << (i & 31));
+    const int RW = (m + 31) >> 5;
+    while (!x) {
+        if (++w >= RW) return m;
+        x = rows[w];
+    }
+    return (w << 5) + __ffs(x) - 1;
+}
+
+__device__ __forceinline__ int prev_row_at_or_before(const uint32_t* rows, int i) {
+    if (i < 0) return -1;
+    int w = i >> 5;
+    uint32_t x = rows[w] & (0xffffffffu >> (31 - (i & 31)));
+    while (!x) {
+        if (--w < 0) return -1;
+        x = rows[w];
+    }
+    return (w << 5) + 31 - __clz(x);
+}
+
+__device__ __forceinline__ float row_best_cos(float4 c, const uint32_t* clr, int i, int j0, const GridDev& g,
+                                              const float* __restrict__ tab) {
+    const int W = g.W, n = g.n;
+    const uint32_t* row = clr + i * W;
+    // first clear cell at or after j0 (circular; the row has one)
+    int w = j0 >> 5;
+    uint32_t x = row[w] & (0xffffffffu << (j0 & 31));
+    while (!x) {
+        w = (w + 1 == W) ? 0 : w + 1;
+        x = row[w];
+    }
+    const int jr = (w << 5) + __ffs(x) - 1;
+    // last clear cell at or before j0 - 1 (circular)
+    const int jl0 = j0 == 0 ? n - 1 : j0 - 1;
+    w = jl0 >> 5;
+    x = row[w] & (0xffffffffu >> (31 - (jl0 & 31)));
+    while (!x) {
+        w = (w == 0) ? W - 1 : w - 1;
+        x = row[w];
+    }
+    const int jl = (w << 5) + 31 - __clz(x);
+    const float cph = __ldg(tab + i), sph = __ldg(tab + g.m + i);
+    const float* cg = tab + 2 * g.m;
+    const float* sg = cg + n;
+    const float br = fmaf(cph, c.z, sph * fmaf(c.x, __ldg(cg + jr), c.y * __ldg(sg + jr)));
+    const float bl = fmaf(cph, c.z, sph * fmaf(c.x, __ldg(cg + jl), c.y * __ldg(sg + jl)));
+    return fmaxf(br, bl);
+}
+
+__device__ float nearest_clear_rows(float4 c, const uint32_t* clr, const uint32_t* rows, const GridDev& g,
+                                    const float* __restrict__ tab) {
+    const int m = g.m, n = g.n;
+    const float cz = fminf(fmaxf(c.z, -1.f), 1.f);
+    const float sc = sqrtf(fmaf(c.x, c.x, c.y * c.y));
+    const float phic = acosf(cz);
+    float gc = atan2f(c.y, c.x);
+    if (gc < 0.f) gc += 6.2831853071795865f;
+    int j0 = (int)ceilf(fmaf(gc, g.inv_dgam, -0.5f));
+    j0 = j0 < 0 ? 0 : (j0 >= n ? 0 : j0);
+    // row ic: phi_ic <= phi_c < phi_ic+1 (up to rounding: ub is then non-monotone only at rounding level)
+    const int ic = min(m - 1, max(-1, (int)floorf(fmaf(phic, g.inv_dphi, -0.5f))));
+    int id = prev_row_at_or_before(rows, ic);
+    int iu = next_row_at_or_after(rows, ic + 1, m);
+    float best = -2.f;
+    for (;;) {
+        const float ud = id >= 0 ? fmaf(__ldg(tab + id), cz, __ldg(tab + m + id) * sc) : -3.f;
+        const float uu = iu < m ? fmaf(__ldg(tab + iu), cz, __ldg(tab + m + iu) * sc) : -3.f;
+        const bool down = ud >= uu;
+        const float ub = down ? ud : uu;
+        if (ub < best - 1e-6f || ub < -2.5f) break;
+        const int i = down ? id : iu;
+        best = fmaxf(best, row_best_cos(c, clr, i, j0, g, tab));
+        if (down)
+            id = prev_row_at_or_before(rows, id - 1);
+        else
+            iu = next_row_at_or_after(rows, iu + 1, m);
+    }
+    return best;
 }
 
 // The cells still clear in sAM as directions in sDirs, by the whole CTA; returns
@@ -290,6 +391,70 @@ __device__ int clear_list_rows_cta(const uint32_t* sAM, const GridDev& g, const 
     return total;
 }
 
+// Coarse-block path for B x B texel blocks (B = 8), one warp per block:
+// lane l holds the texels (l % B, l / B + k 32/B), k < B^2/32.  The block centre
+// c (normalised sum of its texel centres) and radius rho (max angle from c to
+// a texel centre, rounded up) bound the search: with theta_C = the angle from
+// c to its nearest clear direction, every texel's nearest clear direction lies
+// within theta_C + 2 rho of c (triangle inequality), so only those candidates
+// (found by one ballot pass over the list) are tried per texel.
+template <int B>
+__device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float* __restrict__ V,
+                                 const float4* sDirs, int total, int w0, int wstride) {
+    constexpr int TPL = B * B / 32, ROWS = 32 / B;
+    const int lane = threadIdx.x & 31;
+    const int Tc = T / B, nct = 6 * Tc * Tc;
+    for (int ct = w0; ct < nct; ct += wstride) {
+        const int face = ct / (Tc * Tc), rem = ct - face * Tc * Tc, cw = rem / Tc, cu = rem - cw * Tc;
+        const int t0 = (face * T + B * cw + lane / B) * T + B * cu + lane % B;
+        float4 f[TPL];
+        float sx = 0.f, sy = 0.f, sz = 0.f;
+#pragma unroll
+        for (int k = 0; k < TPL; ++k) {
+            f[k] = texels[t0 + k * ROWS * T];
+            sx += f[k].x;
+            sy += f[k].y;
+            sz += f[k].z;
+        }
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            sx += __shfl_xor_sync(0xffffffffu, sx, o);
+            sy += __shfl_xor_sync(0xffffffffu, sy, o);
+            sz += __shfl_xor_sync(0xffffffffu, sz, o);
+        }
+        const float inv = rsqrtf(fmaf(sx, sx, fmaf(sy, sy, sz * sz)));
+        const float4 c = make_float4(sx * inv, sy * inv, sz * inv, 0.f);
+        // rho from the smallest cosine (acos decreasing), rounded up
+        float cmin = 2.f;
+#pragma unroll
+        for (int k = 0; k < TPL; ++k) cmin = fminf(cmin, dot3(f[k], c));
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) cmin = fminf(cmin, __shfl_xor_sync(0xffffffffu, cmin, o));
+        const float rho = acosf(fmaxf(cmin - 1e-6f, -1.f));
+        float bc = -2.f;
+        for (int e = lane; e < total; e += 32) bc = fmaxf(bc, dot3(c, sDirs[e]));
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) bc = fmaxf(bc, __shfl_xor_sync(0xffffffffu, bc, o));
+        const float th = acosf(fmaxf(bc - 1e-6f, -1.f)) + 2.f * rho + 1e-4f;
+        const float thr = th >= 3.14159f ? -2.f : cosf(th) - 1e-6f;
+        float bf[TPL];
+#pragma unroll
+        for (int k = 0; k < TPL; ++k) bf[k] = -2.f;
+        for (int base = 0; base < total; base += 32) {
+            const int e = base + lane;
+            unsigned int mask = __ballot_sync(0xffffffffu, e < total && dot3(c, sDirs[e]) >= thr);
+            while (mask) {
+                const float4 d = sDirs[base + __ffs(mask) - 1];
+                mask &= mask - 1u;
+#pragma unroll
+                for (int k = 0; k < TPL; ++k) bf[k] = fmaxf(bf[k], dot3(f[k], d));
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < TPL; ++k) V[t0 + k * ROWS * T] = clear_map_value(bf[k], f[k].w);
+    }
+}
+
 // The clear-direction map of `gam` into V (6 T^2 texels), computed by the CTAs
 // gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
 // (kMapDirs), sN.
@@ -311,7 +476,31 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
     __syncthreads();
     const int total = *sN;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    if (total > kMapBrute && total <= kMapDirs && (T & 3) == 0) {
+    if (total > g.rowscan) {
+        // clear masks in place (sAM is re-seeded by every caller before reuse),
+        // one bit per row with a clear cell in the sDirs space
+        uint32_t* sRows = reinterpret_cast<uint32_t*>(sDirs);
+        for (int w = threadIdx.x; w < ((g.m + 31) >> 5); w += blockDim.x) sRows[w] = 0u;
+        __syncthreads();
+        for (int w = threadIdx.x; w < MW; w += blockDim.x) {
+            const int i = w / g.W;
+            const uint32_t cl = ~sAM[w] & row_word_mask(w - i * g.W, g.n);
+            sAM[w] = cl;
+            if (cl) atomicOr(sRows + (i >> 5), 1u << (i & 31));
+        }
+        __syncthreads();
+        for (int t = gb * blockDim.x + threadIdx.x; t < ntex; t += gn * blockDim.x) {
+            const float4 c = texels[t];
+            V[t] = clear_map_value(nearest_clear_rows(c, sAM, sRows, g, tab), c.w);
+        }
+        return;
+    }
+    if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
+        compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
+        clear_map_blocks<8>(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps);
+        return;
+    }
+    if (total > g.brute && total <= kMapDirs && (T & 3) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
         const int Tc = T >> 2, nct = 6 * Tc * Tc;
         const int half = lane >> 4, sub = lane & 15;

@@ -261,6 +261,20 @@ def test_phases_and_tunables_give_identical_maps(am, name):
         assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
     with pytest.raises(am.AMError):
         ctx.set_option(am.binding.OPT_CMAP_T1, 129)  # larger than cmap_T
+    # the clear map by the row-ordered nearest-clear search always (0), never, or by default
+    for rs in (0, 128, 1 << 21):
+        ctx.set_option(am.binding.OPT_CMAP_ROWSCAN, rs)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+    with pytest.raises(am.AMError):
+        ctx.set_option(am.binding.OPT_CMAP_ROWSCAN, -1)
+    # every clear-map search path: all pairs, or candidates bounded per 4x4 / 8x8 texel block
+    for brute, block in ((1 << 21, 8), (0, 4), (0, 8), (64, 4), (64, 8)):
+        ctx.set_option(am.binding.OPT_CMAP_BRUTE, brute)
+        ctx.set_option(am.binding.OPT_CMAP_BLOCK, block)
+        assert np.array_equal(ctx.compute_batch(P), ref), (brute, block)
+    with pytest.raises(am.AMError):
+        ctx.set_option(am.binding.OPT_CMAP_BLOCK, 16)
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
