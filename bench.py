@@ -265,6 +265,8 @@ def run_ours(args):
         ctx.set_option(B.OPT_CMAP_BLOCK, args.cmap_block)
     if args.map_ctas >= 0:
         ctx.set_option(B.OPT_MAP_CTAS, args.map_ctas)
+    if args.subbricks >= 0:
+        ctx.set_option(B.OPT_SUBBRICKS, args.subbricks)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
     if args.band_subdiv:
@@ -524,6 +526,7 @@ def main():
     ap.add_argument("--cmap-brute", type=int, default=-1, help="AM_OPT_CMAP_BRUTE (-1 = library default)")
     ap.add_argument("--cmap-block", type=int, default=0, help="AM_OPT_CMAP_BLOCK (0 = library default)")
     ap.add_argument("--map-ctas", type=int, default=-1, help="AM_OPT_MAP_CTAS (-1 = library default)")
+    ap.add_argument("--subbricks", type=int, default=-1, help="AM_OPT_SUBBRICKS (-1 = library default)")
     ap.add_argument("--phases", type=int, default=None, help="AM_OPT_PHASES (coarse levels, 1 or 2)")
     ap.add_argument("--band-subdiv", type=int, default=0,
                     help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")

@@ -120,9 +120,13 @@ enum {
                                     whose centre bounds the candidate cells on that path: 4 or 8
                                     (default 8; a map resolution that is not a multiple falls
                                     back to 4, then to every texel x every cell).  Same map      */
-    AM_OPT_MAP_CTAS = 18         /* batched path: CTAs per pivot of the (final) clear-direction
+    AM_OPT_MAP_CTAS = 18,        /* batched path: CTAs per pivot of the (final) clear-direction
                                     map launch, 0..4096 (0 = one per 1024 texels; default 48).
                                     Same map                                                    */
+    AM_OPT_SUBBRICKS = 19        /* fused and batched paths: 1 = inside a kept brick, skip each
+                                    32-voxel sub-brick (one warp's voxels) whose bounding sphere
+                                    reaches no clear cell before its voxels are read (default);
+                                    0 = read them.  Same map                                    */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

@@ -29,6 +29,9 @@ using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
 // level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_BRICK_STEPS
+#define AM_BRICK_STEPS 4  // brick-test steps (256 bricks each) per CTA of the batched path
+#endif
 #ifndef AM_MAP_CTAS
 #define AM_MAP_CTAS 48
 #endif
@@ -106,9 +109,11 @@ struct am_ctx {
     float4* d_texels1 = nullptr;
     int phases = 2;
     float4* d_bricks = nullptr;            // bounding spheres of 256-voxel bricks of d_vox
-    unsigned int* d_brick_list = nullptr;  // bricks kept per map (capacity nbricks)
+    unsigned int* d_brick_list = nullptr;  // kept bricks (stream path) / sub-bricks (fused path) per map (capacity 8 nbricks)
     unsigned int nbricks = 0;
     int bricks_on = 1;
+    float4* d_subs = nullptr;              // bounding spheres of 32-voxel sub-bricks (warps of a brick)
+    int subs_on = 1;                       // AM_OPT_SUBBRICKS
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
@@ -321,7 +326,7 @@ int ensure_slots(am_ctx* ctx, int K) {
     CK(cudaMalloc(&ctx->d_tasks, (size_t)K * kTaskCap * sizeof(unsigned long long)));
     CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float)));
     if (ctx->vox_cap > 0) CK(cudaMalloc(&ctx->d_live, (size_t)K * ctx->vox_cap * sizeof(unsigned int)));
-    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * ctx->nbricks * sizeof(unsigned int)));
+    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * 8 * ctx->nbricks * sizeof(unsigned int)));
     return AM_OK;
 }
 
@@ -493,6 +498,7 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.main.cmap = ctx->d_cmap;
     F.main.bricks = ctx->d_bricks;
     F.main.nbricks = ctx->nbricks;
+    F.main.subs = ctx->subs_on ? ctx->d_subs : nullptr;
     F.main.brick_list = ctx->d_brick_list;
     F.main.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
     F.main.recs = ctx->d_recs;
@@ -630,7 +636,7 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
     F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
     F.cmap_stride = (unsigned long long)ntex * sizeof(float);
-    F.blist_stride = (unsigned long long)ctx->nbricks * sizeof(unsigned int);
+    F.blist_stride = 8ull * ctx->nbricks * sizeof(unsigned int);
     F.piv = ctx->d_piv;
     F.npiv = (unsigned int)P;
     F.gam0 = gam0;
@@ -684,7 +690,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
         F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
         F.cmap_stride = (unsigned long long)ntex * sizeof(float);
-        F.blist_stride = (unsigned long long)ctx->nbricks * sizeof(unsigned int);
+        F.blist_stride = 8ull * ctx->nbricks * sizeof(unsigned int);
         F.piv = ctx->d_piv + c0;
         F.npiv = (unsigned int)kk;
         F.gam0 = g;
@@ -728,7 +734,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
         }
-        if ((rc = L(bk_bricks, grid(ctx->nbricks, 4 * kThreads, 1 << 16), 0))) return rc;
+        if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
         AM_KM(AM_K_BRICKS);
         if ((rc = L(bk_voxels, grid(1 << 30, 1, ctx->bk_voxel_ctas), 0))) return rc;
         AM_KM(AM_K_VOXELS);
@@ -1061,10 +1067,21 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     ctx->d_brick_list = nullptr;
     ctx->nbricks = (unsigned int)((N + kThreads - 1) / kThreads);
     UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
-    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * ctx->nbricks * sizeof(unsigned int)));
+    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * 8 * ctx->nbricks * sizeof(unsigned int)));
     brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
                                                                                         ctx->nbricks, kThreads);
     UK(cudaGetLastError());
+    cudaFree(ctx->d_subs);
+    ctx->d_subs = nullptr;
+    {
+        const unsigned int nsub = (unsigned int)((N + 31) / 32);
+        if (nsub > 0) {
+            UK(cudaMalloc(&ctx->d_subs, (size_t)nsub * sizeof(float4)));
+            brick_bounds_kernel<<<(unsigned)(((long long)nsub * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_subs,
+                                                                                         nsub, 32);
+            UK(cudaGetLastError());
+        }
+    }
     // coarse levels for the clear-direction map: level 0 = the n0 largest
     // voxels, level 1 = the next ones up to n1 plus every 512th voxel
     cudaFree(ctx->d_coarse);
@@ -1147,7 +1164,10 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
         // every voxel goes through the filter once; the rest of it was dropped
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
-        stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks) ? (int64_t)h[kCtrBricks] : (int64_t)ctx->nbricks;
+        // (fused path: kept bricks in the high word, kept sub-bricks -- the list length -- in the low word)
+        stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks)
+                                 ? (int64_t)(fused_ok(ctx) ? (h[kCtrBricks] >> 32) : (h[kCtrBricks] & 0xffffffffull))
+                                 : (int64_t)ctx->nbricks;
         stats->level_voxels = ctx->phases == 0 ? 0 : ctx->phases == 1 ? ctx->n_l0 : ctx->n_l1;
         if ((rc = print_phase_times(ctx)) != AM_OK) return rc;
     } else if (!dst_is_device) {
@@ -1308,6 +1328,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_MAP_CTAS:
         if (value < 0 || value > 4096) return fail(ctx, AM_EINVAL, "map_ctas must be in [0, 4096]");
         ctx->bk_map_ctas = (int)value;
+        return AM_OK;
+    case AM_OPT_SUBBRICKS:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "subbricks must be 0 or 1");
+        ctx->subs_on = (int)value;
         return AM_OK;
     case AM_OPT_CMAP_T1:
         if (value < 4 || value > ctx->cmapT) return fail(ctx, AM_EINVAL, "cmap_T1 must be in [4, cmap_T]");
@@ -1634,6 +1658,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_live);
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);
+    cudaFree(ctx->d_subs);
     cudaFree(ctx->d_bricks);
     cudaFree(ctx->d_brick_list);
     cudaFree(ctx->d_texels);

@@ -180,27 +180,17 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
                   gridDim.x);
 }
 
-// Brick test: bricks whose bounding sphere may still reach a clear cell.
+// Brick test: bricks, then their 32-voxel sub-bricks, whose bounding sphere may
+// still reach a clear cell (fused.cuh brick_step).
 __global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
-    __shared__ FusedScratch sc;
     const int p = blockIdx.y;
     pivot_params(sP, F, p, false);
     const StreamParams& P = sP;
-    const unsigned int nb = P.nbricks;
-    for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
-        const unsigned int b = b0 + threadIdx.x;
-        bool keep = false;
-        if (b < nb) {
-            const float4 s = __ldg(P.bricks + b);
-            keep = !sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
-        }
-        const unsigned int pos = cta_reserve<unsigned int>(keep ? 1u : 0u, P.brick_count, sc.r32);
-        if (keep) P.brick_list[pos] = b;
-    }
+    for (unsigned int b0 = blockIdx.x * kThreads; b0 < P.nbricks; b0 += gridDim.x * kThreads) brick_step(P, b0);
 }
 
-// Kept bricks' voxels through the filter; live voxels to the live list.
+// Kept sub-bricks' voxels through the filter; live voxels to the live list.
 __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     __shared__ FusedScratch sc;
@@ -210,35 +200,10 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
     pivot_params(sP, F, p, false);
     const StreamParams& P = sP;
     const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
-    if (blockIdx.x * kVPT >= nk) return;  // CTA-uniform
+    if (blockIdx.x * (kVPT * kWarps) >= nk) return;  // CTA-uniform
     unsigned int nculled = 0, npassed = 0, streamed = 0;
-    for (unsigned int k0 = blockIdx.x * kVPT; k0 < nk; k0 += gridDim.x * kVPT) {
-        float4 q[kVPT];
-        unsigned int idx[kVPT];
-        bool ok[kVPT];
-#pragma unroll
-        for (int k = 0; k < kVPT; ++k) {
-            ok[k] = k0 + k < nk;
-            idx[k] = ok[k] ? P.brick_list[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
-            ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
-            q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
-        }
-        bool live[kVPT];
-        unsigned int nl = 0;
-#pragma unroll
-        for (int k = 0; k < kVPT; ++k) {
-            const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
-            nculled += f >> 1;
-            streamed += ok[k];
-            live[k] = f == F_LIVE;
-            nl += live[k];
-        }
-        npassed += nl;
-        unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
-#pragma unroll
-        for (int k = 0; k < kVPT; ++k)
-            if (live[k]) P.live_idx[pos++] = idx[k];
-    }
+    for (unsigned int k0 = blockIdx.x * (kVPT * kWarps); k0 < nk; k0 += gridDim.x * (kVPT * kWarps))
+        voxel_step(P, k0, nk, sc, nculled, npassed, streamed);
     npassed = __reduce_add_sync(0xffffffffu, npassed);
     nculled = __reduce_add_sync(0xffffffffu, nculled);
     streamed = __reduce_add_sync(0xffffffffu, streamed);

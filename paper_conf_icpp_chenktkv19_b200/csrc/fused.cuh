@@ -226,6 +226,85 @@ struct FusedScratch {
     unsigned long long r64[kWarps + 1];
 };
 
+// Brick phase (the paper's octree pruning, Alg. 2
+// L218-219, as bounding spheres over the Morton order), one brick of 256
+// voxels per thread of the CTA step starting at brick b0: a brick whose sphere
+// may still reach a clear cell is kept (counted in the high word of the brick
+// counter, for am_stats) and its 8 sub-bricks of 32 voxels are tested the same
+// way, warp-cooperatively (4 kept bricks x 8 sub-bricks per pass); the kept
+// sub-bricks are appended to brick_list (count in the low word).  Without
+// sub-brick spheres (AM_OPT_SUBBRICKS = 0) every sub-brick of a kept brick is
+// kept.  Exact-safe: a voxel's cube lies inside each enclosing sphere.
+__device__ __forceinline__ bool node_dropped(const StreamParams& P, const float4* __restrict__ spheres, unsigned int k) {
+    if (!spheres) return false;
+    const float4 s = __ldg(spheres + k);
+    return sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
+}
+
+__device__ __forceinline__ void brick_step(const StreamParams& P, unsigned int b0) {
+    __shared__ unsigned int sKept[kWarps][32];  // per warp: its kept bricks
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const unsigned int lt = (1u << lane) - 1u;
+    const unsigned int b = b0 + threadIdx.x;
+    const unsigned long long nsub = ((unsigned long long)P.N + 31) >> 5;
+    const bool kb = b < P.nbricks && !node_dropped(P, P.bricks, b);
+    const unsigned int mb = __ballot_sync(0xffffffffu, kb);
+    if (!mb) return;
+    if (lane == 0) atomicAdd(P.brick_count + 1, (unsigned int)__popc(mb));
+    if (kb) sKept[warp][__popc(mb & lt)] = b;
+    __syncwarp();
+    const int n = __popc(mb);
+    for (int u = 0; u < n; u += 4) {  // 4 kept bricks x 8 sub-bricks per pass
+        const int j = u + (lane >> 3);
+        const unsigned int sb = j < n ? sKept[warp][j] * 8u + (lane & 7) : 0u;
+        const bool sk = j < n && sb < nsub && !node_dropped(P, P.subs, sb);
+        const unsigned int mk = __ballot_sync(0xffffffffu, sk);
+        if (mk) {
+            unsigned int base = 0;
+            if (lane == 0) base = atomicAdd(P.brick_count, (unsigned int)__popc(mk));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (sk) P.brick_list[base + __popc(mk & lt)] = sb;
+        }
+    }
+    __syncwarp();
+}
+
+// Voxel phase, one CTA step over the kept sub-bricks [k0, k0 + kVPT kWarps):
+// warp w reads sub-bricks k0 + k kWarps + w (k < kVPT), one voxel per lane (a
+// coalesced 512-byte read each), through fast_filter; live voxels are appended
+// to the live list with one reservation per CTA step (CTA-uniform call).
+__device__ __forceinline__ void voxel_step(const StreamParams& P, unsigned int k0, unsigned int nk,
+                                           FusedScratch& sc, unsigned int& nculled, unsigned int& npassed,
+                                           unsigned int& streamed) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    float4 q[kVPT];
+    unsigned int idx[kVPT];
+    bool ok[kVPT];
+#pragma unroll
+    for (int k = 0; k < kVPT; ++k) {
+        const unsigned int e = k0 + k * kWarps + warp;
+        ok[k] = e < nk;
+        idx[k] = ok[k] ? P.brick_list[e] * 32u + lane : 0u;
+        ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
+        q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
+    }
+    bool live[kVPT];
+    unsigned int nl = 0;
+#pragma unroll
+    for (int k = 0; k < kVPT; ++k) {
+        const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
+        nculled += f >> 1;
+        streamed += ok[k];
+        live[k] = f == F_LIVE;
+        nl += live[k];
+    }
+    npassed += nl;
+    unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
+#pragma unroll
+    for (int k = 0; k < kVPT; ++k)
+        if (live[k]) P.live_idx[pos++] = idx[k];
+}
+
 // Rows i0 .. i0 + nrows - 1 that are not yet full, word w of the row-full bits.
 __device__ __forceinline__ uint32_t open_rows_word(const uint32_t* rowfull, int i0, int i1, int w) {
     uint32_t b = ~rowfull[w];
@@ -427,55 +506,17 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
         gsync();
         if (!BATCH || gb == 0) fused_mark(F, 6);
     }
-    // 7. brick test
-    {
-        const unsigned int nb = P.nbricks;
-        for (unsigned int b0 = gb * kThreads; b0 < nb; b0 += gn * kThreads) {
-            const unsigned int b = b0 + threadIdx.x;
-            bool keep = false;
-            if (b < nb) {
-                const float4 s = __ldg(P.bricks + b);
-                keep = !sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
-            }
-            const unsigned int pos = cta_reserve<unsigned int>(keep ? 1u : 0u, P.brick_count, sc.r32);
-            if (keep) P.brick_list[pos] = b;
-        }
-    }
+    // 7. brick test (kept bricks -> kept 32-voxel sub-bricks)
+    for (unsigned int b0 = gb * kThreads; b0 < P.nbricks; b0 += gn * kThreads) brick_step(P, b0);
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 7);
-    // 8a. kept bricks: filter (kVPT bricks per CTA step); live voxels go to the
-    //     global live list with one atomic per CTA step
+    // 8a. kept sub-bricks: filter (kVPT x kWarps sub-bricks per CTA step); live voxels go
+    //     to the global live list with one atomic per CTA step
     {
-        unsigned int nculled = 0, npassed = 0;
-        unsigned long long streamed = 0;
+        unsigned int nculled = 0, npassed = 0, streamed = 0;
         const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
-        for (unsigned int k0 = gb * kVPT; k0 < nk; k0 += gn * kVPT) {
-            float4 q[kVPT];
-            unsigned int idx[kVPT];
-            bool ok[kVPT];
-#pragma unroll
-            for (int k = 0; k < kVPT; ++k) {
-                ok[k] = k0 + k < nk;
-                idx[k] = ok[k] ? P.brick_list[k0 + k] * (unsigned int)kThreads + threadIdx.x : 0u;
-                ok[k] = ok[k] && idx[k] < (unsigned long long)P.N;
-                q[k] = ok[k] ? __ldcs(P.vox + idx[k]) : make_float4(0.f, 0.f, 0.f, 1.f);
-            }
-            bool live[kVPT];
-            unsigned int nl = 0;
-#pragma unroll
-            for (int k = 0; k < kVPT; ++k) {
-                const int f = ok[k] ? fast_filter(P, q[k], P.gam) : F_DROP;
-                nculled += f >> 1;
-                streamed += ok[k];
-                live[k] = f == F_LIVE;
-                nl += live[k];
-            }
-            npassed += nl;
-            unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
-#pragma unroll
-            for (int k = 0; k < kVPT; ++k)
-                if (live[k]) P.live_idx[pos++] = idx[k];
-        }
+        for (unsigned int k0 = gb * (kVPT * kWarps); k0 < nk; k0 += gn * (kVPT * kWarps))
+            voxel_step(P, k0, nk, sc, nculled, npassed, streamed);
         // warp sums, one shared atomic per warp (a 64-bit shared atomic would be a CAS loop)
         npassed = __reduce_add_sync(0xffffffffu, npassed);
         nculled = __reduce_add_sync(0xffffffffu, nculled);

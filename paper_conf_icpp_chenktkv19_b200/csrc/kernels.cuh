@@ -72,6 +72,9 @@ struct StreamParams {
     unsigned int* brick_list;      // bricks kept by brick_test_kernel (capacity nbricks)
     unsigned int* brick_count;     // zeroed per map
     int band_vdepth;               // band pairs: virtual sub-cube levels before CHECKBOX (§4.3)
+    // sub-bricks of 32 consecutive voxels (one warp of a brick): bounding spheres;
+    // nullptr = not tested
+    const float4* __restrict__ subs;
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,

@@ -275,6 +275,10 @@ def test_phases_and_tunables_give_identical_maps(am, name):
         assert np.array_equal(ctx.compute_batch(P), ref), (brute, block)
     with pytest.raises(am.AMError):
         ctx.set_option(am.binding.OPT_CMAP_BLOCK, 16)
+    ctx.set_option(am.binding.OPT_SUBBRICKS, 0)  # read every voxel of a kept brick
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+    ctx.set_option(am.binding.OPT_SUBBRICKS, 1)
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
