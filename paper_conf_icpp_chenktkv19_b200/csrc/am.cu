@@ -863,6 +863,15 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         T.Rin[k] = T.Rin[n_cyl - 1];
         T.Rpm[k] = T.Rpm[n_cyl - 1];
     }
+    for (int k = 0; k < AM_MAX_CYL; ++k)
+        for (int set = 0; set < 2; ++set)
+            for (int e = 0; e < 2; ++e) {
+                const double zc = k < n_cyl ? (double)(e ? T.z1[k] : T.z0[k]) : 1.0;
+                const double Rc = k < n_cyl ? (double)(set ? T.Rin[k] : T.R[k]) : 1.0;
+                const double dc = std::sqrt(zc * zc + Rc * Rc);
+                T.cD[set][e][k] = (float)dc;
+                T.ciD[set][e][k] = (float)(1.0 / dc);
+            }
     T.R_first = T.Rpm[0];
     T.nbp = 0;
     for (int k = 0; k < AM_MAX_CYL; ++k) {

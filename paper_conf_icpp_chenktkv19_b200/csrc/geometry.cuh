@@ -39,6 +39,10 @@ struct ToolDev {
     float R_first;
     float bp_z[AM_MAX_CYL];
     float bp_R[AM_MAX_CYL];
+    // rounded corners of the expanded rectangles (L175): distance from the pivot of
+    // (z0_k | z1_k, R_k | Rin_k) and its reciprocal, [radius set][end][k] (host, fp64)
+    float cD[2][2][AM_MAX_CYL];
+    float ciD[2][2][AM_MAX_CYL];
 };
 
 // An upper bound on the radius of every cylinder that starts within `reach`
@@ -80,7 +84,8 @@ constexpr float kClearSlack = 1e-4f;   // cosine slack of the live voxels' clear
 //   cmin = cos(largest blocked angle)   (2 if nothing is blocked)
 //   cmax = cos(smallest blocked angle)  (-2 if nothing is blocked).
 __device__ __forceinline__ void ica_cylinder(float D, float D2, float invD, float r, float z0,
-                                             float z1, float R, float& cmin, float& cmax) {
+                                             float z1, float R, const ToolDev& T, int set, int k,
+                                             float& cmin, float& cmax) {
     cmin = 2.f;
     cmax = -2.f;
     if (D + z0 <= r) cmin = -1.f;               // theta = pi lies inside
@@ -119,19 +124,19 @@ __device__ __forceinline__ void ica_cylinder(float D, float D2, float invD, floa
 #pragma unroll
     for (int e = 0; e < 2; ++e) {  // rounded corners centred (zc, R), radius r
         const float zc = e ? z1 : z0;
-        const float Dc = sqrtf(zc * zc + R2);
+        const float Dc = T.cD[set][e][k], iDc = T.ciD[set][e][k];  // |(zc, R)|, 1 / |(zc, R)|
         const float dd = D - Dc;
         if (fabsf(dd) <= r) {
             // arc of radius D meets the corner circle at theta_c +- beta with
             // cos(beta) = (D^2 + Dc^2 - r^2) / (2 D Dc); 1 -+ cos(beta) factored
             // so sin(beta) keeps its relative accuracy near tangency
-            const float inv2 = 0.5f / (D * Dc);
+            const float inv2 = 0.5f * invD * iDc;
             const float omc = (r - dd) * (r + dd) * inv2;               // 1 - cos(beta)
             const float sp = D + Dc;
             const float opc = (sp - r) * (sp + r) * inv2;               // 1 + cos(beta)
             const float cb = 0.5f * (opc - omc);
             const float sb = sqrtf(fmaxf(omc * opc, 0.f));
-            const float ct = zc / Dc, st = R / Dc;
+            const float ct = zc * iDc, st = R * iDc;
             const float s_hi = st * cb + ct * sb;                       // sin(theta_c + beta)
             const float c_hi = (s_hi < 0.f) ? -1.f : (ct * cb - st * sb);
             const float s_lo = st * cb - ct * sb;                       // sin(theta_c - beta)
@@ -164,7 +169,7 @@ __device__ __forceinline__ Cones tool_cones(float D, float h, const ToolDev& T) 
         float cm = 2.f;
         for (int k = 0; k < T.ncyl; ++k) {
             float a, b;
-            ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], a, b);
+            ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], T, 1, k, a, b);
             cm = fminf(cm, a);
         }
         c.cin = (cm <= 1.f) ? cm + kCosGuard : 2.f;
@@ -172,7 +177,7 @@ __device__ __forceinline__ Cones tool_cones(float D, float h, const ToolDev& T) 
     float co = 2.f, cx = -2.f;
     for (int k = 0; k < T.ncyl; ++k) {
         float a, b;
-        ica_cylinder(D, D2, invD, r2, T.z0[k], T.z1[k], T.R[k], a, b);
+        ica_cylinder(D, D2, invD, r2, T.z0[k], T.z1[k], T.R[k], T, 0, k, a, b);
         co = fminf(co, a);
         cx = fmaxf(cx, b);
     }
@@ -193,7 +198,7 @@ __device__ __forceinline__ float inner_cone(float D, float h, const ToolDev& T) 
     float cm = 2.f;
     for (int k = 0; k < T.ncyl; ++k) {
         float a, b;
-        ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], a, b);
+        ica_cylinder(D, D2, invD, r1, T.z0[k], T.z1[k], T.Rin[k], T, 1, k, a, b);
         cm = fminf(cm, a);
     }
     return (cm <= 1.f) ? cm + kCosGuard : 2.f;
