@@ -4,8 +4,9 @@
 
 A step is one am_compute_batch call: the whole hot path (a1-a8 of SURVEY.md
 8(a)) for --batch (default 64) consecutive pivots of the seeded 1 mm path over
-the resident voxel model, computed phase by phase with --slots (default 64)
-pivots per launch (8(f) NEXT 2, csrc/batch.cuh).  Default workload: C3
+the resident voxel model, computed phase by phase (8(f) NEXT 2, csrc/batch.cuh)
+in chunks of --slots / --lanes (default 64 / 8) pivots per launch that go
+round-robin to --lanes internal streams, so the chunks' short phases overlap.  Default workload: C3
 (head-like, ~27M leaf voxels, 3-cylinder tool, 64 x 64 = 4096 orientations),
 the configuration BASELINE.json's metric is quoted on.  The one-pivot latency
 (am_compute) is reported beside it.  For N > 1 (torchrun), every rank computes
@@ -171,7 +172,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch, args.slots),
+        "data": "synthetic", "config": _config_dict(cfg, len(H), not args.no_flush, args.batch, args.slots, args.lanes),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                          "sample": f"{cells} cells of {args.steps} maps (seeded cells, pivots of the 1 mm path), "
                                    f"every voxel per cell, fp64 clip-project-hull test with exact-safe shortcuts"},
@@ -181,14 +182,14 @@ def run_reference(args):
     return 0
 
 
-def _config_dict(cfg, N, flushed=True, batch=1, slots=1):
+def _config_dict(cfg, N, flushed=True, batch=1, slots=1, lanes=1):
     return {"workload": f"{cfg.name}: {cfg.note}, {len(cfg.tool)}-cylinder tool, {cfg.m}x{cfg.n} AM, "
                         f"pivots on the {cfg.offset:g} mm path",
             "voxels": int(N), "m": cfg.m, "n": cfg.n, "cylinders": [list(t) for t in cfg.tool],
             "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
                    f"every timed step, outside the per-step CUDA events") if flushed else
                   f"inputs {16 * N / 1e6:.0f} MB; no flush",
-            "pivots_per_step": batch, "pivots_per_launch": slots,
+            "pivots_per_step": batch, "pivots_per_launch": max(1, slots // lanes), "streams": lanes,
             "parallelism": "pivot-sharded (weak)"}
 
 
@@ -267,6 +268,7 @@ def run_ours(args):
         ctx.set_option(B.OPT_MAP_CTAS, args.map_ctas)
     if args.subbricks >= 0:
         ctx.set_option(B.OPT_SUBBRICKS, args.subbricks)
+    ctx.set_option(B.OPT_BATCH_LANES, args.lanes)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
     if args.band_subdiv:
@@ -399,7 +401,7 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N, flush is not None, bsz, args.slots),
+            "config": _config_dict(cfg, N, flush is not None, bsz, args.slots, args.lanes),
             "ms_per_am": ms_max / args.steps / bsz,
             "roofline": dom_roof,
             "step_roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -527,6 +529,8 @@ def main():
     ap.add_argument("--cmap-block", type=int, default=0, help="AM_OPT_CMAP_BLOCK (0 = library default)")
     ap.add_argument("--map-ctas", type=int, default=-1, help="AM_OPT_MAP_CTAS (-1 = library default)")
     ap.add_argument("--subbricks", type=int, default=-1, help="AM_OPT_SUBBRICKS (-1 = library default)")
+    ap.add_argument("--lanes", type=int, default=8,
+                    help="AM_OPT_BATCH_LANES: streams the step's chunks of slots / lanes pivots go to")
     ap.add_argument("--phases", type=int, default=None, help="AM_OPT_PHASES (coarse levels, 1 or 2)")
     ap.add_argument("--band-subdiv", type=int, default=0,
                     help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")

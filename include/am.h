@@ -123,10 +123,15 @@ enum {
     AM_OPT_MAP_CTAS = 18,        /* batched path: CTAs per pivot of the (final) clear-direction
                                     map launch, 0..4096 (0 = one per 1024 texels; default 48).
                                     Same map                                                    */
-    AM_OPT_SUBBRICKS = 19        /* fused and batched paths: 1 = inside a kept brick, skip each
+    AM_OPT_SUBBRICKS = 19,       /* fused and batched paths: 1 = inside a kept brick, skip each
                                     32-voxel sub-brick (one warp's voxels) whose bounding sphere
                                     reaches no clear cell before its voxels are read (default);
                                     0 = read them.  Same map                                    */
+    AM_OPT_BATCH_LANES = 20      /* am_compute_batch: chunks of AM_OPT_BATCH / lanes pivots go
+                                    round-robin to this many internal streams (forked from and
+                                    joined to the caller's stream), so one chunk's short phases
+                                    overlap another's (1..8, default 8; 1 while
+                                    AM_OPT_KERNEL_TIMING = 2).  Same maps                       */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

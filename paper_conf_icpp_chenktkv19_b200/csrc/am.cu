@@ -29,6 +29,10 @@ using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
 // level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_BATCH_LANES
+#define AM_BATCH_LANES 8
+#endif
+constexpr int kMaxLanes = 8;
 #ifndef AM_BRICK_STEPS
 #define AM_BRICK_STEPS 4  // brick-test steps (256 bricks each) per CTA of the batched path
 #endif
@@ -118,6 +122,9 @@ struct am_ctx {
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
     int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
+    int lanes = AM_BATCH_LANES;            // streams of the batched path (AM_OPT_BATCH_LANES)
+    cudaStream_t lane_s[kMaxLanes] = {};
+    cudaEvent_t lane_ev[kMaxLanes + 1] = {};
     int bk_map_ctas = AM_MAP_CTAS;         // per pivot, batched clear map (AM_OPT_MAP_CTAS; 0 = texels / 1024)
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
@@ -658,6 +665,45 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
 // P maps (pivots[3P]) into gam0 + k * MW, phase by phase over chunks of up to
 // ctx->batch pivots (batch.cuh): each phase is one launch with blockIdx.y =
 // pivot of the chunk.
+// Host mirror of fused.cuh slot_params for a whole launch: advance the slot-0
+// per-map pointers of F by `base` slots, so that launch pivot y uses slot base + y.
+template <typename T>
+T* hshift(T* p, unsigned long long b) {
+    return p ? reinterpret_cast<T*>(reinterpret_cast<uintptr_t>(p) + b) : p;
+}
+
+void shift_slots(FusedParams& F, int base) {
+    if (base == 0) return;
+    const unsigned long long b = (unsigned long long)base;
+    for (int which = 0; which < 2; ++which) {
+        StreamParams& p = which ? F.lvl : F.main;
+        p.qcount = hshift(p.qcount, b * F.ctr_stride);
+        p.stats = hshift(p.stats, b * F.ctr_stride);
+        p.live_count = hshift(p.live_count, b * F.ctr_stride);
+        p.rec_count = hshift(p.rec_count, b * F.ctr_stride);
+        p.task_count = hshift(p.task_count, b * F.ctr_stride);
+        p.brick_count = hshift(p.brick_count, b * F.ctr_stride);
+        p.queue = hshift(p.queue, b * F.q_stride);
+        p.live_idx = hshift(p.live_idx, b * F.live_stride);
+        p.recs = hshift(p.recs, b * F.rec_stride);
+        p.tasks = hshift(p.tasks, b * F.task_stride);
+        p.brick_list = hshift(p.brick_list, b * F.blist_stride);
+        if (!which) p.cmap = hshift(p.cmap, b * F.cmap_stride);
+    }
+    F.rec1 = hshift(F.rec1, b * F.ctr_stride);
+    F.task1 = hshift(F.task1, b * F.ctr_stride);
+    F.ctr0 = hshift(F.ctr0, b * F.ctr_stride);
+}
+
+// Streams (and fork/join events) of the batched path's lanes.
+int ensure_lanes(am_ctx* ctx, int lanes) {
+    for (int l = 0; l < lanes; ++l)
+        if (!ctx->lane_s[l]) CK(cudaStreamCreateWithFlags(&ctx->lane_s[l], cudaStreamNonBlocking));
+    for (int l = 0; l <= kMaxLanes; ++l)
+        if (!ctx->lane_ev[l]) CK(cudaEventCreateWithFlags(&ctx->lane_ev[l], cudaEventDisableTiming));
+    return AM_OK;
+}
+
 int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* gam0, cudaStream_t s) {
     const int K = (int)std::min<int64_t>(P, ctx->batch);
     int rc;
@@ -677,11 +723,12 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv.data(), (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
     const size_t sm_rows = (size_t)(ctx->MW + ((ctx->grid.m + 31) >> 5) + 1) * sizeof(uint32_t);
-    for (int64_t c0 = 0; c0 < P; c0 += K) {
-        const int kk = (int)std::min<int64_t>(K, P - c0);
+    // one chunk of kk pivots from c0 on, slots [sb, sb + kk), on stream s
+    auto run_chunk = [&](int64_t c0, int kk, int sb, cudaStream_t s) -> int {
+        int rc;
         uint32_t* g = gam0 + c0 * ctx->MW;
         CK(cudaMemsetAsync(g, 0, (size_t)kk * ctx->MW * sizeof(uint32_t), s));
-        CK(cudaMemsetAsync(ctx->d_ctr, 0, (size_t)kk * kCtrStride * sizeof(unsigned long long), s));
+        CK(cudaMemsetAsync(ctx->d_ctr + (size_t)sb * kCtrStride, 0, (size_t)kk * kCtrStride * sizeof(unsigned long long), s));
         FusedParams F = fused_params(ctx, pivots + 3 * c0, g);
         F.nslot = kk;
         F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
@@ -696,7 +743,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.gam0 = g;
         F.ctr0 = ctx->d_ctr;
         F.ctr_words = kCtrStride;
-        if ((rc = timed_begin(ctx, s))) return rc;
+        shift_slots(F, sb);
         if ((rc = kchain(ctx, s))) return rc;
         auto grid = [&](long long items, long long per_cta, int cap) {
             long long gx = (items + per_cta - 1) / per_cta;
@@ -746,9 +793,32 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         if ((rc = L(bk_band, grid(1 << 30, 1, AM_BAND_CTAS), 0, dim3(AM_BAND_THREADS)))) return rc;
         AM_KM(AM_K_BAND);
 #undef AM_KM
-        if ((rc = timed_end(ctx, s))) return rc;
+        return AM_OK;
+    };
+    // chunks of Kl pivots round-robin over `lanes` streams, lane l on slots
+    // [l Kl, (l + 1) Kl): one lane's phase tails overlap another's launches
+    // (per-kernel timing keeps one stream so its events bracket single kernels)
+    const int lanes = ctx->timing == 2 ? 1 : (int)std::max<int64_t>(1, std::min<int64_t>(ctx->lanes, K));
+    const int Kl = K / lanes;  // (lanes <= K: lane slots stay inside the K allocated)
+    if ((rc = timed_begin(ctx, s))) return rc;
+    if (lanes == 1) {
+        for (int64_t c0 = 0; c0 < P; c0 += K)
+            if ((rc = run_chunk(c0, (int)std::min<int64_t>(K, P - c0), 0, s))) return rc;
+        return timed_end(ctx, s);
     }
-    return AM_OK;
+    if ((rc = ensure_lanes(ctx, lanes))) return rc;
+    CK(cudaEventRecord(ctx->lane_ev[lanes], s));
+    for (int l = 0; l < lanes; ++l) CK(cudaStreamWaitEvent(ctx->lane_s[l], ctx->lane_ev[lanes], 0));
+    int64_t chunk = 0;
+    for (int64_t c0 = 0; c0 < P; c0 += Kl, ++chunk) {
+        const int l = (int)(chunk % lanes);
+        if ((rc = run_chunk(c0, (int)std::min<int64_t>(Kl, P - c0), l * Kl, ctx->lane_s[l]))) return rc;
+    }
+    for (int l = 0; l < lanes; ++l) {
+        CK(cudaEventRecord(ctx->lane_ev[l], ctx->lane_s[l]));
+        CK(cudaStreamWaitEvent(s, ctx->lane_ev[l], 0));
+    }
+    return timed_end(ctx, s);
 }
 
 int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s) {
@@ -1342,6 +1412,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "subbricks must be 0 or 1");
         ctx->subs_on = (int)value;
         return AM_OK;
+    case AM_OPT_BATCH_LANES:
+        if (value < 1 || value > kMaxLanes) return fail(ctx, AM_EINVAL, "batch_lanes must be in [1, %d]", kMaxLanes);
+        ctx->lanes = (int)value;
+        return AM_OK;
     case AM_OPT_CMAP_T1:
         if (value < 4 || value > ctx->cmapT) return fail(ctx, AM_EINVAL, "cmap_T1 must be in [4, cmap_T]");
         return set_texels1(ctx, (int)value);
@@ -1658,6 +1732,10 @@ void am_destroy(am_ctx* ctx) {
     int prev = -1;
     cudaGetDevice(&prev);
     cudaSetDevice(ctx->device);
+    for (int l = 0; l < kMaxLanes; ++l)
+        if (ctx->lane_s[l]) cudaStreamDestroy(ctx->lane_s[l]);
+    for (int l = 0; l <= kMaxLanes; ++l)
+        if (ctx->lane_ev[l]) cudaEventDestroy(ctx->lane_ev[l]);
     cudaFree(ctx->d_vox);
     cudaFree(ctx->d_tab);
     cudaFree(ctx->d_am);

@@ -299,8 +299,10 @@ def test_batched_launch_matches_single_maps(am, batch, diag):
     single = np.stack([ctx.compute(p)[0] for p in P])
     ctx.set_option(am.binding.OPT_DIAG, diag)
     ctx.set_option(am.binding.OPT_BATCH, batch)
-    assert np.array_equal(ctx.compute_batch(P), single)
-    assert np.array_equal(ctx.compute_batch(P[::-1]), single[::-1])  # slots see other pivots
+    for lanes in (1, 2, 3):  # chunks round-robin over internal streams, each lane its own slots
+        ctx.set_option(am.binding.OPT_BATCH_LANES, lanes)
+        assert np.array_equal(ctx.compute_batch(P), single), lanes
+        assert np.array_equal(ctx.compute_batch(P[::-1]), single[::-1]), lanes  # slots see other pivots
     ctx.close()
 
 
