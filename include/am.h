@@ -127,11 +127,15 @@ enum {
                                     32-voxel sub-brick (one warp's voxels) whose bounding sphere
                                     reaches no clear cell before its voxels are read (default);
                                     0 = read them.  Same map                                    */
-    AM_OPT_BATCH_LANES = 20      /* am_compute_batch: chunks of AM_OPT_BATCH / lanes pivots go
+    AM_OPT_BATCH_LANES = 20,     /* am_compute_batch: chunks of AM_OPT_BATCH / lanes pivots go
                                     round-robin to this many internal streams (forked from and
                                     joined to the caller's stream), so one chunk's short phases
                                     overlap another's (1..8, default 8; 1 while
                                     AM_OPT_KERNEL_TIMING = 2).  Same maps                       */
+    AM_OPT_GRAPH = 21            /* am_compute_batch: 1 = capture the batch's launch chain as a
+                                    CUDA graph and replay it while the options, the pivot count,
+                                    the output buffer and the model are unchanged (default);
+                                    0 = launch every kernel from the host.  Same maps           */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

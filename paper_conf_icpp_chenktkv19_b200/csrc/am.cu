@@ -123,6 +123,15 @@ struct am_ctx {
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
     int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
     int lanes = AM_BATCH_LANES;            // streams of the batched path (AM_OPT_BATCH_LANES)
+    int use_graph = 1;                     // AM_OPT_GRAPH: replay the batched launch chain as a CUDA graph
+    unsigned long long gen = 1;            // bumped by every option / upload / reallocation (graph key)
+    cudaStream_t cap_s = nullptr;          // capture stream
+    cudaGraphExec_t g_exec = nullptr;      // the captured chain and its key
+    unsigned long long g_gen = 0;
+    int64_t g_P = 0;
+    const void* g_dst = nullptr;
+    const void* g_piv = nullptr;
+    long long g_launches[AM_K_COUNT] = {};  // kernel launches per replay (am_kernel_stats)
     cudaStream_t lane_s[kMaxLanes] = {};
     cudaEvent_t lane_ev[kMaxLanes + 1] = {};
     int bk_map_ctas = AM_MAP_CTAS;         // per pivot, batched clear map (AM_OPT_MAP_CTAS; 0 = texels / 1024)
@@ -310,6 +319,7 @@ int set_texels1(am_ctx* ctx, int T1) {
 // batched launch; the single-map paths use slot 0).
 int ensure_slots(am_ctx* ctx, int K) {
     if (ctx->slots >= K) return AM_OK;
+    ++ctx->gen;
     const size_t ntex = (size_t)6 * ctx->cmapT * ctx->cmapT;
     cudaFree(ctx->d_ctr);
     cudaFree(ctx->d_queue);
@@ -800,23 +810,67 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     // (per-kernel timing keeps one stream so its events bracket single kernels)
     const int lanes = ctx->timing == 2 ? 1 : (int)std::max<int64_t>(1, std::min<int64_t>(ctx->lanes, K));
     const int Kl = K / lanes;  // (lanes <= K: lane slots stay inside the K allocated)
+    auto chain = [&](cudaStream_t cs) -> int {
+        int rc;
+        if (lanes == 1) {
+            for (int64_t c0 = 0; c0 < P; c0 += K)
+                if ((rc = run_chunk(c0, (int)std::min<int64_t>(K, P - c0), 0, cs))) return rc;
+            return AM_OK;
+        }
+        if ((rc = ensure_lanes(ctx, lanes))) return rc;
+        CK(cudaEventRecord(ctx->lane_ev[lanes], cs));
+        for (int l = 0; l < lanes; ++l) CK(cudaStreamWaitEvent(ctx->lane_s[l], ctx->lane_ev[lanes], 0));
+        int64_t chunk = 0;
+        for (int64_t c0 = 0; c0 < P; c0 += Kl, ++chunk) {
+            const int l = (int)(chunk % lanes);
+            if ((rc = run_chunk(c0, (int)std::min<int64_t>(Kl, P - c0), l * Kl, ctx->lane_s[l]))) return rc;
+        }
+        for (int l = 0; l < lanes; ++l) {
+            CK(cudaEventRecord(ctx->lane_ev[l], ctx->lane_s[l]));
+            CK(cudaStreamWaitEvent(cs, ctx->lane_ev[l], 0));
+        }
+        return AM_OK;
+    };
     if ((rc = timed_begin(ctx, s))) return rc;
-    if (lanes == 1) {
-        for (int64_t c0 = 0; c0 < P; c0 += K)
-            if ((rc = run_chunk(c0, (int)std::min<int64_t>(K, P - c0), 0, s))) return rc;
-        return timed_end(ctx, s);
-    }
-    if ((rc = ensure_lanes(ctx, lanes))) return rc;
-    CK(cudaEventRecord(ctx->lane_ev[lanes], s));
-    for (int l = 0; l < lanes; ++l) CK(cudaStreamWaitEvent(ctx->lane_s[l], ctx->lane_ev[lanes], 0));
-    int64_t chunk = 0;
-    for (int64_t c0 = 0; c0 < P; c0 += Kl, ++chunk) {
-        const int l = (int)(chunk % lanes);
-        if ((rc = run_chunk(c0, (int)std::min<int64_t>(Kl, P - c0), l * Kl, ctx->lane_s[l]))) return rc;
-    }
-    for (int l = 0; l < lanes; ++l) {
-        CK(cudaEventRecord(ctx->lane_ev[l], ctx->lane_s[l]));
-        CK(cudaStreamWaitEvent(s, ctx->lane_ev[l], 0));
+    // CUDA graph: the whole chain (memsets, ~11 launches per chunk, the lane fork /
+    // join) captured once per (options, P, output, pivot buffer) and replayed: one
+    // host call per batch instead of ~100 (not with per-kernel timing or diagnostics)
+    if (ctx->use_graph && ctx->timing != 2 && ctx->diag == 0) {
+        if (!(ctx->g_exec && ctx->g_gen == ctx->gen && ctx->g_P == P && ctx->g_dst == gam0 &&
+              ctx->g_piv == ctx->d_piv)) {
+            if (ctx->g_exec) cudaGraphExecDestroy(ctx->g_exec);
+            ctx->g_exec = nullptr;
+            if (!ctx->cap_s) CK(cudaStreamCreateWithFlags(&ctx->cap_s, cudaStreamNonBlocking));
+            long long before[AM_K_COUNT];
+            std::copy(ctx->k_launches, ctx->k_launches + AM_K_COUNT, before);
+            CK(cudaStreamBeginCapture(ctx->cap_s, cudaStreamCaptureModeThreadLocal));
+            const int crc = chain(ctx->cap_s);
+            cudaGraph_t graph = nullptr;
+            const cudaError_t ce = cudaStreamEndCapture(ctx->cap_s, &graph);
+            for (int k = 0; k < AM_K_COUNT; ++k) {  // the capture launched nothing
+                ctx->g_launches[k] = ctx->k_launches[k] - before[k];
+                ctx->k_launches[k] = before[k];
+            }
+            if (crc != AM_OK) {
+                if (graph) cudaGraphDestroy(graph);
+                return crc;
+            }
+            if (ce != cudaSuccess) return fail(ctx, AM_ECUDA, "graph capture: %s", cudaGetErrorString(ce));
+            const cudaError_t ie = cudaGraphInstantiate(&ctx->g_exec, graph, 0);
+            cudaGraphDestroy(graph);
+            if (ie != cudaSuccess) {
+                ctx->g_exec = nullptr;
+                return fail(ctx, AM_ECUDA, "graph instantiate: %s", cudaGetErrorString(ie));
+            }
+            ctx->g_gen = ctx->gen;
+            ctx->g_P = P;
+            ctx->g_dst = gam0;
+            ctx->g_piv = ctx->d_piv;
+        }
+        CK(cudaGraphLaunch(ctx->g_exec, s));
+        for (int k = 0; k < AM_K_COUNT; ++k) ctx->k_launches[k] += ctx->g_launches[k];
+    } else {
+        if ((rc = chain(s))) return rc;
     }
     return timed_end(ctx, s);
 }
@@ -1036,6 +1090,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     if (N < 0) return fail(ctx, AM_EINVAL, "N < 0");
     if (N > 0x7fffffffLL) return fail(ctx, AM_EINVAL, "N exceeds 2^31 - 1");
     if (N > 0 && (!centers_xyz || !half_sizes)) return fail(ctx, AM_EINVAL, "NULL voxel array");
+    ++ctx->gen;
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
     ctx->uploaded = false;
@@ -1335,6 +1390,7 @@ int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int
 int am_set_option(am_ctx* ctx, int key, int64_t value) {
     if (!ctx) return AM_EINVAL;
     DeviceGuard dg(ctx->device);
+    ++ctx->gen;  // any option may change the launch chain: recapture the batch graph
     switch (key) {
     case AM_OPT_GRID_CTAS:
         if (value < 0 || value > (1 << 20)) return fail(ctx, AM_EINVAL, "grid_ctas out of range");
@@ -1411,6 +1467,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_SUBBRICKS:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "subbricks must be 0 or 1");
         ctx->subs_on = (int)value;
+        return AM_OK;
+    case AM_OPT_GRAPH:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "graph must be 0 or 1");
+        ctx->use_graph = (int)value;
         return AM_OK;
     case AM_OPT_BATCH_LANES:
         if (value < 1 || value > kMaxLanes) return fail(ctx, AM_EINVAL, "batch_lanes must be in [1, %d]", kMaxLanes);
@@ -1732,6 +1792,8 @@ void am_destroy(am_ctx* ctx) {
     int prev = -1;
     cudaGetDevice(&prev);
     cudaSetDevice(ctx->device);
+    if (ctx->g_exec) cudaGraphExecDestroy(ctx->g_exec);
+    if (ctx->cap_s) cudaStreamDestroy(ctx->cap_s);
     for (int l = 0; l < kMaxLanes; ++l)
         if (ctx->lane_s[l]) cudaStreamDestroy(ctx->lane_s[l]);
     for (int l = 0; l <= kMaxLanes; ++l)

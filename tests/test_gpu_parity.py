@@ -306,6 +306,36 @@ def test_batched_launch_matches_single_maps(am, batch, diag):
     ctx.close()
 
 
+def test_batch_graph_replay(am):
+    """The batch launch chain replayed as a CUDA graph (AM_OPT_GRAPH): replays with new
+    pivots into the same device buffer, a new buffer, host outputs and an option change
+    (each forcing a recapture) all give the one-pivot maps."""
+    import torch
+    cfg = scenes.CONFIGS["C2"]
+    C, H = cfg.leaves()
+    P = cfg.pivots(24)
+    ctx = _ctx(am, cfg, C, H)
+    single = np.stack([ctx.compute(p)[0] for p in P])
+    ctx.set_option(am.binding.OPT_BATCH, 8)
+    ctx.set_option(am.binding.OPT_BATCH_LANES, 2)
+    dev = torch.zeros((8, ctx.words), dtype=torch.int32, device="cuda:0")
+    for rep in range(2):
+        for c in range(3):  # same buffer, new pivots each call: replay
+            ctx.compute_batch(P[8 * c:8 * c + 8], out=dev)
+            torch.cuda.synchronize()
+            assert np.array_equal(dev.cpu().numpy().view(np.uint32), single[8 * c:8 * c + 8]), (rep, c)
+    dev2 = torch.zeros_like(dev)  # another buffer: recapture
+    ctx.compute_batch(P[8:16], out=dev2)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev2.cpu().numpy().view(np.uint32), single[8:16])
+    assert np.array_equal(ctx.compute_batch(P[16:24]), single[16:24])  # host output
+    ctx.set_option(am.binding.OPT_BATCH_LANES, 4)  # option change: recapture
+    assert np.array_equal(ctx.compute_batch(P[:8]), single[:8])
+    ctx.set_option(am.binding.OPT_GRAPH, 0)
+    assert np.array_equal(ctx.compute_batch(P), single)
+    ctx.close()
+
+
 def _check_sampled(cfg, C, H, p, g, rng, nclear=64, nblocked=32):
     clear = np.nonzero(g == 0)[0]
     blocked = np.nonzero(g == 1)[0]
