@@ -29,6 +29,15 @@ using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
 // level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+#ifndef AM_ROWS_CTAS
+#define AM_ROWS_CTAS 64
+#endif
+#ifndef AM_VOXEL_CTAS
+#define AM_VOXEL_CTAS 64
+#endif
+#ifndef AM_CONE_CTAS
+#define AM_CONE_CTAS 64
+#endif
 #ifndef AM_BATCH_LANES
 #define AM_BATCH_LANES 8
 #endif
@@ -121,7 +130,7 @@ struct am_ctx {
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
-    int bk_rows_ctas = 32, bk_voxel_ctas = 64, bk_cone_ctas = 32;  // per pivot, batched phases
+    int bk_rows_ctas = AM_ROWS_CTAS, bk_voxel_ctas = AM_VOXEL_CTAS, bk_cone_ctas = AM_CONE_CTAS;  // per pivot, batched phases
     int lanes = AM_BATCH_LANES;            // streams of the batched path (AM_OPT_BATCH_LANES)
     int use_graph = 1;                     // AM_OPT_GRAPH: replay the batched launch chain as a CUDA graph
     unsigned long long gen = 1;            // bumped by every option / upload / reallocation (graph key)
