@@ -326,6 +326,8 @@ def run_ours(args):
         ctx.set_option(B.OPT_FUSED, 0)
         ctx.set_option(B.OPT_BRICKS, 0)
         kf = max(1, min(args.steps, 50))
+        _timed_maps(ctx, piv, out, stream, 3, None, torch, 1)  # warm-up (first launches of these kernels)
+        ctx.kernel_time()
         fms, _ = _timed_maps(ctx, piv, out, stream, kf, flush, torch, 1)
         fk, fl = ctx.kernel_time()
         ctx.set_option(B.OPT_BRICKS, 1)
