@@ -299,6 +299,43 @@ std::vector<float> make_texels(int T) {
                 out[t + 2] = (float)c[2];
                 out[t + 3] = (float)(r + 2e-5);
             }
+    // the clear map's 8 x 8-texel blocks (kernels.cuh clear_map_blocks), 2 float4 each after
+    // the texels: (c, cos 2rho'), (sin 2rho', 0, 0, 0) with c the normalised sum of the
+    // block's (fp32) texel centres and 2rho' = 2 max angle(c, texel centre) + 1e-6 + 1e-4
+    if (T % 8 == 0) {
+        const int Tc = T / 8;
+        const size_t ntex = (size_t)6 * T * T;
+        out.resize((ntex + (size_t)2 * 6 * Tc * Tc) * 4, 0.f);
+        for (int ct = 0; ct < 6 * Tc * Tc; ++ct) {
+            const int f = ct / (Tc * Tc), rem = ct % (Tc * Tc), cw = rem / Tc, cu = rem % Tc;
+            double sum[3] = {0, 0, 0};
+            for (int a = 0; a < 8; ++a)
+                for (int b = 0; b < 8; ++b) {
+                    const size_t t = ((size_t)(f * T + 8 * cw + a) * T + 8 * cu + b) * 4;
+                    for (int k = 0; k < 3; ++k) sum[k] += (double)out[t + k];
+                }
+            const double nn = std::sqrt(sum[0] * sum[0] + sum[1] * sum[1] + sum[2] * sum[2]);
+            float cf[3];
+            for (int k = 0; k < 3; ++k) cf[k] = (float)(sum[k] / nn);
+            double rho = 0.0;
+            for (int a = 0; a < 8; ++a)
+                for (int b = 0; b < 8; ++b) {
+                    const size_t t = ((size_t)(f * T + 8 * cw + a) * T + 8 * cu + b) * 4;
+                    const double d0 = out[t], d1 = out[t + 1], d2 = out[t + 2];
+                    const double dn = std::sqrt(d0 * d0 + d1 * d1 + d2 * d2);
+                    const double cn = std::sqrt((double)cf[0] * cf[0] + (double)cf[1] * cf[1] + (double)cf[2] * cf[2]);
+                    const double dp = (cf[0] * d0 + cf[1] * d1 + cf[2] * d2) / (dn * cn);
+                    rho = std::max(rho, std::acos(std::max(-1.0, std::min(1.0, dp))));
+                }
+            const double a2 = 2.0 * (rho + 1e-6) + 1e-4;
+            const size_t o = (ntex + 2 * (size_t)ct) * 4;
+            out[o] = cf[0];
+            out[o + 1] = cf[1];
+            out[o + 2] = cf[2];
+            out[o + 3] = (float)std::cos(a2);
+            out[o + 4] = (float)std::sin(a2);
+        }
+    }
     return out;
 }
 

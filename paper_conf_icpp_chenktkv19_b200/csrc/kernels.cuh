@@ -400,46 +400,35 @@ __device__ int clear_list_rows_cta(const uint32_t* sAM, const GridDev& g, const 
 // a texel centre, rounded up) bound the search: with theta_C = the angle from
 // c to its nearest clear direction, every texel's nearest clear direction lies
 // within theta_C + 2 rho of c (triangle inequality), so only those candidates
-// (found by one ballot pass over the list) are tried per texel.
-template <int B>
+// (found by one ballot pass over the list) are tried per texel.  c and
+// cos / sin(2 rho + slack) come from the host-made block table after the texels.
 __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float* __restrict__ V,
                                  const float4* sDirs, int total, int w0, int wstride) {
-    constexpr int TPL = B * B / 32, ROWS = 32 / B;
+    constexpr int B = 8, TPL = B * B / 32, ROWS = 32 / B;
     const int lane = threadIdx.x & 31;
     const int Tc = T / B, nct = 6 * Tc * Tc;
+    const float inv1 = 1.f / (float)(Tc * Tc), inv2 = 1.f / (float)Tc;
+    const float4* __restrict__ blocks = texels + 6 * T * T;  // host-made block table (am.cu make_texels)
     for (int ct = w0; ct < nct; ct += wstride) {
-        const int face = ct / (Tc * Tc), rem = ct - face * Tc * Tc, cw = rem / Tc, cu = rem - cw * Tc;
+        // (ct < 2^22: the float quotients floor exactly)
+        const int face = (int)(((float)ct + 0.5f) * inv1), rem = ct - face * Tc * Tc;
+        const int cw = (int)(((float)rem + 0.5f) * inv2), cu = rem - cw * Tc;
         const int t0 = (face * T + B * cw + lane / B) * T + B * cu + lane % B;
         float4 f[TPL];
-        float sx = 0.f, sy = 0.f, sz = 0.f;
 #pragma unroll
-        for (int k = 0; k < TPL; ++k) {
-            f[k] = texels[t0 + k * ROWS * T];
-            sx += f[k].x;
-            sy += f[k].y;
-            sz += f[k].z;
-        }
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            sx += __shfl_xor_sync(0xffffffffu, sx, o);
-            sy += __shfl_xor_sync(0xffffffffu, sy, o);
-            sz += __shfl_xor_sync(0xffffffffu, sz, o);
-        }
-        const float inv = rsqrtf(fmaf(sx, sx, fmaf(sy, sy, sz * sz)));
-        const float4 c = make_float4(sx * inv, sy * inv, sz * inv, 0.f);
-        // rho from the smallest cosine (acos decreasing), rounded up
-        float cmin = 2.f;
-#pragma unroll
-        for (int k = 0; k < TPL; ++k) cmin = fminf(cmin, dot3(f[k], c));
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) cmin = fminf(cmin, __shfl_xor_sync(0xffffffffu, cmin, o));
-        const float rho = acosf(fmaxf(cmin - 1e-6f, -1.f));
+        for (int k = 0; k < TPL; ++k) f[k] = texels[t0 + k * ROWS * T];
+        const float4 A = blocks[2 * ct];   // block centre c, cos(2 rho')
+        const float sR = blocks[2 * ct + 1].x;  // sin(2 rho')
+        const float4 c = make_float4(A.x, A.y, A.z, 0.f);
         float bc = -2.f;
         for (int e = lane; e < total; e += 32) bc = fmaxf(bc, dot3(c, sDirs[e]));
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) bc = fmaxf(bc, __shfl_xor_sync(0xffffffffu, bc, o));
-        const float th = acosf(fmaxf(bc - 1e-6f, -1.f)) + 2.f * rho + 1e-4f;
-        const float thr = th >= 3.14159f ? -2.f : cosf(th) - 1e-6f;
+        // thr = cos(theta_C' + 2 rho') - 1e-6 with cos theta_C' = b (rounded down): the sum
+        // formula, sin theta_C' = sqrt((1 - b)(1 + b)); -2 (every candidate) past pi
+        const float b = fmaxf(bc - 1e-6f, -1.f);
+        const float thr = (b <= -A.w) ? -2.f
+                                      : fmaf(b, A.w, -sqrtf(fmaxf((1.f - b) * (1.f + b), 0.f)) * sR) - 1e-6f;
         float bf[TPL];
 #pragma unroll
         for (int k = 0; k < TPL; ++k) bf[k] = -2.f;
@@ -500,7 +489,7 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
     }
     if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
-        clear_map_blocks<8>(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps);
+        clear_map_blocks(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps);
         return;
     }
     if (total > g.brute && total <= kMapDirs && (T & 3) == 0) {
