@@ -42,6 +42,9 @@ using namespace am;
 #define AM_BATCH_LANES 8
 #endif
 constexpr int kMaxLanes = 8;
+#ifndef AM_L1_STEPS
+#define AM_L1_STEPS 8  // level-1 cone steps (256 voxels each) per CTA of the batched path
+#endif
 #ifndef AM_BRICK_STEPS
 #define AM_BRICK_STEPS 4  // brick-test steps (256 bricks each) per CTA of the batched path
 #endif
@@ -830,7 +833,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
-            if ((rc = L(bk_cones<BK_L1>, grid(ctx->n_l1 - ctx->n_l0, 4 * kThreads, 1 << 16), sm_rows))) return rc;
+            if ((rc = L(bk_cones<BK_L1>, grid(ctx->n_l1 - ctx->n_l0, AM_L1_STEPS * kThreads, 1 << 16), sm_rows))) return rc;
             AM_KM(AM_K_L1_CONES);
             if ((rc = L(bk_rows<BK_L1>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
             AM_KM(AM_K_L1_ROWS);
