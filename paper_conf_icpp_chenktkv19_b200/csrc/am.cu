@@ -73,13 +73,13 @@ constexpr int kMaxLanes = 8;
 #define AM_BAND_THREADS 256
 #endif
 #ifndef AM_L0_DIV
-#define AM_L0_DIV 8192
+#define AM_L0_DIV 16384
 #endif
 #ifndef AM_L1_DIV
-#define AM_L1_DIV 256
+#define AM_L1_DIV 4096
 #endif
 #ifndef AM_L1_STRIDE
-#define AM_L1_STRIDE 512
+#define AM_L1_STRIDE 384
 #endif
 
 struct am_ctx {
