@@ -123,10 +123,11 @@ enum {
     AM_OPT_MAP_CTAS = 18,        /* batched path: CTAs per pivot of the (final) clear-direction
                                     map launch, 0..4096 (0 = one per 1024 texels; default 48).
                                     Same map                                                    */
-    AM_OPT_SUBBRICKS = 19,       /* fused and batched paths: 1 = inside a kept brick, skip each
-                                    32-voxel sub-brick (one warp's voxels) whose bounding sphere
-                                    reaches no clear cell before its voxels are read (default);
-                                    0 = read them.  Same map                                    */
+    AM_OPT_SUBBRICKS = 19,       /* fused and batched paths, bit 0: skip each 32-voxel sub-brick
+                                    of a kept brick (one warp's voxels) whose bounding sphere
+                                    reaches no clear cell before its voxels are read; bit 1
+                                    (batched path): test super-bricks of 8 bricks first and only
+                                    the bricks of kept ones (0..3, default 3).  Same map        */
     AM_OPT_BATCH_LANES = 20,     /* am_compute_batch: chunks of AM_OPT_BATCH / lanes pivots go
                                     round-robin to this many internal streams (forked from and
                                     joined to the caller's stream), so one chunk's short phases
@@ -145,7 +146,8 @@ enum {
     AM_K_CLEAR_MAP,     /* clear-direction map of the partial AM                 */
     AM_K_L1_CONES,      /* level-1 filter + inner cones                                        */
     AM_K_L1_ROWS,       /* their rows                                                          */
-    AM_K_BRICKS,        /* brick bounding-sphere test, a1-a2 (8(f) NEXT 1)                     */
+    AM_K_BRICKS,        /* brick bounding-sphere test, a1-a2 (8(f) NEXT 1; batched path: the
+                           super-brick launch and the brick launch)                            */
     AM_K_VOXELS,        /* kept bricks' voxels through the filter -> live list, a1-a3          */
     AM_K_LIVE_CONES,    /* live voxels' inner + outer cones, a3-a4                             */
     AM_K_LIVE_ROWS,     /* their rows + band queue, a5-a7                                      */

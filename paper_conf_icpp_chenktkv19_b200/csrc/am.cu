@@ -129,7 +129,8 @@ struct am_ctx {
     unsigned int nbricks = 0;
     int bricks_on = 1;
     float4* d_subs = nullptr;              // bounding spheres of 32-voxel sub-bricks (warps of a brick)
-    int subs_on = 1;                       // AM_OPT_SUBBRICKS
+    float4* d_supers = nullptr;            // bounding spheres of 2048-voxel super-bricks (8 bricks)
+    int subs_on = 3;                       // AM_OPT_SUBBRICKS: bit 0 sub-bricks, bit 1 super-bricks
     int fused = 1;                         // one cooperative launch per map (fused.cuh)
     int batch = 32;                        // pivots per batched launch (AM_OPT_BATCH)
     int band_vdepth = 0;                   // AM_OPT_BAND_SUBDIV
@@ -186,7 +187,8 @@ namespace {
 constexpr int kCtrTiles = 1 + ST_COUNT;      // live count: full stream (+0), level 1 (+4)
 constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, task count at +2s+1
 constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
-constexpr int kCtrWords = kCtrBricks + 1;
+constexpr int kCtrSupers = kCtrBricks + 1;   // super-bricks kept (batched path)
+constexpr int kCtrWords = kCtrSupers + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
 constexpr int kCtrStride = kCtrAll;          // 64-bit words per slot
 constexpr int kMaxBatch = 64;                // pivots per layered batch launch (slots)
@@ -342,6 +344,11 @@ std::vector<float> make_texels(int T) {
     return out;
 }
 
+// Words per slot of d_brick_list: kept sub-bricks (8 per brick), then kept super-bricks.
+unsigned long long blist_words(const am_ctx* ctx) {
+    return 8ull * ctx->nbricks + (ctx->nbricks + 7) / 8;
+}
+
 int ensure_queue(am_ctx* ctx, long long cap) {
     if (ctx->d_queue && ctx->qcap == cap) return AM_OK;
     if (ctx->d_queue) cudaFree(ctx->d_queue);
@@ -392,7 +399,7 @@ int ensure_slots(am_ctx* ctx, int K) {
     CK(cudaMalloc(&ctx->d_tasks, (size_t)K * kTaskCap * sizeof(unsigned long long)));
     CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float)));
     if (ctx->vox_cap > 0) CK(cudaMalloc(&ctx->d_live, (size_t)K * ctx->vox_cap * sizeof(unsigned int)));
-    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * 8 * ctx->nbricks * sizeof(unsigned int)));
+    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * blist_words(ctx) * sizeof(unsigned int)));
     return AM_OK;
 }
 
@@ -564,7 +571,10 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.main.cmap = ctx->d_cmap;
     F.main.bricks = ctx->d_bricks;
     F.main.nbricks = ctx->nbricks;
-    F.main.subs = ctx->subs_on ? ctx->d_subs : nullptr;
+    F.main.subs = (ctx->subs_on & 1) ? ctx->d_subs : nullptr;
+    F.main.supers = (ctx->subs_on & 2) ? ctx->d_supers : nullptr;
+    F.main.super_list = ctx->d_brick_list + 8ull * ctx->nbricks;
+    F.main.super_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrSupers);
     F.main.brick_list = ctx->d_brick_list;
     F.main.brick_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrBricks);
     F.main.recs = ctx->d_recs;
@@ -702,7 +712,7 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
     F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
     F.cmap_stride = (unsigned long long)ntex * sizeof(float);
-    F.blist_stride = 8ull * ctx->nbricks * sizeof(unsigned int);
+    F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
     F.piv = ctx->d_piv;
     F.npiv = (unsigned int)P;
     F.gam0 = gam0;
@@ -747,6 +757,8 @@ void shift_slots(FusedParams& F, int base) {
         p.recs = hshift(p.recs, b * F.rec_stride);
         p.tasks = hshift(p.tasks, b * F.task_stride);
         p.brick_list = hshift(p.brick_list, b * F.blist_stride);
+        p.super_list = hshift(p.super_list, b * F.blist_stride);
+        p.super_count = hshift(p.super_count, b * F.ctr_stride);
         if (!which) p.cmap = hshift(p.cmap, b * F.cmap_stride);
     }
     F.rec1 = hshift(F.rec1, b * F.ctr_stride);
@@ -796,7 +808,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
         F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
         F.cmap_stride = (unsigned long long)ntex * sizeof(float);
-        F.blist_stride = 8ull * ctx->nbricks * sizeof(unsigned int);
+        F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
         F.piv = ctx->d_piv + c0;
         F.npiv = (unsigned int)kk;
         F.gam0 = g;
@@ -839,6 +851,10 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             AM_KM(AM_K_L1_ROWS);
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
+        }
+        if (F.main.supers) {
+            if ((rc = L(bk_supers, grid((ctx->nbricks + 7) / 8, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
+            AM_KM(AM_K_BRICKS);
         }
         if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
         AM_KM(AM_K_BRICKS);
@@ -1250,13 +1266,21 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     ctx->d_brick_list = nullptr;
     ctx->nbricks = (unsigned int)((N + kThreads - 1) / kThreads);
     UK(cudaMalloc(&ctx->d_bricks, (size_t)ctx->nbricks * sizeof(float4)));
-    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * 8 * ctx->nbricks * sizeof(unsigned int)));
+    UK(cudaMalloc(&ctx->d_brick_list, (size_t)ctx->slots * blist_words(ctx) * sizeof(unsigned int)));
     brick_bounds_kernel<<<(unsigned)(((long long)ctx->nbricks * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_bricks,
                                                                                         ctx->nbricks, kThreads);
     UK(cudaGetLastError());
     cudaFree(ctx->d_subs);
-    ctx->d_subs = nullptr;
+    cudaFree(ctx->d_supers);
+    ctx->d_subs = ctx->d_supers = nullptr;
     {
+        const unsigned int nsup = (ctx->nbricks + 7) / 8;
+        if (nsup > 0) {
+            UK(cudaMalloc(&ctx->d_supers, (size_t)nsup * sizeof(float4)));
+            brick_bounds_kernel<<<(unsigned)(((long long)nsup * 32 + 255) / 256), 256>>>(ctx->d_vox, N, ctx->d_supers,
+                                                                                         nsup, 8 * kThreads);
+            UK(cudaGetLastError());
+        }
         const unsigned int nsub = (unsigned int)((N + 31) / 32);
         if (nsub > 0) {
             UK(cudaMalloc(&ctx->d_subs, (size_t)nsub * sizeof(float4)));
@@ -1514,7 +1538,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->bk_map_ctas = (int)value;
         return AM_OK;
     case AM_OPT_SUBBRICKS:
-        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "subbricks must be 0 or 1");
+        if (value < 0 || value > 3) return fail(ctx, AM_EINVAL, "subbricks must be in [0, 3]");
         ctx->subs_on = (int)value;
         return AM_OK;
     case AM_OPT_GRAPH:
@@ -1857,6 +1881,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);
     cudaFree(ctx->d_subs);
+    cudaFree(ctx->d_supers);
     cudaFree(ctx->d_bricks);
     cudaFree(ctx->d_brick_list);
     cudaFree(ctx->d_texels);

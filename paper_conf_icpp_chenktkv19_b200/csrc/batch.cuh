@@ -180,14 +180,45 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
                   gridDim.x);
 }
 
-// Brick test: bricks, then their 32-voxel sub-bricks, whose bounding sphere may
-// still reach a clear cell (fused.cuh brick_step).
+// Super-brick test (P.supers set): super-bricks of 8 bricks whose bounding
+// sphere may still reach a clear cell go to the map's super list.
+__global__ void __launch_bounds__(kThreads) bk_supers(const __grid_constant__ FusedParams F) {
+    __shared__ StreamParams sP;
+    const int p = blockIdx.y;
+    pivot_params(sP, F, p, false);
+    const StreamParams& P = sP;
+    const int lane = threadIdx.x & 31;
+    const unsigned int nsup = (P.nbricks + 7) >> 3;
+    for (unsigned int s0 = blockIdx.x * kThreads; s0 < nsup; s0 += gridDim.x * kThreads) {
+        const unsigned int sp = s0 + threadIdx.x;
+        const bool keep = sp < nsup && !node_dropped(P, P.supers, sp);
+        const unsigned int mk = __ballot_sync(0xffffffffu, keep);
+        if (!mk) continue;
+        unsigned int base = 0;
+        if (lane == 0) base = atomicAdd(P.super_count, (unsigned int)__popc(mk));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (keep) P.super_list[base + __popc(mk & ((1u << lane) - 1u))] = sp;
+    }
+}
+
+// Brick test: bricks (all, or the 8 of each kept super-brick), then their
+// 32-voxel sub-bricks, whose bounding sphere may still reach a clear cell
+// (fused.cuh brick_test).
 __global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
     pivot_params(sP, F, p, false);
     const StreamParams& P = sP;
-    for (unsigned int b0 = blockIdx.x * kThreads; b0 < P.nbricks; b0 += gridDim.x * kThreads) brick_step(P, b0);
+    if (P.supers) {
+        const unsigned int ne = 8u * *reinterpret_cast<const volatile unsigned int*>(P.super_count);
+        for (unsigned int e0 = blockIdx.x * kThreads; e0 < ne; e0 += gridDim.x * kThreads) {
+            const unsigned int e = e0 + threadIdx.x;
+            const unsigned int b = e < ne ? P.super_list[e >> 3] * 8u + (e & 7u) : 0u;
+            brick_test(P, b, e < ne);
+        }
+    } else {
+        for (unsigned int b0 = blockIdx.x * kThreads; b0 < P.nbricks; b0 += gridDim.x * kThreads) brick_step(P, b0);
+    }
 }
 
 // Kept sub-bricks' voxels through the filter; live voxels to the live list.

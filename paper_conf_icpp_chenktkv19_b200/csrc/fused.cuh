@@ -89,6 +89,8 @@ __device__ void slot_params(StreamParams& p, const FusedParams& F, int s, bool o
     p.recs = shift_bytes(p.recs, s * F.rec_stride);
     p.tasks = shift_bytes(p.tasks, s * F.task_stride);
     p.brick_list = shift_bytes(p.brick_list, s * F.blist_stride);
+    p.super_list = shift_bytes(p.super_list, s * F.blist_stride);
+    p.super_count = shift_bytes(p.super_count, c);
     if (own_cmap) p.cmap = shift_bytes(p.cmap, s * F.cmap_stride);
 }
 
@@ -241,13 +243,12 @@ __device__ __forceinline__ bool node_dropped(const StreamParams& P, const float4
     return sphere_dropped(P, s.x - P.px, s.y - P.py, s.z - P.pz, s.w);
 }
 
-__device__ __forceinline__ void brick_step(const StreamParams& P, unsigned int b0) {
+__device__ __forceinline__ void brick_test(const StreamParams& P, unsigned int b, bool valid) {
     __shared__ unsigned int sKept[kWarps][32];  // per warp: its kept bricks
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const unsigned int lt = (1u << lane) - 1u;
-    const unsigned int b = b0 + threadIdx.x;
     const unsigned long long nsub = ((unsigned long long)P.N + 31) >> 5;
-    const bool kb = b < P.nbricks && !node_dropped(P, P.bricks, b);
+    const bool kb = valid && b < P.nbricks && !node_dropped(P, P.bricks, b);
     const unsigned int mb = __ballot_sync(0xffffffffu, kb);
     if (!mb) return;
     if (lane == 0) atomicAdd(P.brick_count + 1, (unsigned int)__popc(mb));
@@ -267,6 +268,10 @@ __device__ __forceinline__ void brick_step(const StreamParams& P, unsigned int b
         }
     }
     __syncwarp();
+}
+
+__device__ __forceinline__ void brick_step(const StreamParams& P, unsigned int b0) {
+    brick_test(P, b0 + threadIdx.x, true);
 }
 
 // Voxel phase, one CTA step over the kept sub-bricks [k0, k0 + kVPT kWarps):

@@ -75,6 +75,11 @@ struct StreamParams {
     // sub-bricks of 32 consecutive voxels (one warp of a brick): bounding spheres;
     // nullptr = not tested
     const float4* __restrict__ subs;
+    // super-bricks of 8 bricks (batched path): bounding spheres (nullptr = not tested),
+    // kept super-bricks of this map and their count (zeroed per map)
+    const float4* __restrict__ supers;
+    unsigned int* super_list;
+    unsigned int* super_count;
 };
 
 // Cube-map texel of direction v (any length): face = dominant axis and sign,

@@ -275,10 +275,11 @@ def test_phases_and_tunables_give_identical_maps(am, name):
         assert np.array_equal(ctx.compute_batch(P), ref), (brute, block)
     with pytest.raises(am.AMError):
         ctx.set_option(am.binding.OPT_CMAP_BLOCK, 16)
-    ctx.set_option(am.binding.OPT_SUBBRICKS, 0)  # read every voxel of a kept brick
-    assert np.array_equal(ctx.compute_batch(P), ref)
-    assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
-    ctx.set_option(am.binding.OPT_SUBBRICKS, 1)
+    for sub in (0, 1, 2):  # without the sub-brick and / or super-brick levels
+        ctx.set_option(am.binding.OPT_SUBBRICKS, sub)
+        assert np.array_equal(ctx.compute_batch(P), ref), sub
+        assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref), sub
+    ctx.set_option(am.binding.OPT_SUBBRICKS, 3)
     ctx.set_option(am.binding.OPT_CMAP_T, 16)
     ctx.set_option(am.binding.OPT_GRID_CTAS, 7)
     ctx.set_option(am.binding.OPT_REFRESH_TILES, 1)
