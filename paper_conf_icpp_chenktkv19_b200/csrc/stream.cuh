@@ -347,13 +347,21 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
         const float lo = c.cout - kClearSlack, hi = c.clo + kClearSlack;
         bool any = false;
         const int e0 = rowStart ? rowStart[a0] : 0, e1 = rowStart ? rowStart[a1 + 1] : nclear;
-        for (int e = e0; e < e1; ++e) {
+        auto dotc = [&](int e) {
             const float4 d = clear[e];
-            const float cd = fmaf(ux, d.x, fmaf(uy, d.y, uz * d.z));
-            if (cd >= lo && cd <= hi) {
-                any = true;
-                break;
-            }
+            return fmaf(ux, d.x, fmaf(uy, d.y, uz * d.z));
+        };
+        int e = e0;
+        if (hi > 1.5f) {  // no ring (the common case): only the outer cone, 4 cells per test
+            for (; e + 4 <= e1; e += 4)
+                if (fmaxf(fmaxf(dotc(e), dotc(e + 1)), fmaxf(dotc(e + 2), dotc(e + 3))) >= lo) {
+                    any = true;
+                    break;
+                }
+        }
+        for (; e < e1 && !any; ++e) {
+            const float cd = dotc(e);
+            any = cd >= lo && cd <= hi;
         }
         if (!any) return 0;
     }
