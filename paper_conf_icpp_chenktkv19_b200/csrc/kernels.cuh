@@ -440,11 +440,14 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
         for (int base = 0; base < total; base += 32) {
             const int e = base + lane;
             unsigned int mask = __ballot_sync(0xffffffffu, e < total && dot3(c, sDirs[e]) >= thr);
-            while (mask) {
-                const float4 d = sDirs[base + __ffs(mask) - 1];
+            while (mask) {  // two candidates per pass (the second repeats the first when alone)
+                const int k1 = __ffs(mask) - 1;
                 mask &= mask - 1u;
+                const int k2 = mask ? __ffs(mask) - 1 : k1;
+                mask &= mask - 1u;
+                const float4 d1 = sDirs[base + k1], d2 = sDirs[base + k2];
 #pragma unroll
-                for (int k = 0; k < TPL; ++k) bf[k] = fmaxf(bf[k], dot3(f[k], d));
+                for (int k = 0; k < TPL; ++k) bf[k] = fmaxf(bf[k], fmaxf(dot3(f[k], d1), dot3(f[k], d2)));
             }
         }
 #pragma unroll
