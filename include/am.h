@@ -107,11 +107,12 @@ enum {
     AM_OPT_CMAP_T1 = 14,         /* resolution of the clear-direction map built after level 0,
                                     which only filters level 1 (4..AM_OPT_CMAP_T, default 32).
                                     Same map                                                    */
-    AM_OPT_CMAP_ROWSCAN = 15,    /* clear-direction map: with more clear cells than this, each
+    AM_OPT_CMAP_ROWSCAN = 15,    /* clear-direction map: with more clear cells than this -- and
+                                    always with more than fit in shared memory (2048) -- each
                                     texel finds its nearest clear cell row by row (nearest clear
                                     gamma per phi-row, rows outward from the texel's phi, early
-                                    stop); otherwise every texel tries every clear cell
-                                    (0..2^21, default 2^21: off).                               */
+                                    stop); otherwise the block / all-pairs search (0..2^21,
+                                    default 2^21).  Same map                                    */
     AM_OPT_CMAP_BRUTE = 16,      /* clear-direction map: with at most this many clear cells every
                                     texel tries every one; above, texel blocks first bound   
                                     the candidates from the block centre (0..2^21, default

@@ -476,7 +476,12 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
     __syncthreads();
     const int total = *sN;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    if (total > g.rowscan) {
+#ifndef AM_ROWSCAN_OVER_DIRS
+#define AM_ROWSCAN_OVER_DIRS 1
+#endif
+    // (more clear cells than fit in shared memory: clear cells are dense, so the
+    // row-ordered nearest-clear search stops after a few rows)
+    if (total > g.rowscan || (AM_ROWSCAN_OVER_DIRS && total > kMapDirs)) {
         // clear masks in place (sAM is re-seeded by every caller before reuse),
         // one bit per row with a clear cell in the sDirs space
         uint32_t* sRows = reinterpret_cast<uint32_t*>(sDirs);
