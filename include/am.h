@@ -112,7 +112,7 @@ enum {
                                     texel finds its nearest clear cell row by row (nearest clear
                                     gamma per phi-row, rows outward from the texel's phi, early
                                     stop); otherwise the block / all-pairs search (0..2^21,
-                                    default 2^21).  Same map                                    */
+                                    default 1024).  Same map                                    */
     AM_OPT_CMAP_BRUTE = 16,      /* clear-direction map: with at most this many clear cells every
                                     texel tries every one; above, texel blocks first bound   
                                     the candidates from the block centre (0..2^21, default

@@ -58,7 +58,7 @@ constexpr int kMaxLanes = 8;
 #define AM_CMAP_BRUTE 0
 #endif
 #ifndef AM_CMAP_ROWSCAN
-#define AM_CMAP_ROWSCAN 2097152
+#define AM_CMAP_ROWSCAN 1024
 #endif
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 32
