@@ -87,3 +87,14 @@ def test_kernel_names_match_header(am):
     assert len(set(am.binding.KERNEL_NAMES)) == am.binding.K_COUNT
     assert am.lib.am_kernel_name(am.binding.K_COUNT) is None
     assert am.lib.am_kernel_name(-1) is None
+
+
+def test_option_keys_match_header(am):
+    """Every AM_OPT_* key of include/am.h has the same value in the binding (OPT_*), and the
+    binding defines no key the header lacks."""
+    src = open(os.path.join(ROOT, "include", "am.h")).read()
+    header = {k[len("AM_OPT_"):]: int(v)
+              for k, v in re.findall(r"^\s*(AM_OPT_[A-Z0-9_]+)\s*=\s*(\d+)\s*,?\s*/\*", src, re.M)}
+    binding = {k[len("OPT_"):]: getattr(am.binding, k) for k in dir(am.binding) if k.startswith("OPT_")}
+    assert header == binding
+    assert sorted(header.values()) == list(range(1, len(header) + 1))
