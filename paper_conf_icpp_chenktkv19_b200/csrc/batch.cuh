@@ -44,11 +44,19 @@ namespace am {
 // a __grid_constant__ parameter is not a global address); `lvl` selects the
 // clear-map-level copy.  Ends with a barrier.
 __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParams& F, int p, bool lvl) {
+    // the copy one word per thread (a ~1 KB struct copied by one thread is a long
+    // serial chain in every CTA's prologue), then thread 0 applies slot and pivot
+    constexpr int kWords = (int)(sizeof(StreamParams) / 4);
+    uint32_t* dst = reinterpret_cast<uint32_t*>(&out);
+    if (lvl) {
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(&F.lvl);
+        for (int w = threadIdx.x; w < kWords; w += blockDim.x) dst[w] = src[w];
+    } else {
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(&F.main);
+        for (int w = threadIdx.x; w < kWords; w += blockDim.x) dst[w] = src[w];
+    }
+    __syncthreads();
     if (threadIdx.x == 0) {
-        if (lvl)
-            out = F.lvl;
-        else
-            out = F.main;
         slot_params(out, F, p, !lvl);
         set_pivot(out, F.piv[p], F.gam0 + (size_t)p * F.main.grid.m * F.main.grid.W);
     }
@@ -251,7 +259,10 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
     }
 }
 
-// Band: exact test of the queued pairs whose bit is still clear.
+// Band: exact test of the queued pairs whose bit is still clear.  Each pair
+// is tested by 4 lanes, lane q taking cylinders q, q + 4, ... (the test is an
+// OR over cylinders), so the long serial CHECKBOX chain is ~ncyl times
+// shorter; a warp takes 8 pairs per pass.
 __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
@@ -260,19 +271,55 @@ __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ Fuse
     const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
     const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
     unsigned long long tests = 0, hits = 0;
-    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += stride) {
-        const unsigned long long e = P.queue[k];
-        const unsigned int vidx = (unsigned int)(e >> 32);
-        const int cell = (int)(e & 0xffffffffu);
-        const int i = cell / P.grid.n, j = cell - i * P.grid.n;
-        uint32_t* wp = P.gam + i * P.grid.W + (j >> 5);
-        const uint32_t bit = 1u << (j & 31);
-        if (ld_cg(wp) & bit) continue;
-        ++tests;
-        if (exact_pair(P, P.vox_main[vidx], cell)) {
-            ++hits;
-            atomicOr(wp, bit);
+    const int lane = threadIdx.x & 31, sub = lane & 3;
+    if (P.band_vdepth > 0) {  // corner-case expansion: one pair per thread (exact_pair)
+        const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+        for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += stride) {
+            const unsigned long long e = P.queue[k];
+            const unsigned int vidx = (unsigned int)(e >> 32);
+            const int cell = (int)(e & 0xffffffffu);
+            const int i = cell / P.grid.n, j = cell - i * P.grid.n;
+            uint32_t* wp = P.gam + i * P.grid.W + (j >> 5);
+            const uint32_t bit = 1u << (j & 31);
+            if (ld_cg(wp) & bit) continue;
+            ++tests;
+            if (exact_pair(P, P.vox_main[vidx], cell)) {
+                ++hits;
+                atomicOr(wp, bit);
+            }
+        }
+    } else {
+        const unsigned long long stride = ((unsigned long long)gridDim.x * blockDim.x) >> 2;
+        for (unsigned long long k0 = ((unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) >> 2; k0 < n;
+             k0 += stride) {  // warp-uniform
+            const unsigned long long k = k0 + (lane >> 2);
+            bool test = false, hit = false;
+            uint32_t* wp = nullptr;
+            uint32_t bit = 0u;
+            if (k < n) {
+                const unsigned long long e = P.queue[k];
+                const unsigned int vidx = (unsigned int)(e >> 32);
+                const int cell = (int)(e & 0xffffffffu);
+                const int i = cell / P.grid.n, j = cell - i * P.grid.n;
+                wp = P.gam + i * P.grid.W + (j >> 5);
+                bit = 1u << (j & 31);
+                test = !(ld_cg(wp) & bit);
+                if (test) {
+                    const float4 q = P.vox_main[vidx];
+                    const float* t = P.tab;
+                    const float cph = __ldg(t + i), sph = __ldg(t + P.grid.m + i);
+                    const float cg = __ldg(t + 2 * P.grid.m + j), sg = __ldg(t + 2 * P.grid.m + P.grid.n + j);
+                    hit = exact_hit(q.x - P.px, q.y - P.py, q.z - P.pz, q.w, sph * cg, sph * sg, cph, P.tool, sub, 4);
+                }
+            }
+            const unsigned int hm = __ballot_sync(0xffffffffu, hit);
+            if (sub == 0 && test) {
+                ++tests;
+                if ((hm >> lane) & 0xfu) {
+                    ++hits;
+                    atomicOr(wp, bit);
+                }
+            }
         }
     }
     if (tests) atomicAdd(P.stats + ST_EXACT, tests);

@@ -317,7 +317,7 @@ __device__ __forceinline__ void edge_vertices(int e, int& a, int& b) {
 }
 
 __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, float dx, float dy,
-                                       float dz, const ToolDev& T) {
+                                       float dz, const ToolDev& T, int c0 = 0, int cs = 1) {
     // frame: e1 = normalize(d x a), a = the world axis least aligned with d; e2 = d x e1
     const float adx = fabsf(dx), ady = fabsf(dy), adz = fabsf(dz);
     float e1x, e1y, e1z;
@@ -340,7 +340,7 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
         Y[k] = cY + sx * e2x + sy * e2y + sz * e2z;
         Z[k] = cZ + sx * dx + sy * dy + sz * dz;
     }
-    for (int c = 0; c < T.ncyl; ++c) {
+    for (int c = c0; c < T.ncyl; c += cs) {  // (cylinders c0, c0 + cs, ...: a lane's share of the OR)
         const float z0 = T.z0[c], z1 = T.z1[c], R = T.R[c], R2 = R * R;
         // (0) the axis segment crosses the box: slab test in world coordinates
         {
