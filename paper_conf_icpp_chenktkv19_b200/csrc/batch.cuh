@@ -28,7 +28,7 @@
 
 // CTAs per SM each stage is compiled for (register budget vs occupancy)
 #ifndef AM_LIVE_MIN_BLOCKS
-#define AM_LIVE_MIN_BLOCKS 6
+#define AM_LIVE_MIN_BLOCKS 5
 #endif
 #ifndef AM_LEVEL_ROWS_MIN_BLOCKS
 #define AM_LEVEL_ROWS_MIN_BLOCKS 8
