@@ -133,18 +133,21 @@ def cpu_oracle_sample(cfg, C, H, pivot, seconds=12.0, seed=0, max_cells=None):
     t0 = time.perf_counter()
     used = 0
     chunk = 8
+    states = []
     while True:
         cells = cells_all[done: done + chunk]
         if len(cells) == 0:
             break
-        _, used = oracle.am_states(C, H, cfg.tool, pivot, cfg.m, cfg.n, cells=cells, return_threads=True)
+        st, used = oracle.am_states(C, H, cfg.tool, pivot, cfg.m, cfg.n, cells=cells, return_threads=True)
+        states.append(np.asarray(st))
         done += len(cells)
         el = time.perf_counter() - t0
         if el >= seconds or (max_cells and done >= max_cells):
             break
         chunk = min(256, chunk * 2)
     el = time.perf_counter() - t0
-    return {"tests": float(len(H)) * done, "cells": done, "seconds": el, "threads": used}
+    return {"tests": float(len(H)) * done, "cells": done, "seconds": el, "threads": used,
+            "cell_ids": cells_all[:done], "states": np.concatenate(states) if states else np.zeros(0, np.int8)}
 
 
 def run_reference(args):
@@ -305,6 +308,7 @@ def run_ours(args):
     torch.cuda.synchronize(dev)
     kms, klaunch = ctx.kernel_time()
     kstats_timed = {k: v for k, v in ctx.kernel_stats().items() if v[1] > 0}  # launch counts of the timed region
+    timed_maps = out[:bsz].cpu().numpy().view(np.uint32).copy()  # the maps the timed steps produced
     # ---- the same K steps again with a CUDA event after every kernel launch
     #      (AM_OPT_KERNEL_TIMING = 2): per-kernel device times for `kernels` / `roofline`
     ctx.set_option(B.OPT_KERNEL_TIMING, 2)
@@ -384,11 +388,22 @@ def run_ours(args):
         stream.synchronize()
         baseline_ms = e0.elapsed_time(e1)
     cpu = None
+    parity = None
+    # blocked fraction of the maps the timed path produced (SURVEY 8(d) metrics)
+    blocked_frac = float(np.mean([am.unpack(timed_maps[k], cfg.m, cfg.n).mean() for k in range(len(timed_maps))]))
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         r = cpu_oracle_sample(cfg, C, H, piv[0], seconds=args.cpu_seconds)
         cpu = {"value": r["tests"] / r["seconds"], "unit": UNIT, "cores": r["threads"], "kind": "oracle",
                "sample": f"{r['cells']} seeded cells of one {cfg.name} map (pivot 0), every voxel per cell, "
                          f"{r['seconds']:.1f} s"}
+        # the same oracle cells against the timed path's own map of pivot 0 (north_star parity rule:
+        # zero mismatches on robust cells; band cells counted)
+        g0 = am.unpack(timed_maps[0], cfg.m, cfg.n).reshape(-1)
+        st = r["states"]
+        robust = st != 1
+        parity = {"pivot": 0, "cells": int(len(st)), "mismatches": int(((g0[r["cell_ids"]] == 1) != (st == 2))[robust].sum()),
+                  "band_cells": int((~robust).sum()), "oracle_blocked": int((st == 2).sum()),
+                  "source": "the cpu_baseline sample's fp64 oracle states vs the map the timed am_compute_batch produced"}
     if rank == 0:
         full_roof = None
         if full:
@@ -431,7 +446,9 @@ def run_ours(args):
                         for k, v in sorted(kstats.items(), key=lambda kv: -kv[1][0])},
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
+            "parity_sample": parity,
             "detail": {"stats_mean_over_pivots": mean, "upload_s": upload_s, "scene_gen_s": gen_s,
+                       "blocked_fraction_mean": blocked_frac,
                        "pivots_per_rank": len(piv), "baseline_ms_per_am": baseline_ms,
                        "single_pivot_ms_per_am": ms_single / ks,
                        "single_pivot_kernel_ms": ks_k / max(ks_l, 1),
