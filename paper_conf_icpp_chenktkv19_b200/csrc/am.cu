@@ -151,7 +151,9 @@ struct am_ctx {
     int slots = 1;                         // per-map buffer slots allocated (d_ctr ... d_brick_list)
     float4* d_piv = nullptr;               // batched launch: pivots (xyz, may_cull)
     long long piv_cap = 0;
-    std::vector<float4> h_piv;
+    float4* h_piv = nullptr;               // pinned staging of the batch's pivots (xyz, may_cull)
+    long long h_piv_cap = 0;
+    cudaEvent_t piv_ev = nullptr;          // the last pivot upload (the staging is reused after it)
     unsigned long long* d_bctl = nullptr;  // batched launch: group barriers, pivot queue
     int fused_grid = 0;
     size_t smem_fused = 0;
@@ -685,6 +687,27 @@ int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s)
     return AM_OK;
 }
 
+// The batch's pivots (xyz + may_cull) into ctx->d_piv, from pinned host staging
+// (the async copy of the previous call is waited for before the staging is rewritten).
+int upload_pivots(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* gam0, cudaStream_t s) {
+    if (!ctx->piv_ev) CK(cudaEventCreateWithFlags(&ctx->piv_ev, cudaEventDisableTiming));
+    CK(cudaEventSynchronize(ctx->piv_ev));
+    if (ctx->h_piv_cap < P) {
+        if (ctx->h_piv) cudaFreeHost(ctx->h_piv);
+        ctx->h_piv = nullptr;
+        ctx->h_piv_cap = 0;
+        CK(cudaMallocHost(&ctx->h_piv, (size_t)P * sizeof(float4)));
+        ctx->h_piv_cap = P;
+    }
+    for (int64_t k = 0; k < P; ++k) {
+        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
+        ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    }
+    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv, (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
+    CK(cudaEventRecord(ctx->piv_ev, s));
+    return AM_OK;
+}
+
 // P maps (pivots[3P]) into gam0 + k * MW with ONE fused launch: K groups of
 // CTAs (K <= ctx->slots) take pivots from a device queue (fused.cuh).
 int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint32_t* gam0, cudaStream_t s) {
@@ -696,12 +719,10 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
         ctx->piv_cap = P;
     }
     if (!ctx->d_bctl) CK(cudaMalloc(&ctx->d_bctl, kBctlWords * sizeof(unsigned long long)));
-    ctx->h_piv.resize((size_t)P);
-    for (int64_t k = 0; k < P; ++k) {
-        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
-        ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    {
+        int rc;
+        if ((rc = upload_pivots(ctx, pivots, P, gam0, s)) != AM_OK) return rc;
     }
-    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv.data(), (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
     CK(cudaMemsetAsync(ctx->d_bctl, 0, kBctlWords * sizeof(unsigned long long), s));
     FusedParams F = fused_params(ctx, pivots, gam0);
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
@@ -786,12 +807,10 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         CK(cudaMalloc(&ctx->d_piv, (size_t)P * sizeof(float4)));
         ctx->piv_cap = P;
     }
-    ctx->h_piv.resize((size_t)P);
-    for (int64_t k = 0; k < P; ++k) {
-        const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
-        ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
+    {
+        int rc;
+        if ((rc = upload_pivots(ctx, pivots, P, gam0, s)) != AM_OK) return rc;
     }
-    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv.data(), (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
     const size_t sm_rows = (size_t)(ctx->MW + ((ctx->grid.m + 31) >> 5) + 1) * sizeof(uint32_t);
     // one chunk of kk pivots from c0 on, slots [sb, sb + kk), on stream s
@@ -1867,6 +1886,8 @@ void am_destroy(am_ctx* ctx) {
     cudaSetDevice(ctx->device);
     if (ctx->g_exec) cudaGraphExecDestroy(ctx->g_exec);
     if (ctx->cap_s) cudaStreamDestroy(ctx->cap_s);
+    if (ctx->piv_ev) cudaEventDestroy(ctx->piv_ev);
+    if (ctx->h_piv) cudaFreeHost(ctx->h_piv);
     for (int l = 0; l < kMaxLanes; ++l)
         if (ctx->lane_s[l]) cudaStreamDestroy(ctx->lane_s[l]);
     for (int l = 0; l <= kMaxLanes; ++l)
