@@ -45,6 +45,9 @@ constexpr int kMaxLanes = 8;
 #ifndef AM_L1_STEPS
 #define AM_L1_STEPS 8  // level-1 cone steps (256 voxels each) per CTA of the batched path
 #endif
+#ifndef AM_BRICKS_CTAS
+#define AM_BRICKS_CTAS 16  // per pivot, brick launch after the super-brick test (entries = 8 x kept supers)
+#endif
 #ifndef AM_BRICK_STEPS
 #define AM_BRICK_STEPS 4  // brick-test steps (256 bricks each) per CTA of the batched path
 #endif
@@ -875,7 +878,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             if ((rc = L(bk_supers, grid((ctx->nbricks + 7) / 8, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
             AM_KM(AM_K_BRICKS);
         }
-        if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
+        if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, F.main.supers ? AM_BRICKS_CTAS : (1 << 16)), 0))) return rc;
         AM_KM(AM_K_BRICKS);
         if ((rc = L(bk_voxels, grid(1 << 30, 1, ctx->bk_voxel_ctas), 0))) return rc;
         AM_KM(AM_K_VOXELS);
