@@ -5,12 +5,13 @@
 // map keeps the GPU busy only in bursts, and the fused kernel's register
 // budget (the heaviest phase sets it for all) caps occupancy at 16 warps/SM.
 // For a toolpath batch the same phases run here as
-// separate kernels over ALL pivots of the batch at once: blockIdx.y is the
-// pivot, each pivot owns slot blockIdx.y of every per-map buffer (the slot-0
-// pointers of FusedParams advanced by the slot strides), and each kernel gets
-// the registers -- and so the occupancy -- its own phase needs.  Kernel
-// boundaries replace the grid barriers, and the block scheduler balances
-// pivots of different cost.
+// separate kernels over a chunk of pivots at once: blockIdx.y is the pivot,
+// each pivot owns slot blockIdx.y of every per-map buffer (the slot-0 pointers
+// of FusedParams advanced by the slot strides; am.cu shifts them per stream
+// lane), and each kernel gets the registers -- and so the occupancy -- its
+// own phase needs.  Kernel boundaries replace the grid barriers, and the
+// block scheduler balances pivots of different cost.  The host runs the
+// chunks on several streams and replays the whole chain as a CUDA graph.
 //
 // Phases (same device functions as fused.cuh, so the maps are bit-identical):
 //   bk_cones<L0>  level-0 inner cones        -> stage-0 records/tasks
@@ -18,8 +19,9 @@
 //   bk_map        clear-direction map
 //   bk_cones<L1>  level-1 filter + cones     -> stage-1 records/tasks
 //   bk_rows<1>, bk_map
-//   bk_bricks     brick test                 -> kept bricks
-//   bk_voxels     kept bricks' voxels filter -> live list
+//   bk_supers     super-brick test           -> kept super-bricks
+//   bk_bricks     their bricks, then the kept bricks' sub-bricks -> kept sub-bricks
+//   bk_voxels     kept sub-bricks' voxels filter -> live list
 //   bk_cones<LIVE> both cones of live voxels -> stage-2 records/tasks
 //   bk_rows<2>    rows + band queue
 //   bk_band       exact test of queued band pairs still clear
