@@ -117,13 +117,13 @@ struct am_ctx {
     unsigned long long* d_tasks = nullptr;
     long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
     float4* d_texels = nullptr;            // cube-map texel centres (xyz) + angular radius (w)
-    float* d_cmap = nullptr;
-    float* d_cmap_ones = nullptr;          // the all-clear map (no voxel can be dropped)
+    float4* d_cmap = nullptr;              // per slot: per texel (cos, sin of the nearest-clear angle, U_t |U_t|, 0)
+    float4* d_cmap_ones = nullptr;         // the all-clear map (no voxel can be dropped): (1, 0, 1, 0)
     uint32_t* d_prev = nullptr;            // diagnostics: copy of the last map
     unsigned long long* d_ts = nullptr;    // diagnostics: fused-phase timestamps
     int diag = 0;
     int diag_ts = 0;
-    int cmapT = 160;
+    int cmapT = 112;
     int cmapT1 = AM_CMAP_T1;               // map after level 0 (AM_OPT_CMAP_T1, <= cmapT)
     float4* d_texels1 = nullptr;
     int phases = 2;
@@ -259,6 +259,7 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.vox_main = c->d_vox;
     p.vox_coarse = c->d_coarse;
     p.cmapT = c->cmapT;
+    p.cmap_tex = c->d_texels;
     p.cull_dist = c->tool.rho_max * (1.f + 1e-5f) + 1e-6f;
     p.band_vdepth = c->band_vdepth;
     // the reach cull can only fire when some voxel centre lies farther than
@@ -402,7 +403,7 @@ int ensure_slots(am_ctx* ctx, int K) {
     CK(cudaMalloc(&ctx->d_queue, (size_t)K * ctx->qcap * sizeof(unsigned long long)));
     CK(cudaMalloc(&ctx->d_recs, (size_t)K * kRecCap * sizeof(ConeRec)));
     CK(cudaMalloc(&ctx->d_tasks, (size_t)K * kTaskCap * sizeof(unsigned long long)));
-    CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float)));
+    CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float4)));
     if (ctx->vox_cap > 0) CK(cudaMalloc(&ctx->d_live, (size_t)K * ctx->vox_cap * sizeof(unsigned int)));
     if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * blist_words(ctx) * sizeof(unsigned int)));
     return AM_OK;
@@ -483,7 +484,7 @@ int launch_cones_rows(am_ctx* ctx, StreamParams p, bool coarse, int stage, cudaS
 }
 
 // The full voxel stream over vox[0, n) with clear-direction map `cmap`.
-int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, bool timed,
+int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float4* cmap, bool timed,
                   cudaStream_t s, bool coarse = false) {
     if (n <= 0) return AM_OK;
     p.vox = vox;
@@ -533,7 +534,7 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
 }
 
 // A coarse level: inner cones of every voxel of vox[0, n) (no filter).
-int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float* cmap, int stage,
+int launch_coarse(am_ctx* ctx, StreamParams p, const float4* vox, long long n, const float4* cmap, int stage,
                   cudaStream_t s) {
     if (n <= 0) return AM_OK;
     p.vox = vox;
@@ -735,7 +736,7 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
     F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
     F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
-    F.cmap_stride = (unsigned long long)ntex * sizeof(float);
+    F.cmap_stride = (unsigned long long)ntex * sizeof(float4);
     F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
     F.piv = ctx->d_piv;
     F.npiv = (unsigned int)P;
@@ -829,7 +830,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
         F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
         F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
-        F.cmap_stride = (unsigned long long)ntex * sizeof(float);
+        F.cmap_stride = (unsigned long long)ntex * sizeof(float4);
         F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
         F.piv = ctx->d_piv + c0;
         F.npiv = (unsigned int)kk;
@@ -970,7 +971,7 @@ int launch_aica(am_ctx* ctx, const float pivot[3], uint32_t* gam, cudaStream_t s
     StreamParams p = make_params(ctx, pivot, gam);
     int rc;
     if ((rc = kchain(ctx, s))) return rc;
-    const float* cm = ctx->d_cmap_ones;
+    const float4* cm = ctx->d_cmap_ones;
     if (ctx->diag & 2) {
         // diagnostic: clear map from the previous map computed on this context
         // (exact only when the previous call used the same pivot)
@@ -1145,16 +1146,16 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         const std::vector<float> tex = make_texels(ctx->cmapT);
         if (cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)) != cudaSuccess ||
             cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMalloc(&ctx->d_cmap, tex.size() / 4 * sizeof(float)) != cudaSuccess ||
-            cudaMalloc(&ctx->d_cmap_ones, tex.size() / 4 * sizeof(float)) != cudaSuccess) {
+            cudaMalloc(&ctx->d_cmap, tex.size() / 4 * sizeof(float4)) != cudaSuccess ||
+            cudaMalloc(&ctx->d_cmap_ones, tex.size() / 4 * sizeof(float4)) != cudaSuccess) {
             cudaGetLastError();
             return bail(AM_ENOMEM);
         }
     }
     if (set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT)) != AM_OK) return bail(AM_ENOMEM);
     {
-        const std::vector<float> ones((size_t)6 * ctx->cmapT * ctx->cmapT, 1.0f);
-        if (cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice) !=
+        const std::vector<float4> ones((size_t)6 * ctx->cmapT * ctx->cmapT, make_float4(1.f, 0.f, 1.f, 0.f));
+        if (cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float4), cudaMemcpyHostToDevice) !=
             cudaSuccess) {
             cudaGetLastError();
             return bail(AM_ECUDA);
@@ -1578,7 +1579,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
         {
             const std::vector<float> tex = make_texels((int)value);
-            const std::vector<float> ones(tex.size() / 4, 1.0f);
+            const std::vector<float4> ones(tex.size() / 4, make_float4(1.f, 0.f, 1.f, 0.f));
             cudaFree(ctx->d_texels);
             cudaFree(ctx->d_cmap);
             cudaFree(ctx->d_cmap_ones);
@@ -1586,9 +1587,9 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
             ctx->d_cmap = ctx->d_cmap_ones = nullptr;
             CK(cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)));
             CK(cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
-            CK(cudaMalloc(&ctx->d_cmap, (size_t)ctx->slots * ones.size() * sizeof(float)));
-            CK(cudaMalloc(&ctx->d_cmap_ones, ones.size() * sizeof(float)));
-            CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float), cudaMemcpyHostToDevice));
+            CK(cudaMalloc(&ctx->d_cmap, (size_t)ctx->slots * ones.size() * sizeof(float4)));
+            CK(cudaMalloc(&ctx->d_cmap_ones, ones.size() * sizeof(float4)));
+            CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float4), cudaMemcpyHostToDevice));
             ctx->cmapT = (int)value;
         }
         return set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT));

@@ -117,8 +117,8 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
                 nrows = cone_of_voxel<true>(P, P.vox[e], (unsigned int)e, r, counted);
             } else if (STAGE == BK_L1) {
                 const float4 q = F.l1[e];
-                if (fast_filter(P, q, P.gam, F.cmapT1) == F_LIVE)
-                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1);
+                if (fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
+                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1, nullptr, F.texels1);
             } else {
                 const unsigned int vidx = P.live_idx[e];
                 nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear, 0, sRowStart);
@@ -186,7 +186,7 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
     float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
     clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
-                  const_cast<float*>(P.cmap), sAM, sDirs, &sN, blockIdx.x,
+                  const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x,
                   gridDim.x);
 }
 

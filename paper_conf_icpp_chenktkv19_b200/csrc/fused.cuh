@@ -466,7 +466,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     if (!BATCH || gb == 0) fused_mark(F, 2);
     // 3. clear-direction map (at cmapT1 texels per face when level 1 follows: it only filters level 1)
     clear_map_cta(P.gam, P.grid, P.tab, F.use_l1 ? F.texels1 : F.texels, F.use_l1 ? F.cmapT1 : P.cmapT,
-                  const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
+                  const_cast<float4*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 3);
     if (F.use_l1) {
@@ -480,8 +480,8 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             ConeRec r;
             if (e < F.n1) {
                 const float4 q = F.l1[e];
-                if (fast_filter(P, q, P.gam, F.cmapT1) == F_LIVE)
-                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1);
+                if (fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
+                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1, nullptr, F.texels1);
             }
             emit_cones_cta<true>(P, rec1, task1, P.rec_cap / 2, P.task_cap / 2, P.rec_cap, P.task_cap, nrows, r,
                                  counted, &sc, nullptr, sRowFull);
@@ -507,7 +507,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
         gsync();
         if (!BATCH || gb == 0) fused_mark(F, 5);
         // 6. clear-direction map again
-        clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
+        clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float4*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
         gsync();
         if (!BATCH || gb == 0) fused_mark(F, 6);
     }

@@ -50,8 +50,10 @@ struct StreamParams {
     const float4* __restrict__ vox_coarse;
     unsigned int vtag;             // OR-ed into queued indices by this launch
     unsigned int vbase;            // index of vox[0] within its array
-    // clear-direction map; nullptr = not yet built
-    const float* __restrict__ cmap;
+    // clear-direction map: per texel (cos, sin) of the angle from
+    // its centre to the nearest cell still clear, rounded down; the texel centres of that map
+    const float4* __restrict__ cmap;
+    const float4* __restrict__ cmap_tex;
     int cmapT;                     // texels per cube-face side
     float cull_dist;               // rho_max, grown by the fp32 guard (reach cull)
     int tile;                      // voxels per tile of this launch (<= kTile, multiple of 4)
@@ -194,22 +196,17 @@ __device__ __forceinline__ float dot3(float4 a, float4 b) { return fmaf(a.x, b.x
 
 // V_t from the best cosine of texel (c, r): the nearest-cell angle rounded
 // down and the bound rounded up (fp32 guards).
-__device__ __forceinline__ float clear_map_value(float best, float r) {
-    float u = -2.f;
-    if (best >= -1.5f) {
-        // cos(max(0, th - r)) with cos th = b, without acos/cos: b cos r + sin th sin r
-        // (sin th = sqrt((1 - b)(1 + b)) >= 0); the error of the fast sin/cos and of
-        // the square root (< 1e-6 here: sin th is multiplied by sin r) is inside the guard
-        const float b = fminf(best + 2e-6f, 1.f);
-        const float cr = __cosf(r), sr = __sinf(r);
-        if (b >= cr) {
-            u = 1.f;
-        } else {
-            const float st = sqrtf(fmaxf((1.f - b) * (1.f + b), 0.f));
-            u = fminf(fmaf(b, cr, st * sr) + 4e-6f, 1.f);
-        }
-    }
-    return u * fabsf(u);
+__device__ __forceinline__ float4 clear_map_value(float best, float r) {
+    // (cos theta, sin theta, U_t |U_t|, 0): theta = the texel centre's nearest-clear angle, cos
+    // rounded up (theta down); U_t = cos(max(0, theta - r)) bounds every direction of the texel
+    // (r = its radius), evaluated as b cos r + sin theta sin r without acos/cos (the fast sin/cos
+    // and square-root errors, < 1e-6, are inside the guard).  No clear cell: (-2, 0, -4, 0).
+    if (best < -1.5f) return make_float4(-2.f, 0.f, -4.f, 0.f);
+    const float b = fminf(best + 2e-6f, 1.f);
+    const float st = sqrtf(fmaxf((1.f - b) * (1.f + b), 0.f));
+    const float cr = __cosf(r), sr = __sinf(r);
+    const float u = (b >= cr) ? 1.f : fminf(fmaf(b, cr, st * sr) + 4e-6f, 1.f);
+    return make_float4(b, st, u * fabsf(u), 0.f);
 }
 
 // Compact the directions of the clear cells of words [w0, w1) of sAM into
@@ -407,7 +404,7 @@ __device__ int clear_list_rows_cta(const uint32_t* sAM, const GridDev& g, const 
 // within theta_C + 2 rho of c (triangle inequality), so only those candidates
 // (found by one ballot pass over the list) are tried per texel.  c and
 // cos / sin(2 rho + slack) come from the host-made block table after the texels.
-__device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float* __restrict__ V,
+__device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float4* __restrict__ V,
                                  const float4* sDirs, int total, int w0, int wstride) {
     constexpr int B = 8, TPL = B * B / 32, ROWS = 32 / B;
     const int lane = threadIdx.x & 31;
@@ -459,7 +456,7 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
 // gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
 // (kMapDirs), sN.
 __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
-                              const float4* __restrict__ texels, int T, float* __restrict__ V, uint32_t* sAM,
+                              const float4* __restrict__ texels, int T, float4* __restrict__ V, uint32_t* sAM,
                               float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
     const int MW = g.m * g.W;
     const int ntex = 6 * T * T;
@@ -594,7 +591,7 @@ __host__ __device__ inline size_t clear_map_smem_bytes(int MW) {
 __global__ void __launch_bounds__(256) clear_map_kernel(const uint32_t* __restrict__ gam, GridDev g,
                                                         const float* __restrict__ tab,
                                                         const float4* __restrict__ texels, int T,
-                                                        float* __restrict__ V) {
+                                                        float4* __restrict__ V) {
     extern __shared__ __align__(16) unsigned char smem_cm[];
     __shared__ int sN;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_cm);

@@ -47,6 +47,34 @@ enum { F_DROP = 0, F_LIVE = 1, F_CULLED = 2 };
 
 __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T);
 
+// Can a sphere / voxel whose blocked directions all satisfy U |U| >= thr (thr = the squared-sign
+// cosine of its cheap or exact outer cone) be dropped, from the clear-direction map (m, texel
+// centres tex, T per side)?  First the texel-wide bound U_t (as every direction of the texel);
+// when that keeps it, the bound for v itself: with theta' = the stored (rounded-down) nearest-clear
+// angle of the texel centre c and a = angle(v, c), every cell still clear is at least theta' - a
+// from v (triangle inequality, for ANY texel), so U = cos(max(0, theta' - a)) = cos theta' cos a +
+// sin theta' sin a (a < theta'), guarded.  sin a from |v x c| (accurate for small a).
+#ifndef AM_SPHERE_REFINE
+#define AM_SPHERE_REFINE true  // brick / sub-brick spheres too (false: the texel-wide bound only)
+#endif
+template <bool REFINE = true>
+__device__ __forceinline__ bool cmap_drop(const float4* __restrict__ m, const float4* __restrict__ tex, int T,
+                                          float vx, float vy, float vz, float thr) {
+    const int t = texel_of(vx, vy, vz, T);
+    const float4 cs = __ldg(m + t);
+    if (cs.z < thr) return true;
+    if (!REFINE) return false;
+    if (cs.y == 0.f) return false;  // theta' = 0 (a clear cell at the texel centre): U = 1
+    const float4 c = __ldg(tex + t);
+    const float inv = rsqrtf(fmaf(vx, vx, fmaf(vy, vy, vz * vz)));
+    const float ca = fmaf(vx, c.x, fmaf(vy, c.y, vz * c.z)) * inv;
+    if (ca <= cs.x) return false;  // a >= theta': U = 1
+    const float x = fmaf(vy, c.z, -vz * c.y), y = fmaf(vz, c.x, -vx * c.z), z = fmaf(vx, c.y, -vy * c.x);
+    const float sa = sqrtf(fmaf(x, x, fmaf(y, y, z * z))) * inv;
+    const float u = fminf(fmaf(cs.x, ca, cs.y * sa) + 4e-6f, 1.f);
+    return u * fabsf(u) < thr;
+}
+
 // a2 + cheap cone vs clear-direction map (p.cmap is never null: before any map
 // is built it is the all-clear map).  The map stores V = U |U|, where U bounds
 // from above the cosine of the angle from any direction of the texel to the
@@ -55,7 +83,8 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T);
 // F_DROP otherwise.  A voxel holding the pivot blocks every orientation: it
 // fills `am` (shared or global) directly.
 // T: texels per face of the clear-direction map in p.cmap (0 = p.cmapT).
-__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am, int T = 0) {
+__device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint32_t* am, int T = 0,
+                                           const float4* tex = nullptr) {
     const float vx = q.x - p.px, vy = q.y - p.py, vz = q.z - p.pz, h = q.w;
     const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
     const float r2 = kSqrt3 * h;
@@ -77,7 +106,7 @@ __device__ __forceinline__ int fast_filter(const StreamParams& p, float4 q, uint
     const float s = fmaf((Reff + r2) * invD, 1.f + 1.6e-5f, 1e-6f);
     const float c = fmaf(r2 * invD, 1.f + 1.6e-5f, 1e-6f);
     const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
-    return __ldg(p.cmap + texel_of(vx, vy, vz, T ? T : p.cmapT)) < thr ? F_DROP : F_LIVE;
+    return cmap_drop(p.cmap, T ? tex : p.cmap_tex, T ? T : p.cmapT, vx, vy, vz, thr) ? F_DROP : F_LIVE;
 }
 
 // Cube-map texel of v (cube_texel of kernels.cuh with an approximate
@@ -172,7 +201,7 @@ __device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, 
     const float s = fmaf((Reff + r) * invD, 1.f + 1.6e-5f, 1e-6f);
     const float c = fmaf(r * invD, 1.f + 1.6e-5f, 1e-6f);
     const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
-    return __ldg(p.cmap + texel_of(vx, vy, vz, p.cmapT)) < thr;
+    return cmap_drop<AM_SPHERE_REFINE>(p.cmap, p.cmap_tex, p.cmapT, vx, vy, vz, thr);
 }
 
 // Full stream with brick culling (the paper's octree
@@ -313,7 +342,8 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
 template <bool COARSE>
 __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, unsigned int vidx, ConeRec& r,
                                              bool& counted, const float4* clear = nullptr, int nclear = -1,
-                                             int cmT = 0, const int* rowStart = nullptr) {
+                                             int cmT = 0, const int* rowStart = nullptr,
+                                             const float4* cmTex = nullptr) {
     const ToolDev& T = p.tool;
     const GridDev& g = p.grid;
     counted = false;
@@ -333,7 +363,9 @@ __device__ __forceinline__ int cone_of_voxel(const StreamParams& p, float4 q, un
     }
     // the exact outer cone against the clear-direction map: no clear cell
     // within it means this voxel cannot change the map
-    if (c.cout > 1.f || __ldg(p.cmap + texel_of(vx, vy, vz, cmT ? cmT : p.cmapT)) < c.cout * fabsf(c.cout)) return 0;
+    if (c.cout > 1.f || cmap_drop(p.cmap, cmT ? cmTex : p.cmap_tex, cmT ? cmT : p.cmapT, vx, vy, vz,
+                                  c.cout * fabsf(c.cout)))
+        return 0;
     const float rxy = sqrtf(vx * vx + vy * vy);
     const float phv = atan2f(rxy, vz);
     const float ao = acosf(fmaxf(c.cout, -1.f));
