@@ -123,7 +123,7 @@ struct am_ctx {
     unsigned long long* d_ts = nullptr;    // diagnostics: fused-phase timestamps
     int diag = 0;
     int diag_ts = 0;
-    int cmapT = 112;
+    int cmapT = 96;
     int cmapT1 = AM_CMAP_T1;               // map after level 0 (AM_OPT_CMAP_T1, <= cmapT)
     float4* d_texels1 = nullptr;
     int phases = 2;
