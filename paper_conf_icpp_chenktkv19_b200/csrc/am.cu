@@ -28,7 +28,8 @@
 using namespace am;
 
 // coarse-level sizes (upload): level 0 = the N / AM_L0_DIV largest voxels,
-// level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel
+// level 1 = the next up to N / AM_L1_DIV plus every AM_L1_STRIDE-th voxel (a sample of at
+// least AM_L1_MIN_SAMPLE voxels: small models, tools/ab.sh on C2)
 #ifndef AM_ROWS_CTAS
 #define AM_ROWS_CTAS 64
 #endif
@@ -83,6 +84,9 @@ constexpr int kMaxLanes = 8;
 #endif
 #ifndef AM_L1_STRIDE
 #define AM_L1_STRIDE 384
+#endif
+#ifndef AM_L1_MIN_SAMPLE
+#define AM_L1_MIN_SAMPLE 24576
 #endif
 
 struct am_ctx {
@@ -1320,7 +1324,10 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     if (N >= 2048) {
         const long long n0 = std::min<long long>(N, std::max<long long>(1024, N / AM_L0_DIV));
         const long long n1 = std::min<long long>(N, std::max<long long>(8192, N / AM_L1_DIV));
-        const long long stride = AM_L1_STRIDE, ns = N / stride;
+        // strided sample: every AM_L1_STRIDE-th voxel, at least AM_L1_MIN_SAMPLE voxels (small models)
+        long long stride = AM_L1_STRIDE;
+        if (N / stride < AM_L1_MIN_SAMPLE) stride = std::max<long long>(1, N / AM_L1_MIN_SAMPLE);
+        const long long ns = std::min<long long>(N / stride, N - n1);  // level 1 fits the live lists (N)
         unsigned int *sk = nullptr, *sk2 = nullptr, *si = nullptr, *si2 = nullptr, *cid = nullptr;
         void* ct = nullptr;
         auto cfree = [&]() {
