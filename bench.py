@@ -261,6 +261,8 @@ def run_ours(args):
         ctx.set_option(B.OPT_CMAP_T, args.cmap_t)
     if args.cmap_t1:
         ctx.set_option(B.OPT_CMAP_T1, args.cmap_t1)
+    if args.l1_sample:
+        ctx.set_option(B.OPT_L1_SAMPLE, args.l1_sample)
     if args.cmap_rowscan >= 0:
         ctx.set_option(B.OPT_CMAP_ROWSCAN, args.cmap_rowscan)
     if args.cmap_brute >= 0:
@@ -548,6 +550,7 @@ def main():
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps")
     ap.add_argument("--cmap-t", type=int, default=0, help="AM_OPT_CMAP_T (0 = library default)")
     ap.add_argument("--cmap-t1", type=int, default=0, help="AM_OPT_CMAP_T1 (0 = library default)")
+    ap.add_argument("--l1-sample", type=int, default=0, help="AM_OPT_L1_SAMPLE (0 = library default)")
     ap.add_argument("--cmap-rowscan", type=int, default=-1, help="AM_OPT_CMAP_ROWSCAN (-1 = library default)")
     ap.add_argument("--cmap-brute", type=int, default=-1, help="AM_OPT_CMAP_BRUTE (-1 = library default)")
     ap.add_argument("--cmap-block", type=int, default=0, help="AM_OPT_CMAP_BLOCK (0 = library default)")

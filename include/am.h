@@ -134,10 +134,15 @@ enum {
                                     joined to the caller's stream), so one chunk's short phases
                                     overlap another's (1..8, default 8; 1 while
                                     AM_OPT_KERNEL_TIMING = 2).  Same maps                       */
-    AM_OPT_GRAPH = 21            /* am_compute_batch: 1 = capture the batch's launch chain as a
+    AM_OPT_GRAPH = 21,           /* am_compute_batch: 1 = capture the batch's launch chain as a
                                     CUDA graph and replay it while the options, the pivot count,
                                     the output buffer and the model are unchanged (default);
                                     0 = launch every kernel from the host.  Same maps           */
+    AM_OPT_L1_SAMPLE = 22        /* coarse level 1's strided sample of the model, in voxels, taken
+                                    at the NEXT am_upload_voxels (0..2^31-1; 0 = library default:
+                                    every 384th voxel, at least 24,576).  Only the culling
+                                    changes (scene-dependent best: profiles/r2x_level_sizes.txt).
+                                    Same maps                                                   */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

@@ -128,6 +128,7 @@ struct am_ctx {
     int diag = 0;
     int diag_ts = 0;
     int cmapT = 96;
+    long long l1_sample = 0;               // AM_OPT_L1_SAMPLE (0 = N / AM_L1_STRIDE, >= AM_L1_MIN_SAMPLE)
     int cmapT1 = AM_CMAP_T1;               // map after level 0 (AM_OPT_CMAP_T1, <= cmapT)
     float4* d_texels1 = nullptr;
     int phases = 2;
@@ -1327,6 +1328,7 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
         // strided sample: every AM_L1_STRIDE-th voxel, at least AM_L1_MIN_SAMPLE voxels (small models)
         long long stride = AM_L1_STRIDE;
         if (N / stride < AM_L1_MIN_SAMPLE) stride = std::max<long long>(1, N / AM_L1_MIN_SAMPLE);
+        if (ctx->l1_sample > 0) stride = std::max<long long>(1, N / ctx->l1_sample);  // AM_OPT_L1_SAMPLE
         const long long ns = std::min<long long>(N / stride, N - n1);  // level 1 fits the live lists (N)
         unsigned int *sk = nullptr, *sk2 = nullptr, *si = nullptr, *si2 = nullptr, *cid = nullptr;
         void* ct = nullptr;
@@ -1578,6 +1580,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_BATCH_LANES:
         if (value < 1 || value > kMaxLanes) return fail(ctx, AM_EINVAL, "batch_lanes must be in [1, %d]", kMaxLanes);
         ctx->lanes = (int)value;
+        return AM_OK;
+    case AM_OPT_L1_SAMPLE:
+        if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "l1_sample must be in [0, 2^31-1]");
+        ctx->l1_sample = value;  // taken at the next am_upload_voxels
         return AM_OK;
     case AM_OPT_CMAP_T1:
         if (value < 4 || value > ctx->cmapT) return fail(ctx, AM_EINVAL, "cmap_T1 must be in [4, cmap_T]");

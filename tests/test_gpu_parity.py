@@ -308,6 +308,29 @@ def test_batched_launch_matches_single_maps(am, batch, diag):
     ctx.close()
 
 
+@pytest.mark.gpu
+def test_l1_sample_option_same_maps(am):
+    """AM_OPT_L1_SAMPLE only resizes coarse level 1 (culling): the maps stay bit-identical,
+    from a 1-voxel sample to the whole model, and the option takes effect at the next upload."""
+    cfg = scenes.CONFIGS["C2"]
+    C, H = cfg.leaves()
+    P = cfg.pivots(9)
+    ctx = _ctx(am, cfg, C, H)
+    ref = ctx.compute_batch(P)
+    base_levels = ctx.compute(P[0], stats=True)[1].level_voxels
+    for sample in (1, 5000, 100000, len(H), 0):
+        ctx.set_option(am.binding.OPT_L1_SAMPLE, sample)
+        ctx.upload(C, H)
+        assert np.array_equal(ctx.compute_batch(P), ref), sample
+        lv = ctx.compute(P[0], stats=True)[1].level_voxels
+        assert 0 < lv <= len(H), (sample, lv)
+        if sample == 0:
+            assert lv == base_levels
+    with pytest.raises(Exception):
+        ctx.set_option(am.binding.OPT_L1_SAMPLE, -1)
+    ctx.close()
+
+
 def test_batch_graph_replay(am):
     """The batch launch chain replayed as a CUDA graph (AM_OPT_GRAPH): replays with new
     pivots into the same device buffer, a new buffer, host outputs and an option change
