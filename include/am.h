@@ -92,7 +92,7 @@ enum {
                                     of the coarse levels (a lower-bound probe of the filter; the
                                     result is exact only when that map had the same pivot)       */
     AM_OPT_CMAP_T = 9,           /* clear-direction map resolution: texels per cube-face side
-                                    (4..256, default 96)                                         */
+                                    (4..256, default 96; 80 when m·n >= 128·128)                 */
     AM_OPT_BRICKS = 10,          /* 1 = skip whole 256-voxel bricks whose bounding sphere reaches
                                     no clear cell (default); 0 = read every voxel.  Same map     */
     AM_OPT_FUSED = 11,           /* 1 = the whole map in one persistent cooperative launch when

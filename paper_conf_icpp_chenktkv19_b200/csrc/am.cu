@@ -1147,6 +1147,9 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
         return bail(AM_ENOMEM);
     }
     ctx->am_cap_maps = 1;
+    // finer orientation grids (C4, 128 x 128) are faster with a coarser default map (B200 sweep,
+    // profiles/r2v_sweep.txt: 12.50 -> 12.28 us per map at T = 80)
+    if ((long long)m * n >= 128ll * 128) ctx->cmapT = 80;
     {
         const std::vector<float> tex = make_texels(ctx->cmapT);
         if (cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)) != cudaSuccess ||
