@@ -29,9 +29,14 @@
  * Ownership: the library copies whatever it is given; caller buffers are never
  * retained.  Errors: every int-returning call returns AM_OK (0) or a negative
  * AM_E* code, and am_last_error() describes the last failure on that context.
- * Threading: calls on one context are not thread-safe; use one context per
- * device (per rank).  No call falls back to the CPU: a missing or failing GPU
- * is reported as AM_ECUDA.
+ * Threading and streams: calls on one context are not thread-safe; use one
+ * context per device (per rank).  Asynchronous calls share the context's
+ * scratch (per-map slots, staged pivots), so a compute call issued on another
+ * stream than the previous compute call first waits (on the device) for that
+ * call to finish; calls on one stream are ordered by the stream.  No call falls
+ * back to the CPU: a missing or failing GPU is reported as AM_ECUDA.
+ * Allocation failures (AM_ENOMEM) leave the context usable as it was: e.g. a
+ * batch whose AM_OPT_BATCH slots do not fit can be retried with fewer.
  */
 #ifndef AM_H_
 #define AM_H_
@@ -61,9 +66,12 @@ typedef struct {
     int64_t exact_tests;       /* exact cylinder-box tests actually run (CHECKBOX, L97)         */
     int64_t exact_hits;        /* of which collided                                             */
     int64_t queue_overflow;    /* band pairs resolved inline because the queue was full         */
-    int64_t early_exit;        /* 1 if the AM filled up and the stream stopped early (a7)       */
+    int64_t early_exit;        /* 1 if the AM filled up before the full stream, which then read
+                                  no voxel (a7: "stop when popcount(AM) = m n")               */
     int64_t bricks_kept;       /* 256-voxel bricks whose voxels were read (AM_OPT_BRICKS)       */
     int64_t level_voxels;      /* voxels of the clear-map levels (read once more per map)       */
+    int64_t rows_skipped_full; /* (live voxel, phi-row) pairs of the full stream skipped because
+                                  the row was already full (a5: "rows already full are skipped") */
 } am_stats;
 
 enum {
@@ -140,7 +148,9 @@ enum {
                                     0 = launch every kernel from the host.  Same maps           */
     AM_OPT_L1_SAMPLE = 22        /* coarse level 1's strided sample of the model, in voxels, taken
                                     at the NEXT am_upload_voxels (0..2^31-1; 0 = library default:
-                                    every 384th voxel, at least 24,576).  Only the culling
+                                    every 384th voxel, at least 24,576).  Approximate: every
+                                    floor(N / sample)-th voxel is taken, so the realised sample is
+                                    between sample and 2 sample - 1 voxels.  Only the culling
                                     changes (scene-dependent best: profiles/r2x_level_sizes.txt).
                                     Same maps                                                   */
 };
@@ -164,6 +174,7 @@ enum {
     AM_K_LAYOUT,        /* am_unpack_cells / am_pack_cells                                     */
     AM_K_ICA_MEMO,      /* am_compute_octree: parallel ICA calculation of the top S levels     */
     AM_K_OCTREE,        /* am_compute_octree: one thread per orientation, Alg. 2               */
+    AM_K_INIT,          /* batched path: zero a chunk's maps and per-map counters              */
     AM_K_COUNT
 };
 
@@ -181,7 +192,8 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
  * (src_is_device = 0) or on `device` (1).  Replaces any previous model.  The
  * library may reorder voxels (Morton sort); the AM is order-independent.
  * AM_EINVAL if N < 0, a pointer is NULL while N > 0, or any value is non-finite
- * or a half size is <= 0.  N = 0 is legal (every AM is then all-zero).
+ * or a half size is <= 0.  N = 0 is legal (every AM is then all-zero).  A failed
+ * upload leaves no model: compute calls return AM_ESTATE until an upload succeeds.
  * Synchronous: returns after the model is resident (upload time is excluded
  * from AM timings).
  */

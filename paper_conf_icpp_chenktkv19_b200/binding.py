@@ -21,7 +21,7 @@ LIB_PATH = os.environ.get("AM_LIBRARY") or os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
-K_COUNT = 16  # AM_K_COUNT (include/am.h)
+K_COUNT = 17  # AM_K_COUNT (include/am.h)
 SCHEME_PBOX, SCHEME_PBOX_AABB, SCHEME_PICA, SCHEME_MICA, SCHEME_AICA = 0, 1, 2, 3, 4  # AM_SCHEME_*
 SCHEMES = {"pbox": 0, "pbox_aabb": 1, "pica": 2, "mica": 3, "aica": 4}
 OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
@@ -47,7 +47,7 @@ class _Stats(ctypes.Structure):
     _fields_ = [(k, ctypes.c_int64) for k in (
         "voxels_streamed", "voxels_culled", "voxels_skipped", "voxels_live", "rows_rasterised",
         "band_pairs", "exact_tests", "exact_hits", "queue_overflow", "early_exit", "bricks_kept",
-        "level_voxels")]
+        "level_voxels", "rows_skipped_full")]
 
 
 @dataclass
@@ -64,6 +64,7 @@ class Stats:
     early_exit: int
     bricks_kept: int
     level_voxels: int
+    rows_skipped_full: int
 
 
 lib = ctypes.CDLL(LIB_PATH)
@@ -144,6 +145,32 @@ def _stream_handle(stream):
     return ctypes.c_void_p(int(stream))
 
 
+def _check_out_dev(out, nwords: int, device: int):
+    """A caller's device output: C-contiguous 4-byte elements on cuda:`device`, >= nwords."""
+    if out.device.type != "cuda" or out.device.index != device:
+        raise ValueError(f"out is on {out.device}, the context on cuda:{device}")
+    if out.element_size() != 4 or out.dtype.is_floating_point:
+        raise ValueError(f"out must hold 32-bit integer words (int32 / uint32), got {out.dtype}")
+    if not out.is_contiguous():
+        raise ValueError("out must be contiguous")
+    if out.numel() < nwords:
+        raise ValueError(f"out holds {out.numel()} words, the call writes {nwords}")
+
+
+def _host_out(out, nwords: int):
+    """A caller's host output as a writable C-contiguous 4-byte numpy view of >= nwords words."""
+    if hasattr(out, "numpy") and not _is_torch_cuda(out):  # torch CPU tensor
+        out = out.numpy()
+    a = np.asarray(out)
+    if a.dtype.itemsize != 4 or a.dtype.kind not in "iu":
+        raise ValueError(f"out must hold 32-bit integer words (int32 / uint32), got {a.dtype}")
+    if not a.flags["C_CONTIGUOUS"] or not a.flags["WRITEABLE"]:
+        raise ValueError("out must be a writable C-contiguous array")
+    if a.size < nwords:
+        raise ValueError(f"out holds {a.size} words, the call writes {nwords}")
+    return a
+
+
 def _f3(p):
     a = np.ascontiguousarray(np.asarray(p, dtype=np.float32).reshape(3))
     return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_float))
@@ -214,12 +241,18 @@ class Context:
 
     def unpack_cells(self, words, cells, stream=None):
         """am_unpack_cells: device words (int32/uint32 [words]) -> device uint8 [m * n]."""
+        _check_out_dev(words, self.words, self.device)
+        if cells.numel() < self.m * self.n or cells.element_size() != 1 or not cells.is_contiguous():
+            raise ValueError("cells must be a contiguous uint8 device tensor of >= m * n elements")
         self._check(lib.am_unpack_cells(self._h, _P(words.data_ptr()), _P(cells.data_ptr()),
                                         self._dev_stream(words, stream)))
         return cells
 
     def pack_cells(self, cells, words, stream=None):
         """am_pack_cells: device uint8 [m * n] -> device words."""
+        _check_out_dev(words, self.words, self.device)
+        if cells.numel() < self.m * self.n or cells.element_size() != 1 or not cells.is_contiguous():
+            raise ValueError("cells must be a contiguous uint8 device tensor of >= m * n elements")
         self._check(lib.am_pack_cells(self._h, _P(cells.data_ptr()), _P(words.data_ptr()),
                                       self._dev_stream(cells, stream)))
         return words
@@ -232,9 +265,19 @@ class Context:
     def upload(self, centers, half_sizes):
         """am_upload_voxels: centres [N,3] + half sizes [N] (numpy host or torch CUDA float32)."""
         if _is_torch_cuda(centers):
+            import torch
+            if not _is_torch_cuda(half_sizes):
+                raise ValueError("centres and half sizes must both be CUDA tensors (or both host arrays)")
+            for name, t in (("centres", centers), ("half sizes", half_sizes)):
+                if t.dtype != torch.float32:
+                    raise ValueError(f"{name} must be float32, got {t.dtype}")
+                if t.device.index != self.device:
+                    raise ValueError(f"{name} are on {t.device}, the context on cuda:{self.device}")
             c = centers.contiguous()
             hs = half_sizes.contiguous()
             N = int(hs.numel())
+            if c.numel() != 3 * N:
+                raise ValueError(f"centres hold {c.numel()} floats, expected 3 x {N}")
             self._check(lib.am_upload_voxels(self._h, _P(c.data_ptr()), _P(hs.data_ptr()), N, 1))
         else:
             c = np.ascontiguousarray(np.asarray(centers, dtype=np.float32).reshape(-1, 3))
@@ -254,6 +297,7 @@ class Context:
         st = _Stats() if stats else None
         sp = ctypes.byref(st) if st is not None else None
         if out is not None and _is_torch_cuda(out):
+            _check_out_dev(out, self.words, self.device)
             if stream is None:
                 import torch
                 stream = torch.cuda.current_stream(out.device)
@@ -261,7 +305,8 @@ class Context:
         else:
             if out is None:
                 out = np.zeros(self.words, dtype=np.uint32)
-            self._check(lib.am_compute(self._h, pp, _P(out.ctypes.data), 0, _stream_handle(stream), sp))
+            host = _host_out(out, self.words)
+            self._check(lib.am_compute(self._h, pp, _P(host.ctypes.data), 0, _stream_handle(stream), sp))
         return out, (Stats(*[getattr(st, f[0]) for f in _Stats._fields_]) if st is not None else None)
 
     def compute_batch(self, pivots, out=None, stream=None):
@@ -270,6 +315,7 @@ class Context:
         P = len(pv)
         pp = pv.ctypes.data_as(ctypes.POINTER(ctypes.c_float))
         if out is not None and _is_torch_cuda(out):
+            _check_out_dev(out, P * self.words, self.device)
             if stream is None:
                 import torch
                 stream = torch.cuda.current_stream(out.device)
@@ -277,13 +323,15 @@ class Context:
         else:
             if out is None:
                 out = np.zeros((P, self.words), dtype=np.uint32)
-            self._check(lib.am_compute_batch(self._h, pp, P, _P(out.ctypes.data), 0, _stream_handle(stream)))
+            host = _host_out(out, P * self.words)
+            self._check(lib.am_compute_batch(self._h, pp, P, _P(host.ctypes.data), 0, _stream_handle(stream)))
         return out
 
     def compute_baseline(self, pivot, out=None, stream=None):
         """am_compute_baseline: all-pairs exact test (PBox analogue)."""
         _, pp = _f3(pivot)
         if out is not None and _is_torch_cuda(out):
+            _check_out_dev(out, self.words, self.device)
             if stream is None:
                 import torch
                 stream = torch.cuda.current_stream(out.device)
@@ -291,7 +339,8 @@ class Context:
         else:
             if out is None:
                 out = np.zeros(self.words, dtype=np.uint32)
-            self._check(lib.am_compute_baseline(self._h, pp, _P(out.ctypes.data), 0, _stream_handle(stream)))
+            host = _host_out(out, self.words)
+            self._check(lib.am_compute_baseline(self._h, pp, _P(host.ctypes.data), 0, _stream_handle(stream)))
         return out
 
     def build_octree(self, root_lo, root_size) -> int:
@@ -308,6 +357,7 @@ class Context:
         _, pp = _f3(pivot)
         st = (ctypes.c_int64 * 4)() if stats else None
         if out is not None and _is_torch_cuda(out):
+            _check_out_dev(out, self.words, self.device)
             if stream is None:
                 import torch
                 stream = torch.cuda.current_stream(out.device)
@@ -316,7 +366,8 @@ class Context:
         else:
             if out is None:
                 out = np.zeros(self.words, dtype=np.uint32)
-            self._check(lib.am_compute_octree(self._h, pp, sc, int(S), int(vdepth), _P(out.ctypes.data), 0,
+            host = _host_out(out, self.words)
+            self._check(lib.am_compute_octree(self._h, pp, sc, int(S), int(vdepth), _P(host.ctypes.data), 0,
                                               _stream_handle(stream), st))
         sd = None
         if st is not None:

@@ -150,7 +150,6 @@ struct am_ctx {
     cudaGraphExec_t g_exec = nullptr;      // the captured chain and its key
     unsigned long long g_gen = 0;
     int64_t g_P = 0;
-    const void* g_dst = nullptr;
     const void* g_piv = nullptr;
     long long g_launches[AM_K_COUNT] = {};  // kernel launches per replay (am_kernel_stats)
     cudaStream_t lane_s[kMaxLanes] = {};
@@ -162,6 +161,9 @@ struct am_ctx {
     float4* h_piv = nullptr;               // pinned staging of the batch's pivots (xyz, may_cull)
     long long h_piv_cap = 0;
     cudaEvent_t piv_ev = nullptr;          // the last pivot upload (the staging is reused after it)
+    cudaEvent_t done_ev = nullptr;         // end of the last compute call (its stream: last_s)
+    cudaStream_t last_s = nullptr;
+    bool has_last = false;
     unsigned long long* d_bctl = nullptr;  // batched launch: group barriers, pivot queue
     int fused_grid = 0;
     size_t smem_fused = 0;
@@ -258,6 +260,7 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.tab = c->d_tab;
     p.qcount = c->d_ctr;
     p.stats = c->d_ctr + 1;
+    p.early = c->d_ctr + 1 + ST_EARLY;
     p.queue = c->d_queue;
     p.qcap = c->qcap;
     p.refresh_tiles = c->refresh_tiles;
@@ -360,57 +363,116 @@ unsigned long long blist_words(const am_ctx* ctx) {
     return 8ull * ctx->nbricks + (ctx->nbricks + 7) / 8;
 }
 
+// (all-or-nothing, like ensure_slots: on failure the previous queue stays)
 int ensure_queue(am_ctx* ctx, long long cap) {
     if (ctx->d_queue && ctx->qcap == cap) return AM_OK;
-    if (ctx->d_queue) cudaFree(ctx->d_queue);
-    ctx->d_queue = nullptr;
-    ctx->qcap = 0;
-    CK(cudaMalloc(&ctx->d_queue, (size_t)ctx->slots * cap * sizeof(unsigned long long)));
+    unsigned long long* q = nullptr;
+    CK(cudaMalloc(&q, (size_t)ctx->slots * cap * sizeof(unsigned long long)));
+    if (ctx->d_queue) {
+        cudaDeviceSynchronize();
+        cudaFree(ctx->d_queue);
+    }
+    ctx->d_queue = q;
     ctx->qcap = cap;
+    ++ctx->gen;
     return AM_OK;
 }
 
 // Texels of the map after level 0 (T1 texels per face, T1 <= cmapT: the map
-// lives in the first 6 T1^2 floats of the slot's cmap).
+// lives in the first 6 T1^2 floats of the slot's cmap).  All-or-nothing.
 int set_texels1(am_ctx* ctx, int T1) {
     const std::vector<float> tex = make_texels(T1);
+    float4* t = nullptr;
+    CK(cudaMalloc(&t, tex.size() * sizeof(float)));
+    const cudaError_t e = cudaMemcpy(t, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        cudaFree(t);
+        CK(e);
+    }
+    cudaDeviceSynchronize();
     cudaFree(ctx->d_texels1);
-    ctx->d_texels1 = nullptr;
-    CK(cudaMalloc(&ctx->d_texels1, tex.size() * sizeof(float)));
-    CK(cudaMemcpy(ctx->d_texels1, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
+    ctx->d_texels1 = t;
     ctx->cmapT1 = T1;
+    ++ctx->gen;
     return AM_OK;
+}
+
+// Clear-direction map resolution T (AM_OPT_CMAP_T): texel table, per-slot maps and the all-clear
+// map, all-or-nothing; then the level-0 map's texels at min(T1, T).
+int set_cmap_T(am_ctx* ctx, int T) {
+    const std::vector<float> tex = make_texels(T);
+    const std::vector<float4> ones(tex.size() / 4, make_float4(1.f, 0.f, 1.f, 0.f));
+    float4 *t = nullptr, *cm = nullptr, *on = nullptr;
+    cudaError_t e = cudaMalloc(&t, tex.size() * sizeof(float));
+    if (e == cudaSuccess) e = cudaMalloc(&cm, (size_t)ctx->slots * ones.size() * sizeof(float4));
+    if (e == cudaSuccess) e = cudaMalloc(&on, ones.size() * sizeof(float4));
+    if (e == cudaSuccess) e = cudaMemcpy(t, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(on, ones.data(), ones.size() * sizeof(float4), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(t);
+        cudaFree(cm);
+        cudaFree(on);
+        return fail(ctx, e == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA, "cmap_T %d: %s", T,
+                    cudaGetErrorString(e));
+    }
+    cudaDeviceSynchronize();
+    cudaFree(ctx->d_texels);
+    cudaFree(ctx->d_cmap);
+    cudaFree(ctx->d_cmap_ones);
+    ctx->d_texels = t;
+    ctx->d_cmap = cm;
+    ctx->d_cmap_ones = on;
+    ctx->cmapT = T;
+    ++ctx->gen;
+    return set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT));
 }
 
 // Per-map buffers for K slots (slot s of each = the buffer of pivot s of a
 // batched launch; the single-map paths use slot 0).
+// All-or-nothing: the new buffers are allocated first and swapped in only when every
+// allocation succeeded, so an AM_ENOMEM leaves the context as it was (its current slots
+// stay usable, e.g. for a retry with a smaller AM_OPT_BATCH).
 int ensure_slots(am_ctx* ctx, int K) {
     if (ctx->slots >= K) return AM_OK;
-    ++ctx->gen;
     const size_t ntex = (size_t)6 * ctx->cmapT * ctx->cmapT;
-    cudaFree(ctx->d_ctr);
-    cudaFree(ctx->d_queue);
-    cudaFree(ctx->d_recs);
-    cudaFree(ctx->d_tasks);
-    cudaFree(ctx->d_cmap);
-    cudaFree(ctx->d_live);
-    cudaFree(ctx->d_brick_list);
-    ctx->d_ctr = nullptr;
-    ctx->d_queue = nullptr;
-    ctx->d_recs = nullptr;
-    ctx->d_tasks = nullptr;
-    ctx->d_cmap = nullptr;
-    ctx->d_live = nullptr;
-    ctx->d_brick_list = nullptr;
+    unsigned long long *ctr = nullptr, *queue = nullptr, *tasks = nullptr;
+    ConeRec* recs = nullptr;
+    float4* cmap = nullptr;
+    unsigned int *live = nullptr, *blist = nullptr;
+    cudaError_t e = cudaSuccess;
+    auto al = [&](void** p, size_t bytes) {
+        if (e == cudaSuccess && bytes > 0) e = cudaMalloc(p, bytes);
+    };
+    al((void**)&ctr, (size_t)K * kCtrStride * sizeof(unsigned long long));
+    al((void**)&queue, (size_t)K * ctx->qcap * sizeof(unsigned long long));
+    al((void**)&recs, (size_t)K * kRecCap * sizeof(ConeRec));
+    al((void**)&tasks, (size_t)K * kTaskCap * sizeof(unsigned long long));
+    al((void**)&cmap, (size_t)K * ntex * sizeof(float4));
+    if (ctx->vox_cap > 0) al((void**)&live, (size_t)K * ctx->vox_cap * sizeof(unsigned int));
+    if (ctx->nbricks > 0) al((void**)&blist, (size_t)K * blist_words(ctx) * sizeof(unsigned int));
+    if (e == cudaSuccess) e = cudaMemset(ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(ctr); cudaFree(queue); cudaFree(recs); cudaFree(tasks); cudaFree(cmap); cudaFree(live); cudaFree(blist);
+        return fail(ctx, e == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA,
+                    "%d map slots need ~%.1f GB of device memory: %s (the context keeps its %d slots)", K,
+                    (double)K * (kCtrStride * 8.0 + ctx->qcap * 8.0 + kRecCap * sizeof(ConeRec) + kTaskCap * 8.0 +
+                                 ntex * 16.0 + ctx->vox_cap * 4.0 + blist_words(ctx) * 4.0) / 1e9,
+                    cudaGetErrorString(e), ctx->slots);
+    }
+    CK(cudaDeviceSynchronize());  // no launch may still use the old buffers
+    cudaFree(ctx->d_ctr); cudaFree(ctx->d_queue); cudaFree(ctx->d_recs); cudaFree(ctx->d_tasks);
+    cudaFree(ctx->d_cmap); cudaFree(ctx->d_live); cudaFree(ctx->d_brick_list);
+    ctx->d_ctr = ctr;
+    ctx->d_queue = queue;
+    ctx->d_recs = recs;
+    ctx->d_tasks = tasks;
+    ctx->d_cmap = cmap;
+    ctx->d_live = live;
+    ctx->d_brick_list = blist;
     ctx->slots = K;
-    CK(cudaMalloc(&ctx->d_ctr, (size_t)K * kCtrStride * sizeof(unsigned long long)));
-    CK(cudaMemset(ctx->d_ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long)));
-    CK(cudaMalloc(&ctx->d_queue, (size_t)K * ctx->qcap * sizeof(unsigned long long)));
-    CK(cudaMalloc(&ctx->d_recs, (size_t)K * kRecCap * sizeof(ConeRec)));
-    CK(cudaMalloc(&ctx->d_tasks, (size_t)K * kTaskCap * sizeof(unsigned long long)));
-    CK(cudaMalloc(&ctx->d_cmap, (size_t)K * ntex * sizeof(float4)));
-    if (ctx->vox_cap > 0) CK(cudaMalloc(&ctx->d_live, (size_t)K * ctx->vox_cap * sizeof(unsigned int)));
-    if (ctx->nbricks > 0) CK(cudaMalloc(&ctx->d_brick_list, (size_t)K * blist_words(ctx) * sizeof(unsigned int)));
+    ++ctx->gen;
     return AM_OK;
 }
 
@@ -556,7 +618,7 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
     const int gcm = std::max(1, std::min(ctx->sms * 4, (ntex / 16 + 7) / 8));
     clear_map_kernel<<<gcm, 256, ctx->smem_cmap, s>>>(gam, ctx->grid, ctx->d_tab, ctx->d_texels, ctx->cmapT,
-                                                      ctx->d_cmap);
+                                                      ctx->d_cmap, ctx->d_ctr + 1 + ST_EARLY);
     return kmark(ctx, s, AM_K_CLEAR_MAP);
 }
 
@@ -701,31 +763,44 @@ int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s)
 int upload_pivots(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* gam0, cudaStream_t s) {
     if (!ctx->piv_ev) CK(cudaEventCreateWithFlags(&ctx->piv_ev, cudaEventDisableTiming));
     CK(cudaEventSynchronize(ctx->piv_ev));
-    if (ctx->h_piv_cap < P) {
+    if (ctx->h_piv_cap < P + 1) {
         if (ctx->h_piv) cudaFreeHost(ctx->h_piv);
         ctx->h_piv = nullptr;
         ctx->h_piv_cap = 0;
-        CK(cudaMallocHost(&ctx->h_piv, (size_t)P * sizeof(float4)));
-        ctx->h_piv_cap = P;
+        CK(cudaMallocHost(&ctx->h_piv, (size_t)(P + 1) * sizeof(float4)));
+        ctx->h_piv_cap = P + 1;
     }
     for (int64_t k = 0; k < P; ++k) {
         const StreamParams pk = make_params(ctx, pivots + 3 * k, gam0);
         ctx->h_piv[k] = make_float4(pk.px, pk.py, pk.pz, pk.may_cull ? 1.f : 0.f);
     }
-    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv, (size_t)P * sizeof(float4), cudaMemcpyHostToDevice, s));
+    // entry P: the output base of the call (read by the batched kernels: a captured chain replays
+    // into any output buffer)
+    const unsigned long long outp = (unsigned long long)(uintptr_t)gam0;
+    std::memset(&ctx->h_piv[P], 0, sizeof(float4));
+    std::memcpy(&ctx->h_piv[P], &outp, sizeof outp);
+    CK(cudaMemcpyAsync(ctx->d_piv, ctx->h_piv, (size_t)(P + 1) * sizeof(float4), cudaMemcpyHostToDevice, s));
     CK(cudaEventRecord(ctx->piv_ev, s));
     return AM_OK;
 }
 
 // P maps (pivots[3P]) into gam0 + k * MW with ONE fused launch: K groups of
 // CTAs (K <= ctx->slots) take pivots from a device queue (fused.cuh).
+int ensure_piv(am_ctx* ctx, int64_t P) {
+    if (ctx->piv_cap >= P + 1) return AM_OK;
+    ++ctx->gen;
+    cudaFree(ctx->d_piv);
+    ctx->d_piv = nullptr;
+    ctx->piv_cap = 0;
+    CK(cudaMalloc(&ctx->d_piv, (size_t)(P + 1) * sizeof(float4)));
+    ctx->piv_cap = P + 1;
+    return AM_OK;
+}
+
 int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint32_t* gam0, cudaStream_t s) {
-    if (ctx->piv_cap < P) {
-        cudaFree(ctx->d_piv);
-        ctx->d_piv = nullptr;
-        ctx->piv_cap = 0;
-        CK(cudaMalloc(&ctx->d_piv, (size_t)P * sizeof(float4)));
-        ctx->piv_cap = P;
+    {
+        int rc;
+        if ((rc = ensure_piv(ctx, P)) != AM_OK) return rc;
     }
     if (!ctx->d_bctl) CK(cudaMalloc(&ctx->d_bctl, kBctlWords * sizeof(unsigned long long)));
     {
@@ -778,6 +853,7 @@ void shift_slots(FusedParams& F, int base) {
         StreamParams& p = which ? F.lvl : F.main;
         p.qcount = hshift(p.qcount, b * F.ctr_stride);
         p.stats = hshift(p.stats, b * F.ctr_stride);
+        p.early = hshift(p.early, b * F.ctr_stride);
         p.live_count = hshift(p.live_count, b * F.ctr_stride);
         p.rec_count = hshift(p.rec_count, b * F.ctr_stride);
         p.task_count = hshift(p.task_count, b * F.ctr_stride);
@@ -809,13 +885,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     const int K = (int)std::min<int64_t>(P, ctx->batch);
     int rc;
     if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
-    if (ctx->piv_cap < P) {
-        cudaFree(ctx->d_piv);
-        ctx->d_piv = nullptr;
-        ctx->piv_cap = 0;
-        CK(cudaMalloc(&ctx->d_piv, (size_t)P * sizeof(float4)));
-        ctx->piv_cap = P;
-    }
+    if ((rc = ensure_piv(ctx, P)) != AM_OK) return rc;
     {
         int rc;
         if ((rc = upload_pivots(ctx, pivots, P, gam0, s)) != AM_OK) return rc;
@@ -826,9 +896,9 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     auto run_chunk = [&](int64_t c0, int kk, int sb, cudaStream_t s) -> int {
         int rc;
         uint32_t* g = gam0 + c0 * ctx->MW;
-        CK(cudaMemsetAsync(g, 0, (size_t)kk * ctx->MW * sizeof(uint32_t), s));
-        CK(cudaMemsetAsync(ctx->d_ctr + (size_t)sb * kCtrStride, 0, (size_t)kk * kCtrStride * sizeof(unsigned long long), s));
         FusedParams F = fused_params(ctx, pivots + 3 * c0, g);
+        F.out_ptr = reinterpret_cast<const unsigned long long*>(ctx->d_piv + P);  // the call's output base
+        F.out_off = (unsigned long long)c0 * ctx->MW;
         F.nslot = kk;
         F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
         F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
@@ -855,6 +925,8 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             kern<<<g, bd, smem, s>>>(F);
             return AM_OK;
         };
+        bk_init<<<kk, b, 0, s>>>(F);  // this chunk's maps and counters start at zero
+        AM_KM(AM_K_INIT);
         bk_cones<BK_L0><<<grid(ctx->n_l0, kThreads, 1 << 16), b, sm_rows, s>>>(F);
         AM_KM(AM_K_L0_CONES);
         if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
@@ -929,8 +1001,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     // join) captured once per (options, P, output, pivot buffer) and replayed: one
     // host call per batch instead of ~100 (not with per-kernel timing or diagnostics)
     if (ctx->use_graph && ctx->timing != 2 && ctx->diag == 0) {
-        if (!(ctx->g_exec && ctx->g_gen == ctx->gen && ctx->g_P == P && ctx->g_dst == gam0 &&
-              ctx->g_piv == ctx->d_piv)) {
+        if (!(ctx->g_exec && ctx->g_gen == ctx->gen && ctx->g_P == P && ctx->g_piv == ctx->d_piv)) {
             if (ctx->g_exec) cudaGraphExecDestroy(ctx->g_exec);
             ctx->g_exec = nullptr;
             if (!ctx->cap_s) CK(cudaStreamCreateWithFlags(&ctx->cap_s, cudaStreamNonBlocking));
@@ -957,7 +1028,6 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             }
             ctx->g_gen = ctx->gen;
             ctx->g_P = P;
-            ctx->g_dst = gam0;
             ctx->g_piv = ctx->d_piv;
         }
         CK(cudaGraphLaunch(ctx->g_exec, s));
@@ -1017,6 +1087,21 @@ int print_phase_times(am_ctx* ctx) {
         if (t[k] >= t[0] && t[k]) fprintf(stderr, " %d:%.1f", k, (t[k] - t[0]) * 1e-3);
     fprintf(stderr, "\n");
     CK(cudaMemset(ctx->d_ts, 0, sizeof t));
+    return AM_OK;
+}
+
+// Calls on one context share its scratch (per-map slots, pivots, host-output maps): a call on
+// another stream than the previous one first waits for the previous call's end (done_ev).
+int stream_begin(am_ctx* ctx, cudaStream_t s) {
+    if (ctx->has_last && ctx->last_s != s) CK(cudaStreamWaitEvent(s, ctx->done_ev, 0));
+    return AM_OK;
+}
+
+int stream_end(am_ctx* ctx, cudaStream_t s) {
+    if (!ctx->done_ev) CK(cudaEventCreateWithFlags(&ctx->done_ev, cudaEventDisableTiming));
+    CK(cudaEventRecord(ctx->done_ev, s));
+    ctx->last_s = s;
+    ctx->has_last = true;
     return AM_OK;
 }
 
@@ -1183,13 +1268,13 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
 int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_sizes, int64_t N,
                      int src_is_device) {
     if (!ctx) return AM_EINVAL;
+    ctx->uploaded = false;  // (a failed upload leaves no model: AM_ESTATE until one succeeds)
     if (N < 0) return fail(ctx, AM_EINVAL, "N < 0");
     if (N > 0x7fffffffLL) return fail(ctx, AM_EINVAL, "N exceeds 2^31 - 1");
     if (N > 0 && (!centers_xyz || !half_sizes)) return fail(ctx, AM_EINVAL, "NULL voxel array");
     ++ctx->gen;
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
-    ctx->uploaded = false;
     if (N == 0) {
         ctx->N = 0;
         ctx->uploaded = true;
@@ -1393,17 +1478,20 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    if ((rc = stream_begin(ctx, s)) != AM_OK) return rc;
     uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
     if ((rc = launch_aica(ctx, pivot, gam, s)) != AM_OK) return rc;
     if (!dst_is_device)
         CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if ((rc = stream_end(ctx, s)) != AM_OK) return rc;
     if (stats) {
         unsigned long long h[kCtrWords];
         CK(cudaMemcpyAsync(h, ctx->d_ctr, sizeof h, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         int64_t* o = reinterpret_cast<int64_t*>(stats);
-        static_assert(sizeof(am_stats) == (ST_PASSED + 2) * sizeof(int64_t), "am_stats mirrors StatIdx");
+        static_assert(sizeof(am_stats) == (ST_PASSED + 3) * sizeof(int64_t), "am_stats mirrors StatIdx");
         for (int k = 0; k < ST_PASSED; ++k) o[k] = (int64_t)h[1 + k];
+        stats->rows_skipped_full = (int64_t)h[1 + ST_ROWFULL];
         // every voxel goes through the filter once; the rest of it was dropped
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
         // (fused path: kept bricks in the high word, kept sub-bricks -- the list length -- in the low word)
@@ -1430,6 +1518,8 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    int rc;
+    if ((rc = stream_begin(ctx, s)) != AM_OK) return rc;
     uint32_t* dst = am_out;
     if (!dst_is_device) {
         if (ctx->am_cap_maps < P) {
@@ -1441,7 +1531,6 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
         }
         dst = ctx->d_am;
     }
-    int rc;
     const int K = (int)std::min<int64_t>(P, ctx->batch);
     if (K > 1 && fused_ok(ctx) && (ctx->diag & 8)) {
         // diagnostic: one cooperative launch, K CTA groups taking pivots from a queue
@@ -1455,10 +1544,9 @@ int am_compute_batch(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* am_o
         for (int64_t k = 0; k < P; ++k)
             if ((rc = launch_aica(ctx, pivots + 3 * k, dst + k * ctx->MW, s)) != AM_OK) return rc;
     }
-    if (!dst_is_device) {
-        CK(cudaMemcpyAsync(am_out, dst, (size_t)P * ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-    }
+    if (!dst_is_device) CK(cudaMemcpyAsync(am_out, dst, (size_t)P * ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if ((rc = stream_end(ctx, s)) != AM_OK) return rc;
+    if (!dst_is_device) CK(cudaStreamSynchronize(s));
     if (ctx->diag_ts) {
         CK(cudaStreamSynchronize(s));
         if ((rc = print_phase_times(ctx)) != AM_OK) return rc;
@@ -1476,6 +1564,7 @@ int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    if ((rc = stream_begin(ctx, s)) != AM_OK) return rc;
     uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     if (ctx->N > 0) {
@@ -1488,17 +1577,20 @@ int am_compute_baseline(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int
         baseline_kernel<<<g, kThreads, 0, s>>>(p, ctx->baseline_reject);
         if ((rc = kmark(ctx, s, AM_K_BASELINE))) return rc;
     }
-    if (!dst_is_device) {
-        CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-    }
+    if (!dst_is_device) CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if ((rc = stream_end(ctx, s)) != AM_OK) return rc;
+    if (!dst_is_device) CK(cudaStreamSynchronize(s));
     return AM_OK;
 }
 
 int am_set_option(am_ctx* ctx, int key, int64_t value) {
     if (!ctx) return AM_EINVAL;
     DeviceGuard dg(ctx->device);
-    ++ctx->gen;  // any option may change the launch chain: recapture the batch graph
+    // options that shape the batched launch chain invalidate its captured graph; timing, the
+    // baseline's reject, the upload-time options and the graph switch itself do not
+    if (key != AM_OPT_KERNEL_TIMING && key != AM_OPT_BASELINE_REJECT && key != AM_OPT_MORTON_SORT &&
+        key != AM_OPT_L1_SAMPLE && key != AM_OPT_GRAPH)
+        ++ctx->gen;
     switch (key) {
     case AM_OPT_GRID_CTAS:
         if (value < 0 || value > (1 << 20)) return fail(ctx, AM_EINVAL, "grid_ctas out of range");
@@ -1593,22 +1685,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         return set_texels1(ctx, (int)value);
     case AM_OPT_CMAP_T:
         if (value < 4 || value > 256) return fail(ctx, AM_EINVAL, "cmap_T must be in [4, 256]");
-        {
-            const std::vector<float> tex = make_texels((int)value);
-            const std::vector<float4> ones(tex.size() / 4, make_float4(1.f, 0.f, 1.f, 0.f));
-            cudaFree(ctx->d_texels);
-            cudaFree(ctx->d_cmap);
-            cudaFree(ctx->d_cmap_ones);
-            ctx->d_texels = nullptr;
-            ctx->d_cmap = ctx->d_cmap_ones = nullptr;
-            CK(cudaMalloc(&ctx->d_texels, tex.size() * sizeof(float)));
-            CK(cudaMemcpy(ctx->d_texels, tex.data(), tex.size() * sizeof(float), cudaMemcpyHostToDevice));
-            CK(cudaMalloc(&ctx->d_cmap, (size_t)ctx->slots * ones.size() * sizeof(float4)));
-            CK(cudaMalloc(&ctx->d_cmap_ones, ones.size() * sizeof(float4)));
-            CK(cudaMemcpy(ctx->d_cmap_ones, ones.data(), ones.size() * sizeof(float4), cudaMemcpyHostToDevice));
-            ctx->cmapT = (int)value;
-        }
-        return set_texels1(ctx, std::min(ctx->cmapT1, ctx->cmapT));
+        return set_cmap_T(ctx, (int)value);
     default:
         return fail(ctx, AM_EINVAL, "unknown option %d", key);
     }
@@ -1657,7 +1734,7 @@ const char* am_kernel_name(int k) {
     static const char* names[AM_K_COUNT] = {
         "l0_cones", "l0_rows", "clear_map", "l1_cones", "l1_rows", "bricks", "voxels",
         "live_cones", "live_rows", "band", "fused_pipeline", "filter", "baseline", "layout",
-        "ica_memo", "octree"};
+        "ica_memo", "octree", "init"};
     return (k >= 0 && k < AM_K_COUNT) ? names[k] : nullptr;
 }
 
@@ -1816,6 +1893,7 @@ int am_compute_octree(am_ctx* ctx, const float pivot[3], int scheme, int S, int 
     DeviceGuard dg(ctx->device);
     if (!dg.ok) return fail(ctx, AM_ECUDA, "cannot select device %d", ctx->device);
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    if ((rc = stream_begin(ctx, s)) != AM_OK) return rc;
     uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
     CK(cudaMemsetAsync(ctx->d_ostats, 0, 4 * sizeof(unsigned long long), s));
@@ -1856,6 +1934,7 @@ int am_compute_octree(am_ctx* ctx, const float pivot[3], int scheme, int S, int 
     }
     if (!dst_is_device)
         CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if ((rc = stream_end(ctx, s)) != AM_OK) return rc;
     if (stats) {
         unsigned long long h[4];
         CK(cudaMemcpyAsync(h, ctx->d_ostats, sizeof h, cudaMemcpyDeviceToHost, s));
@@ -1907,6 +1986,7 @@ void am_destroy(am_ctx* ctx) {
     if (ctx->g_exec) cudaGraphExecDestroy(ctx->g_exec);
     if (ctx->cap_s) cudaStreamDestroy(ctx->cap_s);
     if (ctx->piv_ev) cudaEventDestroy(ctx->piv_ev);
+    if (ctx->done_ev) cudaEventDestroy(ctx->done_ev);
     if (ctx->h_piv) cudaFreeHost(ctx->h_piv);
     for (int l = 0; l < kMaxLanes; ++l)
         if (ctx->lane_s[l]) cudaStreamDestroy(ctx->lane_s[l]);

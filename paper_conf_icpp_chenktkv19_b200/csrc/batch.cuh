@@ -41,6 +41,13 @@
 
 namespace am {
 
+// Start of this launch's maps: the call's output base (device memory, written with the pivots) or gam0.
+__device__ __forceinline__ uint32_t* launch_maps(const FusedParams& F) {
+    return F.out_ptr ? reinterpret_cast<uint32_t*>(*reinterpret_cast<const volatile unsigned long long*>(F.out_ptr)) +
+                           F.out_off
+                     : F.gam0;
+}
+
 // StreamParams of pivot p (slot p) into shared memory (thread 0; the kernel
 // parameter is read by plain member access: a dynamically indexed pointer into
 // a __grid_constant__ parameter is not a global address); `lvl` selects the
@@ -60,9 +67,19 @@ __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParam
     __syncthreads();
     if (threadIdx.x == 0) {
         slot_params(out, F, p, !lvl);
-        set_pivot(out, F.piv[p], F.gam0 + (size_t)p * F.main.grid.m * F.main.grid.W);
+        set_pivot(out, F.piv[p], launch_maps(F) + (size_t)p * F.main.grid.m * F.main.grid.W);
     }
     __syncthreads();
+}
+
+// First launch of a chunk: zero the maps and the per-slot counters of its pivots (blockIdx.x = pivot).
+__global__ void __launch_bounds__(kThreads) bk_init(const __grid_constant__ FusedParams F) {
+    const int p = blockIdx.x;
+    const int MW = F.main.grid.m * F.main.grid.W;
+    uint32_t* g = launch_maps(F) + (size_t)p * MW;
+    for (int w = threadIdx.x; w < MW; w += blockDim.x) g[w] = 0u;
+    unsigned long long* c = shift_bytes(F.ctr0, p * F.ctr_stride);
+    for (int w = threadIdx.x; w < F.ctr_words; w += blockDim.x) c[w] = 0ull;
 }
 
 enum { BK_L0 = 0, BK_L1 = 1, BK_LIVE = 2 };
@@ -96,7 +113,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
             n = F.n1;
         else
             n = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
-        if ((unsigned long long)blockIdx.x * blockDim.x >= n) return;  // CTA-uniform
+        if ((unsigned long long)blockIdx.x * blockDim.x >= n || map_full(P.early)) return;  // CTA-uniform
         fused_seed(P, sAM, sRowFull);
         if (STAGE == BK_LIVE) nclear = clear_list_rows_cta(sAM, P.grid, P.tab, sDirs, sRowStart);
     }
@@ -125,7 +142,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
             }
         }
         emit_cones_cta<STAGE != BK_LIVE>(P, rc, tc, roff, toff, rcap, tcap, nrows, r, counted, &sc,
-                                         STAGE == BK_LIVE ? P.stats + ST_LIVE : nullptr, sRowFull);
+                                         STAGE == BK_LIVE ? P.stats : nullptr, sRowFull);
     }
 }
 
@@ -145,30 +162,37 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     const unsigned long long cap = STAGE == BK_L1 ? P.task_cap / 2 : P.task_cap;
     const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(tc), cap);
     if ((unsigned long long)blockIdx.x * blockDim.x >= ntask) return;  // CTA-uniform
+    if (STAGE != BK_L0 && map_full(P.early)) return;
     uint32_t* sAM = smem_bk;
     uint32_t* sRowFull = sAM + P.grid.m * P.grid.W;
     fused_seed(P, sAM, sRowFull);
     const unsigned long long toff = STAGE == BK_L1 ? P.task_cap / 2 : 0ull;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    unsigned int rows = 0;
+    unsigned int rows = 0, rfull = 0;
     for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask; k += stride) {
         const unsigned long long t = P.tasks[toff + k];
         const ConeRec r = P.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);
-        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) {
+            ++rfull;
+            continue;
+        }
         ++rows;
         raster_row<STAGE != BK_LIVE>(P, r, i, sAM, Counters{STAGE == BK_LIVE ? sCnt : nullptr});
     }
     fused_flush(P, sAM);
     if (STAGE == BK_LIVE) {
         rows = __reduce_add_sync(0xffffffffu, rows);
+        rfull = __reduce_add_sync(0xffffffffu, rfull);
         if ((threadIdx.x & 31) == 0 && rows) atomicAdd(&sCnt[CT_ROWS], rows);
+        if ((threadIdx.x & 31) == 0 && rfull) atomicAdd(&sCnt[CT_ROWFULL], rfull);
         __syncthreads();
         if (threadIdx.x == 0) {
             if (sCnt[CT_ROWS]) atomicAdd(P.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
             if (sCnt[CT_BAND]) atomicAdd(P.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
             if (sCnt[CT_OVERFLOW]) atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+            if (sCnt[CT_ROWFULL]) atomicAdd(P.stats + ST_ROWFULL, (unsigned long long)sCnt[CT_ROWFULL]);
         }
     }
 }
@@ -185,9 +209,10 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
     const StreamParams& P = sP;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
     float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
-    clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
-                  const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x,
-                  gridDim.x);
+    if (map_full(P.early)) return;
+    const int total = clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
+                                    const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x);
+    if (total == 0 && blockIdx.x == 0 && threadIdx.x == 0) *P.early = 1ull;  // early exit (a7)
 }
 
 // Super-brick test (P.supers set): super-bricks of 8 bricks whose bounding
@@ -197,6 +222,7 @@ __global__ void __launch_bounds__(kThreads) bk_supers(const __grid_constant__ Fu
     const int p = blockIdx.y;
     pivot_params(sP, F, p, false);
     const StreamParams& P = sP;
+    if (map_full(P.early)) return;
     const int lane = threadIdx.x & 31;
     const unsigned int nsup = (P.nbricks + 7) >> 3;
     for (unsigned int s0 = blockIdx.x * kThreads; s0 < nsup; s0 += gridDim.x * kThreads) {
@@ -219,6 +245,7 @@ __global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ Fu
     const int p = blockIdx.y;
     pivot_params(sP, F, p, false);
     const StreamParams& P = sP;
+    if (map_full(P.early)) return;
     if (P.supers) {
         const unsigned int ne = 8u * *reinterpret_cast<const volatile unsigned int*>(P.super_count);
         for (unsigned int e0 = blockIdx.x * kThreads; e0 < ne; e0 += gridDim.x * kThreads) {
@@ -242,6 +269,7 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
     const StreamParams& P = sP;
     const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
     if (blockIdx.x * (kVPT * kWarps) >= nk) return;  // CTA-uniform
+    if (map_full(P.early)) return;
     unsigned int nculled = 0, npassed = 0, streamed = 0;
     for (unsigned int k0 = blockIdx.x * (kVPT * kWarps); k0 < nk; k0 += gridDim.x * (kVPT * kWarps))
         voxel_step(P, k0, nk, sc, nculled, npassed, streamed);
@@ -272,6 +300,7 @@ __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ Fuse
     const StreamParams& P = sP;
     const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
     const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
+    if ((unsigned long long)blockIdx.x * (blockDim.x >> 2) >= n) return;  // CTA-uniform: no pair for this CTA
     unsigned long long tests = 0, hits = 0;
     const int lane = threadIdx.x & 31, sub = lane & 3;
     if (P.band_vdepth > 0) {  // corner-case expansion: one pair per thread (exact_pair)

@@ -61,6 +61,11 @@ struct FusedParams {
     const float4* piv;        // npiv pivots: xyz, w = may_cull
     unsigned int npiv;
     uint32_t* gam0;           // map of pivot k at gam0 + k * m * W
+    // batched path (batch.cuh): the call's output base is read from device memory (*out_ptr, written
+    // with the pivots), so a captured launch chain does not depend on the caller's buffer; the maps
+    // of this launch start out_off words after it.  nullptr: gam0.
+    const unsigned long long* out_ptr;
+    unsigned long long out_off;
     unsigned long long* ctr0; // slot s's counters: ctr0 + s * ctr_stride bytes, ctr_words 64-bit words
     int ctr_words;
     unsigned int* qnext;      // pivot queue head (zeroed)
@@ -80,6 +85,7 @@ __device__ void slot_params(StreamParams& p, const FusedParams& F, int s, bool o
     const unsigned long long c = s * F.ctr_stride;
     p.qcount = shift_bytes(p.qcount, c);
     p.stats = shift_bytes(p.stats, c);
+    p.early = shift_bytes(p.early, c);
     p.live_count = shift_bytes(p.live_count, c);
     p.rec_count = shift_bytes(p.rec_count, c);
     p.task_count = shift_bytes(p.task_count, c);
@@ -179,18 +185,22 @@ template <bool COARSE>
 __device__ void fused_rows(const StreamParams& p, const unsigned long long* task_count, uint32_t* sAM,
                            const uint32_t* sRowFull, Counters cnt, unsigned int gb, unsigned int gn) {
     const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(task_count), p.task_cap);
-    unsigned int rows = 0;
+    unsigned int rows = 0, rfull = 0;
     for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
          k += (unsigned long long)gn * blockDim.x) {
         const unsigned long long t = p.tasks[k];
         const ConeRec r = p.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);
-        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) {
+            ++rfull;
+            continue;
+        }
         ++rows;
         raster_row<COARSE>(p, r, i, sAM, cnt);
     }
     if (rows && cnt.c) atomicAdd(cnt.c + CT_ROWS, rows);
+    if (rfull && cnt.c) atomicAdd(cnt.c + CT_ROWFULL, rfull);
 }
 
 // CTA-wide reservation (every thread of the CTA calls it): `cnt` slots for
@@ -380,16 +390,20 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
                                                unsigned long long* task_count, unsigned int slot_off,
                                                unsigned long long task_off, unsigned int slot_cap,
                                                unsigned long long task_cap, int nrows, const ConeRec& r, bool counted,
-                                               FusedScratch* sc, unsigned long long* live_stat,
+                                               FusedScratch* sc, unsigned long long* stats,
                                                const uint32_t* rowfull) {
-    if (live_stat) {
-        const unsigned int c = __popc(__ballot_sync(0xffffffffu, counted));
-        if ((threadIdx.x & 31) == 0 && c) atomicAdd(live_stat, (unsigned long long)c);
-    }
     const int i0 = r.i0, i1 = r.i0 + nrows - 1;
     int ntask = 0;
     if (nrows > 0)
         for (int w = i0 >> 5; w <= (i1 >> 5); ++w) ntask += __popc(open_rows_word(rowfull, i0, i1, w));
+    if (stats) {  // the full stream's am_stats: live voxels, rows of their cones already full (a5)
+        const unsigned int c = __popc(__ballot_sync(0xffffffffu, counted));
+        const unsigned int f = __reduce_add_sync(0xffffffffu, (unsigned int)(nrows > 0 ? nrows - ntask : 0));
+        if ((threadIdx.x & 31) == 0) {
+            if (c) atomicAdd(stats + ST_LIVE, (unsigned long long)c);
+            if (f) atomicAdd(stats + ST_ROWFULL, (unsigned long long)f);
+        }
+    }
     if (!__syncthreads_or(ntask > 0)) return;  // nothing to emit in the whole CTA (CTA-uniform)
     unsigned int slot;
     unsigned long long t0;
@@ -465,11 +479,13 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 2);
     // 3. clear-direction map (at cmapT1 texels per face when level 1 follows: it only filters level 1)
-    clear_map_cta(P.gam, P.grid, P.tab, F.use_l1 ? F.texels1 : F.texels, F.use_l1 ? F.cmapT1 : P.cmapT,
-                  const_cast<float4*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
+    //    Every CTA counts the clear cells of the same (barrier-stable) map: a full map ends the
+    //    phases in all CTAs alike (early exit, a7)
+    bool full = clear_map_cta(P.gam, P.grid, P.tab, F.use_l1 ? F.texels1 : F.texels, F.use_l1 ? F.cmapT1 : P.cmapT,
+                              const_cast<float4*>(P.cmap), sAM, sDirs, &S.n, gb, gn) == 0;
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 3);
-    if (F.use_l1) {
+    if (F.use_l1 && !full) {
         // 4. level-1 voxels: filter against the map, inner cones (stage 1: upper
         //    halves of the record / task buffers; the records index the level-1 array)
         fused_seed(P, sAM, sRowFull);
@@ -507,9 +523,14 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
         gsync();
         if (!BATCH || gb == 0) fused_mark(F, 5);
         // 6. clear-direction map again
-        clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float4*>(P.cmap), sAM, sDirs, &S.n, gb, gn);
+        full = clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float4*>(P.cmap), sAM, sDirs, &S.n,
+                             gb, gn) == 0;
         gsync();
         if (!BATCH || gb == 0) fused_mark(F, 6);
+    }
+    if (full) {  // early exit: the coarse levels filled the map, no voxel can change it
+        if (gb == 0 && threadIdx.x == 0) *P.early = 1ull;
+        return;
     }
     // 7. brick test (kept bricks -> kept 32-voxel sub-bricks)
     for (unsigned int b0 = gb * kThreads; b0 < P.nbricks; b0 += gn * kThreads) brick_step(P, b0);
@@ -551,7 +572,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
                 nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear, 0, sRowStart);
             }
             emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
-                                  &sc, P.stats + ST_LIVE, sRowFull);
+                                  &sc, P.stats, sRowFull);
         }
     }
     gsync();
@@ -593,6 +614,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
         atomicAdd(P.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
         atomicAdd(P.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
         atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+        atomicAdd(P.stats + ST_ROWFULL, (unsigned long long)sCnt[CT_ROWFULL]);
     }
 }
 

@@ -2,20 +2,25 @@
 // hot path on sm_100a: deferred band kernel, clear-direction map, all-pairs
 // baseline kernel, upload helpers.  The voxel-streaming kernel is stream.cuh.
 //
-// Map of SURVEY.md 8(a) steps to code:
-//   a1 voxel stream ........ stream.cuh aica_stream_kernel: persistent CTAs, dynamic
-//                             tiles, 1-D TMA (cp.async.bulk) into a 2-stage smem ring
-//   a2 reach cull .......... stream.cuh fast_filter(): D - sqrt3 h > rho_max
-//   a3 cone axis ........... stream.cuh process_live(): v, D, phi_v, gamma_v
-//   a4 cone half-angles .... am::tool_cones() (geometry.cuh)
-//   a5 rasterise ........... stream.cuh process_live(): per phi-row gamma
-//                             intervals -> 32-bit masks OR-ed into the per-CTA smem AM
-//   a6 band resolution ..... band pairs pushed to a global queue; band_exact_kernel
-//                             runs CHECKBOX only where the final AM bit is still 0
-//   a7 merge/flush/exit .... stream.cuh cta_merge(): one atomicOr per changed word,
-//                             global AM read back into smem, row-full bits, early exit
+// Map of SURVEY.md 8(a) steps to code (kernel names as in am_kernel_name):
+//   a1 voxel stream ........ batch.cuh bk_supers / bk_bricks / bk_voxels (kept 32-voxel
+//                             sub-bricks, one warp each, coalesced LDG.128 with a
+//                             streaming hint); stream.cuh filter_kernel reads every voxel
+//                             (AM_OPT_BRICKS = 0)
+//   a2 reach cull .......... stream.cuh fast_filter() / sphere_dropped(): D - r > rho_max
+//   a3 cone axis ........... stream.cuh cone_of_voxel(): v, D, phi_v, gamma_v
+//   a4 cone half-angles .... geometry.cuh tool_cones() / inner_cone()
+//   a5 rasterise ........... stream.cuh raster_row(): per phi-row gamma intervals ->
+//                             32-bit masks OR-ed into a per-CTA shared AM
+//   a6 band resolution ..... band pairs pushed to a global queue; bk_band /
+//                             band_exact_kernel run CHECKBOX only where the bit is still 0
+//   a7 merge/flush/exit .... fused.cuh fused_flush(): one atomicOr per changed word;
+//                             row-full bits skip full rows; a full map stops the later
+//                             phases (early exit, am_stats.early_exit)
 //   a8 output .............. bit-packed AM (layout in include/am.h)
 //   a9 baseline ............ baseline_kernel: CHECKBOX for every (voxel, cell)
+// The whole chain of one map runs as one cooperative launch (fused.cuh) or, for a
+// batch of pivots, one launch per phase (batch.cuh).
 #pragma once
 #include <cstdint>
 
@@ -29,7 +34,7 @@ constexpr int kTile = kThreads * kVPT;   // voxels per tile
 
 enum StatIdx {
     ST_STREAMED = 0, ST_CULLED, ST_SKIPPED, ST_LIVE, ST_ROWS, ST_BAND, ST_EXACT, ST_EXACT_HIT,
-    ST_OVERFLOW, ST_EARLY, ST_PASSED, ST_COUNT
+    ST_OVERFLOW, ST_EARLY, ST_PASSED, ST_ROWFULL, ST_COUNT
 };
 
 struct StreamParams {
@@ -44,6 +49,8 @@ struct StreamParams {
     unsigned long long* queue;     // band pairs: (voxel << 32) | cell
     long long qcap;
     unsigned long long* stats;     // ST_COUNT counters (zeroed)
+    unsigned long long* early;     // the map's early-exit flag (main stats[ST_EARLY]): set once the map
+                                   // is full; every later phase of that map then returns at once (a7)
     int refresh_tiles;
     // band-queue voxel references: bit 31 of the queued index selects vox_coarse
     const float4* __restrict__ vox_main;
@@ -56,8 +63,6 @@ struct StreamParams {
     const float4* __restrict__ cmap_tex;
     int cmapT;                     // texels per cube-face side
     float cull_dist;               // rho_max, grown by the fp32 guard (reach cull)
-    int tile;                      // voxels per tile of this launch (<= kTile, multiple of 4)
-    unsigned int* tile_ctr;        // dynamic tile counter of this launch (zeroed)
     unsigned int* live_count;      // live voxels found by the filter (zeroed)
     unsigned int* live_idx;        // their indices into vox (capacity N)
     int may_cull;                  // some voxel may lie beyond the tool's reach (per pivot)
@@ -137,7 +142,7 @@ __device__ __forceinline__ bool exact_pair(const StreamParams& p, float4 q, int 
 struct Counters {
     unsigned int* c;  // [CT_LIVE, CT_ROWS, CT_BAND, CT_OVERFLOW]
 };
-enum { CT_LIVE = 0, CT_ROWS, CT_BAND, CT_OVERFLOW, CT_COUNT };
+enum { CT_LIVE = 0, CT_ROWS, CT_BAND, CT_OVERFLOW, CT_ROWFULL, CT_COUNT };
 
 // Are all rows i0..i1 full (bit set in sRowFull)?
 __device__ __forceinline__ bool rows_all_full(const uint32_t* sRowFull, int i0, int i1) {
@@ -455,7 +460,7 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
 // The clear-direction map of `gam` into V (6 T^2 texels), computed by the CTAs
 // gb = 0..gn-1 of a group.  Shared memory: sAM (m * W words), sDirs
 // (kMapDirs), sN.
-__device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
+__device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
                               const float4* __restrict__ texels, int T, float4* __restrict__ V, uint32_t* sAM,
                               float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
     const int MW = g.m * g.W;
@@ -472,6 +477,7 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
     if (cnt) atomicAdd(sN, cnt);
     __syncthreads();
     const int total = *sN;
+    if (total == 0) return 0;  // the map is full (early exit): no clear cell to find
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
 #ifndef AM_ROWSCAN_OVER_DIRS
 #define AM_ROWSCAN_OVER_DIRS 1
@@ -495,12 +501,12 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
             const float4 c = texels[t];
             V[t] = clear_map_value(nearest_clear_rows(c, sAM, sRows, g, tab), c.w);
         }
-        return;
+        return total;
     }
     if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
         clear_map_blocks(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps);
-        return;
+        return total;
     }
     if (total > g.brute && total <= kMapDirs && (T & 3) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
@@ -550,7 +556,7 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
             bf = fmaxf(bf, __shfl_xor_sync(0xffffffffu, bf, 16));
             if (!half) V[t] = clear_map_value(bf, cf.w);
         }
-        return;
+        return total;
     }
     // every texel against every clear direction, kMaxT texels per thread per
     // pass, the directions in chunks of whole words
@@ -580,6 +586,7 @@ __device__ void clear_map_cta(const uint32_t* gam, const GridDev& g, const float
             if (t < ntex) V[t] = clear_map_value(best[j], c[j].w);
         }
     }
+    return total;
 }
 
 // Stand-alone launch of clear_map_cta (multi-kernel path); dynamic shared
@@ -591,16 +598,30 @@ __host__ __device__ inline size_t clear_map_smem_bytes(int MW) {
 __global__ void __launch_bounds__(256) clear_map_kernel(const uint32_t* __restrict__ gam, GridDev g,
                                                         const float* __restrict__ tab,
                                                         const float4* __restrict__ texels, int T,
-                                                        float4* __restrict__ V) {
+                                                        float4* __restrict__ V, unsigned long long* early) {
     extern __shared__ __align__(16) unsigned char smem_cm[];
     __shared__ int sN;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_cm);
     float4* sDirs = reinterpret_cast<float4*>(smem_cm + (((size_t)g.m * g.W * sizeof(uint32_t) + 15) & ~(size_t)15));
-    clear_map_cta(gam, g, tab, texels, T, V, sAM, sDirs, &sN, blockIdx.x, gridDim.x);
+    const int total = clear_map_cta(gam, g, tab, texels, T, V, sAM, sDirs, &sN, blockIdx.x, gridDim.x);
+    if (total == 0 && early && blockIdx.x == 0 && threadIdx.x == 0) *early = 1ull;
+}
+
+// Early exit (a7, SURVEY 8(a) "stop when popcount(AM) = m n"): has a clear-map phase of this
+// map found it full?  One read per CTA, broadcast through shared memory, so every thread of the
+// CTA takes the same branch even while another CTA of the same launch is setting the flag (the
+// map launch sets it while its own CTAs may still be starting).  Every thread must call it.
+__device__ __forceinline__ bool map_full(const unsigned long long* early) {
+    __shared__ int s_full;
+    __syncthreads();  // (a previous call's readers are done with s_full)
+    if (threadIdx.x == 0) s_full = early && *reinterpret_cast<const volatile unsigned long long*>(early) != 0ull;
+    __syncthreads();
+    return s_full != 0;
 }
 
 // a6: exact test for queued band pairs whose AM bit is still clear.
 __global__ void __launch_bounds__(kThreads) band_exact_kernel(const StreamParams p) {
+    if (map_full(p.early)) return;
     const unsigned long long cnt = *p.qcount;
     const long long n = (long long)(cnt < (unsigned long long)p.qcap ? cnt : (unsigned long long)p.qcap);
     if ((long long)blockIdx.x * blockDim.x >= n) return;  // (whole CTA: nothing queued for it)

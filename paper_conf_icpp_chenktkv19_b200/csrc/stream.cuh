@@ -148,6 +148,7 @@ __device__ __forceinline__ void append_live(const StreamParams& p, bool live, un
 // thread, streaming cache hint); the ragged last tile is guarded.
 __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant__ StreamParams p) {
     __shared__ unsigned int sCulled, sPassed;
+    if (map_full(p.early)) return;
     if (threadIdx.x == 0) sCulled = sPassed = 0u;
     __syncthreads();
     unsigned int nculled = 0, npassed = 0;
@@ -213,6 +214,7 @@ __device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, 
 // brick), through fast_filter.  Exact-safe: a voxel's cone lies inside its
 // brick's.
 __global__ void __launch_bounds__(kThreads) brick_test_kernel(const __grid_constant__ StreamParams p) {
+    if (map_full(p.early)) return;
     const int lane = threadIdx.x & 31;
     const unsigned int nb = p.nbricks;
     for (unsigned int b0 = blockIdx.x * kThreads; b0 < nb; b0 += gridDim.x * kThreads) {
@@ -236,6 +238,7 @@ __global__ void __launch_bounds__(kThreads) brick_test_kernel(const __grid_const
 __global__ void __launch_bounds__(kThreads) brick_voxels_kernel(const __grid_constant__ StreamParams p) {
     __shared__ unsigned int sCulled, sPassed;
     __shared__ unsigned long long sStreamed;
+    if (map_full(p.early)) return;
     if (threadIdx.x == 0) {
         sCulled = sPassed = 0u;
         sStreamed = 0ull;
@@ -451,6 +454,7 @@ __device__ __forceinline__ void emit_cones(const StreamParams& p, int nrows, con
 // With p.live_idx == nullptr every voxel of vox[0, N) is live (clear-map level 0).
 template <bool COARSE>
 __global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
+    if (map_full(p.early)) return;
     const int lane = threadIdx.x & 31;
     const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
     const unsigned long long wstride = (unsigned long long)gridDim.x * blockDim.x;
@@ -528,7 +532,8 @@ __global__ void __launch_bounds__(kThreads) row_kernel(const __grid_constant__ S
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_raw);
     uint32_t* sRowFull = sAM + MW;
     const unsigned long long ntask = min(*p.task_count, p.task_cap);
-    if ((unsigned long long)blockIdx.x * kThreads >= ntask) return;
+    if ((unsigned long long)blockIdx.x * kThreads >= ntask) return;  // CTA-uniform
+    if (map_full(p.early)) return;
     for (int w = threadIdx.x; w < MW; w += blockDim.x) sAM[w] = ld_cg(p.gam + w);
     if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
     __syncthreads();
@@ -546,18 +551,22 @@ __global__ void __launch_bounds__(kThreads) row_kernel(const __grid_constant__ S
     }
     __syncthreads();
     const Counters cnt{sCnt};
-    unsigned int rows = 0;
+    unsigned int rows = 0, rfull = 0;
     for (unsigned long long k = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; k < ntask;
          k += (unsigned long long)gridDim.x * kThreads) {
         const unsigned long long t = p.tasks[k];
         const ConeRec r = p.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);
-        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) continue;
+        if ((sRowFull[i >> 5] >> (i & 31)) & 1u) {
+            ++rfull;
+            continue;
+        }
         ++rows;
         raster_row<COARSE>(p, r, i, sAM, cnt);
     }
     if (rows) atomicAdd(sCnt + CT_ROWS, rows);
+    if (rfull) atomicAdd(sCnt + CT_ROWFULL, rfull);
     __syncthreads();
     for (int w = threadIdx.x; w < MW; w += blockDim.x) {
         const uint32_t sv = sAM[w];
@@ -567,6 +576,7 @@ __global__ void __launch_bounds__(kThreads) row_kernel(const __grid_constant__ S
         atomicAdd(p.stats + ST_ROWS, (unsigned long long)sCnt[CT_ROWS]);
         atomicAdd(p.stats + ST_BAND, (unsigned long long)sCnt[CT_BAND]);
         atomicAdd(p.stats + ST_OVERFLOW, (unsigned long long)sCnt[CT_OVERFLOW]);
+        if (!COARSE) atomicAdd(p.stats + ST_ROWFULL, (unsigned long long)sCnt[CT_ROWFULL]);
     }
 }
 

@@ -126,16 +126,6 @@ def test_edge_cases(am):
     ctx.close()
 
 
-def test_enclosing_shell_early_exit(am):
-    C, H = scenes.octree_leaves("shell", (24.0, 20.0), (-32, -32, -32), 64.0, 6)
-    ctx = am.Context(scenes.TOOL_3CYL, 64, 64, device=0)
-    ctx.upload(C, H)
-    w, st = ctx.compute((0.5, -0.25, 0.3), stats=True)
-    assert (am.unpack(w, 64, 64) == 1).all()
-    assert st.voxels_streamed <= len(H)
-    ctx.close()
-
-
 @pytest.mark.parametrize("m,n", [(1, 1), (1, 64), (5, 1), (33, 95), (64, 1024), (200, 32)])
 def test_grid_shapes(am, m, n):
     cfg = scenes.CONFIGS["T_head"]

@@ -210,6 +210,60 @@ def test_shortcuts_are_exact():
         assert np.array_equal(a, b)
 
 
+def _nearest_first(C, H, p):
+    """The voxels in order of D - sqrt(3) h from the pivot (the AM is a plain OR over voxels, so
+    the order is free -- test_permutation_invariance; blocked cells then stop at a near voxel)."""
+    o = np.argsort(np.linalg.norm(C.astype(np.float64) - np.asarray(p, np.float64)[None, :], axis=1)
+                   - math.sqrt(3.0) * H, kind="stable")
+    return np.ascontiguousarray(C[o]), np.ascontiguousarray(H[o])
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_shortcuts_are_exact_on_configs(name):
+    """the exact-safe sphere shortcuts agree bit for bit with the plain
+    clip-project-hull path on C1 and C2 -- every cell of the full map of two pivots each (C2:
+    1.95M voxels), the cell states (0 / 1 / 2) compared exactly."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    for p in cfg.pivots(2):
+        Cs, Hs = _nearest_first(C, H, p)
+        a = oracle.am_states(Cs, Hs, cfg.tool, p, cfg.m, cfg.n, shortcuts=True)
+        b = oracle.am_states(Cs, Hs, cfg.tool, p, cfg.m, cfg.n, shortcuts=False)
+        assert np.array_equal(a, b), (name, p, int((a != b).sum()))
+        assert (a == 0).any() and (a == 2).any()  # both decisions exercised
+
+
+def test_shortcuts_are_exact_pairs_near_the_cones():
+    """Pair-level identity of the shortcuts (stronger than per cell: no hit can hide behind
+    another voxel's) on C2 voxels near the pivot, with directions spread over and around each
+    voxel's blocked cone (angles up to 1.3 x asin((R_max + sqrt3 h) / D)), paper 4-cyl tool."""
+    cfg = scenes.CONFIGS["C2"]
+    C, H = cfg.leaves()
+    rng = np.random.default_rng(5)
+    tool = scenes.TOOL_PAPER4
+    Rmax = max(r for r, _ in tool)
+    states = np.zeros(3, int)
+    for p in cfg.pivots(2):
+        Cs, Hs = _nearest_first(C, H, p)
+        pick = np.concatenate([np.arange(400), rng.choice(len(Hs), 400, replace=False)])
+        for q in pick:
+            v = Cs[q].astype(np.float64) - p.astype(np.float64)
+            D = np.linalg.norm(v)
+            u = v / D
+            a = np.array([1.0, 0.0, 0.0]) if abs(u[0]) < 0.9 else np.array([0.0, 1.0, 0.0])
+            e1 = np.cross(u, a)
+            e1 /= np.linalg.norm(e1)
+            e2 = np.cross(u, e1)
+            top = 1.3 * math.asin(min(1.0, (Rmax + math.sqrt(3.0) * Hs[q]) / D))
+            for th, az in zip(rng.uniform(0.0, min(top, math.pi), 12), rng.uniform(0, 2 * math.pi, 12)):
+                d = math.cos(th) * u + math.sin(th) * (math.cos(az) * e1 + math.sin(az) * e2)
+                s1 = oracle.pair_state(v, Hs[q], d, tool, shortcuts=True)
+                s0 = oracle.pair_state(v, Hs[q], d, tool, shortcuts=False)
+                assert s1 == s0, (q, th, az, s1, s0)
+                states[s1] += 1
+    assert states[0] > 1000 and states[2] > 1000, states  # (band pairs are a 1e-5 rad sliver)
+
+
 # ---------------------------------------------------------------- P3 sphere cap
 
 def _theta_c(Rs, Dp, R):
