@@ -183,6 +183,18 @@ class Config:
         extra = path_pivots(self.model, self.params, count - len(fixed), off, seed0, self.centre)
         return np.concatenate([np.stack(fixed) if fixed else np.zeros((0, 3), np.float32), extra])
 
+    def pivots_at(self, indices):
+        """Pivots number k of the path for k in `indices` (pivots_at(range(n)) == pivots(n)):
+        a rank of a pivot-sharded run generates only its own."""
+        fixed = [np.asarray(p, dtype=np.float32) for p in self.fixed_pivots]
+        off = max(self.offset, 2.0 * np.sqrt(3.0) * self.min_half() + 0.05)
+        out = np.zeros((len(indices), 3), np.float32)
+        for r, k in enumerate(indices):
+            k = int(k)
+            out[r] = fixed[k] if k < len(fixed) else path_pivots(self.model, self.params, 1, off,
+                                                                   1 + k - len(fixed), self.centre)[0]
+        return out
+
 
 def _cfg(**kw):
     return Config(**kw)

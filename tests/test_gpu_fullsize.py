@@ -39,12 +39,18 @@ def full_oracle_map(cfg, C, H, p):
     return oracle.am_states(Cs, Hs, cfg.tool, p, cfg.m, cfg.n)
 
 
-@pytest.mark.parametrize("name,npiv,check", [
-    ("C3", 64, (0, 1, 2, 3)),
-    ("C4", 16, (0, 1)),
-    ("C5", 64, (0, 9, 18, 27, 36, 45, 54, 63)),
-])
-def test_full_size_every_cell(am, name, npiv, check):
+def _pick(maps, cfg, am, n_open):
+    """The first n_open maps that still have clear cells (where a wrong cone or a missed exact test
+    shows), the map with the most clear cells, and the first fully blocked map (early exit)."""
+    clear = [int((am.unpack(w, cfg.m, cfg.n) == 0).sum()) for w in maps]
+    open_ = [k for k, c in enumerate(clear) if c > 0]
+    full = [k for k, c in enumerate(clear) if c == 0]
+    pick = open_[:n_open] + ([int(np.argmax(clear))] if clear else []) + full[:1]
+    return sorted(set(pick))
+
+
+@pytest.mark.parametrize("name,npiv,n_open", [("C3", 64, 4), ("C4", 16, 2), ("C5", 64, 7)])
+def test_full_size_every_cell(am, name, npiv, n_open):
     import torch
     cfg = scenes.CONFIGS[name]
     C, H = cfg.leaves()
@@ -57,6 +63,8 @@ def test_full_size_every_cell(am, name, npiv, check):
     torch.cuda.synchronize()
     maps = out.cpu().numpy().view(np.uint32)
     report = []
+    check = _pick(maps, cfg, am, n_open)
+    assert len(check) >= n_open
     for k in check:
         t = time.time()
         S = full_oracle_map(cfg, C, H, P[k])

@@ -3,7 +3,8 @@
     python tools/summarize_ncu.py <tag> [config] [maps per captured launch]
 reads gpurun_out/prof_<tag>.ncu-rep and gpurun_out/launches_<tag>.csv, writes
 profiles/<tag>_launches.txt, profiles/<tag>_<kernel>_ncu.txt and merges each captured
-kernel's DRAM bytes into profiles/ncu_summary.json, which bench.py reads for `traffic`.
+kernel's DRAM bytes into profiles/ncu_summary.json (by_config[config][kernel]), which bench.py reads
+for `traffic` and `warp_inst_per_launch`.
 """
 import csv
 import io
@@ -124,7 +125,7 @@ def main():
             if "gpu__time_duration.sum" in rawrow:
                 ent["ncu_duration_us"] = tobytes(rawrow["gpu__time_duration.sum"], "") / (
                     1e3 if rawu.get("gpu__time_duration.sum") == "nsecond" else 1)
-            old = summ.get("kernels", {}).get(kname)
+            old = summ.get("by_config", {}).get(config, {}).get(kname)
             if old and old.get("tag") == tag:  # same stage captured twice (clear_map): average
                 for k2 in ("dram_bytes_per_launch", "dram_read", "dram_write", "warp_inst_per_launch",
                            "ncu_duration_us"):
@@ -132,8 +133,10 @@ def main():
                         n_ = old.get("launches_averaged", 1)
                         ent[k2] = (old[k2] * n_ + ent[k2]) / (n_ + 1)
                 ent["launches_averaged"] = old.get("launches_averaged", 1) + 1
-            summ.setdefault("kernels", {})[kname] = ent
-            json.dump({"kernels": summ["kernels"]}, open(sp, "w"), indent=1)
+            summ.setdefault("by_config", {}).setdefault(config, {})[kname] = ent
+            if config == "C3":  # (the default workload's entries also under "kernels")
+                summ.setdefault("kernels", {})[kname] = ent
+            json.dump({"kernels": summ.get("kernels", {}), "by_config": summ["by_config"]}, open(sp, "w"), indent=1)
 
 if __name__ == "__main__":
     main()
