@@ -20,6 +20,7 @@
 #include "stream.cuh"
 #include "fused.cuh"
 #include "batch.cuh"
+#include "latency.cuh"
 #include "octree.cuh"
 
 #include <algorithm>
@@ -166,6 +167,7 @@ struct am_ctx {
     bool has_last = false;
     unsigned long long* d_bctl = nullptr;  // batched launch: group barriers, pivot queue
     int fused_grid = 0;
+    int lat_grid = 0;                      // am_latency_kernel: co-resident CTAs (cooperative launch)
     size_t smem_fused = 0;
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -510,6 +512,13 @@ int configure_launch(am_ctx* ctx) {
                                                           ctx->smem_fused) == cudaSuccess &&
             occf > 0 && occb > 0)
             ctx->fused_grid = std::min(occf, occb) * ctx->sms;
+        int occl = 0;
+        if (cudaFuncSetAttribute(am_latency_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)ctx->smem_fused) == cudaSuccess &&
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occl, am_latency_kernel, kThreads, ctx->smem_fused) ==
+                cudaSuccess &&
+            occl > 0)
+            ctx->lat_grid = occl * ctx->sms;
     }
     cudaGetLastError();
     // batched phases (batch.cuh)
@@ -630,9 +639,12 @@ int launch_clear_map(am_ctx* ctx, const uint32_t* gam, cudaStream_t s) {
 //   subsets of the model, so the map is the same with any number of them
 //   (AM_OPT_PHASES = 0, 1 or 2 levels).
 // Can the whole map run as one fused cooperative launch?
+// Small models (latency.cuh): level 0 is the whole model, no clear-direction maps or bricks.
+bool small_model(const am_ctx* ctx) { return ctx->N <= kSmallModel || ctx->n_l0 == 0; }
+
 bool fused_ok(const am_ctx* ctx) {
-    return ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->phases >= 1 && ctx->n_l0 > 0 &&
-           ctx->bricks_on && ctx->d_bricks && ctx->N > 0;
+    return ctx->fused && ctx->fused_grid > 0 && !(ctx->diag & 3) && ctx->N > 0 &&
+           (small_model(ctx) || (ctx->phases >= 1 && ctx->n_l0 > 0 && ctx->bricks_on && ctx->d_bricks));
 }
 
 // The fused launch parameters for slot 0 and the map gam.
@@ -742,15 +754,33 @@ int kmark(am_ctx* ctx, cudaStream_t s, int k) {
 
 // One map (pivot) into gam with one fused cooperative launch over the whole grid.
 int launch_fused(am_ctx* ctx, const float* pivot, uint32_t* gam, cudaStream_t s) {
+    const bool lat = ctx->lat_grid > 0 && !(ctx->diag & 16);
     CK(cudaMemsetAsync(gam, 0, (size_t)ctx->MW * sizeof(uint32_t), s));
-    CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrStride * sizeof(unsigned long long), s));
+    if (!lat) CK(cudaMemsetAsync(ctx->d_ctr, 0, kCtrStride * sizeof(unsigned long long), s));
     FusedParams F = fused_params(ctx, pivot, gam);
+    F.ctr0 = ctx->d_ctr;  // (am_latency_kernel zeroes the map's counters itself)
+    F.ctr_words = kCtrStride;
+    if (small_model(ctx)) {  // level 0 = every voxel; the all-clear map (no map is built)
+        F.small = 1;
+        F.lvl.vox = ctx->d_vox;
+        F.lvl.N = ctx->N;
+        F.n0 = (unsigned int)ctx->N;
+        F.n1 = 0;
+        F.use_l1 = 0;
+        F.main.cmap = ctx->d_cmap_ones;
+    }
     int rc;
     if ((rc = timed_begin(ctx, s))) return rc;
     if ((rc = kchain(ctx, s))) return rc;
     void* args[] = {&F};
-    CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads), args,
-                                   ctx->smem_fused, s));
+    if (lat) {
+        CK(cudaLaunchCooperativeKernel((const void*)am_latency_kernel, dim3(ctx->lat_grid), dim3(kThreads), args,
+                                       ctx->smem_fused, s));
+    } else {  // (AM_OPT_DIAG bit 4: the previous single-pivot kernel, for comparison)
+        F.small = 0;
+        CK(cudaLaunchCooperativeKernel((const void*)am_pipeline_kernel<false>, dim3(ctx->fused_grid), dim3(kThreads),
+                                       args, ctx->smem_fused, s));
+    }
     if ((rc = kmark(ctx, s, AM_K_FUSED))) return rc;
     if ((rc = timed_end(ctx, s))) return rc;
     if (ctx->d_prev)
@@ -1495,9 +1525,9 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
         // every voxel goes through the filter once; the rest of it was dropped
         o[ST_SKIPPED] = (int64_t)ctx->N - (int64_t)h[1 + ST_CULLED] - (int64_t)h[1 + ST_PASSED];
         // (fused path: kept bricks in the high word, kept sub-bricks -- the list length -- in the low word)
-        stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks)
+        stats->bricks_kept = (ctx->bricks_on && ctx->d_bricks && !(fused_ok(ctx) && small_model(ctx)))
                                  ? (int64_t)(fused_ok(ctx) ? (h[kCtrBricks] >> 32) : (h[kCtrBricks] & 0xffffffffull))
-                                 : (int64_t)ctx->nbricks;
+                                 : (int64_t)ctx->nbricks;  // (small models: every brick is read)
         stats->level_voxels = ctx->phases == 0 ? 0 : ctx->phases == 1 ? ctx->n_l0 : ctx->n_l1;
         if ((rc = print_phase_times(ctx)) != AM_OK) return rc;
     } else if (!dst_is_device) {
@@ -1620,7 +1650,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
-        if (value < 0 || value > 15) return fail(ctx, AM_EINVAL, "diag must be in [0, 15]");
+        if (value < 0 || value > 31) return fail(ctx, AM_EINVAL, "diag must be in [0, 31]");
         if ((value & 3) && !ctx->d_prev) {
             CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));

@@ -289,10 +289,11 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
     }
 }
 
-// Band: exact test of the queued pairs whose bit is still clear.  Each pair
-// is tested by 4 lanes, lane q taking cylinders q, q + 4, ... (the test is an
-// OR over cylinders), so the long serial CHECKBOX chain is ~ncyl times
-// shorter; a warp takes 8 pairs per pass.
+// Band: exact test of the queued pairs whose bit is still clear.  Each warp checks 32 pairs (one
+// per lane; lane j of warp w takes pair w + j W of the W warps of the pivot, so that the open
+// pairs, neighbours in the queue, land on different warps) and runs CHECKBOX on the still-clear
+// ones with the whole warp (exact_hit_warp: the sub-tests side by side, ~4x less latency than one
+// thread's chain).
 __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
@@ -300,61 +301,53 @@ __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ Fuse
     const StreamParams& P = sP;
     const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
     const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
-    if ((unsigned long long)blockIdx.x * (blockDim.x >> 2) >= n) return;  // CTA-uniform: no pair for this CTA
+    const unsigned long long nw = (unsigned long long)gridDim.x * (blockDim.x >> 5);  // warps of this pivot
+    const unsigned long long gw = (unsigned long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (gw >= n) return;  // (warp-uniform: no pair for this warp)
+    const int lane = threadIdx.x & 31;
     unsigned long long tests = 0, hits = 0;
-    const int lane = threadIdx.x & 31, sub = lane & 3;
-    if (P.band_vdepth > 0) {  // corner-case expansion: one pair per thread (exact_pair)
-        const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-        for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < n; k += stride) {
-            const unsigned long long e = P.queue[k];
-            const unsigned int vidx = (unsigned int)(e >> 32);
+    for (unsigned long long k0 = 0; k0 < n; k0 += nw * 32) {  // warp-uniform
+        const unsigned long long k = k0 + lane * nw + gw;
+        unsigned long long e = 0;
+        bool open = false;
+        if (k < n) {
+            e = P.queue[k];
             const int cell = (int)(e & 0xffffffffu);
+            const int i = cell / P.grid.n, j = cell - i * P.grid.n;
+            open = !(ld_cg(P.gam + i * P.grid.W + (j >> 5)) & (1u << (j & 31)));
+        }
+        unsigned int mo = __ballot_sync(0xffffffffu, open);
+        while (mo) {
+            const int src = __ffs(mo) - 1;
+            mo &= mo - 1u;
+            const unsigned long long es = __shfl_sync(0xffffffffu, e, src);
+            const unsigned int vidx = (unsigned int)(es >> 32);
+            const int cell = (int)(es & 0xffffffffu);
             const int i = cell / P.grid.n, j = cell - i * P.grid.n;
             uint32_t* wp = P.gam + i * P.grid.W + (j >> 5);
             const uint32_t bit = 1u << (j & 31);
-            if (ld_cg(wp) & bit) continue;
+            if (ld_cg(wp) & bit) continue;  // (blocked meanwhile; warp-uniform)
             ++tests;
-            if (exact_pair(P, P.vox_main[vidx], cell)) {
+            const float4 q = P.vox_main[vidx];
+            bool hit;
+            if (P.band_vdepth > 0) {  // corner-case expansion (§4.3): one lane (exact_pair)
+                hit = __shfl_sync(0xffffffffu, lane == 0 && exact_pair(P, q, cell), 0);
+            } else {
+                const float* t = P.tab;
+                const float cph = __ldg(t + i), sph = __ldg(t + P.grid.m + i);
+                const float cg = __ldg(t + 2 * P.grid.m + j), sg = __ldg(t + 2 * P.grid.m + P.grid.n + j);
+                hit = exact_hit_warp(q.x - P.px, q.y - P.py, q.z - P.pz, q.w, sph * cg, sph * sg, cph, P.tool);
+            }
+            if (hit) {
                 ++hits;
-                atomicOr(wp, bit);
-            }
-        }
-    } else {
-        const unsigned long long stride = ((unsigned long long)gridDim.x * blockDim.x) >> 2;
-        for (unsigned long long k0 = ((unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) >> 2; k0 < n;
-             k0 += stride) {  // warp-uniform
-            const unsigned long long k = k0 + (lane >> 2);
-            bool test = false, hit = false;
-            uint32_t* wp = nullptr;
-            uint32_t bit = 0u;
-            if (k < n) {
-                const unsigned long long e = P.queue[k];
-                const unsigned int vidx = (unsigned int)(e >> 32);
-                const int cell = (int)(e & 0xffffffffu);
-                const int i = cell / P.grid.n, j = cell - i * P.grid.n;
-                wp = P.gam + i * P.grid.W + (j >> 5);
-                bit = 1u << (j & 31);
-                test = !(ld_cg(wp) & bit);
-                if (test) {
-                    const float4 q = P.vox_main[vidx];
-                    const float* t = P.tab;
-                    const float cph = __ldg(t + i), sph = __ldg(t + P.grid.m + i);
-                    const float cg = __ldg(t + 2 * P.grid.m + j), sg = __ldg(t + 2 * P.grid.m + P.grid.n + j);
-                    hit = exact_hit(q.x - P.px, q.y - P.py, q.z - P.pz, q.w, sph * cg, sph * sg, cph, P.tool, sub, 4);
-                }
-            }
-            const unsigned int hm = __ballot_sync(0xffffffffu, hit);
-            if (sub == 0 && test) {
-                ++tests;
-                if ((hm >> lane) & 0xfu) {
-                    ++hits;
-                    atomicOr(wp, bit);
-                }
+                if (lane == 0) atomicOr(wp, bit);
             }
         }
     }
-    if (tests) atomicAdd(P.stats + ST_EXACT, tests);
-    if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
+    if (lane == 0) {
+        if (tests) atomicAdd(P.stats + ST_EXACT, tests);
+        if (hits) atomicAdd(P.stats + ST_EXACT_HIT, hits);
+    }
 }
 
 }  // namespace am

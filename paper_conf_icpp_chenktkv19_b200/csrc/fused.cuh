@@ -52,6 +52,7 @@ struct FusedParams {
     int cmapT1;
     int ntex;
     int use_l1;
+    int small;                // am_latency_kernel: level 0 is the whole model, no maps / bricks (latency.cuh)
     unsigned long long* ts;   // diagnostics: %globaltimer after each phase (CTA 0), or nullptr
     // batched launch (am_pipeline_kernel<true>): the CTAs form nslot groups; group s
     // owns slot s of every per-map buffer (the slot-0 pointers above advanced by

@@ -316,8 +316,12 @@ __device__ __forceinline__ void edge_vertices(int e, int& a, int& b) {
     b = v | (1 << ax);
 }
 
+// The test is an OR of 15 sub-tests per cylinder c -- (0) the axis crossing the box, (1..12) box
+// edge e clipped to the slab, (13, 14) the cap planes -- so it can be split over the lanes of a
+// group: sub-test s = 15 c + k is done by the lane with s % nparts == part (default: all of them,
+// one lane).  The OR of the parts is the whole test, value for value.
 __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, float dx, float dy,
-                                       float dz, const ToolDev& T, int c0 = 0, int cs = 1) {
+                                       float dz, const ToolDev& T, int part = 0, int nparts = 1) {
     // frame: e1 = normalize(d x a), a = the world axis least aligned with d; e2 = d x e1
     const float adx = fabsf(dx), ady = fabsf(dy), adz = fabsf(dz);
     float e1x, e1y, e1z;
@@ -340,10 +344,11 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
         Y[k] = cY + sx * e2x + sy * e2y + sz * e2z;
         Z[k] = cZ + sx * dx + sy * dy + sz * dz;
     }
-    for (int c = c0; c < T.ncyl; c += cs) {  // (cylinders c0, c0 + cs, ...: a lane's share of the OR)
+    for (int c = 0; c < T.ncyl; ++c) {
+        const int s0 = 15 * c;  // this cylinder's sub-tests s0 .. s0 + 14
         const float z0 = T.z0[c], z1 = T.z1[c], R = T.R[c], R2 = R * R;
         // (0) the axis segment crosses the box: slab test in world coordinates
-        {
+        if (s0 % nparts == part) {
             float tlo = z0, thi = z1;
             const float dv[3] = {dx, dy, dz}, vv[3] = {vx, vy, vz};
 #pragma unroll
@@ -363,6 +368,7 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
         // (1) box edges clipped to the slab
 #pragma unroll
         for (int e = 0; e < 12; ++e) {
+            if ((s0 + 1 + e) % nparts != part) continue;
             int a, b;
             edge_vertices(e, a, b);
             const float za = Z[a], zb = Z[b];
@@ -383,6 +389,7 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
         }
         // (2) on each cap plane, segments between crossing points of one face's edges
         for (int cap = 0; cap < 2; ++cap) {
+            if ((s0 + 13 + cap) % nparts != part) continue;
             const float zc = cap ? z1 : z0;
             float PX[12], PY[12];
             bool ok[12];
@@ -421,6 +428,115 @@ __device__ __noinline__ bool exact_hit(float vx, float vy, float vz, float h, fl
                 }
             }
         }
+    }
+    return false;
+}
+
+// The same test by a whole warp (warp-uniform call, every lane gets the result): the sub-tests run
+// side by side instead of one after the other -- lane k & 7 holds box vertex k, lane e < 12 clips
+// edge e to the slab, lanes 16 cap + e put edge e's crossing of cap plane `cap`, and the 2 x 36
+// polygon sides between crossings on one face are spread over the lanes -- with the very same
+// arithmetic per sub-test as exact_hit, so the OR is the same value for value.  A latency path:
+// one test costs a few hundred cycles instead of ~10^4 (exact_hit is ~8K dependent instructions for
+// 3 cylinders, and lanes that branch on different sub-tests of one warp run serially).
+__device__ __forceinline__ int face_side(int u) {  // (edge p) | (edge q) << 4 of polygon side u < 36
+    const unsigned long long w = u < 8    ? 0x9575a8a686a48464ull
+                                 : u < 16 ? 0x82908020b9b797b5ull
+                                 : u < 24 ? 0xbab3a3b1a1319892ull
+                                 : u < 32 ? 0x6232545141504010ull
+                                          : 0x76736372ull;
+    return (int)((w >> ((u & 7) * 8)) & 0xffull);
+}
+
+__device__ __noinline__ bool exact_hit_warp(float vx, float vy, float vz, float h, float dx, float dy, float dz,
+                                            const ToolDev& T) {
+    const int lane = threadIdx.x & 31;
+    const float adx = fabsf(dx), ady = fabsf(dy), adz = fabsf(dz);
+    float e1x, e1y, e1z;
+    if (adx <= ady && adx <= adz) { e1x = 0.f; e1y = dz; e1z = -dy; }      // d x (1,0,0)
+    else if (ady <= adz)          { e1x = -dz; e1y = 0.f; e1z = dx; }      // d x (0,1,0)
+    else                          { e1x = dy; e1y = -dx; e1z = 0.f; }      // d x (0,0,1)
+    const float in1 = rsqrtf(e1x * e1x + e1y * e1y + e1z * e1z);
+    e1x *= in1; e1y *= in1; e1z *= in1;
+    const float e2x = dy * e1z - dz * e1y, e2y = dz * e1x - dx * e1z, e2z = dx * e1y - dy * e1x;
+    const float cX = vx * e1x + vy * e1y + vz * e1z;
+    const float cY = vx * e2x + vy * e2y + vz * e2z;
+    const float cZ = vx * dx + vy * dy + vz * dz;
+    // vertex k = lane & 7
+    const int k = lane & 7;
+    const float sx = (k & 1) ? h : -h, sy = (k & 2) ? h : -h, sz = (k & 4) ? h : -h;
+    const float Xk = cX + sx * e1x + sy * e1y + sz * e1z;
+    const float Yk = cY + sx * e2x + sy * e2y + sz * e2z;
+    const float Zk = cZ + sx * dx + sy * dy + sz * dz;
+    // edge lanes (e = lane < 12) and cap-crossing lanes (cap = lane >> 4, e = lane & 15 < 12)
+    int a, b;
+    edge_vertices(lane < 12 ? lane : 0, a, b);
+    const float Xa = __shfl_sync(0xffffffffu, Xk, a), Xb = __shfl_sync(0xffffffffu, Xk, b);
+    const float Ya = __shfl_sync(0xffffffffu, Yk, a), Yb = __shfl_sync(0xffffffffu, Yk, b);
+    const float za = __shfl_sync(0xffffffffu, Zk, a), zb = __shfl_sync(0xffffffffu, Zk, b);
+    const int ec = lane & 15;
+    int ca, cb;
+    edge_vertices(ec < 12 ? ec : 0, ca, cb);
+    const float cXa = __shfl_sync(0xffffffffu, Xk, ca), cXb = __shfl_sync(0xffffffffu, Xk, cb);
+    const float cYa = __shfl_sync(0xffffffffu, Yk, ca), cYb = __shfl_sync(0xffffffffu, Yk, cb);
+    const float cza = __shfl_sync(0xffffffffu, Zk, ca), czb = __shfl_sync(0xffffffffu, Zk, cb);
+    for (int c = 0; c < T.ncyl; ++c) {
+        const float z0 = T.z0[c], z1 = T.z1[c], R = T.R[c], R2 = R * R;
+        bool hit;
+        {   // (0) the axis segment crosses the box (every lane, the same values)
+            float tlo = z0, thi = z1;
+            const float dv[3] = {dx, dy, dz}, vv[3] = {vx, vy, vz};
+#pragma unroll
+            for (int ax = 0; ax < 3; ++ax) {
+                if (dv[ax] != 0.f) {
+                    const float inv = 1.f / dv[ax];
+                    float t0 = (vv[ax] - h) * inv, t1 = (vv[ax] + h) * inv;
+                    if (t0 > t1) { const float t = t0; t0 = t1; t1 = t; }
+                    tlo = fmaxf(tlo, t0);
+                    thi = fminf(thi, t1);
+                } else if (fabsf(vv[ax]) > h) {
+                    thi = -1e30f;
+                }
+            }
+            hit = tlo <= thi;
+        }
+        if (lane < 12) {  // (1) box edge `lane` clipped to the slab
+            float t0, t1;
+            bool valid;
+            if (za == zb) {
+                valid = !(za < z0 || za > z1);
+                t0 = 0.f; t1 = 1.f;
+            } else {
+                const float inv = 1.f / (zb - za);
+                float ta = (z0 - za) * inv, tb = (z1 - za) * inv;
+                t0 = fmaxf(fminf(ta, tb), 0.f);
+                t1 = fminf(fmaxf(ta, tb), 1.f);
+                valid = !(t0 > t1);
+            }
+            const float ux = Xb - Xa, uy = Yb - Ya;
+            if (valid && seg_dist2(fmaf(t0, ux, Xa), fmaf(t0, uy, Ya), fmaf(t1, ux, Xa), fmaf(t1, uy, Ya)) <= R2)
+                hit = true;
+        }
+        // (2) cap planes: crossing of edge ec with plane zc, then the cross-section's vertices and
+        //     the sides between crossings on one face
+        const float zc = (lane >> 4) ? z1 : z0;
+        const bool ok = ec < 12 && (cza != czb) && ((cza - zc) * (czb - zc) <= 0.f);
+        const float t = ok ? (zc - cza) / (czb - cza) : 0.f;
+        const float PX = fmaf(t, cXb - cXa, cXa), PY = fmaf(t, cYb - cYa, cYa);
+        if (ok && PX * PX + PY * PY <= R2) hit = true;
+        const int okm = (int)ok;
+#pragma unroll
+        for (int u0 = 0; u0 < 72; u0 += 32) {
+            const int u = u0 + lane;
+            const int cap = u >= 36 ? 1 : 0;
+            const int sd = face_side(u < 72 ? u - 36 * cap : 0);
+            const int lp = 16 * cap + (sd & 15), lq = 16 * cap + (sd >> 4);
+            const float px = __shfl_sync(0xffffffffu, PX, lp), py = __shfl_sync(0xffffffffu, PY, lp);
+            const float qx = __shfl_sync(0xffffffffu, PX, lq), qy = __shfl_sync(0xffffffffu, PY, lq);
+            const int op = __shfl_sync(0xffffffffu, okm, lp), oq = __shfl_sync(0xffffffffu, okm, lq);
+            if (u < 72 && op && oq && seg_dist2(px, py, qx, qy) <= R2) hit = true;
+        }
+        if (__any_sync(0xffffffffu, hit)) return true;
     }
     return false;
 }

@@ -462,7 +462,7 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
 // (kMapDirs), sN.
 __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
                               const float4* __restrict__ texels, int T, float4* __restrict__ V, uint32_t* sAM,
-                              float4* sDirs, int* sN, unsigned int gb, unsigned int gn) {
+                              float4* sDirs, int* sN, unsigned int gb, unsigned int gn, bool warp_texel = false) {
     const int MW = g.m * g.W;
     const int ntex = 6 * T * T;
     __syncthreads();
@@ -479,6 +479,23 @@ __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float*
     const int total = *sN;
     if (total == 0) return 0;  // the map is full (early exit): no clear cell to find
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    // few texels for the grid's warps (the map after level 0 of ONE pivot): one WARP per texel, the
+    // lanes share the clear directions (the same maximum as every other path)
+    if (warp_texel && total <= kMapDirs && ntex <= 4 * (int)(gn * nwarps)) {
+        compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
+        for (int t = gb * nwarps + warp; t < ntex; t += gn * nwarps) {
+            const float4 c = texels[t];
+            float best = -2.f;
+            for (int e = lane; e < total; e += 32) best = fmaxf(best, dot3(c, sDirs[e]));
+            best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, 16));
+            best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, 8));
+            best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, 4));
+            best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, 2));
+            best = fmaxf(best, __shfl_xor_sync(0xffffffffu, best, 1));
+            if (lane == 0) V[t] = clear_map_value(best, c.w);
+        }
+        return total;
+    }
 #ifndef AM_ROWSCAN_OVER_DIRS
 #define AM_ROWSCAN_OVER_DIRS 1
 #endif

@@ -114,7 +114,10 @@ def test_enclosing_shell_early_exit(am):
     """P5 / a7: a closed voxel shell around the pivot within the tool's reach blocks every
     orientation; the coarse levels fill the map and the full stream then reads no voxel
     (am_stats.early_exit = 1), on the fused path and on the stage-by-stage path."""
-    C, H = scenes.octree_leaves("shell", (24.0, 20.0), (-32, -32, -32), 64.0, 6)
+    # (0.25 mm cells: ~150K leaves, above the small-model size whose single-pivot kernel has no
+    #  coarse levels)
+    C, H = scenes.octree_leaves("shell", (24.0, 20.0), (-32, -32, -32), 64.0, 8)
+    assert len(H) > 65536
     pivot = (0.5, -0.25, 0.3)
     S = oracle.am_states(C, H, scenes.TOOL_3CYL, pivot, 64, 64)
     assert (S == 2).all()
