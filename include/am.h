@@ -150,13 +150,23 @@ enum {
                                     CUDA graph and replay it while the options, the pivot count,
                                     the output buffer and the model are unchanged (default);
                                     0 = launch every kernel from the host.  Same maps           */
-    AM_OPT_L1_SAMPLE = 22        /* coarse level 1's strided sample of the model, in voxels, taken
+    AM_OPT_L1_SAMPLE = 22,       /* coarse level 1's strided sample of the model, in voxels, taken
                                     at the NEXT am_upload_voxels (0..2^31-1; 0 = library default:
                                     every 384th voxel, at least 24,576).  Approximate: every
                                     floor(N / sample)-th voxel is taken, so the realised sample is
                                     between sample and 2 sample - 1 voxels.  Only the culling
                                     changes (scene-dependent best: profiles/r2x_level_sizes.txt).
                                     Same maps                                                   */
+    AM_OPT_REUSE = 23            /* am_compute_batch, AM reuse between neighbouring pivots
+                                    ("reuse the AM values
+                                    among nearby pivots"): 1 = every map slot remembers the voxels
+                                    whose inner cone set new cells of its map, and the slot's next
+                                    map rasterises their inner cones -- recomputed at the new pivot,
+                                    so exactly -- before level 0, which tightens every clear-
+                                    direction map after it.  Pays when slot s of consecutive calls
+                                    gets consecutive pivots of a toolpath (e.g. call t computes
+                                    pivots s L + t of 64 path segments of L pivots).  0 = off
+                                    (default).  Same maps                                         */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

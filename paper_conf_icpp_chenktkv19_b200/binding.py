@@ -27,6 +27,7 @@ SCHEMES = {"pbox": 0, "pbox_aabb": 1, "pica": 2, "mica": 3, "aica": 4}
 OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
 OPT_BAND_SUBDIV, OPT_CMAP_T1, OPT_CMAP_ROWSCAN, OPT_CMAP_BRUTE, OPT_CMAP_BLOCK, OPT_MAP_CTAS, OPT_SUBBRICKS, OPT_BATCH_LANES, OPT_GRAPH = 13, 14, 15, 16, 17, 18, 19, 20, 21
 OPT_L1_SAMPLE = 22
+OPT_REUSE = 23
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

@@ -48,6 +48,11 @@ __device__ __forceinline__ uint32_t* launch_maps(const FusedParams& F) {
                      : F.gam0;
 }
 
+// AM_OPT_REUSE: the parity of this call (word 2 of the output-base entry written with the pivots).
+__device__ __forceinline__ unsigned int reuse_parity(const FusedParams& F) {
+    return reinterpret_cast<const volatile unsigned int*>(F.out_ptr)[2] & 1u;
+}
+
 // StreamParams of pivot p (slot p) into shared memory (thread 0; the kernel
 // parameter is read by plain member access: a dynamically indexed pointer into
 // a __grid_constant__ parameter is not a global address); `lvl` selects the
@@ -68,6 +73,12 @@ __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParam
     if (threadIdx.x == 0) {
         slot_params(out, F, p, !lvl);
         set_pivot(out, F.piv[p], launch_maps(F) + (size_t)p * F.main.grid.m * F.main.grid.W);
+        if (F.contrib0) {  // AM_OPT_REUSE: this map's contributor list (parity q)
+            const unsigned int q = reuse_parity(F);
+            out.contrib = F.contrib0 + (2ull * p + q) * out.contrib_cap;
+            out.contrib_n = F.contrib_n0 + 2 * p + q;
+            out.contrib_seen = F.seen0 + (unsigned long long)p * F.seen_words;
+        }
     }
     __syncthreads();
 }
@@ -80,6 +91,11 @@ __global__ void __launch_bounds__(kThreads) bk_init(const __grid_constant__ Fuse
     for (int w = threadIdx.x; w < MW; w += blockDim.x) g[w] = 0u;
     unsigned long long* c = shift_bytes(F.ctr0, p * F.ctr_stride);
     for (int w = threadIdx.x; w < F.ctr_words; w += blockDim.x) c[w] = 0ull;
+    if (F.contrib0) {  // (AM_OPT_REUSE) this map's list starts empty
+        if (threadIdx.x == 0) F.contrib_n0[2 * p + reuse_parity(F)] = 0u;
+        unsigned int* seen = F.seen0 + (unsigned long long)p * F.seen_words;
+        for (unsigned int w = threadIdx.x; w < F.seen_words; w += blockDim.x) seen[w] = 0u;
+    }
 }
 
 enum { BK_L0 = 0, BK_L1 = 1, BK_LIVE = 2 };
@@ -101,8 +117,14 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     int* sRowStart = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_rows_offset(m, P.grid.W));
     int nclear = -1;
     unsigned long long n;
+    const unsigned int* prev = nullptr;  // AM_OPT_REUSE: the previous map's contributors of this slot
     if (STAGE == BK_L0) {
         n = F.n0;
+        if (F.contrib0) {
+            const unsigned int q1 = 1u - reuse_parity(F);
+            prev = F.contrib0 + (2ull * p + q1) * P.contrib_cap;
+            n += min(*reinterpret_cast<const volatile unsigned int*>(F.contrib_n0 + 2 * p + q1), P.contrib_cap);
+        }
         for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
         __syncthreads();
     } else {
@@ -131,11 +153,16 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
         ConeRec r;
         if (e < n) {
             if (STAGE == BK_L0) {
-                nrows = cone_of_voxel<true>(P, P.vox[e], (unsigned int)e, r, counted);
+                // level 0, then the previous map's contributors (AM_OPT_REUSE): their inner cones at this
+                // pivot.  Ids: bit 31 = the coarse array (levels 0 and 1), else the model
+                const unsigned int id = e < F.n0 ? (0x80000000u | (unsigned int)e) : prev[e - F.n0];
+                const float4 q = (id & 0x80000000u) ? P.vox_coarse[id & 0x7fffffffu] : P.vox_main[id];
+                nrows = cone_of_voxel<true>(P, q, id, r, counted);
             } else if (STAGE == BK_L1) {
                 const float4 q = F.l1[e];
                 if (fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
-                    nrows = cone_of_voxel<true>(P, q, (unsigned int)e, r, counted, nullptr, -1, F.cmapT1, nullptr, F.texels1);
+                    nrows = cone_of_voxel<true>(P, q, 0x80000000u | (F.n0 + (unsigned int)e), r, counted, nullptr, -1,
+                                                F.cmapT1, nullptr, F.texels1);
             } else {
                 const unsigned int vidx = P.live_idx[e];
                 nrows = cone_of_voxel<false>(P, P.vox[vidx], vidx, r, counted, sDirs, nclear, 0, sRowStart);
@@ -171,6 +198,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     unsigned int rows = 0, rfull = 0;
     for (unsigned long long k = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; k < ntask; k += stride) {
         const unsigned long long t = P.tasks[toff + k];
+        if (t == kInertTask) continue;  // (a cone rasterised inline: see emit_cones)
         const ConeRec r = P.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);

@@ -67,6 +67,13 @@ struct FusedParams {
     // of this launch start out_off words after it.  nullptr: gam0.
     const unsigned long long* out_ptr;
     unsigned long long out_off;
+    // AM_OPT_REUSE (batched path): per slot two contributor lists of contrib_cap voxel indices and two
+    // counts, at contrib0 + (2 slot + parity) contrib_cap and contrib_n0 + 2 slot + parity; a call writes
+    // parity q (read with the output base, word 2 of *out_ptr) and reads 1 - q.  nullptr: off.
+    unsigned int* contrib0;
+    unsigned int* contrib_n0;
+    unsigned int* seen0;      // per slot seen_words words: the listed-coarse-voxel bits (zeroed per map)
+    unsigned int seen_words;
     unsigned long long* ctr0; // slot s's counters: ctr0 + s * ctr_stride bytes, ctr_words 64-bit words
     int ctr_words;
     unsigned int* qnext;      // pivot queue head (zeroed)
@@ -190,6 +197,7 @@ __device__ void fused_rows(const StreamParams& p, const unsigned long long* task
     for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
          k += (unsigned long long)gn * blockDim.x) {
         const unsigned long long t = p.tasks[k];
+        if (t == kInertTask) continue;  // (a cone rasterised inline: see emit_cones)
         const ConeRec r = p.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);
@@ -424,8 +432,11 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
                 }
             }
         } else {
+            // buffers full: rasterise inline, and make the task entries reserved for this cone that lie
+            // inside the task buffer inert (the row pass reads every entry below the capacity)
             for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
             if (slot < slot_cap) p.recs[slot].i0 = -1;
+            for (unsigned long long t = t0; t < t0 + ntask && t < task_cap; ++t) p.tasks[t] = kInertTask;
         }
     }
 }
@@ -513,6 +524,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             for (unsigned long long k = gb * (unsigned long long)blockDim.x + threadIdx.x; k < ntask;
                  k += gstride) {
                 const unsigned long long t = P.tasks[P.task_cap / 2 + k];
+                if (t == kInertTask) continue;
                 const ConeRec r = P.recs[t >> 16];
                 if (r.i0 < 0) continue;
                 const int i = r.i0 + (int)(t & 0xffffu);

@@ -316,6 +316,9 @@ __host__ __device__ inline size_t live_smem_bytes(int m, int W) {
     return (size_t)(m * W + ((m + 31) >> 5)) * sizeof(uint32_t);
 }
 
+// A task entry that names no cone (its cone was rasterised inline when the buffers were full).
+constexpr unsigned long long kInertTask = ~0ull;
+
 // A live voxel's cones and phi-row range, as the row kernel needs them.
 struct ConeRec {
     float cin, cout, clo;  // guarded cone cosines (geometry.cuh Cones)
@@ -444,8 +447,11 @@ __device__ __forceinline__ void emit_cones(const StreamParams& p, int nrows, con
             p.recs[slot] = r;
             for (int k = 0; k < nrows; ++k) p.tasks[t0 + k] = ((unsigned long long)slot << 16) | (unsigned int)k;
         } else {
+            // buffers full: rasterise inline; the record slot and the reserved task entries inside the
+            // buffers are made inert (the row pass reads every entry below the capacities)
             for (int k = 0; k < nrows; ++k) raster_row<COARSE>(p, r, r.i0 + k, p.gam, Counters{nullptr});
-            if (slot < p.rec_cap) p.recs[slot].i0 = -1;  // keep the slot inert
+            if (slot < p.rec_cap) p.recs[slot].i0 = -1;
+            for (unsigned long long t = t0; t < t0 + nrows && t < p.task_cap; ++t) p.tasks[t] = kInertTask;
         }
     }
 }
@@ -484,10 +490,24 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
     if (COARSE) {
         const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
         if (In.len == 0) return;
+        bool fresh_set = false;
         for (int w = 0; w < W; ++w) {
             const uint32_t ib = interval_bits(In, w, g.n);
             uint32_t* wp = am + i * W + w;
-            if (ib & ~*reinterpret_cast<volatile uint32_t*>(wp)) atomicOr(wp, ib);
+            if (ib & ~*reinterpret_cast<volatile uint32_t*>(wp)) {
+                atomicOr(wp, ib);
+                fresh_set = true;
+            }
+        }
+        // (AM_OPT_REUSE: coarse records carry the voxel's id -- bit 31 + index in the coarse array;
+        //  level 0 is processed by every map anyway, the others are listed once)
+        if (fresh_set && p.contrib) {
+            const unsigned int c = r.vidx & 0x7fffffffu;
+            if (!(r.vidx & 0x80000000u) ||
+                (c >= p.contrib_l0 && !(atomicOr(p.contrib_seen + (c >> 5), 1u << (c & 31)) & (1u << (c & 31))))) {
+                const unsigned int pos = atomicAdd(p.contrib_n, 1u);
+                if (pos < p.contrib_cap) p.contrib[pos] = r.vidx;
+            }
         }
         return;
     }
@@ -501,6 +521,7 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
     }
     const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
     const Interval X = gamma_interval(r.clo, rb, rd, r.gv, -1, g);
+    bool fresh_set = false;
     for (int w = 0; w < W; ++w) {
         uint32_t ob = interval_bits(O, w, g.n);
         if (!ob) continue;
@@ -512,6 +533,7 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
         if (ib & ~cur) {
             atomicOr(wp, ib);
             cur |= ib;
+            fresh_set = true;
         }
         uint32_t band = ob & ~ib & ~cur;
         while (band) {
@@ -519,6 +541,10 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
             band &= band - 1u;
             push_band(p, am, r.vidx, p.vox_main[r.vidx], i * g.n + (w << 5) + b, wp, 1u << b, cnt);
         }
+    }
+    if (fresh_set && p.contrib) {  // (AM_OPT_REUSE) this voxel blocked cells: the next map tries it first
+        const unsigned int pos = atomicAdd(p.contrib_n, 1u);
+        if (pos < p.contrib_cap) p.contrib[pos] = r.vidx;
     }
 }
 
@@ -555,6 +581,7 @@ __global__ void __launch_bounds__(kThreads) row_kernel(const __grid_constant__ S
     for (unsigned long long k = blockIdx.x * (unsigned long long)kThreads + threadIdx.x; k < ntask;
          k += (unsigned long long)gridDim.x * kThreads) {
         const unsigned long long t = p.tasks[k];
+        if (t == kInertTask) continue;  // (a cone rasterised inline: see emit_cones)
         const ConeRec r = p.recs[t >> 16];
         if (r.i0 < 0) continue;
         const int i = r.i0 + (int)(t & 0xffffu);

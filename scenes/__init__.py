@@ -110,6 +110,34 @@ def sdf(model: str, points, params=()) -> np.ndarray:
     return out.reshape(np.asarray(points).shape[:-1])
 
 
+def _march_to_offset(model, params, u, offset, c):
+    """The first point along c + t u (0.25 mm steps, then bisection) whose distance bound reaches
+    `offset` and stays there for 2 mm (skips blade gaps); f(pivot) >= offset."""
+    ts = np.arange(0.0, 400.0, 0.25)
+    f = sdf(model, c[None, :] + ts[:, None] * u[None, :], params)
+    idx = np.nonzero(f >= offset)[0]
+    j = None
+    for i in idx:
+        if i > 0 and np.all(f[i: i + 8] >= offset):
+            j = i
+            break
+    if j is None:
+        j = idx[-1]
+    a, b = ts[j - 1], ts[j]
+    for _ in range(50):
+        mid = 0.5 * (a + b)
+        if sdf(model, (c + mid * u)[None, :], params)[0] >= offset:
+            b = mid
+        else:
+            a = mid
+    p = (c + b * u).astype(np.float32)
+    # float32 rounding must not bring the pivot closer than the offset
+    while sdf(model, p.astype(np.float64)[None, :], params)[0] < offset:
+        b += 1e-4
+        p = (c + b * u).astype(np.float32)
+    return p
+
+
 def path_pivots(model: str, params, count: int, offset: float, seed0: int = 1,
                 centre=(0.0, 0.0, 0.0)):
     """Pivots on the offset path: pivot k uses seed seed0 + k.
@@ -124,30 +152,23 @@ def path_pivots(model: str, params, count: int, offset: float, seed0: int = 1,
         rng = np.random.default_rng(seed0 + k)
         u = rng.normal(size=3)
         u /= np.linalg.norm(u)
-        ts = np.arange(0.0, 400.0, 0.25)
-        f = sdf(model, c[None, :] + ts[:, None] * u[None, :], params)
-        idx = np.nonzero(f >= offset)[0]
-        # first crossing that stays outside afterwards for 2 mm (skip blade gaps)
-        j = None
-        for i in idx:
-            if i > 0 and np.all(f[i: i + 8] >= offset):
-                j = i
-                break
-        if j is None:
-            j = idx[-1]
-        a, b = ts[j - 1], ts[j]
-        for _ in range(50):
-            mid = 0.5 * (a + b)
-            if sdf(model, (c + mid * u)[None, :], params)[0] >= offset:
-                b = mid
-            else:
-                a = mid
-        p = (c + b * u).astype(np.float32)
-        # float32 rounding must not bring the pivot closer than the offset
-        while sdf(model, p.astype(np.float64)[None, :], params)[0] < offset:
-            b += 1e-4
-            p = (c + b * u).astype(np.float32)
-        out[k] = p
+        out[k] = _march_to_offset(model, params, u, offset, c)
+    return out
+
+
+def toolpath_pivots(model: str, params, count: int, offset: float, centre=(0.0, 0.0, 0.0), turns: float = 16.0):
+    """A continuous toolpath on the offset surface (PAPER.md L311, 8(f) NEXT 2): directions on a
+    spherical spiral (z from +1 to -1, `turns` turns), each marched from ``centre`` to the offset
+    surface like path_pivots, so consecutive pivots are neighbours (about 0.5 mm apart for 4096
+    pivots on the head) except where the spiral crosses into another sheet of the surface."""
+    out = np.empty((count, 3), dtype=np.float32)
+    c = np.asarray(centre, dtype=np.float64)
+    for k in range(count):
+        z = 1.0 - 2.0 * (k + 0.5) / count
+        phi = 2.0 * np.pi * turns * k / count
+        rxy = np.sqrt(max(0.0, 1.0 - z * z))
+        u = np.array([rxy * np.cos(phi), rxy * np.sin(phi), z])
+        out[k] = _march_to_offset(model, params, u, offset, c)
     return out
 
 
@@ -182,6 +203,11 @@ class Config:
         off = max(self.offset, 2.0 * np.sqrt(3.0) * self.min_half() + 0.05)
         extra = path_pivots(self.model, self.params, count - len(fixed), off, seed0, self.centre)
         return np.concatenate([np.stack(fixed) if fixed else np.zeros((0, 3), np.float32), extra])
+
+    def toolpath(self, count: int, turns: float = 16.0):
+        """`count` consecutive pivots of a continuous toolpath (toolpath_pivots)."""
+        off = max(self.offset, 2.0 * np.sqrt(3.0) * self.min_half() + 0.05)
+        return toolpath_pivots(self.model, self.params, count, off, self.centre, turns)
 
     def pivots_at(self, indices):
         """Pivots number k of the path for k in `indices` (pivots_at(range(n)) == pivots(n)):

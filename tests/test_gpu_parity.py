@@ -413,3 +413,56 @@ def test_band_subdivision_matches_oracle(am, name, subdiv):
         assert mism == 0
         assert int((g != am.unpack(ref[k], cfg.m, cfg.n))[S != 1].sum()) == 0
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "C2"])
+def test_reuse_between_neighbouring_pivots_same_maps(am, name):
+    """AM_OPT_REUSE (8(f) NEXT 2): each slot first rasterises the inner cones, at its
+    new pivot, of the voxels that set cells of its previous map.  Any voxel's inner cone at the new
+    pivot is exact, so the maps stay bit-identical -- on a continuous toolpath in slot-segment order
+    (the intended use), on random pivots, after an option change and after a re-upload."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    path = cfg.toolpath(64)
+    ctx = _ctx(am, cfg, C, H)
+    ref = np.stack([ctx.compute(p)[0] for p in path])
+    ctx.set_option(am.binding.OPT_BATCH, 16)
+    ctx.set_option(am.binding.OPT_REUSE, 1)
+    seg = path.reshape(16, 4, 3)  # 16 slots, each 4 consecutive path pivots
+    for t in range(4):
+        got = ctx.compute_batch(seg[:, t])
+        assert np.array_equal(got, ref.reshape(16, 4, -1)[:, t]), t
+    rnd = cfg.pivots(16)
+    ref_r = np.stack([ctx.compute(p)[0] for p in rnd])
+    assert np.array_equal(ctx.compute_batch(rnd), ref_r)
+    ctx.set_option(am.binding.OPT_BATCH_LANES, 2)
+    assert np.array_equal(ctx.compute_batch(seg[:, 0]), ref.reshape(16, 4, -1)[:, 0])
+    ctx.upload(C, H)
+    assert np.array_equal(ctx.compute_batch(seg[:, 1]), ref.reshape(16, 4, -1)[:, 1])
+    ctx.close()
+
+
+def test_record_and_task_overflow_is_exact(am):
+    """When the cone-record / row-task buffers of a stage overflow (C3 with only one coarse level,
+    so that ~10^5 voxels per map reach the live stage), the cones that do not fit are rasterised
+    inline and the task entries reserved for them are made inert; the batched maps then equal the
+    single-pivot maps (whose kernel rasterises in shared memory) and the oracle on every robust cell.
+    These toolpath pivots gave robust-clear cells marked blocked before the inert entries (stale
+    tasks of an earlier map)."""
+    import torch
+    cfg = scenes.CONFIGS["C3"]
+    C, H = cfg.leaves()
+    path = cfg.toolpath(4096)
+    P = path[[75, 2322, 2897, 3226, 3250, 3915]]
+    ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=0)
+    ctx.upload(torch.from_numpy(C).cuda(), torch.from_numpy(H).cuda())
+    ctx.set_option(am.binding.OPT_PHASES, 1)
+    ctx.set_option(am.binding.OPT_BATCH, 64)
+    got = ctx.compute_batch(P)
+    single = np.stack([ctx.compute(p)[0] for p in P])
+    assert np.array_equal(got, single)
+    from test_gpu_fullsize import full_oracle_map
+    S = full_oracle_map(cfg, C, H, P[-1])
+    mism, _ = _compare(am.unpack(got[-1], cfg.m, cfg.n), S)
+    assert mism == 0
+    ctx.close()
