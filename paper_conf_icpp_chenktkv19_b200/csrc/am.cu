@@ -169,15 +169,13 @@ struct am_ctx {
     unsigned long long* d_bctl = nullptr;  // batched launch: group barriers, pivot queue
     int fused_grid = 0;
     int lat_grid = 0;                      // am_latency_kernel: co-resident CTAs (cooperative launch)
-    // AM_OPT_REUSE (8(f) NEXT 2): per slot, two lists of the voxels that set bits of its last maps
+    // AM_OPT_REUSE (8(f) NEXT 2): per slot, two per-cell witness arrays and a dedupe set
     int reuse = 0;
-    unsigned int* d_contrib = nullptr;     // slots x 2 x kContribCap voxel indices
-    unsigned int* d_contrib_n = nullptr;   // slots x 2 counts
-    unsigned int* d_seen = nullptr;        // slots x seen_words: coarse voxels already listed
-    unsigned int seen_words = 0;
+    unsigned int* d_wit = nullptr;         // slots x 2 x m n voxel ids
+    unsigned int* d_hash = nullptr;        // slots x hash_words
+    unsigned int hash_words = 0;
     int contrib_slots = 0;
     unsigned int reuse_parity = 0;         // the list this call writes (the other is read)
-    bool reuse_warm = false;               // the slots hold lists: level 1 and the first map are skipped
     size_t smem_fused = 0;
     float bbox[6] = {0, 0, 0, 0, 0, 0};    // centre bounding box of the resident model
     // kernel timing (AM_OPT_KERNEL_TIMING)
@@ -219,7 +217,6 @@ constexpr int kMaxBatch = 64;                // pivots per layered batch launch 
 constexpr int kBctlWords = 2 * kMaxSlots + 1 + kMaxSlots / 2;  // bars, then queue head + per-group pivot (u32)
 constexpr unsigned int kRecCap = 1u << 20;   // cone records per stage (more: rows rasterised inline)
 constexpr unsigned long long kTaskCap = 1ull << 22;  // (voxel, row) tasks per stage
-constexpr unsigned int kContribCap = 16384;  // AM_OPT_REUSE: contributors kept per map
 
 int fail(am_ctx* c, int code, const char* fmt, ...) {
     if (c) {
@@ -681,7 +678,6 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.main.task_cap = kTaskCap;
     F.main.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
     F.main.live_idx = ctx->d_live;
-    F.main.contrib_cap = kContribCap;
     F.lvl = F.main;
     F.lvl.vox = ctx->d_coarse;
     F.lvl.N = ctx->n_l0;
@@ -913,10 +909,9 @@ void shift_slots(FusedParams& F, int base) {
     F.rec1 = hshift(F.rec1, b * F.ctr_stride);
     F.task1 = hshift(F.task1, b * F.ctr_stride);
     F.ctr0 = hshift(F.ctr0, b * F.ctr_stride);
-    if (F.contrib0) {
-        F.contrib0 += b * 2 * kContribCap;
-        F.contrib_n0 += b * 2;
-        F.seen0 += b * F.seen_words;
+    if (F.wit0) {
+        F.wit0 += b * 2 * (unsigned long long)F.main.grid.m * F.main.grid.n;
+        F.hash0 += b * F.hash_words;
     }
 }
 
@@ -934,23 +929,20 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
     int rc;
     if ((rc = ensure_slots(ctx, K)) != AM_OK) return rc;
     if ((rc = ensure_piv(ctx, P)) != AM_OK) return rc;
-    const unsigned int seen_words = (unsigned int)((ctx->n_l1 + 31) / 32) + 1;
-    if (ctx->reuse && (ctx->contrib_slots < ctx->slots || ctx->seen_words < seen_words)) {  // AM_OPT_REUSE lists
-        cudaFree(ctx->d_contrib);
-        cudaFree(ctx->d_contrib_n);
-        cudaFree(ctx->d_seen);
-        ctx->d_contrib = nullptr;
-        ctx->d_contrib_n = nullptr;
-        ctx->d_seen = nullptr;
+    const size_t mn = (size_t)ctx->grid.m * ctx->grid.n;
+    if (ctx->reuse && ctx->contrib_slots < ctx->slots) {  // AM_OPT_REUSE witness arrays (no witness at first)
+        cudaFree(ctx->d_wit);
+        cudaFree(ctx->d_hash);
+        ctx->d_wit = nullptr;
+        ctx->d_hash = nullptr;
         ctx->contrib_slots = 0;
-        ctx->seen_words = 0;
-        CK(cudaMalloc(&ctx->d_contrib, (size_t)ctx->slots * 2 * kContribCap * sizeof(unsigned int)));
-        CK(cudaMalloc(&ctx->d_contrib_n, (size_t)ctx->slots * 2 * sizeof(unsigned int)));
-        CK(cudaMalloc(&ctx->d_seen, (size_t)ctx->slots * seen_words * sizeof(unsigned int)));
-        ctx->seen_words = seen_words;
-        CK(cudaMemset(ctx->d_contrib_n, 0, (size_t)ctx->slots * 2 * sizeof(unsigned int)));
+        unsigned int hw = 1;
+        while (hw < 2 * mn) hw <<= 1;
+        CK(cudaMalloc(&ctx->d_wit, (size_t)ctx->slots * 2 * mn * sizeof(unsigned int)));
+        CK(cudaMalloc(&ctx->d_hash, (size_t)ctx->slots * hw * sizeof(unsigned int)));
+        CK(cudaMemset(ctx->d_wit, 0xff, (size_t)ctx->slots * 2 * mn * sizeof(unsigned int)));
+        ctx->hash_words = hw;
         ctx->contrib_slots = ctx->slots;
-        ctx->reuse_warm = false;
         ++ctx->gen;
     }
     {
@@ -958,7 +950,6 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         if ((rc = upload_pivots(ctx, pivots, P, gam0, s)) != AM_OK) return rc;
     }
     if (ctx->reuse) ctx->reuse_parity ^= 1u;  // (the next call reads what this one writes)
-    const bool warm_next = ctx->reuse != 0;    // after this call every slot it used holds a list
     const int ntex = 6 * ctx->cmapT * ctx->cmapT;
     const size_t sm_rows = (size_t)(ctx->MW + ((ctx->grid.m + 31) >> 5) + 1) * sizeof(uint32_t);
     // one chunk of kk pivots from c0 on, slots [sb, sb + kk), on stream s
@@ -969,14 +960,9 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.out_ptr = reinterpret_cast<const unsigned long long*>(ctx->d_piv + P);  // the call's output base
         F.out_off = (unsigned long long)c0 * ctx->MW;
         if (ctx->reuse) {
-            F.contrib0 = ctx->d_contrib;
-            F.contrib_n0 = ctx->d_contrib_n;
-            F.seen0 = ctx->d_seen;
-            F.seen_words = ctx->seen_words;
-            F.main.contrib_l0 = F.lvl.contrib_l0 = (unsigned int)ctx->n_l0;
-            // warm slots: level 0 and the previous map's contributors already give nearly the final
-            // map, so the map after them is built once at full resolution and level 1 is skipped
-            if (ctx->reuse_warm && !(ctx->diag & 32)) F.use_l1 = 0;
+            F.wit0 = ctx->d_wit;
+            F.hash0 = ctx->d_hash;
+            F.hash_words = ctx->hash_words;
         }
         F.nslot = kk;
         F.ctr_stride = (unsigned long long)kCtrStride * sizeof(unsigned long long);
@@ -1006,7 +992,8 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         };
         bk_init<<<kk, b, 0, s>>>(F);  // this chunk's maps and counters start at zero
         AM_KM(AM_K_INIT);
-        bk_cones<BK_L0><<<grid(ctx->n_l0 + (ctx->reuse ? kContribCap : 0), kThreads, 1 << 16), b, sm_rows, s>>>(F);
+        bk_cones<BK_L0><<<grid(ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0), kThreads, 1 << 16), b, sm_rows,
+                          s>>>(F);
         AM_KM(AM_K_L0_CONES);
         if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
         AM_KM(AM_K_L0_ROWS);
@@ -1113,18 +1100,6 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         for (int k = 0; k < AM_K_COUNT; ++k) ctx->k_launches[k] += ctx->g_launches[k];
     } else {
         if ((rc = chain(s))) return rc;
-    }
-    if (ctx->reuse && getenv("AM_DEBUG_REUSE")) {  // (temporary debug)
-        std::vector<unsigned int> cn((size_t)ctx->contrib_slots * 2);
-        cudaStreamSynchronize(s);
-        cudaMemcpy(cn.data(), ctx->d_contrib_n, cn.size() * 4, cudaMemcpyDeviceToHost);
-        fprintf(stderr, "reuse warm %d parity-written %u counts:", (int)ctx->reuse_warm, ctx->reuse_parity ^ 1u);
-        for (int k = 0; k < 8; ++k) fprintf(stderr, " %u/%u", cn[2 * k], cn[2 * k + 1]);
-        fprintf(stderr, "\n");
-    }
-    if (warm_next != ctx->reuse_warm) {  // (the chain changes: a new graph)
-        ctx->reuse_warm = warm_next;
-        ++ctx->gen;
     }
     return timed_end(ctx, s);
 }
@@ -1550,9 +1525,8 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
         ctx->n_l0 = n0;
         ctx->n_l1 = n1 + ns;
     }
-    if (ctx->d_contrib_n)  // (AM_OPT_REUSE lists name voxels of the previous model)
-        UK(cudaMemset(ctx->d_contrib_n, 0, (size_t)ctx->contrib_slots * 2 * sizeof(unsigned int)));
-    ctx->reuse_warm = false;
+    if (ctx->d_wit)  // (AM_OPT_REUSE witnesses name voxels of the previous model)
+        UK(cudaMemset(ctx->d_wit, 0xff, (size_t)ctx->contrib_slots * 2 * ctx->grid.m * ctx->grid.n * sizeof(unsigned int)));
     UK(cudaDeviceSynchronize());
 #undef UK
     cleanup();
@@ -1714,7 +1688,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
-        if (value < 0 || value > 63) return fail(ctx, AM_EINVAL, "diag must be in [0, 63]");
+        if (value < 0 || value > 31) return fail(ctx, AM_EINVAL, "diag must be in [0, 31]");
         if ((value & 3) && !ctx->d_prev) {
             CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
@@ -1773,7 +1747,6 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_REUSE:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "reuse must be 0 or 1");
         ctx->reuse = (int)value;
-        ctx->reuse_warm = false;
         return AM_OK;
     case AM_OPT_L1_SAMPLE:
         if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "l1_sample must be in [0, 2^31-1]");
@@ -2116,9 +2089,8 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_olink);
     cudaFree(ctx->d_omemo);
     cudaFree(ctx->d_ostats);
-    cudaFree(ctx->d_contrib);
-    cudaFree(ctx->d_contrib_n);
-    cudaFree(ctx->d_seen);
+    cudaFree(ctx->d_wit);
+    cudaFree(ctx->d_hash);
     for (auto e : ctx->kev) cudaEventDestroy(e);
     for (auto e : ctx->ev_start) cudaEventDestroy(e);
     for (auto e : ctx->ev_stop) cudaEventDestroy(e);

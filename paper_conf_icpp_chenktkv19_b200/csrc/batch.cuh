@@ -48,6 +48,21 @@ __device__ __forceinline__ uint32_t* launch_maps(const FusedParams& F) {
                      : F.gam0;
 }
 
+constexpr unsigned int kNoWitness = 0xffffffffu;
+
+// Insert id into the open-addressing set hs (nwords a power of 2, empty = kNoWitness): true when it
+// was not there yet (the caller then owns the id).
+__device__ __forceinline__ bool hash_insert(unsigned int* hs, unsigned int nwords, unsigned int id) {
+    unsigned int h = (id * 2654435761u) & (nwords - 1u);
+    for (unsigned int k = 0; k < nwords; ++k) {
+        const unsigned int old = atomicCAS(hs + h, kNoWitness, id);
+        if (old == kNoWitness) return true;
+        if (old == id) return false;
+        h = (h + 1u) & (nwords - 1u);
+    }
+    return true;  // (full: process it anyway)
+}
+
 // AM_OPT_REUSE: the parity of this call (word 2 of the output-base entry written with the pivots).
 __device__ __forceinline__ unsigned int reuse_parity(const FusedParams& F) {
     return reinterpret_cast<const volatile unsigned int*>(F.out_ptr)[2] & 1u;
@@ -73,12 +88,8 @@ __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParam
     if (threadIdx.x == 0) {
         slot_params(out, F, p, !lvl);
         set_pivot(out, F.piv[p], launch_maps(F) + (size_t)p * F.main.grid.m * F.main.grid.W);
-        if (F.contrib0) {  // AM_OPT_REUSE: this map's contributor list (parity q)
-            const unsigned int q = reuse_parity(F);
-            out.contrib = F.contrib0 + (2ull * p + q) * out.contrib_cap;
-            out.contrib_n = F.contrib_n0 + 2 * p + q;
-            out.contrib_seen = F.seen0 + (unsigned long long)p * F.seen_words;
-        }
+        if (F.wit0)  // AM_OPT_REUSE: this map's witnesses (parity q)
+            out.wit = F.wit0 + (2ull * p + reuse_parity(F)) * (out.grid.m * out.grid.n);
     }
     __syncthreads();
 }
@@ -91,10 +102,12 @@ __global__ void __launch_bounds__(kThreads) bk_init(const __grid_constant__ Fuse
     for (int w = threadIdx.x; w < MW; w += blockDim.x) g[w] = 0u;
     unsigned long long* c = shift_bytes(F.ctr0, p * F.ctr_stride);
     for (int w = threadIdx.x; w < F.ctr_words; w += blockDim.x) c[w] = 0ull;
-    if (F.contrib0) {  // (AM_OPT_REUSE) this map's list starts empty
-        if (threadIdx.x == 0) F.contrib_n0[2 * p + reuse_parity(F)] = 0u;
-        unsigned int* seen = F.seen0 + (unsigned long long)p * F.seen_words;
-        for (unsigned int w = threadIdx.x; w < F.seen_words; w += blockDim.x) seen[w] = 0u;
+    if (F.wit0) {  // (AM_OPT_REUSE) no witness yet; an empty dedupe set
+        const int mn = F.main.grid.m * F.main.grid.n;
+        unsigned int* wit = F.wit0 + (2ull * p + reuse_parity(F)) * mn;
+        for (int w = threadIdx.x; w < mn; w += blockDim.x) wit[w] = kNoWitness;
+        unsigned int* hs = F.hash0 + (unsigned long long)p * F.hash_words;
+        for (unsigned int w = threadIdx.x; w < F.hash_words; w += blockDim.x) hs[w] = kNoWitness;
     }
 }
 
@@ -117,13 +130,15 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     int* sRowStart = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_rows_offset(m, P.grid.W));
     int nclear = -1;
     unsigned long long n;
-    const unsigned int* prev = nullptr;  // AM_OPT_REUSE: the previous map's contributors of this slot
+    const unsigned int* prev = nullptr;  // AM_OPT_REUSE: the previous map's witnesses of this slot
+    unsigned int* hs = nullptr;
     if (STAGE == BK_L0) {
         n = F.n0;
-        if (F.contrib0) {
-            const unsigned int q1 = 1u - reuse_parity(F);
-            prev = F.contrib0 + (2ull * p + q1) * P.contrib_cap;
-            n += min(*reinterpret_cast<const volatile unsigned int*>(F.contrib_n0 + 2 * p + q1), P.contrib_cap);
+        if (F.wit0) {
+            const unsigned int mn = (unsigned int)(P.grid.m * P.grid.n);
+            prev = F.wit0 + (2ull * p + (1u - reuse_parity(F))) * mn;
+            hs = F.hash0 + (unsigned long long)p * F.hash_words;
+            n += mn;
         }
         for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
         __syncthreads();
@@ -153,11 +168,14 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
         ConeRec r;
         if (e < n) {
             if (STAGE == BK_L0) {
-                // level 0, then the previous map's contributors (AM_OPT_REUSE): their inner cones at this
-                // pivot.  Ids: bit 31 = the coarse array (levels 0 and 1), else the model
-                const unsigned int id = e < F.n0 ? (0x80000000u | (unsigned int)e) : prev[e - F.n0];
-                const float4 q = (id & 0x80000000u) ? P.vox_coarse[id & 0x7fffffffu] : P.vox_main[id];
-                nrows = cone_of_voxel<true>(P, q, id, r, counted);
+                // level 0, then the previous map's witnesses (AM_OPT_REUSE), each once: their inner cones
+                // at this pivot.  Ids: bit 31 = the coarse array (levels 0 and 1), else the model
+                unsigned int id = e < F.n0 ? (0x80000000u | (unsigned int)e) : prev[e - F.n0];
+                if (e >= F.n0 && (id == kNoWitness || !hash_insert(hs, F.hash_words, id))) id = kNoWitness;
+                if (id != kNoWitness) {
+                    const float4 q = (id & 0x80000000u) ? P.vox_coarse[id & 0x7fffffffu] : P.vox_main[id];
+                    nrows = cone_of_voxel<true>(P, q, id, r, counted);
+                }
             } else if (STAGE == BK_L1) {
                 const float4 q = F.l1[e];
                 if (fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)

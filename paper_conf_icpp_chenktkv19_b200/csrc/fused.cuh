@@ -67,13 +67,12 @@ struct FusedParams {
     // of this launch start out_off words after it.  nullptr: gam0.
     const unsigned long long* out_ptr;
     unsigned long long out_off;
-    // AM_OPT_REUSE (batched path): per slot two contributor lists of contrib_cap voxel indices and two
-    // counts, at contrib0 + (2 slot + parity) contrib_cap and contrib_n0 + 2 slot + parity; a call writes
-    // parity q (read with the output base, word 2 of *out_ptr) and reads 1 - q.  nullptr: off.
-    unsigned int* contrib0;
-    unsigned int* contrib_n0;
-    unsigned int* seen0;      // per slot seen_words words: the listed-coarse-voxel bits (zeroed per map)
-    unsigned int seen_words;
+    // AM_OPT_REUSE (batched path): per slot two witness arrays of m n voxel ids at wit0 + (2 slot +
+    // parity) m n (a call writes parity q -- read with the output base, word 2 of *out_ptr -- and
+    // reads 1 - q) and a hash set of hash_words ids (power of 2) that dedupes the witnesses it reads.
+    unsigned int* wit0;
+    unsigned int* hash0;
+    unsigned int hash_words;
     unsigned long long* ctr0; // slot s's counters: ctr0 + s * ctr_stride bytes, ctr_words 64-bit words
     int ctr_words;
     unsigned int* qnext;      // pivot queue head (zeroed)

@@ -79,14 +79,11 @@ struct StreamParams {
     unsigned int* brick_list;      // bricks kept by brick_test_kernel (capacity nbricks)
     unsigned int* brick_count;     // zeroed per map
     int band_vdepth;               // band pairs: virtual sub-cube levels before CHECKBOX (§4.3)
-    // AM reuse between neighbouring pivots (AM_OPT_REUSE; 8(f) NEXT 2): the live voxels
-    // whose inner cone set new bits of this map are appended here (nullptr: off); the slot's next map
-    // rasterises their inner cones -- at its own pivot, so exactly -- before level 0
-    unsigned int* contrib;
-    unsigned int* contrib_n;
-    unsigned int contrib_cap;
-    unsigned int* contrib_seen;    // one bit per coarse voxel already listed (a voxel sets cells in many rows)
-    unsigned int contrib_l0;       // coarse ids below this (level 0, processed anyway) are not listed
+    // AM reuse between neighbouring pivots (AM_OPT_REUSE; 8(f) NEXT 2): per cell of this
+    // map, the id of a voxel whose inner cone set it (nullptr: off; ids: bit 31 = coarse array).  The
+    // slot's next map rasterises the inner cones of these witnesses -- at its own pivot, so exactly --
+    // with level 0
+    unsigned int* wit;
     // sub-bricks of 32 consecutive voxels (one warp of a brick): bounding spheres;
     // nullptr = not tested
     const float4* __restrict__ subs;

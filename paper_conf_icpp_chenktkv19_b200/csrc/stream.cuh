@@ -327,6 +327,18 @@ struct ConeRec {
     int i0;                // first phi-row of the outer cone
 };
 
+// AM_OPT_REUSE: voxel `id` set the cells `fresh` of word w of row i (in this CTA's view): it becomes
+// their witness (any voxel whose inner cone holds a cell is a valid one; the last writer wins).
+__device__ __forceinline__ void note_witness(const StreamParams& p, unsigned int id, int i, int w, uint32_t fresh) {
+    if (!p.wit) return;
+    unsigned int* row = p.wit + i * p.grid.n + (w << 5);
+    while (fresh) {
+        const int b = __ffs(fresh) - 1;
+        fresh &= fresh - 1u;
+        row[b] = id;
+    }
+}
+
 // Rows of a voxel processed inline when the record/task buffers are full
 // (correct, only slower).
 template <bool COARSE>
@@ -490,23 +502,13 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
     if (COARSE) {
         const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
         if (In.len == 0) return;
-        bool fresh_set = false;
         for (int w = 0; w < W; ++w) {
             const uint32_t ib = interval_bits(In, w, g.n);
             uint32_t* wp = am + i * W + w;
-            if (ib & ~*reinterpret_cast<volatile uint32_t*>(wp)) {
+            const uint32_t fresh = ib & ~*reinterpret_cast<volatile uint32_t*>(wp);
+            if (fresh) {
                 atomicOr(wp, ib);
-                fresh_set = true;
-            }
-        }
-        // (AM_OPT_REUSE: coarse records carry the voxel's id -- bit 31 + index in the coarse array;
-        //  level 0 is processed by every map anyway, the others are listed once)
-        if (fresh_set && p.contrib) {
-            const unsigned int c = r.vidx & 0x7fffffffu;
-            if (!(r.vidx & 0x80000000u) ||
-                (c >= p.contrib_l0 && !(atomicOr(p.contrib_seen + (c >> 5), 1u << (c & 31)) & (1u << (c & 31))))) {
-                const unsigned int pos = atomicAdd(p.contrib_n, 1u);
-                if (pos < p.contrib_cap) p.contrib[pos] = r.vidx;
+                note_witness(p, r.vidx, i, w, fresh);
             }
         }
         return;
@@ -521,7 +523,6 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
     }
     const Interval In = gamma_interval(r.cin, rb, rd, r.gv, -1, g);
     const Interval X = gamma_interval(r.clo, rb, rd, r.gv, -1, g);
-    bool fresh_set = false;
     for (int w = 0; w < W; ++w) {
         uint32_t ob = interval_bits(O, w, g.n);
         if (!ob) continue;
@@ -532,8 +533,8 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
         uint32_t cur = *reinterpret_cast<volatile uint32_t*>(wp);
         if (ib & ~cur) {
             atomicOr(wp, ib);
+            note_witness(p, r.vidx, i, w, ib & ~cur);
             cur |= ib;
-            fresh_set = true;
         }
         uint32_t band = ob & ~ib & ~cur;
         while (band) {
@@ -541,10 +542,6 @@ __device__ void raster_row(const StreamParams& p, const ConeRec& r, int i, uint3
             band &= band - 1u;
             push_band(p, am, r.vidx, p.vox_main[r.vidx], i * g.n + (w << 5) + b, wp, 1u << b, cnt);
         }
-    }
-    if (fresh_set && p.contrib) {  // (AM_OPT_REUSE) this voxel blocked cells: the next map tries it first
-        const unsigned int pos = atomicAdd(p.contrib_n, 1u);
-        if (pos < p.contrib_cap) p.contrib[pos] = r.vidx;
     }
 }
 
