@@ -157,7 +157,7 @@ enum {
                                     between sample and 2 sample - 1 voxels.  Only the culling
                                     changes (scene-dependent best: profiles/r2x_level_sizes.txt).
                                     Same maps                                                   */
-    AM_OPT_REUSE = 23            /* am_compute_batch, AM reuse between neighbouring pivots
+    AM_OPT_REUSE = 23,           /* am_compute_batch, AM reuse between neighbouring pivots
                                     ("reuse the AM values
                                     among nearby pivots"): 1 = every map slot remembers the voxels
                                     whose inner cone set new cells of its map, and the slot's next
@@ -167,6 +167,13 @@ enum {
                                     gets consecutive pivots of a toolpath (e.g. call t computes
                                     pivots s L + t of 64 path segments of L pivots).  0 = off
                                     (default).  Same maps                                         */
+    AM_OPT_STAGE_FUSION = 24     /* am_compute_batch: 1 = each stage (level 0, level 1, the kept
+                                    voxels) is ONE launch whose filter survivors, cones and rows
+                                    stay in shared memory (stage.cuh); 0 = cone and row kernels
+                                    with records and tasks in device memory (default: measured
+                                    faster with 64 maps in flight, C3 6.4 vs 10.8 us per map --
+                                    the one-launch stages pay off for ONE map, am_compute).  Same
+                                    maps                                                         */
 };
 
 /* Kernels of the library, for am_kernel_stats. */
@@ -189,6 +196,9 @@ enum {
     AM_K_ICA_MEMO,      /* am_compute_octree: parallel ICA calculation of the top S levels     */
     AM_K_OCTREE,        /* am_compute_octree: one thread per orientation, Alg. 2               */
     AM_K_INIT,          /* batched path: zero a chunk's maps and per-map counters              */
+    AM_K_LEVEL0,        /* batched, AM_OPT_STAGE_FUSION: level 0 (+ reuse witnesses), cones + rows  */
+    AM_K_LEVEL1,        /* batched, AM_OPT_STAGE_FUSION: level-1 filter, cones + rows             */
+    AM_K_STREAM,        /* batched, AM_OPT_STAGE_FUSION: kept voxels' filter, cones, rows, band queue */
     AM_K_COUNT
 };
 

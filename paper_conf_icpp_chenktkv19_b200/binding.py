@@ -21,13 +21,14 @@ LIB_PATH = os.environ.get("AM_LIBRARY") or os.path.join(_HERE, "libam.so")
 
 AM_OK, AM_EINVAL, AM_ENOMEM, AM_ECUDA, AM_ESTATE = 0, -1, -2, -3, -4
 OPT_GRID_CTAS, OPT_REFRESH_TILES, OPT_MORTON_SORT, OPT_BASELINE_REJECT, OPT_BAND_QUEUE = 1, 2, 3, 4, 5
-K_COUNT = 17  # AM_K_COUNT (include/am.h)
+K_COUNT = 20  # AM_K_COUNT (include/am.h)
 SCHEME_PBOX, SCHEME_PBOX_AABB, SCHEME_PICA, SCHEME_MICA, SCHEME_AICA = 0, 1, 2, 3, 4  # AM_SCHEME_*
 SCHEMES = {"pbox": 0, "pbox_aabb": 1, "pica": 2, "mica": 3, "aica": 4}
 OPT_KERNEL_TIMING, OPT_PHASES, OPT_DIAG, OPT_CMAP_T, OPT_BRICKS, OPT_FUSED, OPT_BATCH = 6, 7, 8, 9, 10, 11, 12
 OPT_BAND_SUBDIV, OPT_CMAP_T1, OPT_CMAP_ROWSCAN, OPT_CMAP_BRUTE, OPT_CMAP_BLOCK, OPT_MAP_CTAS, OPT_SUBBRICKS, OPT_BATCH_LANES, OPT_GRAPH = 13, 14, 15, 16, 17, 18, 19, 20, 21
 OPT_L1_SAMPLE = 22
 OPT_REUSE = 23
+OPT_STAGE_FUSION = 24
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

@@ -22,6 +22,7 @@
 #include "fused.cuh"
 #include "batch.cuh"
 #include "latency.cuh"
+#include "stage.cuh"
 #include "octree.cuh"
 
 #include <algorithm>
@@ -171,6 +172,7 @@ struct am_ctx {
     int lat_grid = 0;                      // am_latency_kernel: co-resident CTAs (cooperative launch)
     // AM_OPT_REUSE (8(f) NEXT 2): per slot, two per-cell witness arrays and a dedupe set
     int reuse = 0;
+    int stage_fusion = 0;                  // AM_OPT_STAGE_FUSION: one kernel per batched stage (stage.cuh)
     unsigned int* d_wit = nullptr;         // slots x 2 x m n voxel ids
     unsigned int* d_hash = nullptr;        // slots x hash_words
     unsigned int hash_words = 0;
@@ -539,6 +541,9 @@ int configure_launch(am_ctx* ctx) {
     CK(cudaFuncSetAttribute(bk_rows<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_map<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     CK(cudaFuncSetAttribute(bk_map<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_level0, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     return AM_OK;
 }
 
@@ -992,11 +997,16 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         };
         bk_init<<<kk, b, 0, s>>>(F);  // this chunk's maps and counters start at zero
         AM_KM(AM_K_INIT);
-        bk_cones<BK_L0><<<grid(ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0), kThreads, 1 << 16), b, sm_rows,
-                          s>>>(F);
-        AM_KM(AM_K_L0_CONES);
-        if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
-        AM_KM(AM_K_L0_ROWS);
+        const long long n0e = ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0);  // (+ reuse witnesses)
+        if (ctx->stage_fusion) {
+            if ((rc = L(bk_level0, grid(n0e, kThreads, 32), ctx->smem_fused))) return rc;
+            AM_KM(AM_K_LEVEL0);
+        } else {
+            bk_cones<BK_L0><<<grid(n0e, kThreads, 1 << 16), b, sm_rows, s>>>(F);
+            AM_KM(AM_K_L0_CONES);
+            if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
+            AM_KM(AM_K_L0_ROWS);
+        }
         if (F.use_l1) {
             // (few texels, many clear cells after level 0: spread them over more CTAs -- one
             // warp per 4 x 4 coarse texel on the coarse-block path)
@@ -1011,10 +1021,17 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
-            if ((rc = L(bk_cones<BK_L1>, grid(ctx->n_l1 - ctx->n_l0, AM_L1_STEPS * kThreads, 1 << 16), sm_rows))) return rc;
-            AM_KM(AM_K_L1_CONES);
-            if ((rc = L(bk_rows<BK_L1>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
-            AM_KM(AM_K_L1_ROWS);
+            if (ctx->stage_fusion) {
+                if ((rc = L(bk_level1, grid(ctx->n_l1 - ctx->n_l0, kThreads, ctx->bk_cone_ctas), ctx->smem_fused)))
+                    return rc;
+                AM_KM(AM_K_LEVEL1);
+            } else {
+                if ((rc = L(bk_cones<BK_L1>, grid(ctx->n_l1 - ctx->n_l0, AM_L1_STEPS * kThreads, 1 << 16), sm_rows)))
+                    return rc;
+                AM_KM(AM_K_L1_CONES);
+                if ((rc = L(bk_rows<BK_L1>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
+                AM_KM(AM_K_L1_ROWS);
+            }
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
         }
@@ -1024,12 +1041,17 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, F.main.supers ? AM_BRICKS_CTAS : (1 << 16)), 0))) return rc;
         AM_KM(AM_K_BRICKS);
-        if ((rc = L(bk_voxels, grid(1 << 30, 1, ctx->bk_voxel_ctas), 0))) return rc;
-        AM_KM(AM_K_VOXELS);
-        if ((rc = L(bk_cones<BK_LIVE>, grid(1 << 30, 1, ctx->bk_cone_ctas), ctx->smem_fused))) return rc;
-        AM_KM(AM_K_LIVE_CONES);
-        if ((rc = L(bk_rows<BK_LIVE>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
-        AM_KM(AM_K_LIVE_ROWS);
+        if (ctx->stage_fusion) {
+            if ((rc = L(bk_stream, grid(1 << 30, 1, ctx->bk_voxel_ctas), ctx->smem_fused))) return rc;
+            AM_KM(AM_K_STREAM);
+        } else {
+            if ((rc = L(bk_voxels, grid(1 << 30, 1, ctx->bk_voxel_ctas), 0))) return rc;
+            AM_KM(AM_K_VOXELS);
+            if ((rc = L(bk_cones<BK_LIVE>, grid(1 << 30, 1, ctx->bk_cone_ctas), ctx->smem_fused))) return rc;
+            AM_KM(AM_K_LIVE_CONES);
+            if ((rc = L(bk_rows<BK_LIVE>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
+            AM_KM(AM_K_LIVE_ROWS);
+        }
         // (few pairs, each a long exact test: small CTAs spread them over the SMs)
         if ((rc = L(bk_band, grid(1 << 30, 1, AM_BAND_CTAS), 0, dim3(AM_BAND_THREADS)))) return rc;
         AM_KM(AM_K_BAND);
@@ -1748,6 +1770,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "reuse must be 0 or 1");
         ctx->reuse = (int)value;
         return AM_OK;
+    case AM_OPT_STAGE_FUSION:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "stage_fusion must be 0 or 1");
+        ctx->stage_fusion = (int)value;
+        return AM_OK;
     case AM_OPT_L1_SAMPLE:
         if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "l1_sample must be in [0, 2^31-1]");
         ctx->l1_sample = value;  // taken at the next am_upload_voxels
@@ -1806,7 +1832,7 @@ const char* am_kernel_name(int k) {
     static const char* names[AM_K_COUNT] = {
         "l0_cones", "l0_rows", "clear_map", "l1_cones", "l1_rows", "bricks", "voxels",
         "live_cones", "live_rows", "band", "fused_pipeline", "filter", "baseline", "layout",
-        "ica_memo", "octree", "init"};
+        "ica_memo", "octree", "init", "level0", "level1", "stream"};
     return (k >= 0 && k < AM_K_COUNT) ? names[k] : nullptr;
 }
 

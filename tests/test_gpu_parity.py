@@ -466,3 +466,24 @@ def test_record_and_task_overflow_is_exact(am):
     mism, _ = _compare(am.unpack(got[-1], cfg.m, cfg.n), S)
     assert mism == 0
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "T_imp", "C2"])
+def test_stage_fusion_same_maps(am, name):
+    """AM_OPT_STAGE_FUSION (stage.cuh): one launch per batched stage with survivors, cones and rows
+    in shared memory gives the maps of the split cone / row kernels bit for bit, with and without
+    AM_OPT_REUSE, on random pivots and on a toolpath."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_BATCH, 16)
+    for P in (cfg.pivots(16), cfg.toolpath(16)):
+        ctx.set_option(am.binding.OPT_STAGE_FUSION, 0)
+        ref = ctx.compute_batch(P)
+        ctx.set_option(am.binding.OPT_STAGE_FUSION, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 0)
+    ctx.close()
