@@ -180,7 +180,12 @@ def _config_dict(cfg, N, flushed=True, batch=1, slots=1, lanes=1, split="pivot",
          "l2": (f"inputs {16 * N / 1e6:.0f} MB; L2 (126 MB) flushed by a {2 * L2_BYTES >> 20} MB write before "
                 f"every timed step, outside the per-step CUDA events") if flushed else
                f"inputs {16 * N / 1e6:.0f} MB; no flush"}
-    if split == "pivot":
+    if split == "toolpath":
+        d.update({"pivots_per_step": batch, "pivots_per_launch": max(1, slots // lanes), "streams": lanes,
+                  "distinct_pivots_per_rank": npiv,
+                  "parallelism": "pivot-sharded (weak): rank r a contiguous sub-path; step t = pivot s L + t of "
+                                 "each of the batch's path segments (AM_OPT_REUSE)"})
+    elif split == "pivot":
         d.update({"pivots_per_step": batch, "pivots_per_launch": max(1, slots // lanes), "streams": lanes,
                   "distinct_pivots_per_rank": npiv, "parallelism": "pivot-sharded (weak)"})
     else:
@@ -343,6 +348,8 @@ def _apply_options(ctx, B, args):
         if getattr(args, flag) >= 0:
             ctx.set_option(key, getattr(args, flag))
     ctx.set_option(B.OPT_BATCH_LANES, args.lanes)
+    if args.stage_fusion >= 0:
+        ctx.set_option(B.OPT_STAGE_FUSION, args.stage_fusion)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
 
@@ -371,10 +378,20 @@ def _run_pivot_split(args, am, torch, dist, dev, cfg, C, H, gen_s, ws, rank):
     npiv = args.pivots or min(4096, max(args.steps, 1) * bsz)
     npiv = max(npiv, bsz) // bsz * bsz
     t = time.time()
-    piv = cfg.pivots_at(range(rank, npiv * ws, ws))  # pivot sharding: rank r takes pivots r, r + G, ...
+    if args.toolpath:
+        # a continuous toolpath (8(f) NEXT 2): rank r takes the contiguous sub-path r; within it, step
+        # t computes pivot s L + t of its bsz segments of L pivots, so slot s of consecutive steps gets
+        # neighbouring pivots (AM_OPT_REUSE reuses the slot's previous map)
+        path = cfg.toolpath(npiv * ws)[rank * npiv:(rank + 1) * npiv]
+        L = npiv // bsz
+        piv = np.ascontiguousarray(path.reshape(bsz, L, 3).transpose(1, 0, 2).reshape(-1, 3))
+    else:
+        piv = cfg.pivots_at(range(rank, npiv * ws, ws))  # pivot sharding: rank r takes pivots r, r + G, ...
     piv_s = time.time() - t
     ctx = am.Context(cfg.tool, cfg.m, cfg.n, device=dev.index)
     _apply_options(ctx, B, args)
+    if args.toolpath:
+        ctx.set_option(B.OPT_REUSE, 1)
     t0 = time.time()
     ctx.upload(torch.from_numpy(C).to(dev), torch.from_numpy(H).to(dev))
     torch.cuda.synchronize(dev)
@@ -423,6 +440,17 @@ def _run_pivot_split(args, am, torch, dist, dev, cfg, C, H, gen_s, ws, rank):
     kw = max(1, min(args.steps, 200))
     ms_warm, _ = _timed_maps(ctx, piv, out, stream, kw, None, torch, bsz)
     ctx.kernel_time()
+    reuse_off = None
+    if args.toolpath:  # the same steps without AM_OPT_REUSE (maps checked equal)
+        ctx.set_option(B.OPT_REUSE, 0)
+        o2 = torch.zeros_like(out)
+        _timed_maps(ctx, piv, o2, stream, 3, None, torch, bsz)
+        ms_off, _ = _timed_maps(ctx, piv, o2, stream, args.steps, flush, torch, bsz)
+        ctx.kernel_time()
+        same = bool(torch.equal(o2[:steps_done * bsz], out[:steps_done * bsz]))
+        reuse_off = {"ms_per_am": ms_off / args.steps / bsz, "reuse_speedup": ms_off / ms, "maps_identical": same,
+                     "median_step_mm": float(np.median(np.linalg.norm(np.diff(path, axis=0), axis=1)))}
+        ctx.set_option(B.OPT_REUSE, 1)
     # ---- full-scan leg: every voxel read by filter_kernel (no brick skipping, one launch per stage)
     full = None
     if not args.no_full_scan:
@@ -521,7 +549,8 @@ def _run_pivot_split(args, am, torch, dist, dev, cfg, C, H, gen_s, ws, rank):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": _config_dict(cfg, N, flush is not None, bsz, args.slots, args.lanes, "pivot", len(piv)),
+            "config": _config_dict(cfg, N, flush is not None, bsz, args.slots, args.lanes,
+                                   "toolpath" if args.toolpath else "pivot", len(piv)),
             "ms_per_am": ms_max / args.steps / bsz,
             "roofline": dom_roof,
             "step_roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -556,6 +585,7 @@ def _run_pivot_split(args, am, torch, dist, dev, cfg, C, H, gen_s, ws, rank):
                        "scene_gen_s": gen_s, "pivot_gen_s": piv_s,
                        "blocked_fraction_mean": blocked_frac, "distinct_pivots_timed": steps_done * bsz,
                        "pivots_per_rank": len(piv),
+                       "toolpath_reuse_off": reuse_off,
                        "single_pivot_ms_per_am": ms_single / ks,
                        "single_pivot_kernel_ms": ks_k / max(ks_l, 1),
                        "warm_l2_ms_per_am": ms_warm / kw / bsz, "timed_wall_ms_incl_flush": wall_ms,
@@ -762,6 +792,10 @@ def main(argv=None):
     ap.add_argument("--band-subdiv", type=int, default=0,
                     help="AM_OPT_BAND_SUBDIV: virtual sub-cube levels before CHECKBOX (PAPER.md 4.3)")
     ap.add_argument("--no-full-scan", action="store_true", help="skip the full-scan (filter_kernel) leg")
+    ap.add_argument("--toolpath", action="store_true",
+                    help="pivots of a continuous toolpath in slot-segment order, AM_OPT_REUSE on (8(f) NEXT 2); "
+                         "the same steps without reuse in detail.toolpath_reuse_off")
+    ap.add_argument("--stage-fusion", type=int, default=-1, help="AM_OPT_STAGE_FUSION (-1 = library default)")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3
