@@ -487,3 +487,21 @@ def test_stage_fusion_same_maps(am, name):
         assert np.array_equal(ctx.compute_batch(P), ref)
         ctx.set_option(am.binding.OPT_REUSE, 0)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["C1", "T_head", "T_imp", "C2"])
+def test_latency_kernel_matches_previous_single_pivot_kernel(am, name):
+    """am_compute's single-pivot kernel (am_latency_kernel: 7 phases, CTA raster, warp-parallel
+    CHECKBOX) gives the maps of the previous cooperative kernel (AM_OPT_DIAG bit 4) and of the
+    batched path bit for bit, including the small-model variant (no coarse levels)."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    P = cfg.pivots(6)
+    ctx = _ctx(am, cfg, C, H)
+    new = np.stack([ctx.compute(p)[0] for p in P])
+    ctx.set_option(am.binding.OPT_DIAG, 16)
+    old = np.stack([ctx.compute(p)[0] for p in P])
+    ctx.set_option(am.binding.OPT_DIAG, 0)
+    assert np.array_equal(new, old)
+    assert np.array_equal(ctx.compute_batch(P), new)
+    ctx.close()
