@@ -31,19 +31,29 @@ for w in $WHAT; do
     launches)
       timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
         --log-file $OUT/launches_$TAG.csv python bench.py --steps 20 --warmup 3 > $OUT/launches_$TAG.log 2>&1
-      echo "launches rc=$?" ;;
+      echo "launches rc=$?"
+      mkdir -p $OUT/prof_summ; PROF_DIR=$OUT/prof_summ python tools/summarize_ncu.py $TAG C3 64 > /dev/null 2>&1
+      gzip -f $OUT/launches_$TAG.csv ;;
     full)
       for c in C3 C2 C4 C5; do
         timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bk_ -s ${KSKIP:-26} -c 13 \
           -o $OUT/prof_${TAG}_$c -f python bench.py --config $c --steps 4 --warmup 3 --lanes 1 --no-cpu-baseline \
           --no-baseline --e2e-steps 1 --no-full-scan > $OUT/full_${TAG}_$c.log 2>&1
         echo "full $c rc=$?"
+        # (summarised here: the reports would exceed what gpurun brings back)
+        mkdir -p $OUT/prof_summ; [ -f $OUT/prof_summ/ncu_summary.json ] || cp profiles/ncu_summary.json $OUT/prof_summ/
+        PROF_DIR=$OUT/prof_summ python tools/summarize_ncu.py ${TAG}_$c $c 64 > /dev/null 2>&1
+        rm -f $OUT/prof_${TAG}_$c.ncu-rep
       done ;;
     latency)
       for c in C3 C1; do
         timeout 600 ncu --set full --clock-control none --import-source on -k regex:am_latency_kernel -s 4 -c 1 \
           -o $OUT/prof_${TAG}_lat_$c -f python tools/sp_one.py $c 2 > $OUT/lat_${TAG}_$c.log 2>&1
         echo "latency $c rc=$?"
+        mkdir -p $OUT/prof_summ
+        PROF_DIR=$OUT/prof_summ python tools/summarize_ncu.py ${TAG}_lat_$c $c 1 > /dev/null 2>&1
+        python tools/ncu_src.py $OUT/prof_${TAG}_lat_$c.ncu-rep 40 > $OUT/prof_summ/${TAG}_lat_${c}_source_top.txt 2>&1
+        [ "$c" = "C3" ] || rm -f $OUT/prof_${TAG}_lat_$c.ncu-rep
       done ;;
     sp)
       for c in C1 C2 C3 C5; do SP_PER_PIVOT=1 timeout 300 python tools/sp_sweep.py $c "" "OPT_DIAG=16"; done > $OUT/sp_$TAG.txt 2>&1

@@ -25,7 +25,8 @@ def base_name(k):
 
 
 _STAGES = {"bk_cones": ("l0_cones", "l1_cones", "live_cones"), "bk_rows": ("l0_rows", "l1_rows", "live_rows")}
-_PLAIN = {"bk_map": "clear_map", "bk_bricks": "bricks", "bk_voxels": "voxels", "bk_band": "band",
+_PLAIN = {"am_latency_kernel": "fused_pipeline", "bk_init": "init", "bk_level0": "level0", "bk_level1": "level1",
+          "bk_stream": "stream", "bk_map": "clear_map", "bk_bricks": "bricks", "bk_voxels": "voxels", "bk_band": "band",
           "am_pipeline_kernel": "fused_pipeline", "filter_kernel": "filter", "baseline_kernel": "baseline",
           "clear_map_kernel": "clear_map", "band_exact_kernel": "band", "brick_test_kernel": "bricks",
           "brick_voxels_kernel": "voxels"}
@@ -50,7 +51,7 @@ def main():
     tag = sys.argv[1]
     config = sys.argv[2] if len(sys.argv) > 2 else "C3"
     maps = int(sys.argv[3]) if len(sys.argv) > 3 else 1  # AMs computed by the captured launch
-    prof = os.path.join(ROOT, "profiles")
+    prof = os.environ.get("PROF_DIR") or os.path.join(ROOT, "profiles")  # (on the GPU box: under gpurun_out/)
     os.makedirs(prof, exist_ok=True)
     lc = os.path.join(ROOT, "gpurun_out", f"launches_{tag}.csv")
     if os.path.exists(lc):
