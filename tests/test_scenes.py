@@ -54,3 +54,22 @@ def test_pivots_are_on_the_offset_path_and_outside_the_voxels():
         assert not inside.any()
     # seeded: same seeds -> same pivots
     assert np.array_equal(P, cfg.pivots(6))
+
+
+def test_pivots_at_matches_pivots_and_toolpath_is_continuous():
+    """pivots_at(indices) gives pivots(n)[indices] (a rank generates only its own); the toolpath's
+    pivots are on the offset surface, outside every voxel, and consecutive ones are neighbours."""
+    cfg = scenes.CONFIGS["T_head"]
+    P = cfg.pivots(7)
+    assert np.array_equal(cfg.pivots_at(range(7)), P)
+    assert np.array_equal(cfg.pivots_at([5, 2]), P[[5, 2]])
+    C, H = cfg.leaves()
+    T = cfg.toolpath(1024)
+    off = max(cfg.offset, 2 * np.sqrt(3) * cfg.min_half() + 0.05)
+    f = scenes.sdf(cfg.model, T.astype(np.float64))
+    assert (f >= off).all()
+    for p in T[::64]:
+        assert not np.all(np.abs(C - p[None, :]) <= H[:, None], axis=1).any()
+    step = np.linalg.norm(np.diff(T, axis=0), axis=1)
+    rnd = np.linalg.norm(P[:, None, :] - P[None, :, :], axis=2)[np.triu_indices(7, 1)]
+    assert np.median(step) < 0.1 * np.median(rnd)  # neighbours, unlike the seeded pivots (~40 mm apart)

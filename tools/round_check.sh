@@ -20,7 +20,8 @@ for w in $WHAT; do
     bench) timeout 900 python bench.py --steps 20 --warmup 3 > $OUT/bench_$TAG.log 2>&1; echo "bench rc=$?"; tail -c 400 $OUT/bench_$TAG.log; echo ;;
     others)
       for c in C2 C4 C5; do
-        timeout 600 python bench.py --config $c --steps 20 --warmup 3 --no-cpu-baseline > $OUT/bench_${TAG}_$c.log 2>&1; echo "bench $c rc=$?"
+        S=20; [ "$c" = "C5" ] && S=64  # (C5: the whole 4096-pivot toolpath batch of BASELINE configs[4])
+        timeout 600 python bench.py --config $c --steps $S --pivots 4096 --warmup 3 --no-cpu-baseline > $OUT/bench_${TAG}_$c.log 2>&1; echo "bench $c rc=$?"
       done ;;
     toolpath)
       for c in C5 C4 C3; do
