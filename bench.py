@@ -142,6 +142,13 @@ def launch_ranks(argv, gpus):
     return subprocess.call(cmd)
 
 
+def _device_index(local):
+    """One GPU per rank; more ranks than GPUs share them round robin (a plumbing check only --
+    AM_BENCH_BACKEND=gloo then, NCCL refuses two ranks on one GPU)."""
+    import torch
+    return local % max(1, torch.cuda.device_count())
+
+
 def _init_dist(ws, local, cuda):
     """Process group of the ranks: NCCL over NVLink on GPUs, gloo on CPU (tests)."""
     if ws <= 1:
@@ -149,8 +156,8 @@ def _init_dist(ws, local, cuda):
     import torch
     import torch.distributed as dist
     if cuda:
-        torch.cuda.set_device(local)
-    dist.init_process_group("nccl" if cuda else "gloo")
+        torch.cuda.set_device(_device_index(local))
+    dist.init_process_group(os.environ.get("AM_BENCH_BACKEND") or ("nccl" if cuda else "gloo"))
     return dist
 
 
@@ -358,7 +365,7 @@ def run_ours(args):
     import torch
     ws, rank, local = _dist_env()
     dist = _init_dist(ws, local, cuda=True)
-    dev = torch.device("cuda", local if ws > 1 else 0)
+    dev = torch.device("cuda", _device_index(local) if ws > 1 else 0)
     torch.cuda.set_device(dev)
     import paper_conf_icpp_chenktkv19_b200 as am
     cfg, C, H, gen_s = _scene(args.config)
