@@ -167,13 +167,28 @@ enum {
                                     gets consecutive pivots of a toolpath (e.g. call t computes
                                     pivots s L + t of 64 path segments of L pivots).  0 = off
                                     (default).  Same maps                                         */
-    AM_OPT_STAGE_FUSION = 24     /* am_compute_batch: 1 = each stage (level 0, level 1, the kept
+    AM_OPT_STAGE_FUSION = 24,    /* am_compute_batch: 1 = each stage (level 0, level 1, the kept
                                     voxels) is ONE launch whose filter survivors, cones and rows
                                     stay in shared memory (stage.cuh); 0 = cone and row kernels
                                     with records and tasks in device memory (default: measured
                                     faster with 64 maps in flight, C3 6.4 vs 10.8 us per map --
                                     the one-launch stages pay off for ONE map, am_compute).  Same
                                     maps                                                         */
+    AM_OPT_STREAM_TMA = 25,      /* full-stream filter (AM_OPT_BRICKS = 0): north_star "voxel loads
+                                    staged via TMA".  1..3 = filter_tma(_ws)_kernel: persistent CTAs
+                                    whose 16 KB voxel tiles arrive in shared memory by 1-D bulk
+                                    copies (cp.async.bulk completing on an mbarrier, L2 evict-first)
+                                    -- 1: a producer warp refills a 2-stage ring as soon as the 8
+                                    consumer warps release a stage (empty mbarriers); 2: 2 stages,
+                                    thread 0 refills after a CTA barrier; 3: as 1 with 4 stages.
+                                    0 = filter_kernel, 4 LDG.128 per thread (default: the filter is
+                                    issue-bound, ~85 instructions per voxel, so the TMA rings measure
+                                    0.56-0.61 of HBM on C3 against 0.65).  Same maps              */
+    AM_OPT_PDL = 26              /* am_compute_batch: 1 = each phase kernel of a lane is a
+                                    programmatic dependent launch (griddepcontrol): its CTAs are
+                                    scheduled under the previous phase's tail and copy their
+                                    parameters there, then wait for the previous phase's writes
+                                    (default); 0 = plain stream order.  Same maps                 */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

@@ -29,6 +29,8 @@ OPT_BAND_SUBDIV, OPT_CMAP_T1, OPT_CMAP_ROWSCAN, OPT_CMAP_BRUTE, OPT_CMAP_BLOCK, 
 OPT_L1_SAMPLE = 22
 OPT_REUSE = 23
 OPT_STAGE_FUSION = 24
+OPT_STREAM_TMA = 25
+OPT_PDL = 26
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

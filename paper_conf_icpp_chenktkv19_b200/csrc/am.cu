@@ -92,6 +92,23 @@ constexpr int kMaxLanes = 8;
 #define AM_L1_MIN_SAMPLE 24576
 #endif
 
+// AM_OPT_STREAM_TMA ring shapes of filter_tma_kernel: (voxels per thread per tile, stages)
+// AM_OPT_STREAM_TMA values: ring shapes of the TMA-staged full-stream filter (stream.cuh), as
+// (voxels per thread per tile, stages); measured on B200 (C3, profiles/r5_tma_sweep.txt) all below
+// the LDG filter_kernel, which is the default (0)
+constexpr int kTmaShapes = 3;
+inline const void* tma_kernel(int k) {
+    switch (k) {
+        case 1: return (const void*)filter_tma_ws_kernel<4, 2>;  // warp-specialised producer, 32 KB ring
+        case 2: return (const void*)filter_tma_kernel<4, 2>;     // CTA barrier per tile, 32 KB ring
+        default: return (const void*)filter_tma_ws_kernel<4, 4>; // warp-specialised producer, 64 KB ring
+    }
+}
+inline int tma_stages(int k) { return k == 3 ? 4 : 2; }
+inline size_t tma_smem(int k) { return (size_t)tma_stages(k) * 4 * kThreads * sizeof(float4); }
+inline int tma_threads(int k) { return k == 2 ? kThreads : kThreads + 32; }
+inline long long tma_tile_vox(int) { return 4ll * kThreads; }
+
 struct am_ctx {
     int device = 0;
     int sms = 0;
@@ -173,6 +190,9 @@ struct am_ctx {
     // AM_OPT_REUSE (8(f) NEXT 2): per slot, two per-cell witness arrays and a dedupe set
     int reuse = 0;
     int stage_fusion = 0;                  // AM_OPT_STAGE_FUSION: one kernel per batched stage (stage.cuh)
+    int stream_tma = 0;                    // AM_OPT_STREAM_TMA: full-stream filter with TMA-staged tiles
+    int pdl = 1;                           // AM_OPT_PDL: batched phases as programmatic dependent launches
+    int occ_tma[8] = {};                   // filter_tma_kernel: CTAs per SM, per ring shape
     unsigned int* d_wit = nullptr;         // slots x 2 x m n voxel ids
     unsigned int* d_hash = nullptr;        // slots x hash_words
     unsigned int hash_words = 0;
@@ -507,6 +527,16 @@ int configure_launch(am_ctx* ctx) {
                     ctx->grid.n, ctx->smem);
     }
     ctx->occ = occ;
+    // the TMA-staged full-stream filter (one ring shape per AM_OPT_STREAM_TMA value)
+    for (int k = 1; k <= kTmaShapes; ++k) {
+        ctx->occ_tma[k] = 0;
+        const void* fn = tma_kernel(k);
+        const size_t sm = tma_smem(k);
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm) != cudaSuccess ||
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ_tma[k], fn, tma_threads(k), sm) != cudaSuccess)
+            ctx->occ_tma[k] = 0;
+    }
+    cudaGetLastError();
     // the fused pipeline: all CTAs co-resident (cooperative launch)
     ctx->smem_fused = fused_smem_bytes(m, ctx->grid.W);
     ctx->fused_grid = 0;
@@ -613,6 +643,16 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
         if ((rc = kmark(ctx, s, AM_K_BRICKS))) return rc;
         brick_voxels_kernel<<<(unsigned)gmax, kThreads, 0, s>>>(p);
         if ((rc = kmark(ctx, s, AM_K_VOXELS))) return rc;
+    } else if (ctx->stream_tma && ctx->occ_tma[ctx->stream_tma] > 0) {
+        const int k = ctx->stream_tma;
+        const long long tiles = (n + tma_tile_vox(k) - 1) / tma_tile_vox(k);
+        long long gt = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ_tma[k];
+        if (gt > tiles) gt = tiles;
+        if (gt < 1) gt = 1;
+        void* args[] = {&p};
+        CK(cudaLaunchKernel(tma_kernel(k), dim3((unsigned)gt), dim3(tma_threads(k)), args, tma_smem(k), s));
+        int rc;
+        if ((rc = kmark(ctx, s, AM_K_FILTER))) return rc;
     } else {
         filter_kernel<<<(unsigned)g, kThreads, 0, s>>>(p);
         int rc;
@@ -991,8 +1031,24 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         const dim3 b(kThreads);
         const int map_cap = ctx->bk_map_ctas > 0 ? ctx->bk_map_ctas : (1 << 16);
 #define AM_KM(k) if ((rc = kmark(ctx, s, k))) return rc
+        // (AM_OPT_PDL: programmatic stream serialisation -- the kernel's CTAs may start under the previous
+        //  kernel's tail and run their parameter prologue there; batch.cuh grid_dep_wait orders the rest)
         auto L = [&](auto kern, dim3 g, size_t smem, dim3 bd = dim3(kThreads)) -> int {
-            kern<<<g, bd, smem, s>>>(F);
+            if (ctx->pdl) {
+                cudaLaunchConfig_t lc{};
+                lc.gridDim = g;
+                lc.blockDim = bd;
+                lc.dynamicSmemBytes = smem;
+                lc.stream = s;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+                at[0].val.programmaticStreamSerializationAllowed = 1;
+                lc.attrs = at;
+                lc.numAttrs = 1;
+                CK(cudaLaunchKernelEx(&lc, kern, F));
+            } else {
+                kern<<<g, bd, smem, s>>>(F);
+            }
             return AM_OK;
         };
         bk_init<<<kk, b, 0, s>>>(F);  // this chunk's maps and counters start at zero
@@ -1002,7 +1058,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             if ((rc = L(bk_level0, grid(n0e, kThreads, 32), ctx->smem_fused))) return rc;
             AM_KM(AM_K_LEVEL0);
         } else {
-            bk_cones<BK_L0><<<grid(n0e, kThreads, 1 << 16), b, sm_rows, s>>>(F);
+            if ((rc = L(bk_cones<BK_L0>, grid(n0e, kThreads, 1 << 16), sm_rows))) return rc;
             AM_KM(AM_K_L0_CONES);
             if ((rc = L(bk_rows<BK_L0>, grid(1 << 30, 1, ctx->bk_rows_ctas), sm_rows))) return rc;
             AM_KM(AM_K_L0_ROWS);
@@ -1175,6 +1231,33 @@ int print_phase_times(am_ctx* ctx) {
         if (t[k] >= t[0] && t[k]) fprintf(stderr, " %d:%.1f", k, (t[k] - t[0]) * 1e-3);
     fprintf(stderr, "\n");
     CK(cudaMemset(ctx->d_ts, 0, sizeof t));
+    // am_latency_kernel: per-CTA P6 end (us after the kernel start), live voxels, rows, filter survivors
+    std::vector<unsigned long long> c(4 * kDiagCtas);
+    CK(cudaMemcpy(c.data(), ctx->d_ts + 16, c.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+    std::vector<std::pair<double, int>> ends;
+    for (int b = 0; b < kDiagCtas; ++b)
+        if (c[4 * b] >= t[0] && c[4 * b]) ends.push_back({(c[4 * b] - t[0]) * 1e-3, b});
+    if (!ends.empty()) {
+        std::sort(ends.begin(), ends.end());
+        const size_t nE = ends.size();
+        fprintf(stderr, "am P6 per CTA (%zu): end us min %.1f med %.1f p90 %.1f max %.1f;", nE, ends[0].first,
+                ends[nE / 2].first, ends[(nE * 9) / 10].first, ends[nE - 1].first);
+        for (size_t k = nE >= 3 ? nE - 3 : 0; k < nE; ++k) {
+            const int b = ends[k].second;
+            fprintf(stderr, " cta %d: %.1f us live %llu rows %llu passed %llu;", b, ends[k].first, c[4 * b + 1],
+                    c[4 * b + 2], c[4 * b + 3]);
+        }
+        unsigned long long lmax = 0, lsum = 0, rmax = 0, rsum = 0;
+        for (auto& e : ends) {
+            lmax = std::max(lmax, c[4 * e.second + 1]);
+            lsum += c[4 * e.second + 1];
+            rmax = std::max(rmax, c[4 * e.second + 2]);
+            rsum += c[4 * e.second + 2];
+        }
+        fprintf(stderr, " live max %llu mean %.1f, rows max %llu mean %.1f\n", lmax, (double)lsum / nE, rmax,
+                (double)rsum / nE);
+        CK(cudaMemset(ctx->d_ts + 16, 0, c.size() * sizeof(unsigned long long)));
+    }
     return AM_OK;
 }
 
@@ -1716,8 +1799,8 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
         }
         if ((value & 4) && !ctx->d_ts) {
-            CK(cudaMalloc(&ctx->d_ts, 16 * sizeof(unsigned long long)));
-            CK(cudaMemset(ctx->d_ts, 0, 16 * sizeof(unsigned long long)));
+            CK(cudaMalloc(&ctx->d_ts, (16 + 4 * kDiagCtas) * sizeof(unsigned long long)));
+            CK(cudaMemset(ctx->d_ts, 0, (16 + 4 * kDiagCtas) * sizeof(unsigned long long)));
         }
         ctx->diag = (int)value;
         ctx->diag_ts = (value & 4) != 0;
@@ -1773,6 +1856,14 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_STAGE_FUSION:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "stage_fusion must be 0 or 1");
         ctx->stage_fusion = (int)value;
+        return AM_OK;
+    case AM_OPT_PDL:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "pdl must be 0 or 1");
+        ctx->pdl = (int)value;
+        return AM_OK;
+    case AM_OPT_STREAM_TMA:
+        if (value < 0 || value > kTmaShapes) return fail(ctx, AM_EINVAL, "stream_tma must be in [0, %d]", kTmaShapes);
+        ctx->stream_tma = (int)value;
         return AM_OK;
     case AM_OPT_L1_SAMPLE:
         if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "l1_sample must be in [0, 2^31-1]");

@@ -48,6 +48,15 @@ __device__ __forceinline__ uint32_t* launch_maps(const FusedParams& F) {
                      : F.gam0;
 }
 
+// Programmatic dependent launch (AM_OPT_PDL): the batched kernels of a lane are launched with
+// programmatic stream serialisation, so a kernel's CTAs are scheduled while the previous kernel's
+// last CTAs still run and do their parameter prologue meanwhile; before touching anything the
+// previous kernels wrote (counts, maps, lists) every thread waits here for them to complete and
+// their writes to be visible.  A no-op for a kernel launched without the attribute.  Every CTA of a
+// batched kernel passes it (also on its early-exit paths), so a kernel completes only after its
+// predecessor did -- the dependency stays transitive along the lane.
+__device__ __forceinline__ void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 constexpr unsigned int kNoWitness = 0xffffffffu;
 
 // Insert id into the open-addressing set hs (nwords a power of 2, empty = kNoWitness): true when it
@@ -84,6 +93,7 @@ __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParam
         const uint32_t* src = reinterpret_cast<const uint32_t*>(&F.main);
         for (int w = threadIdx.x; w < kWords; w += blockDim.x) dst[w] = src[w];
     }
+    grid_dep_wait();
     __syncthreads();
     if (threadIdx.x == 0) {
         slot_params(out, F, p, !lvl);
@@ -94,8 +104,66 @@ __device__ __forceinline__ void pivot_params(StreamParams& out, const FusedParam
     __syncthreads();
 }
 
+// The prologue of a batched kernel (every thread calls it; ends CTA-uniformly): pivot_params plus
+// the phase's work count and the early-exit check, with every device-memory read the CTA needs --
+// pivot, output base, reuse parity, the count `cnt` (32- or 64-bit, slot-shifted by the caller from
+// the kernel parameters) and the map's early-exit flag -- issued by thread 0 BEFORE the parameter
+// copy, so their latency overlaps it (pivot_params reads them after its first barrier, and every
+// kernel read its count and the flag after pivot_params).  Returns true when the CTA has nothing to
+// do: the map is full (check_early; a7) or its first item `first` lies at or past the count;
+// n = min(count, cap).
+__device__ __forceinline__ bool bk_prologue(StreamParams& out, const FusedParams& F, int p, bool lvl, const void* cnt,
+                                            bool wide, unsigned long long cap, unsigned long long first,
+                                            bool check_early, unsigned long long& n) {
+    __shared__ unsigned long long s_n;
+    __shared__ int s_exit;
+    constexpr int kWords = (int)(sizeof(StreamParams) / 4);
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    unsigned long long ob = 0ull;
+    unsigned int par = 0u;
+    if (threadIdx.x == 0) {  // (the call's inputs: written before the lane's first kernel)
+        v = F.piv[p];
+        if (F.out_ptr) {
+            ob = *reinterpret_cast<const volatile unsigned long long*>(F.out_ptr);
+            if (F.wit0) par = reinterpret_cast<const volatile unsigned int*>(F.out_ptr)[2] & 1u;
+        }
+    }
+    uint32_t* dst = reinterpret_cast<uint32_t*>(&out);
+    if (lvl) {
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(&F.lvl);
+        for (int w = threadIdx.x; w < kWords; w += blockDim.x) dst[w] = src[w];
+    } else {
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(&F.main);
+        for (int w = threadIdx.x; w < kWords; w += blockDim.x) dst[w] = src[w];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        slot_params(out, F, p, !lvl);
+        uint32_t* base = F.out_ptr ? reinterpret_cast<uint32_t*>(ob) + F.out_off : F.gam0;
+        set_pivot(out, v, base + (size_t)p * F.main.grid.m * F.main.grid.W);
+        if (F.wit0) out.wit = F.wit0 + (2ull * p + par) * (out.grid.m * out.grid.n);
+    }
+    grid_dep_wait();  // (everything below reads what the previous kernels wrote)
+    if (threadIdx.x == 0) {
+        unsigned long long c = ~0ull;
+        if (cnt)
+            c = wide ? *reinterpret_cast<const volatile unsigned long long*>(cnt)
+                     : (unsigned long long)*reinterpret_cast<const volatile unsigned int*>(cnt);
+        const bool full =
+            check_early &&
+            *reinterpret_cast<const volatile unsigned long long*>(shift_bytes(F.main.early, p * F.ctr_stride)) != 0ull;
+        const unsigned long long nn = c < cap ? c : cap;
+        s_n = nn;
+        s_exit = full || first >= nn;
+    }
+    __syncthreads();
+    n = s_n;
+    return s_exit != 0;  // (CTA-uniform)
+}
+
 // First launch of a chunk: zero the maps and the per-slot counters of its pivots (blockIdx.x = pivot).
 __global__ void __launch_bounds__(kThreads) bk_init(const __grid_constant__ FusedParams F) {
+    grid_dep_wait();
     const int p = blockIdx.x;
     const int MW = F.main.grid.m * F.main.grid.W;
     uint32_t* g = launch_maps(F) + (size_t)p * MW;
@@ -121,7 +189,14 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     __shared__ StreamParams sP;
     __shared__ FusedScratch sc;
     const int p = blockIdx.y;
-    pivot_params(sP, F, p, STAGE == BK_L0);
+    unsigned long long n;
+    {
+        const void* cnt = STAGE == BK_LIVE ? (const void*)shift_bytes(F.main.live_count, p * F.ctr_stride) : nullptr;
+        const unsigned long long cap = STAGE == BK_L0 ? ~0ull : (STAGE == BK_L1 ? (unsigned long long)F.n1 : ~0ull);
+        if (bk_prologue(sP, F, p, STAGE == BK_L0, cnt, false, cap, (unsigned long long)blockIdx.x * blockDim.x,
+                        STAGE != BK_L0, n))
+            return;
+    }
     const StreamParams& P = sP;
     const int m = P.grid.m, MW = m * P.grid.W;
     uint32_t* sAM = smem_bk;
@@ -129,7 +204,6 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     float4* sDirs = reinterpret_cast<float4*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_dirs_offset(m, P.grid.W));
     int* sRowStart = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(smem_bk) + fused_rows_offset(m, P.grid.W));
     int nclear = -1;
-    unsigned long long n;
     const unsigned int* prev = nullptr;  // AM_OPT_REUSE: the previous map's witnesses of this slot
     unsigned int* hs = nullptr;
     if (STAGE == BK_L0) {
@@ -143,14 +217,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
         for (int w = threadIdx.x; w < ((m + 31) >> 5); w += blockDim.x) sRowFull[w] = 0u;
         __syncthreads();
     } else {
-        // (two statements: a conditional between a parameter and a volatile load
-        // can be lowered to ONE load through a selected pointer, which is not
-        // valid for a parameter address)
-        if (STAGE == BK_L1)
-            n = F.n1;
-        else
-            n = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
-        if ((unsigned long long)blockIdx.x * blockDim.x >= n || map_full(P.early)) return;  // CTA-uniform
+        // (n: level 1's size, or the live count read by the prologue)
         fused_seed(P, sAM, sRowFull);
         if (STAGE == BK_LIVE) nclear = clear_list_rows_cta(sAM, P.grid, P.tab, sDirs, sRowStart);
     }
@@ -200,14 +267,26 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     __shared__ unsigned int sCnt[CT_COUNT];
     const int p = blockIdx.y;
     if (threadIdx.x < CT_COUNT) sCnt[threadIdx.x] = 0u;
-    pivot_params(sP, F, p, STAGE == BK_L0);
+    unsigned long long ntask;
+    {
+        // (compile-time choices: a run-time select between two kernel-parameter addresses is not valid)
+        const unsigned long long* tc;
+        unsigned long long cap;
+        if constexpr (STAGE == BK_L0) {
+            tc = shift_bytes(F.lvl.task_count, p * F.ctr_stride);
+            cap = F.lvl.task_cap;
+        } else if constexpr (STAGE == BK_L1) {
+            tc = shift_bytes(F.task1, p * F.ctr_stride);
+            cap = F.main.task_cap / 2;
+        } else {
+            tc = shift_bytes(F.main.task_count, p * F.ctr_stride);
+            cap = F.main.task_cap;
+        }
+        if (bk_prologue(sP, F, p, STAGE == BK_L0, tc, true, cap, (unsigned long long)blockIdx.x * blockDim.x,
+                        STAGE != BK_L0, ntask))
+            return;
+    }
     const StreamParams& P = sP;
-    const unsigned long long* tc =
-        STAGE == BK_L1 ? shift_bytes(F.task1, p * F.ctr_stride) : P.task_count;
-    const unsigned long long cap = STAGE == BK_L1 ? P.task_cap / 2 : P.task_cap;
-    const unsigned long long ntask = min(*reinterpret_cast<const volatile unsigned long long*>(tc), cap);
-    if ((unsigned long long)blockIdx.x * blockDim.x >= ntask) return;  // CTA-uniform
-    if (STAGE != BK_L0 && map_full(P.early)) return;
     uint32_t* sAM = smem_bk;
     uint32_t* sRowFull = sAM + P.grid.m * P.grid.W;
     fused_seed(P, sAM, sRowFull);
@@ -251,11 +330,11 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
     __shared__ StreamParams sP;
     __shared__ int sN;
     const int p = blockIdx.y;
-    pivot_params(sP, F, p, false);
+    unsigned long long unused;
+    if (bk_prologue(sP, F, p, false, nullptr, false, ~0ull, 0ull, true, unused)) return;
     const StreamParams& P = sP;
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
     float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
-    if (map_full(P.early)) return;
     const int total = clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
                                     const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x);
     if (total == 0 && blockIdx.x == 0 && threadIdx.x == 0) *P.early = 1ull;  // early exit (a7)
@@ -266,9 +345,9 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
 __global__ void __launch_bounds__(kThreads) bk_supers(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
-    pivot_params(sP, F, p, false);
+    unsigned long long unused;
+    if (bk_prologue(sP, F, p, false, nullptr, false, ~0ull, 0ull, true, unused)) return;
     const StreamParams& P = sP;
-    if (map_full(P.early)) return;
     const int lane = threadIdx.x & 31;
     const unsigned int nsup = (P.nbricks + 7) >> 3;
     for (unsigned int s0 = blockIdx.x * kThreads; s0 < nsup; s0 += gridDim.x * kThreads) {
@@ -289,9 +368,9 @@ __global__ void __launch_bounds__(kThreads) bk_supers(const __grid_constant__ Fu
 __global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
-    pivot_params(sP, F, p, false);
+    unsigned long long unused;
+    if (bk_prologue(sP, F, p, false, nullptr, false, ~0ull, 0ull, true, unused)) return;
     const StreamParams& P = sP;
-    if (map_full(P.early)) return;
     if (P.supers) {
         const unsigned int ne = 8u * *reinterpret_cast<const volatile unsigned int*>(P.super_count);
         for (unsigned int e0 = blockIdx.x * kThreads; e0 < ne; e0 += gridDim.x * kThreads) {
@@ -311,11 +390,12 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
     __shared__ unsigned int sStat[3];
     const int p = blockIdx.y;
     if (threadIdx.x < 3) sStat[threadIdx.x] = 0u;
-    pivot_params(sP, F, p, false);
+    unsigned long long nk64;
+    if (bk_prologue(sP, F, p, false, shift_bytes(F.main.brick_count, p * F.ctr_stride), false, ~0ull,
+                    (unsigned long long)blockIdx.x * (kVPT * kWarps), true, nk64))
+        return;
     const StreamParams& P = sP;
-    const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);
-    if (blockIdx.x * (kVPT * kWarps) >= nk) return;  // CTA-uniform
-    if (map_full(P.early)) return;
+    const unsigned int nk = (unsigned int)nk64;
     unsigned int nculled = 0, npassed = 0, streamed = 0;
     for (unsigned int k0 = blockIdx.x * (kVPT * kWarps); k0 < nk; k0 += gridDim.x * (kVPT * kWarps))
         voxel_step(P, k0, nk, sc, nculled, npassed, streamed);
@@ -343,10 +423,11 @@ __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ Fu
 __global__ void __launch_bounds__(kThreads) bk_band(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;
     const int p = blockIdx.y;
-    pivot_params(sP, F, p, false);
+    unsigned long long n;
+    if (bk_prologue(sP, F, p, false, shift_bytes(F.main.qcount, p * F.ctr_stride), true,
+                    (unsigned long long)F.main.qcap, (unsigned long long)blockIdx.x * (blockDim.x >> 5), false, n))
+        return;
     const StreamParams& P = sP;
-    const unsigned long long cntq = *reinterpret_cast<const volatile unsigned long long*>(P.qcount);
-    const unsigned long long n = cntq < (unsigned long long)P.qcap ? cntq : (unsigned long long)P.qcap;
     const unsigned long long nw = (unsigned long long)gridDim.x * (blockDim.x >> 5);  // warps of this pivot
     const unsigned long long gw = (unsigned long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (gw >= n) return;  // (warp-uniform: no pair for this warp)

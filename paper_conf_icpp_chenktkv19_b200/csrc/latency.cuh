@@ -40,7 +40,8 @@ namespace am {
 
 constexpr long long kSmallModel = 1ll << 16;  // voxels: up to this, no coarse levels / maps / bricks
 
-constexpr int kLiveBuf = 512;  // per CTA: voxels that passed a filter, waiting for their cones
+constexpr int kLiveBuf = 512;
+constexpr int kDiagCtas = 1024;  // AM_OPT_DIAG bit 2: per-CTA P6 records kept for the first CTAs  // per CTA: voxels that passed a filter, waiting for their cones
 
 struct LatShared {
     float4 liveq[kLiveBuf];          // filter survivors of this CTA (voxel) ...
@@ -313,6 +314,14 @@ __device__ void lat_phases(const FusedParams& F, Sync gsync, LatShared& S, unsig
         if (rfull) atomicAdd(&S.cnt[CT_ROWFULL], rfull);
     }
     fused_flush(P, sAM);
+    if (F.ts && threadIdx.x == 0 && gb < kDiagCtas) {  // diagnostics: this CTA's P6 end, live voxels, rows
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        F.ts[16 + 4 * gb] = t;
+        F.ts[16 + 4 * gb + 1] = S.live;
+        F.ts[16 + 4 * gb + 2] = S.cnt[CT_ROWS];
+        F.ts[16 + 4 * gb + 3] = S.passed;
+    }
     gsync();
     fused_mark(F, 6);
     // P7: band -- the exact test of the queued pairs still clear: each warp checks 32 pairs (one per

@@ -188,6 +188,204 @@ __global__ void __launch_bounds__(kThreads) filter_kernel(const __grid_constant_
     }
 }
 
+// ---------------------------------------------------------------------------
+// filter_tma_kernel: the same full-stream filter with the voxel tiles staged
+// in shared memory by the Tensor Memory Accelerator (1-D bulk copies,
+// cp.async.bulk, completing on an mbarrier; north_star: "coalesced 16-byte
+// float4 voxel loads staged via TMA").  Persistent CTAs (SMs x occupancy)
+// each own the tiles blockIdx.x + k gridDim.x; a ring of kTmaStages 16 KB
+// tiles keeps kTmaStages - 1 tiles in flight per CTA while the threads filter
+// the current one, so the HBM stream no longer waits on the filter's
+// registers (the LDG version holds its 4 loads per thread only until the
+// filter starts).  Thread 0 is the producer: it arms the tile's mbarrier with
+// the byte count and issues the copy with an L2 evict-first hint (each voxel
+// is read once per map); every thread waits on the mbarrier's phase, copies
+// its 4 voxels to registers, and after a CTA barrier thread 0 refills the
+// stage with the tile kTmaStages ahead.  Same decisions per voxel as
+// filter_kernel (same fast_filter), so the same live list up to order.
+// ---------------------------------------------------------------------------
+// Ring shapes (AM_OPT_STREAM_TMA value): voxels per thread per tile x stages.
+template <int VPT, int STAGES>
+struct TmaRing {
+    static constexpr int kTileVox = kThreads * VPT;
+    static constexpr unsigned int kBytes = kTileVox * (unsigned int)sizeof(float4);
+    static constexpr size_t kSmem = (size_t)STAGES * kBytes;
+};
+
+__device__ __forceinline__ unsigned int smem_u32(const void* p) {
+    return (unsigned int)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned int count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned int parity) {
+    unsigned int done = 0;
+    do {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+
+// One tile into stage buffer dst: arm bar with the byte count, then one 1-D bulk copy that completes on it.
+__device__ __forceinline__ void tma_tile(void* dst, const void* src, unsigned int bytes, unsigned long long* bar,
+                                         unsigned long long policy) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::
+            "r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy)
+        : "memory");
+}
+
+template <int VPT, int STAGES>
+__global__ void __launch_bounds__(kThreads) filter_tma_kernel(const __grid_constant__ StreamParams p) {
+    using R = TmaRing<VPT, STAGES>;
+    constexpr int kT = R::kTileVox;
+    extern __shared__ __align__(128) unsigned char smem_tma[];
+    __shared__ __align__(8) unsigned long long sBar[STAGES];
+    __shared__ unsigned int sCulled, sPassed;
+    if (map_full(p.early)) return;
+    float4* ring = reinterpret_cast<float4*>(smem_tma);
+    const unsigned int nfull = (unsigned int)(p.N / kT);
+    const unsigned int mine = nfull > blockIdx.x ? (nfull - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
+    unsigned long long policy = 0;
+    if (threadIdx.x == 0) {
+        sCulled = sPassed = 0u;
+        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+        for (int s = 0; s < STAGES; ++s) mbar_init(sBar + s, 1u);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (unsigned int k = 0; k < mine && k < (unsigned int)STAGES; ++k)
+            tma_tile(ring + k * kT, p.vox + (size_t)(blockIdx.x + k * gridDim.x) * kT, R::kBytes, sBar + k, policy);
+    }
+    __syncthreads();
+    unsigned int nculled = 0, npassed = 0;
+    for (unsigned int k = 0; k < mine; ++k) {
+        const int s = (int)(k % STAGES);
+        mbar_wait(sBar + s, (k / STAGES) & 1u);
+        const float4* tile = ring + s * kT;
+        float4 q[VPT];
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) q[j] = tile[j * kThreads + threadIdx.x];
+        __syncthreads();  // every thread holds its voxels: the stage may be refilled
+        if (threadIdx.x == 0 && k + STAGES < mine) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // (generic reads before async writes)
+            tma_tile(ring + s * kT, p.vox + (size_t)(blockIdx.x + (k + STAGES) * gridDim.x) * kT, R::kBytes, sBar + s,
+                     policy);
+        }
+        const unsigned int base = (blockIdx.x + k * gridDim.x) * kT + threadIdx.x;
+        int f[VPT];
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) f[j] = fast_filter(p, q[j], p.gam);
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            nculled += f[j] >> 1;
+            append_live(p, f[j] == F_LIVE, base + j * kThreads, npassed);
+        }
+    }
+    if (blockIdx.x == nfull % gridDim.x && (long long)nfull * kT < p.N) {  // ragged tail: plain loads
+        const unsigned int base = nfull * kT + threadIdx.x;
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const unsigned int idx = base + j * kThreads;
+            const int f = idx < p.N ? fast_filter(p, p.vox[idx], p.gam) : F_DROP;
+            nculled += f >> 1;
+            append_live(p, f == F_LIVE, idx, npassed);
+        }
+    }
+    if ((threadIdx.x & 31) == 0) atomicAdd(&sPassed, npassed);
+    if (nculled) atomicAdd(&sCulled, nculled);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        atomicAdd(p.stats + ST_CULLED, (unsigned long long)sCulled);
+        atomicAdd(p.stats + ST_PASSED, (unsigned long long)sPassed);
+        if (blockIdx.x == 0) atomicAdd(p.stats + ST_STREAMED, (unsigned long long)p.N);  // every voxel is read
+    }
+}
+
+// Warp-specialised variant: a 9th warp is the producer (lane 0 refills a stage as soon as the 8
+// consumer warps have released it on the stage's "empty" mbarrier), so no CTA-wide barrier per tile:
+// each consumer warp runs ahead as far as the ring allows.
+template <int VPT, int STAGES>
+__global__ void __launch_bounds__(kThreads + 32) filter_tma_ws_kernel(const __grid_constant__ StreamParams p) {
+    using R = TmaRing<VPT, STAGES>;
+    constexpr int kT = R::kTileVox;
+    extern __shared__ __align__(128) unsigned char smem_tma[];
+    __shared__ __align__(8) unsigned long long sFull[STAGES], sEmpty[STAGES];
+    __shared__ unsigned int sCulled, sPassed;
+    if (map_full(p.early)) return;
+    float4* ring = reinterpret_cast<float4*>(smem_tma);
+    const unsigned int nfull = (unsigned int)(p.N / kT);
+    const unsigned int mine = nfull > blockIdx.x ? (nfull - blockIdx.x + gridDim.x - 1) / gridDim.x : 0u;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        sCulled = sPassed = 0u;
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(sFull + s, 1u);
+            mbar_init(sEmpty + s, (unsigned int)kWarps);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    unsigned int nculled = 0, npassed = 0;
+    if (warp == kWarps) {  // producer
+        if (lane == 0) {
+            unsigned long long policy;
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+            for (unsigned int k = 0; k < mine; ++k) {
+                const int s = (int)(k % STAGES);
+                if (k >= (unsigned int)STAGES) mbar_wait(sEmpty + s, ((k / STAGES) - 1u) & 1u);
+                tma_tile(ring + s * kT, p.vox + (size_t)(blockIdx.x + k * gridDim.x) * kT, R::kBytes, sFull + s,
+                         policy);
+            }
+        }
+    } else {
+        for (unsigned int k = 0; k < mine; ++k) {
+            const int s = (int)(k % STAGES);
+            mbar_wait(sFull + s, (k / STAGES) & 1u);
+            const float4* tile = ring + s * kT;
+            float4 q[VPT];
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) q[j] = tile[j * kThreads + threadIdx.x];
+            __syncwarp();
+            if (lane == 0)
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(sEmpty + s)) : "memory");
+            const unsigned int base = (blockIdx.x + k * gridDim.x) * kT + threadIdx.x;
+            int f[VPT];
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) f[j] = fast_filter(p, q[j], p.gam);
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                nculled += f[j] >> 1;
+                append_live(p, f[j] == F_LIVE, base + j * kThreads, npassed);
+            }
+        }
+        if (blockIdx.x == nfull % gridDim.x && (long long)nfull * kT < p.N) {  // ragged tail: plain loads
+            const unsigned int base = nfull * kT + threadIdx.x;
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                const unsigned int idx = base + j * kThreads;
+                const int f = idx < p.N ? fast_filter(p, p.vox[idx], p.gam) : F_DROP;
+                nculled += f >> 1;
+                append_live(p, f == F_LIVE, idx, npassed);
+            }
+        }
+        if (lane == 0) atomicAdd(&sPassed, npassed);
+        if (nculled) atomicAdd(&sCulled, nculled);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        atomicAdd(p.stats + ST_CULLED, (unsigned long long)sCulled);
+        atomicAdd(p.stats + ST_PASSED, (unsigned long long)sPassed);
+        if (blockIdx.x == 0) atomicAdd(p.stats + ST_STREAMED, (unsigned long long)p.N);  // every voxel is read
+    }
+}
+
 // The cheap outer cone of a sphere (centre p + v, radius r) against the
 // clear-direction map: true when the sphere -- hence every voxel inside it --
 // can no longer change the AM (all its possibly blocked directions are

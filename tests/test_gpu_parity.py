@@ -505,3 +505,56 @@ def test_latency_kernel_matches_previous_single_pivot_kernel(am, name):
     assert np.array_equal(new, old)
     assert np.array_equal(ctx.compute_batch(P), new)
     ctx.close()
+
+
+@pytest.mark.parametrize("name,ctas", [("C1", 0), ("T_head", 0), ("T_head", 5), ("C2", 0), ("C2", 3)])
+def test_tma_full_stream_same_maps(am, name, ctas):
+    """AM_OPT_STREAM_TMA (stream.cuh filter_tma_kernel): the full-stream filter with its voxel tiles
+    staged by 1-D TMA bulk copies gives the maps and stream counters of the LDG filter_kernel bit for
+    bit, and the robust cells of the oracle.  A few persistent CTAs (ctas > 0) make each CTA's
+    4-stage ring wrap many times (mbarrier phase parity); N is not a multiple of the 1024-voxel
+    tile (ragged tail)."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    assert len(H) % 1024 != 0
+    P = cfg.pivots(3)
+    ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_FUSED, 0)
+    ctx.set_option(am.binding.OPT_BRICKS, 0)
+    if ctas:
+        ctx.set_option(am.binding.OPT_GRID_CTAS, ctas)
+    maps, stats = {}, {}
+    for tma in (0, 1, 2, 3):
+        ctx.set_option(am.binding.OPT_STREAM_TMA, tma)
+        out = [ctx.compute(p, stats=True) for p in P]
+        maps[tma] = np.stack([o[0] for o in out])
+        stats[tma] = [(o[1].voxels_streamed, o[1].voxels_culled, o[1].voxels_live) for o in out]
+    for tma in (1, 2, 3):
+        assert np.array_equal(maps[0], maps[tma]), tma
+        assert stats[0] == stats[tma], tma
+    for p, mp in zip(P[:1], maps[1][:1]):
+        ref = oracle.am_states(C, H, cfg.tool, p, cfg.m, cfg.n)
+        assert _compare(am.unpack(mp, cfg.m, cfg.n), ref)[0] == 0
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "C2"])
+def test_pdl_same_maps(am, name):
+    """AM_OPT_PDL: the batched phases as programmatic dependent launches (CTAs start under the previous
+    phase's tail, griddepcontrol.wait before reading its results) give the maps of plain stream order
+    bit for bit -- 64 pivots in 8 lanes, replayed graph, with and without AM reuse."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_BATCH, 64)
+    for P in (cfg.pivots(64), cfg.toolpath(64)):
+        ctx.set_option(am.binding.OPT_PDL, 0)
+        ref = ctx.compute_batch(P)
+        ctx.set_option(am.binding.OPT_PDL, 1)
+        for _ in range(3):  # (capture, then replays)
+            assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 0)
+    ctx.close()

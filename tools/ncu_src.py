@@ -10,8 +10,8 @@ import subprocess
 import sys
 
 
-def main(rep, top=30):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+def main(rep, top=30, filt=()):
+    out = subprocess.run(["ncu", "-i", rep, *filt, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     fname = "?"
@@ -41,4 +41,5 @@ def main(rep, top=30):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30)
+    # optional 3rd+ args: ncu import filters, e.g. -k regex:bk_voxels --launch-skip 0 --launch-count 1
+    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30, tuple(sys.argv[3:]))
