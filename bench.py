@@ -359,6 +359,9 @@ def _apply_options(ctx, B, args):
         ctx.set_option(B.OPT_STAGE_FUSION, args.stage_fusion)
     if args.phases is not None:
         ctx.set_option(B.OPT_PHASES, args.phases)
+    for kv in args.opt:  # --opt NAME=VALUE: any AM_OPT_* by its binding name (OPT_ prefix optional)
+        k, v = kv.split("=")
+        ctx.set_option(getattr(B, k if k.startswith("OPT_") else "OPT_" + k), int(v))
 
 
 def run_ours(args):
@@ -803,6 +806,8 @@ def main(argv=None):
                     help="pivots of a continuous toolpath in slot-segment order, AM_OPT_REUSE on (8(f) NEXT 2); "
                          "the same steps without reuse in detail.toolpath_reuse_off")
     ap.add_argument("--stage-fusion", type=int, default=-1, help="AM_OPT_STAGE_FUSION (-1 = library default)")
+    ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
+                    help="set any AM_OPT_* (binding name, e.g. CMAP_FAR=120); repeatable")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3

@@ -184,11 +184,18 @@ enum {
                                     0 = filter_kernel, 4 LDG.128 per thread (default: the filter is
                                     issue-bound, ~85 instructions per voxel, so the TMA rings measure
                                     0.56-0.61 of HBM on C3 against 0.65).  Same maps              */
-    AM_OPT_PDL = 26              /* am_compute_batch: 1 = each phase kernel of a lane is a
+    AM_OPT_PDL = 26,             /* am_compute_batch: 1 = each phase kernel of a lane is a
                                     programmatic dependent launch (griddepcontrol): its CTAs are
                                     scheduled under the previous phase's tail and copy their
                                     parameters there, then wait for the previous phase's writes
                                     (default); 0 = plain stream order.  Same maps                 */
+    AM_OPT_CMAP_FAR = 27         /* final clear-direction map, 8x8 texel blocks: a block whose
+                                    centre is farther than this many degrees from every clear cell
+                                    skips the per-texel nearest-clear search and stores for each
+                                    texel the lower bound theta_C - angle(texel, centre) (triangle
+                                    inequality; exact-safe, only less tight).  0 = never; default
+                                    100 (below ~80 the looser map lets many more voxels through)
+                                    Same maps                                                     */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

@@ -31,6 +31,7 @@ OPT_REUSE = 23
 OPT_STAGE_FUSION = 24
 OPT_STREAM_TMA = 25
 OPT_PDL = 26
+OPT_CMAP_FAR = 27
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

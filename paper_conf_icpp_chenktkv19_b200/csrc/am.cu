@@ -67,6 +67,9 @@ constexpr int kMaxLanes = 8;
 #ifndef AM_CMAP_ROWSCAN
 #define AM_CMAP_ROWSCAN 1024
 #endif
+#ifndef AM_CMAP_FAR
+#define AM_CMAP_FAR 100  // degrees (AM_OPT_CMAP_FAR; swept on B200: profiles/r5_sweep_cmap_far.txt)
+#endif
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 32
 #endif
@@ -1371,6 +1374,7 @@ int am_create(const am_cylinder* tool, int n_cyl, int m, int n, int device, am_c
     G.rowscan = AM_CMAP_ROWSCAN;
     G.brute = AM_CMAP_BRUTE;
     G.cblock = AM_CMAP_BLOCK;
+    G.far_cos = AM_CMAP_FAR > 0 ? (float)std::cos(AM_CMAP_FAR * M_PI / 180.0) : -2.f;
     ctx->MW = m * G.W;
     int rc;
     cudaDeviceProp prop;
@@ -1832,6 +1836,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_CMAP_BLOCK:
         if (value != 4 && value != 8) return fail(ctx, AM_EINVAL, "cmap_block must be 4 or 8");
         ctx->grid.cblock = (int)value;
+        return AM_OK;
+    case AM_OPT_CMAP_FAR:
+        if (value < 0 || value > 180) return fail(ctx, AM_EINVAL, "cmap_far must be in [0, 180] degrees");
+        ctx->grid.far_cos = value > 0 ? (float)std::cos((double)value * M_PI / 180.0) : -2.f;
         return AM_OK;
     case AM_OPT_MAP_CTAS:
         if (value < 0 || value > 4096) return fail(ctx, AM_EINVAL, "map_ctas must be in [0, 4096]");

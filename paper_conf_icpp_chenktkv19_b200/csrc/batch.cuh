@@ -336,7 +336,7 @@ __global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ Fused
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
     float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
     const int total = clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
-                                    const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x);
+                                    const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x, false, !FIRST);
     if (total == 0 && blockIdx.x == 0 && threadIdx.x == 0) *P.early = 1ull;  // early exit (a7)
 }
 

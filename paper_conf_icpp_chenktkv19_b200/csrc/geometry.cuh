@@ -62,6 +62,8 @@ struct GridDev {
     int rowscan;            // clear map: above this many clear cells, the row-ordered search (AM_OPT_CMAP_ROWSCAN)
     int brute;              // clear map: up to this many, every texel tries every clear cell (AM_OPT_CMAP_BRUTE)
     int cblock;             // clear map: texel block side of the candidate-bounded path (AM_OPT_CMAP_BLOCK)
+    float far_cos;          // clear map: blocks whose centre is farther than this (cosine) from every clear
+                            // cell store the block-level bound (AM_OPT_CMAP_FAR; -2 = never)
 };
 
 // Guards: the inner cone is shrunk and the outer cone

@@ -415,7 +415,7 @@ __device__ int clear_list_rows_cta(const uint32_t* sAM, const GridDev& g, const 
 // (found by one ballot pass over the list) are tried per texel.  c and
 // cos / sin(2 rho + slack) come from the host-made block table after the texels.
 __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float4* __restrict__ V,
-                                 const float4* sDirs, int total, int w0, int wstride) {
+                                 const float4* sDirs, int total, int w0, int wstride, float far_cos = -2.f) {
     constexpr int B = 8, TPL = B * B / 32, ROWS = 32 / B;
     const int lane = threadIdx.x & 31;
     const int Tc = T / B, nct = 6 * Tc * Tc;
@@ -436,6 +436,21 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
         for (int e = lane; e < total; e += 32) bc = fmaxf(bc, dot3(c, sDirs[e]));
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) bc = fmaxf(bc, __shfl_xor_sync(0xffffffffu, bc, o));
+        if (bc < far_cos) {  // (warp-uniform) a far block: no per-texel search
+            // every clear cell is at least theta_C from c, so at least theta_C - a_t from texel centre t
+            // (a_t = angle(t, c) <= rho < theta_C; triangle inequality): store that lower bound,
+            // cos(theta_C - a_t) = cos theta_C cos a_t + sin theta_C sin a_t, with theta_C and a_t rounded
+            // down / up by 1e-6 in the cosine and the result rounded up
+            const float bg = fminf(bc + 1e-6f, 1.f);
+            const float sb = sqrtf(fmaxf((1.f - bg) * (1.f + bg), 0.f));
+#pragma unroll
+            for (int k = 0; k < TPL; ++k) {
+                const float ca = fmaxf(dot3(f[k], c) - 1e-6f, -1.f);
+                const float sa = sqrtf(fmaxf((1.f - ca) * (1.f + ca), 0.f));
+                V[t0 + k * ROWS * T] = clear_map_value(fminf(fmaf(bg, ca, sb * sa) + 1e-6f, 1.f), f[k].w);
+            }
+            continue;
+        }
         // thr = cos(theta_C' + 2 rho') - 1e-6 with cos theta_C' = b (rounded down): the sum
         // formula, sin theta_C' = sqrt((1 - b)(1 + b)); -2 (every candidate) past pi
         const float b = fmaxf(bc - 1e-6f, -1.f);
@@ -467,7 +482,8 @@ __device__ void clear_map_blocks(const float4* __restrict__ texels, int T, float
 // (kMapDirs), sN.
 __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float* __restrict__ tab,
                               const float4* __restrict__ texels, int T, float4* __restrict__ V, uint32_t* sAM,
-                              float4* sDirs, int* sN, unsigned int gb, unsigned int gn, bool warp_texel = false) {
+                              float4* sDirs, int* sN, unsigned int gb, unsigned int gn, bool warp_texel = false,
+                              bool final_map = false) {
     const int MW = g.m * g.W;
     const int ntex = 6 * T * T;
     __syncthreads();
@@ -527,7 +543,9 @@ __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float*
     }
     if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
-        clear_map_blocks(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps);
+        // (the far-block bound only for the final map: its blocks are small, rho ~ 4 deg at T = 96, where
+        //  the map after level 0, T1 = 32, would give up to 2 rho ~ 30 deg per texel)
+        clear_map_blocks(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps, final_map ? g.far_cos : -2.f);
         return total;
     }
     if (total > g.brute && total <= kMapDirs && (T & 3) == 0) {

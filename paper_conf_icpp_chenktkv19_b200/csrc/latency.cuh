@@ -225,7 +225,7 @@ __device__ void lat_phases(const FusedParams& F, Sync gsync, LatShared& S, unsig
             fused_mark(F, 3);
             // P4: the map again, at full resolution
             full = clear_map_cta(P.gam, P.grid, P.tab, F.texels, P.cmapT, const_cast<float4*>(P.cmap), sAM, sDirs,
-                                 &S.n, gb, gn) == 0;
+                                 &S.n, gb, gn, false, true) == 0;
             gsync();
             fused_mark(F, 4);
         }

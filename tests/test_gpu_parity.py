@@ -558,3 +558,24 @@ def test_pdl_same_maps(am, name):
         assert np.array_equal(ctx.compute_batch(P), ref)
         ctx.set_option(am.binding.OPT_REUSE, 0)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "T_imp", "C2"])
+def test_cmap_far_same_maps(am, name):
+    """AM_OPT_CMAP_FAR: far texel blocks of the final clear-direction map store the block-level bound
+    theta_C - angle(texel, centre) instead of their own nearest-clear angle.  The bound is valid (only
+    looser), so the maps are those without it, batched and single-pivot, down to 1 degree."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    P = cfg.pivots(8)
+    ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_CMAP_FAR, 0)
+    ref = ctx.compute_batch(P)
+    assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+    for far in (100, 60, 1):
+        ctx.set_option(am.binding.OPT_CMAP_FAR, far)
+        assert np.array_equal(ctx.compute_batch(P), ref), far
+        assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref), far
+    with pytest.raises(am.AMError):
+        ctx.set_option(am.binding.OPT_CMAP_FAR, 181)
+    ctx.close()
