@@ -102,7 +102,8 @@ enum {
                                     = per-phase times of the single-pivot kernel on stderr; bit 3
                                     = batches as one cooperative launch of CTA groups; bit 4 =
                                     am_compute with the previous single-pivot kernel (one grid
-                                    barrier per phase) instead of am_latency_kernel; 0..31       */
+                                    barrier per phase) instead of am_latency_kernel; bit 5 =
+                                    am_compute through the batched phase launches (P = 1); 0..63 */
     AM_OPT_CMAP_T = 9,           /* clear-direction map resolution: texels per cube-face side
                                     (4..256, default 96; 80 when m·n >= 128·128)                 */
     AM_OPT_BRICKS = 10,          /* 1 = skip whole 256-voxel bricks whose bounding sphere reaches

@@ -1657,7 +1657,11 @@ int am_compute(am_ctx* ctx, const float pivot[3], uint32_t* am_out, int dst_is_d
     cudaStream_t s = (cudaStream_t)cuda_stream;
     if ((rc = stream_begin(ctx, s)) != AM_OK) return rc;
     uint32_t* gam = dst_is_device ? am_out : ctx->d_am;
-    if ((rc = launch_aica(ctx, pivot, gam, s)) != AM_OK) return rc;
+    if ((ctx->diag & 32) && fused_ok(ctx)) {  // (diagnostics: one pivot through the batched phase launches)
+        if ((rc = launch_batch_layers(ctx, pivot, 1, gam, s)) != AM_OK) return rc;
+    } else if ((rc = launch_aica(ctx, pivot, gam, s)) != AM_OK) {
+        return rc;
+    }
     if (!dst_is_device)
         CK(cudaMemcpyAsync(am_out, gam, (size_t)ctx->MW * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if ((rc = stream_end(ctx, s)) != AM_OK) return rc;
@@ -1797,7 +1801,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->phases = (int)value;
         return AM_OK;
     case AM_OPT_DIAG:
-        if (value < 0 || value > 31) return fail(ctx, AM_EINVAL, "diag must be in [0, 31]");
+        if (value < 0 || value > 63) return fail(ctx, AM_EINVAL, "diag must be in [0, 63]");
         if ((value & 3) && !ctx->d_prev) {
             CK(cudaMalloc(&ctx->d_prev, (size_t)ctx->MW * sizeof(uint32_t)));
             CK(cudaMemset(ctx->d_prev, 0, (size_t)ctx->MW * sizeof(uint32_t)));
