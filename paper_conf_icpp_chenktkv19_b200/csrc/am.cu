@@ -139,6 +139,8 @@ struct am_ctx {
     int occ = 0;
     // coarse levels (largest voxels + a strided sample) and the clear-direction map
     float4* d_coarse = nullptr;
+    float4* d_l1subs = nullptr;            // bounding spheres of every 32 consecutive level-1 voxels
+    int l1_subs = 0;                       // AM_OPT_L1_SUBS: level-1 groups of 32 culled by their sphere
     unsigned int* d_live = nullptr;        // live-voxel list of the full stream (capacity N)
     ConeRec* d_recs = nullptr;             // cone records (kRecCap) and row tasks (kTaskCap)
     unsigned long long* d_tasks = nullptr;
@@ -736,6 +738,7 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.lvl.rec_cap = kRecCap / 2;
     F.lvl.task_cap = kTaskCap / 2;
     F.l1 = ctx->d_coarse + ctx->n_l0;
+    F.l1subs = ctx->l1_subs ? ctx->d_l1subs : nullptr;
     F.n0 = (unsigned int)ctx->n_l0;
     F.n1 = (unsigned int)(ctx->n_l1 - ctx->n_l0);
     F.rec1 = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2);
@@ -1583,7 +1586,8 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     // coarse levels for the clear-direction map: level 0 = the n0 largest
     // voxels, level 1 = the next ones up to n1 plus every 512th voxel
     cudaFree(ctx->d_coarse);
-    ctx->d_coarse = nullptr;
+    cudaFree(ctx->d_l1subs);
+    ctx->d_coarse = ctx->d_l1subs = nullptr;
     ctx->n_l0 = ctx->n_l1 = 0;
     if (N >= 2048) {
         const long long n0 = std::min<long long>(N, std::max<long long>(1024, N / AM_L0_DIV));
@@ -1625,9 +1629,33 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
             strided_ids_kernel<<<blocks, 256>>>(cid + n1, ns, stride);
             CUK(cudaGetLastError());
         }
+        // level 1 (after the n0 largest) in model (Morton) order, so that every 32 consecutive level-1
+        // voxels are a compact group with a useful bounding sphere (the batched level-1 cone launch
+        // skips a group whose sphere cannot reach a clear cell of the map after level 0)
+        if (n1 + ns > n0) {
+            size_t tb1 = 0;
+            const int nl1 = (int)(n1 + ns - n0);
+            CUK(cub::DeviceRadixSort::SortKeys(nullptr, tb1, cid + n0, sk, nl1, 0, 32));
+            if (tb1 > tb) {
+                cudaFree(ct);
+                ct = nullptr;
+                CUK(cudaMalloc(&ct, tb1));
+                tb = tb1;
+            }
+            CUK(cub::DeviceRadixSort::SortKeys(ct, tb, cid + n0, sk, nl1, 0, 32));
+            CUK(cudaMemcpy(cid + n0, sk, (size_t)nl1 * 4, cudaMemcpyDeviceToDevice));
+        }
         CUK(cudaMalloc(&ctx->d_coarse, (size_t)(n1 + ns) * sizeof(float4)));
         gather_kernel<<<blocks, 256>>>(ctx->d_vox, cid, n1 + ns, ctx->d_coarse);
         CUK(cudaGetLastError());
+        if (n1 + ns > n0) {
+            const long long nl1 = n1 + ns - n0;
+            const unsigned int ng = (unsigned int)((nl1 + 31) / 32);
+            CUK(cudaMalloc(&ctx->d_l1subs, (size_t)ng * sizeof(float4)));
+            brick_bounds_kernel<<<(unsigned)(((long long)ng * 32 + 255) / 256), 256>>>(ctx->d_coarse + n0, nl1,
+                                                                                       ctx->d_l1subs, ng, 32);
+            CUK(cudaGetLastError());
+        }
         CUK(cudaDeviceSynchronize());
 #undef CUK
         cfree();
@@ -1868,6 +1896,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_STAGE_FUSION:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "stage_fusion must be 0 or 1");
         ctx->stage_fusion = (int)value;
+        return AM_OK;
+    case AM_OPT_L1_SUBS:
+        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "l1_subs must be 0 or 1");
+        ctx->l1_subs = (int)value;
         return AM_OK;
     case AM_OPT_PDL:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "pdl must be 0 or 1");
@@ -2199,6 +2231,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_ctr);
     cudaFree(ctx->d_queue);
     cudaFree(ctx->d_coarse);
+    cudaFree(ctx->d_l1subs);
     cudaFree(ctx->d_live);
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);

@@ -244,8 +244,15 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
                     nrows = cone_of_voxel<true>(P, q, id, r, counted);
                 }
             } else if (STAGE == BK_L1) {
+                // (the warp's 32 voxels are one level-1 group: skipped together when the group's sphere
+                //  cannot reach a clear cell -- b0 is a multiple of blockDim, so the warp is group-aligned)
+                bool group = true;
+                if (F.l1subs) {
+                    const float4 g = __ldg(F.l1subs + ((b0 + (threadIdx.x & ~31u)) >> 5));
+                    group = !sphere_dropped(P, g.x - P.px, g.y - P.py, g.z - P.pz, g.w, F.cmapT1, F.texels1);
+                }
                 const float4 q = F.l1[e];
-                if (fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
+                if (group && fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
                     nrows = cone_of_voxel<true>(P, q, 0x80000000u | (F.n0 + (unsigned int)e), r, counted, nullptr, -1,
                                                 F.cmapT1, nullptr, F.texels1);
             } else {

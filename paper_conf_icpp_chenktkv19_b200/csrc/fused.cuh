@@ -42,7 +42,8 @@ constexpr int kMaxSlots = 16;  // pivots per batched launch
 struct FusedParams {
     StreamParams main;        // full stream: vox, bricks, cmap (written in phase 3/6), stage-2 counters
     StreamParams lvl;         // clear-map levels: scratch stats, stage-0 counters, vox = level-0 array
-    const float4* l1;         // level-1 voxels (vox_coarse + n_l0) and their count
+    const float4* l1;         // level-1 voxels (vox_coarse + n_l0, model order) and their count
+    const float4* l1subs;     // bounding spheres of every 32 consecutive level-1 voxels (nullptr: not used)
     unsigned int n0, n1;
     unsigned int* rec1;       // stage-1 counters
     unsigned long long* task1;

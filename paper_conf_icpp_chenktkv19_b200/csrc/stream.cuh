@@ -390,7 +390,8 @@ __global__ void __launch_bounds__(kThreads + 32) filter_tma_ws_kernel(const __gr
 // clear-direction map: true when the sphere -- hence every voxel inside it --
 // can no longer change the AM (all its possibly blocked directions are
 // blocked already) or lies beyond the tool's reach.
-__device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, float vy, float vz, float r) {
+__device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, float vy, float vz, float r,
+                                               int T = 0, const float4* tex = nullptr) {
     const float D2 = fmaf(vx, vx, fmaf(vy, vy, vz * vz));
     if (D2 <= r * r * 1.0001f) return false;  // the pivot is (almost) inside: keep
     const float invD = rsqrtf(D2);
@@ -400,7 +401,7 @@ __device__ __forceinline__ bool sphere_dropped(const StreamParams& p, float vx, 
     const float s = fmaf((Reff + r) * invD, 1.f + 1.6e-5f, 1e-6f);
     const float c = fmaf(r * invD, 1.f + 1.6e-5f, 1e-6f);
     const float thr = (s < 1.f) ? fmaf(-s, s, 1.f) : -c * c;
-    return cmap_drop<AM_SPHERE_REFINE>(p.cmap, p.cmap_tex, p.cmapT, vx, vy, vz, thr);
+    return cmap_drop<AM_SPHERE_REFINE>(p.cmap, T ? tex : p.cmap_tex, T ? T : p.cmapT, vx, vy, vz, thr);
 }
 
 // Full stream with brick culling (the paper's octree

@@ -579,3 +579,24 @@ def test_cmap_far_same_maps(am, name):
     with pytest.raises(am.AMError):
         ctx.set_option(am.binding.OPT_CMAP_FAR, 181)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "T_imp", "C2"])
+def test_l1_groups_same_maps(am, name):
+    """AM_OPT_L1_SUBS: level-1 voxels in model order, groups of 32 skipped by their bounding sphere in
+    the batched level-1 launch -- the same maps as filtering every level-1 voxel, batched (random
+    pivots and a toolpath with reuse) and single-pivot."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    for P in (cfg.pivots(16), cfg.toolpath(16)):
+        ctx.set_option(am.binding.OPT_L1_SUBS, 0)
+        ref = ctx.compute_batch(P)
+        assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+        ctx.set_option(am.binding.OPT_L1_SUBS, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 0)
+    ctx.close()
