@@ -168,13 +168,14 @@ enum {
                                     gets consecutive pivots of a toolpath (e.g. call t computes
                                     pivots s L + t of 64 path segments of L pivots).  0 = off
                                     (default).  Same maps                                         */
-    AM_OPT_STAGE_FUSION = 24,    /* am_compute_batch: 1 = each stage (level 0, level 1, the kept
-                                    voxels) is ONE launch whose filter survivors, cones and rows
-                                    stay in shared memory (stage.cuh); 0 = cone and row kernels
-                                    with records and tasks in device memory (default: measured
-                                    faster with 64 maps in flight, C3 6.4 vs 10.8 us per map --
-                                    the one-launch stages pay off for ONE map, am_compute).  Same
-                                    maps                                                         */
+    AM_OPT_STAGE_FUSION = 24,    /* am_compute_batch: stages run as ONE launch each whose filter
+                                    survivors, cones and rows stay in shared memory (stage.cuh),
+                                    by bit: 1 = level 0, 2 = level 1, 4 = the kept voxels (7 =
+                                    all); a clear bit = cone and row kernels with records and
+                                    tasks in device memory (default 0: with 64 maps in flight the
+                                    split kernels measured faster, C3 6.4 vs 10.8 us per map with
+                                    all three fused -- the one-launch stages pay off for ONE map,
+                                    am_compute).  Same maps                                       */
     AM_OPT_STREAM_TMA = 25,      /* full-stream filter (AM_OPT_BRICKS = 0): north_star "voxel loads
                                     staged via TMA".  1..3 = filter_tma(_ws)_kernel: persistent CTAs
                                     whose 16 KB voxel tiles arrive in shared memory by 1-D bulk

@@ -194,7 +194,7 @@ struct am_ctx {
     int lat_grid = 0;                      // am_latency_kernel: co-resident CTAs (cooperative launch)
     // AM_OPT_REUSE (8(f) NEXT 2): per slot, two per-cell witness arrays and a dedupe set
     int reuse = 0;
-    int stage_fusion = 0;                  // AM_OPT_STAGE_FUSION: one kernel per batched stage (stage.cuh)
+    int stage_fusion = 0;                  // AM_OPT_STAGE_FUSION: stages (bit 0 level 0, 1 level 1, 2 kept voxels) as one kernel each (stage.cuh)
     int stream_tma = 0;                    // AM_OPT_STREAM_TMA: full-stream filter with TMA-staged tiles
     int pdl = 1;                           // AM_OPT_PDL: batched phases as programmatic dependent launches
     int occ_tma[8] = {};                   // filter_tma_kernel: CTAs per SM, per ring shape
@@ -1060,7 +1060,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         bk_init<<<kk, b, 0, s>>>(F);  // this chunk's maps and counters start at zero
         AM_KM(AM_K_INIT);
         const long long n0e = ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0);  // (+ reuse witnesses)
-        if (ctx->stage_fusion) {
+        if (ctx->stage_fusion & 1) {
             if ((rc = L(bk_level0, grid(n0e, kThreads, 32), ctx->smem_fused))) return rc;
             AM_KM(AM_K_LEVEL0);
         } else {
@@ -1083,7 +1083,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
-            if (ctx->stage_fusion) {
+            if (ctx->stage_fusion & 2) {
                 if ((rc = L(bk_level1, grid(ctx->n_l1 - ctx->n_l0, kThreads, ctx->bk_cone_ctas), ctx->smem_fused)))
                     return rc;
                 AM_KM(AM_K_LEVEL1);
@@ -1103,7 +1103,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         }
         if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, F.main.supers ? AM_BRICKS_CTAS : (1 << 16)), 0))) return rc;
         AM_KM(AM_K_BRICKS);
-        if (ctx->stage_fusion) {
+        if (ctx->stage_fusion & 4) {
             if ((rc = L(bk_stream, grid(1 << 30, 1, ctx->bk_voxel_ctas), ctx->smem_fused))) return rc;
             AM_KM(AM_K_STREAM);
         } else {
@@ -1894,7 +1894,7 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         ctx->reuse = (int)value;
         return AM_OK;
     case AM_OPT_STAGE_FUSION:
-        if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "stage_fusion must be 0 or 1");
+        if (value < 0 || value > 7) return fail(ctx, AM_EINVAL, "stage_fusion must be in [0, 7]");
         ctx->stage_fusion = (int)value;
         return AM_OK;
     case AM_OPT_L1_SUBS:

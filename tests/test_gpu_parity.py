@@ -480,7 +480,10 @@ def test_stage_fusion_same_maps(am, name):
     for P in (cfg.pivots(16), cfg.toolpath(16)):
         ctx.set_option(am.binding.OPT_STAGE_FUSION, 0)
         ref = ctx.compute_batch(P)
-        ctx.set_option(am.binding.OPT_STAGE_FUSION, 1)
+        for bits in (1, 2, 4):  # one stage at a time
+            ctx.set_option(am.binding.OPT_STAGE_FUSION, bits)
+            assert np.array_equal(ctx.compute_batch(P), ref), bits
+        ctx.set_option(am.binding.OPT_STAGE_FUSION, 7)
         assert np.array_equal(ctx.compute_batch(P), ref)
         ctx.set_option(am.binding.OPT_REUSE, 1)
         assert np.array_equal(ctx.compute_batch(P), ref)

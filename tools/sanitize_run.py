@@ -23,7 +23,7 @@ single = np.stack([ctx.compute(p, stats=True)[0] for p in P])
 ctx.set_option(B.OPT_BATCH, npiv)
 ctx.set_option(B.OPT_BATCH_LANES, 2)
 assert np.array_equal(ctx.compute_batch(P), single)
-ctx.set_option(B.OPT_STAGE_FUSION, 1)
+ctx.set_option(B.OPT_STAGE_FUSION, 7)
 ctx.set_option(B.OPT_REUSE, 1)
 assert np.array_equal(ctx.compute_batch(P), single)
 assert np.array_equal(ctx.compute_batch(P), single)
