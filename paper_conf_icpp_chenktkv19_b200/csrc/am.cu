@@ -68,7 +68,7 @@ constexpr int kMaxLanes = 8;
 #define AM_CMAP_ROWSCAN 1024
 #endif
 #ifndef AM_CMAP_FAR
-#define AM_CMAP_FAR 100  // degrees (AM_OPT_CMAP_FAR; swept on B200: profiles/r5_sweep_cmap_far.txt)
+#define AM_CMAP_FAR 100  // degrees (AM_OPT_CMAP_FAR; swept on B200: profiles/r5_sweeps.txt)
 #endif
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 32
