@@ -172,10 +172,11 @@ enum {
                                     survivors, cones and rows stay in shared memory (stage.cuh),
                                     by bit: 1 = level 0, 2 = level 1, 4 = the kept voxels (7 =
                                     all); a clear bit = cone and row kernels with records and
-                                    tasks in device memory (default 0: with 64 maps in flight the
-                                    split kernels measured faster, C3 6.4 vs 10.8 us per map with
-                                    all three fused -- the one-launch stages pay off for ONE map,
-                                    am_compute).  Same maps                                       */
+                                    tasks in device memory.  Default 1: level 0 fused (its few
+                                    large cones have many rows each, and the CTA raster beats the
+                                    task round trip: C3 6.33 -> 6.17 us per map); levels 1 and the
+                                    kept voxels measured slower fused (their many one-thread cones
+                                    leave a CTA-local drain idle: 7.3 / 9.7 us).  Same maps       */
     AM_OPT_STREAM_TMA = 25,      /* full-stream filter (AM_OPT_BRICKS = 0): north_star "voxel loads
                                     staged via TMA".  1..3 = filter_tma(_ws)_kernel: persistent CTAs
                                     whose 16 KB voxel tiles arrive in shared memory by 1-D bulk

@@ -194,7 +194,7 @@ struct am_ctx {
     int lat_grid = 0;                      // am_latency_kernel: co-resident CTAs (cooperative launch)
     // AM_OPT_REUSE (8(f) NEXT 2): per slot, two per-cell witness arrays and a dedupe set
     int reuse = 0;
-    int stage_fusion = 0;                  // AM_OPT_STAGE_FUSION: stages (bit 0 level 0, 1 level 1, 2 kept voxels) as one kernel each (stage.cuh)
+    int stage_fusion = 1;                  // AM_OPT_STAGE_FUSION: stages (bit 0 level 0, 1 level 1, 2 kept voxels) as one kernel each (stage.cuh)
     int stream_tma = 0;                    // AM_OPT_STREAM_TMA: full-stream filter with TMA-staged tiles
     int pdl = 1;                           // AM_OPT_PDL: batched phases as programmatic dependent launches
     int occ_tma[8] = {};                   // filter_tma_kernel: CTAs per SM, per ring shape
