@@ -576,8 +576,8 @@ int configure_launch(am_ctx* ctx) {
     CK(cudaFuncSetAttribute(bk_rows<BK_LIVE>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_map<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     CK(cudaFuncSetAttribute(bk_map<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
-    CK(cudaFuncSetAttribute(bk_level0, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
-    CK(cudaFuncSetAttribute(bk_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
+    CK(cudaFuncSetAttribute(bk_level0, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
+    CK(cudaFuncSetAttribute(bk_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, sm_rows));
     CK(cudaFuncSetAttribute(bk_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ctx->smem_fused));
     return AM_OK;
 }
@@ -1061,7 +1061,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         AM_KM(AM_K_INIT);
         const long long n0e = ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0);  // (+ reuse witnesses)
         if (ctx->stage_fusion & 1) {
-            if ((rc = L(bk_level0, grid(n0e, kThreads, 32), ctx->smem_fused))) return rc;
+            if ((rc = L(bk_level0, grid(n0e, kThreads, 32), sm_rows))) return rc;  // (AM + row-full bits only)
             AM_KM(AM_K_LEVEL0);
         } else {
             if ((rc = L(bk_cones<BK_L0>, grid(n0e, kThreads, 1 << 16), sm_rows))) return rc;
@@ -1084,7 +1084,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         AM_KM(AM_K_CLEAR_MAP);
         if (F.use_l1) {
             if (ctx->stage_fusion & 2) {
-                if ((rc = L(bk_level1, grid(ctx->n_l1 - ctx->n_l0, kThreads, ctx->bk_cone_ctas), ctx->smem_fused)))
+                if ((rc = L(bk_level1, grid(ctx->n_l1 - ctx->n_l0, kThreads, ctx->bk_cone_ctas), sm_rows)))
                     return rc;
                 AM_KM(AM_K_LEVEL1);
             } else {

@@ -30,6 +30,11 @@
 #ifndef AM_STAGE_MIN_BLOCKS
 #define AM_STAGE_MIN_BLOCKS 3
 #endif
+// the coarse levels (inner cones only, no clear list: launched with the AM + row-full bits as their
+// only dynamic shared memory) fit more CTAs per SM
+#ifndef AM_STAGE_LEVEL_MIN_BLOCKS
+#define AM_STAGE_LEVEL_MIN_BLOCKS 5
+#endif
 
 namespace am {
 
@@ -59,7 +64,7 @@ __device__ __forceinline__ void stage_init(LatShared& S) {
 }
 
 // Level 0 (+ the reuse witnesses) of pivot blockIdx.y: inner cones, rows, straight to the map.
-__global__ void __launch_bounds__(kThreads, AM_STAGE_MIN_BLOCKS) bk_level0(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, AM_STAGE_LEVEL_MIN_BLOCKS) bk_level0(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) unsigned char smem_st[];
     __shared__ StreamParams sP;
     __shared__ LatShared S;
@@ -99,7 +104,7 @@ __global__ void __launch_bounds__(kThreads, AM_STAGE_MIN_BLOCKS) bk_level0(const
 }
 
 // Level 1 of pivot blockIdx.y: filter against the map after level 0, inner cones, rows.
-__global__ void __launch_bounds__(kThreads, AM_STAGE_MIN_BLOCKS) bk_level1(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, AM_STAGE_LEVEL_MIN_BLOCKS) bk_level1(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) unsigned char smem_st[];
     __shared__ StreamParams sP;
     __shared__ LatShared S;
