@@ -199,13 +199,20 @@ enum {
                                     inequality; exact-safe, only less tight).  0 = never; default
                                     100 (below ~80 the looser map lets many more voxels through)
                                     Same maps                                                     */
-    AM_OPT_L1_SUBS = 28          /* am_compute_batch, coarse level 1: 1 = its voxels are kept in
+    AM_OPT_L1_SUBS = 28,         /* am_compute_batch, coarse level 1: 1 = its voxels are kept in
                                     model (Morton) order and every 32 consecutive ones have a
                                     bounding sphere (upload); the level-1 cone launch skips a group
                                     whose sphere cannot reach a clear cell of the map after level 0;
                                     0 = every level-1 voxel filtered (default: the map after level 0
                                     is loose, few groups drop, and the sphere test costs more than it
                                     saves -- l1_cones 0.85 -> 0.90 us per map on C3).  Same maps   */
+    AM_OPT_LIVE_CAP = 29         /* am_compute_batch: live-voxel list entries per map slot, taken
+                                    at the NEXT am_upload_voxels (0 = max(2^20, N / 8), at most N;
+                                    default).  When a map's filter finds more live voxels, its
+                                    live-cone phase streams the kept sub-bricks through the filter
+                                    again and emits every live voxel's cones -- exact, only slower.
+                                    Memory per slot ~4 B x this + ~100 MB (C3, 64 slots: 7.3 GB,
+                                    was 13 GB).  Same maps                                        */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

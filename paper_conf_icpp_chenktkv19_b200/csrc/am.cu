@@ -122,6 +122,8 @@ struct am_ctx {
     float4* d_vox = nullptr;
     long long N = 0;
     long long vox_cap = 0;
+    long long live_cap = 0;                // live list entries per map slot (d_live holds slots x live_cap)
+    long long live_cap_opt = 0;            // AM_OPT_LIVE_CAP (0 = max(2^20, N / 8), at most N)
     bool uploaded = false;
     // per-call state
     float* d_tab = nullptr;                // cos phi, sin phi, cos gamma, sin gamma
@@ -141,7 +143,8 @@ struct am_ctx {
     float4* d_coarse = nullptr;
     float4* d_l1subs = nullptr;            // bounding spheres of every 32 consecutive level-1 voxels
     int l1_subs = 0;                       // AM_OPT_L1_SUBS: level-1 groups of 32 culled by their sphere
-    unsigned int* d_live = nullptr;        // live-voxel list of the full stream (capacity N)
+    unsigned int* d_live = nullptr;        // live-voxel lists of the batched map slots (slots x live_cap)
+    unsigned int* d_live_full = nullptr;   // live-voxel list of the single-pivot paths (capacity N)
     ConeRec* d_recs = nullptr;             // cone records (kRecCap) and row tasks (kTaskCap)
     unsigned long long* d_tasks = nullptr;
     long long n_l0 = 0, n_l1 = 0;          // level 0 = [0, n_l0), level 1 = [n_l0, n_l1)
@@ -303,6 +306,7 @@ StreamParams make_params(am_ctx* c, const float pivot[3], uint32_t* gam) {
     p.refresh_tiles = c->refresh_tiles;
     p.vox_main = c->d_vox;
     p.vox_coarse = c->d_coarse;
+    p.live_cap = (unsigned int)c->vox_cap;  // (d_live_full; the batched path overrides both)
     p.cmapT = c->cmapT;
     p.cmap_tex = c->d_texels;
     p.cull_dist = c->tool.rho_max * (1.f + 1e-5f) + 1e-6f;
@@ -486,7 +490,7 @@ int ensure_slots(am_ctx* ctx, int K) {
     al((void**)&recs, (size_t)K * kRecCap * sizeof(ConeRec));
     al((void**)&tasks, (size_t)K * kTaskCap * sizeof(unsigned long long));
     al((void**)&cmap, (size_t)K * ntex * sizeof(float4));
-    if (ctx->vox_cap > 0) al((void**)&live, (size_t)K * ctx->vox_cap * sizeof(unsigned int));
+    if (ctx->live_cap > 0) al((void**)&live, (size_t)K * ctx->live_cap * sizeof(unsigned int));
     if (ctx->nbricks > 0) al((void**)&blist, (size_t)K * blist_words(ctx) * sizeof(unsigned int));
     if (e == cudaSuccess) e = cudaMemset(ctr, 0, (size_t)K * kCtrStride * sizeof(unsigned long long));
     if (e != cudaSuccess) {
@@ -495,7 +499,7 @@ int ensure_slots(am_ctx* ctx, int K) {
         return fail(ctx, e == cudaErrorMemoryAllocation ? AM_ENOMEM : AM_ECUDA,
                     "%d map slots need ~%.1f GB of device memory: %s (the context keeps its %d slots)", K,
                     (double)K * (kCtrStride * 8.0 + ctx->qcap * 8.0 + kRecCap * sizeof(ConeRec) + kTaskCap * 8.0 +
-                                 ntex * 16.0 + ctx->vox_cap * 4.0 + blist_words(ctx) * 4.0) / 1e9,
+                                 ntex * 16.0 + ctx->live_cap * 4.0 + blist_words(ctx) * 4.0) / 1e9,
                     cudaGetErrorString(e), ctx->slots);
     }
     CK(cudaDeviceSynchronize());  // no launch may still use the old buffers
@@ -618,7 +622,7 @@ int launch_stream(am_ctx* ctx, StreamParams p, const float4* vox, long long n, c
     p.cmap = cmap;
     p.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles + (coarse ? 4 : 0));
     if (coarse) p.stats = ctx->d_ctr + kCtrWords;  // keep am_stats about the full stream
-    p.live_idx = ctx->d_live;
+    p.live_idx = ctx->d_live_full;
     const long long ntiles = (n + kTile - 1) / kTile;
     long long g = ctx->grid_ctas > 0 ? ctx->grid_ctas : (long long)ctx->sms * ctx->occ;
     if (g > ntiles) g = ntiles;
@@ -727,7 +731,7 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.main.rec_cap = kRecCap;
     F.main.task_cap = kTaskCap;
     F.main.live_count = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrTiles);
-    F.main.live_idx = ctx->d_live;
+    F.main.live_idx = ctx->d_live_full;  // (single pivot; launch_batch_layers / launch_fused_batch: d_live)
     F.lvl = F.main;
     F.lvl.vox = ctx->d_coarse;
     F.lvl.N = ctx->n_l0;
@@ -905,7 +909,9 @@ int launch_fused_batch(am_ctx* ctx, const float* pivots, int64_t P, int K, uint3
     F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
     F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
     F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
-    F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
+    F.live_stride = (unsigned long long)ctx->live_cap * sizeof(unsigned int);
+    F.main.live_idx = ctx->d_live;
+    F.main.live_cap = (unsigned int)ctx->live_cap;
     F.cmap_stride = (unsigned long long)ntex * sizeof(float4);
     F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
     F.piv = ctx->d_piv;
@@ -1020,7 +1026,9 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         F.q_stride = (unsigned long long)ctx->qcap * sizeof(unsigned long long);
         F.rec_stride = (unsigned long long)kRecCap * sizeof(ConeRec);
         F.task_stride = (unsigned long long)kTaskCap * sizeof(unsigned long long);
-        F.live_stride = (unsigned long long)ctx->vox_cap * sizeof(unsigned int);
+        F.live_stride = (unsigned long long)ctx->live_cap * sizeof(unsigned int);
+        F.main.live_idx = ctx->d_live;  // (the slots' capped lists; an overflow is re-streamed: live_overflow_rescan)
+        F.main.live_cap = (unsigned int)ctx->live_cap;
         F.cmap_stride = (unsigned long long)ntex * sizeof(float4);
         F.blist_stride = blist_words(ctx) * sizeof(unsigned int);
         F.piv = ctx->d_piv + c0;
@@ -1504,13 +1512,29 @@ int am_upload_voxels(am_ctx* ctx, const float* centers_xyz, const float* half_si
     }
     if (ctx->vox_cap < N) {
         cudaFree(ctx->d_vox);
-        cudaFree(ctx->d_live);
+        cudaFree(ctx->d_live_full);
         ctx->d_vox = nullptr;
-        ctx->d_live = nullptr;
+        ctx->d_live_full = nullptr;
         ctx->vox_cap = 0;
         UK(cudaMalloc(&ctx->d_vox, (size_t)N * sizeof(float4)));
-        UK(cudaMalloc(&ctx->d_live, (size_t)ctx->slots * N * sizeof(unsigned int)));
+        UK(cudaMalloc(&ctx->d_live_full, (size_t)N * sizeof(unsigned int)));
         ctx->vox_cap = N;
+    }
+    {
+        // the live list of each batched map slot: live voxels are a small fraction of the model once the
+        // coarse levels and the clear-direction map are in (~0.04 % at C3), so it holds max(2^20, N / 8)
+        // entries (at most N; AM_OPT_LIVE_CAP), not N -- an overflow is re-streamed (live_overflow_rescan)
+        const long long want = ctx->live_cap_opt > 0
+                                   ? std::min<long long>(ctx->live_cap_opt, ctx->vox_cap)
+                                   : std::min<long long>(ctx->vox_cap, std::max<long long>(1ll << 20, ctx->vox_cap / 8));
+        if (want != ctx->live_cap || !ctx->d_live) {
+            cudaFree(ctx->d_live);
+            ctx->d_live = nullptr;
+            ctx->live_cap = 0;
+            UK(cudaMalloc(&ctx->d_live, (size_t)ctx->slots * want * sizeof(unsigned int)));
+            ctx->live_cap = want;
+            ++ctx->gen;
+        }
     }
     UK(cudaMalloc(&raw, (size_t)N * sizeof(float4)));
     UK(cudaMalloc(&bbox, 6 * sizeof(unsigned int)));
@@ -1901,6 +1925,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "l1_subs must be 0 or 1");
         ctx->l1_subs = (int)value;
         return AM_OK;
+    case AM_OPT_LIVE_CAP:
+        if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "live_cap must be in [0, 2^31-1]");
+        ctx->live_cap_opt = value;  // taken at the next am_upload_voxels
+        return AM_OK;
     case AM_OPT_PDL:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "pdl must be 0 or 1");
         ctx->pdl = (int)value;
@@ -2233,6 +2261,7 @@ void am_destroy(am_ctx* ctx) {
     cudaFree(ctx->d_coarse);
     cudaFree(ctx->d_l1subs);
     cudaFree(ctx->d_live);
+    cudaFree(ctx->d_live_full);
     cudaFree(ctx->d_recs);
     cudaFree(ctx->d_tasks);
     cudaFree(ctx->d_subs);

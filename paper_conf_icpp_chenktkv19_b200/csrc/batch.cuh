@@ -192,7 +192,8 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     unsigned long long n;
     {
         const void* cnt = STAGE == BK_LIVE ? (const void*)shift_bytes(F.main.live_count, p * F.ctr_stride) : nullptr;
-        const unsigned long long cap = STAGE == BK_L0 ? ~0ull : (STAGE == BK_L1 ? (unsigned long long)F.n1 : ~0ull);
+        const unsigned long long cap =
+            STAGE == BK_L0 ? ~0ull : (STAGE == BK_L1 ? (unsigned long long)F.n1 : (unsigned long long)F.main.live_cap);
         if (bk_prologue(sP, F, p, STAGE == BK_L0, cnt, false, cap, (unsigned long long)blockIdx.x * blockDim.x,
                         STAGE != BK_L0, n))
             return;
@@ -262,6 +263,16 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
         }
         emit_cones_cta<STAGE != BK_LIVE>(P, rc, tc, roff, toff, rcap, tcap, nrows, r, counted, &sc,
                                          STAGE == BK_LIVE ? P.stats : nullptr, sRowFull);
+    }
+    if (STAGE == BK_LIVE) {  // the slot's live list overflowed (AM_OPT_LIVE_CAP): fused.cuh live_overflow_rescan
+        __shared__ unsigned int s_count;
+        if (threadIdx.x == 0) s_count = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
+        __syncthreads();
+        const unsigned int count = s_count;
+        if (count > P.live_cap) {  // (CTA-uniform) by the CTAs that did not exit for lack of list entries
+            const unsigned int gn = (unsigned int)min((unsigned long long)gridDim.x, (n + blockDim.x - 1) / blockDim.x);
+            live_overflow_rescan(P, count, blockIdx.x, gn, sDirs, nclear, sRowStart, &sc, sRowFull);
+        }
     }
 }
 

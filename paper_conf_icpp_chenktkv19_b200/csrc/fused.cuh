@@ -326,7 +326,10 @@ __device__ __forceinline__ void voxel_step(const StreamParams& P, unsigned int k
     unsigned int pos = cta_reserve<unsigned int>(nl, P.live_count, sc.r32);
 #pragma unroll
     for (int k = 0; k < kVPT; ++k)
-        if (live[k]) P.live_idx[pos++] = idx[k];
+        if (live[k]) {
+            if (pos < P.live_cap) P.live_idx[pos] = idx[k];  // (past it: live_overflow_rescan)
+            ++pos;
+        }
 }
 
 // Rows i0 .. i0 + nrows - 1 that are not yet full, word w of the row-full bits.
@@ -438,6 +441,33 @@ __device__ __forceinline__ void emit_cones_cta(const StreamParams& p, unsigned i
             if (slot < slot_cap) p.recs[slot].i0 = -1;
             for (unsigned long long t = t0; t < t0 + ntask && t < task_cap; ++t) p.tasks[t] = kInertTask;
         }
+    }
+}
+
+// The live list of a batched map slot holds live_cap entries (AM_OPT_LIVE_CAP); when the filter found
+// more (count > cap) the ones past it were not stored.  Then the CTAs gb = 0 .. gn-1 of the live-cone
+// phase send the kept sub-bricks' voxels through the same filter again and emit the cones of every live
+// one -- the first cap of them a second time, which only repeats work (the map is an OR of per-voxel
+// rows) -- so the map is exact.  CTA-uniform call; counts the overflow once (am_stats.queue_overflow).
+__device__ void live_overflow_rescan(const StreamParams& P, unsigned int count, unsigned int gb, unsigned int gn,
+                                     const float4* sDirs, int nclear, const int* sRowStart, FusedScratch* sc,
+                                     const uint32_t* sRowFull) {
+    if (gb == 0 && threadIdx.x == 0) atomicAdd(P.stats + ST_OVERFLOW, (unsigned long long)(count - P.live_cap));
+    const unsigned int nk = *reinterpret_cast<const volatile unsigned int*>(P.brick_count);  // kept sub-bricks
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (unsigned int k0 = gb * kWarps; k0 < nk; k0 += gn * kWarps) {  // CTA-uniform; a warp per sub-brick
+        const unsigned int e = k0 + warp;
+        const unsigned int idx = e < nk ? P.brick_list[e] * 32u + lane : 0u;
+        int nrows = 0;
+        bool counted = false;
+        ConeRec r;
+        if (e < nk && idx < (unsigned long long)P.N) {
+            const float4 q = P.vox[idx];
+            if (fast_filter(P, q, P.gam) == F_LIVE)
+                nrows = cone_of_voxel<false>(P, q, idx, r, counted, sDirs, nclear, 0, sRowStart);
+        }
+        emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted, sc,
+                              P.stats, sRowFull);
     }
 }
 
@@ -574,7 +604,8 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
     {
         int* sRowStart = reinterpret_cast<int*>(smem_raw + fused_rows_offset(m, P.grid.W));
         const int nclear = clear_list_rows_cta(sAM, P.grid, P.tab, sDirs, sRowStart);
-        const unsigned long long nlive = *reinterpret_cast<const volatile unsigned int*>(P.live_count);
+        const unsigned int count = *reinterpret_cast<const volatile unsigned int*>(P.live_count);  // (uniform)
+        const unsigned long long nlive = min(count, P.live_cap);
         for (unsigned long long b0 = gb * (unsigned long long)blockDim.x; b0 < nlive; b0 += gstride) {
             const unsigned long long e = b0 + threadIdx.x;
             int nrows = 0;
@@ -587,6 +618,7 @@ __device__ __forceinline__ void map_phases(const FusedParams& F, const StreamPar
             emit_cones_cta<false>(P, P.rec_count, P.task_count, 0u, 0ull, P.rec_cap, P.task_cap, nrows, r, counted,
                                   &sc, P.stats, sRowFull);
         }
+        if (count > P.live_cap) live_overflow_rescan(P, count, gb, gn, sDirs, nclear, sRowStart, &sc, sRowFull);
     }
     gsync();
     if (!BATCH || gb == 0) fused_mark(F, 8);

@@ -63,8 +63,9 @@ struct StreamParams {
     const float4* __restrict__ cmap_tex;
     int cmapT;                     // texels per cube-face side
     float cull_dist;               // rho_max, grown by the fp32 guard (reach cull)
-    unsigned int* live_count;      // live voxels found by the filter (zeroed)
-    unsigned int* live_idx;        // their indices into vox (capacity N)
+    unsigned int* live_count;      // live voxels found by the filter (zeroed; may exceed live_cap)
+    unsigned int* live_idx;        // their indices into vox, the first live_cap of them
+    unsigned int live_cap;         // capacity of live_idx; a live voxel past it is rasterised inline (exact)
     int may_cull;                  // some voxel may lie beyond the tool's reach (per pivot)
     // cone records and (voxel, row) tasks between cone_kernel and row_kernel
     struct ConeRec* recs;

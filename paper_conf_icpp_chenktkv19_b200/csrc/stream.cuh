@@ -128,7 +128,8 @@ __device__ __forceinline__ int texel_of(float vx, float vy, float vz, int T) {
     return (face * T + iw) * T + iu;
 }
 
-// Append the live voxels among one warp-row of 32 to the global live list.
+// Append the live voxels among one warp-row of 32 to the global live list (the single-pivot paths'
+// lists hold every voxel of the stream, so live_cap is never reached there).
 __device__ __forceinline__ void append_live(const StreamParams& p, bool live, unsigned int idx,
                                             unsigned int& npassed) {
     const unsigned int mlive = __ballot_sync(0xffffffffu, live);
@@ -139,7 +140,7 @@ __device__ __forceinline__ void append_live(const StreamParams& p, bool live, un
         const int leader = __ffs(mlive) - 1;
         if (lane == leader) pos = atomicAdd(p.live_count, (unsigned int)__popc(mlive));
         pos = __shfl_sync(0xffffffffu, pos, leader) + __popc(mlive & ((1u << lane) - 1u));
-        if (live) p.live_idx[pos] = idx;
+        if (live && pos < p.live_cap) p.live_idx[pos] = idx;
     }
 }
 
@@ -673,7 +674,8 @@ template <bool COARSE>
 __global__ void __launch_bounds__(kThreads) cone_kernel(const __grid_constant__ StreamParams p) {
     if (map_full(p.early)) return;
     const int lane = threadIdx.x & 31;
-    const unsigned long long nlive = p.live_idx ? (unsigned long long)*p.live_count : (unsigned long long)p.N;
+    const unsigned long long nlive =
+        p.live_idx ? (unsigned long long)min(*p.live_count, p.live_cap) : (unsigned long long)p.N;
     const unsigned long long wstride = (unsigned long long)gridDim.x * blockDim.x;
     // warp-uniform loop: the slot reservations are warp-aggregated
     for (unsigned long long e0 = blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x & ~31u); e0 < nlive;

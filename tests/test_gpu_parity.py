@@ -603,3 +603,31 @@ def test_l1_groups_same_maps(am, name):
         assert np.array_equal(ctx.compute_batch(P), ref)
         ctx.set_option(am.binding.OPT_REUSE, 0)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "C2"])
+def test_live_list_overflow_is_exact(am, name):
+    """AM_OPT_LIVE_CAP: batched map slots whose live-voxel list is far too small for the scene (64 entries;
+    these scenes keep hundreds to thousands of live voxels per map): the live-cone phase re-streams the
+    kept sub-bricks and emits every live voxel's cones (live_overflow_rescan) -- the maps equal those with
+    the default list, for the phase launches (8 lanes, graph) and the cooperative batch (AM_OPT_DIAG bit 3),
+    and the single-pivot paths (their list holds every voxel) are unaffected."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    P = cfg.pivots(16)
+    ctx = _ctx(am, cfg, C, H)
+    ref = ctx.compute_batch(P)
+    live = [ctx.compute(p, stats=True)[1].voxels_live for p in P]
+    assert max(live) > 64
+    ctx.set_option(am.binding.OPT_LIVE_CAP, 64)
+    ctx.upload(C, H)
+    ctx.set_option(am.binding.OPT_BATCH, 16)
+    for _ in range(2):  # (capture, replay)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_DIAG, 8)
+    assert np.array_equal(ctx.compute_batch(P), ref)
+    ctx.set_option(am.binding.OPT_DIAG, 0)
+    assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P]), ref)
+    ctx.set_option(am.binding.OPT_FUSED, 0)
+    assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P[:4]]), ref[:4])
+    ctx.close()
