@@ -37,7 +37,7 @@ using namespace am;
 #define AM_ROWS_CTAS 64
 #endif
 #ifndef AM_VOXEL_CTAS
-#define AM_VOXEL_CTAS 64
+#define AM_VOXEL_CTAS 32  // CTAs per pivot of bk_voxels (swept on B200 with PDL: profiles/r5_sweeps.txt)
 #endif
 #ifndef AM_CONE_CTAS
 #define AM_CONE_CTAS 64
