@@ -35,6 +35,9 @@
 #ifndef AM_LEVEL_ROWS_MIN_BLOCKS
 #define AM_LEVEL_ROWS_MIN_BLOCKS 8
 #endif
+#ifndef AM_MAP_MIN_BLOCKS
+#define AM_MAP_MIN_BLOCKS 5  // (48 registers; 6 and 8 measured slower, profiles/r5_sweeps.txt)
+#endif
 #ifndef AM_LEVEL_CONES_MIN_BLOCKS
 #define AM_LEVEL_CONES_MIN_BLOCKS 8
 #endif
@@ -343,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
 // Clear-direction map of pivot p's map (kernels.cuh clear_map_cta); FIRST: the
 // map after level 0 when level 1 follows, at F.cmapT1 texels per face.
 template <bool FIRST>
-__global__ void __launch_bounds__(kThreads) bk_map(const __grid_constant__ FusedParams F) {
+__global__ void __launch_bounds__(kThreads, AM_MAP_MIN_BLOCKS) bk_map(const __grid_constant__ FusedParams F) {
     extern __shared__ __align__(16) unsigned char smem_bm[];
     __shared__ StreamParams sP;
     __shared__ int sN;
