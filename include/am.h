@@ -206,13 +206,20 @@ enum {
                                     0 = every level-1 voxel filtered (default: the map after level 0
                                     is loose, few groups drop, and the sphere test costs more than it
                                     saves -- l1_cones 0.85 -> 0.90 us per map on C3).  Same maps   */
-    AM_OPT_LIVE_CAP = 29         /* am_compute_batch: live-voxel list entries per map slot, taken
+    AM_OPT_LIVE_CAP = 29,        /* am_compute_batch: live-voxel list entries per map slot, taken
                                     at the NEXT am_upload_voxels (0 = max(2^20, N / 8), at most N;
                                     default).  When a map's filter finds more live voxels, its
                                     live-cone phase streams the kept sub-bricks through the filter
                                     again and emits every live voxel's cones -- exact, only slower.
                                     Memory per slot ~4 B x this + ~100 MB (C3, 64 slots: 7.3 GB,
                                     was 13 GB).  Same maps                                        */
+    AM_OPT_L1_SPARSE = 30        /* am_compute_batch: when the map after level 0 of a pivot leaves at
+                                    most this many cells clear, that pivot's level 1 takes every
+                                    2nd voxel (a nearly full map gains little from the rest; the
+                                    coarse levels only decide what is culled).  0 = off (default:
+                                    the clear count does not separate the scenes -- C5 gains 10 %
+                                    only with 2^20 (always), C3 then loses 5 %; r5_sweeps.txt).
+                                    Same maps                                                     */
 };
 
 /* Kernels of the library, for am_kernel_stats. */

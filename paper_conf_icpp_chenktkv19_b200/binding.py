@@ -34,6 +34,7 @@ OPT_PDL = 26
 OPT_CMAP_FAR = 27
 OPT_L1_SUBS = 28
 OPT_LIVE_CAP = 29
+OPT_L1_SPARSE = 30
 
 # every symbol include/am.h declares
 EXPORTS = ("am_create", "am_upload_voxels", "am_compute", "am_compute_batch", "am_compute_baseline",

@@ -143,6 +143,7 @@ struct am_ctx {
     float4* d_coarse = nullptr;
     float4* d_l1subs = nullptr;            // bounding spheres of every 32 consecutive level-1 voxels
     int l1_subs = 0;                       // AM_OPT_L1_SUBS: level-1 groups of 32 culled by their sphere
+    int l1_sparse = 0;                     // AM_OPT_L1_SPARSE: clear cells after level 0 up to which level 1 is halved
     unsigned int* d_live = nullptr;        // live-voxel lists of the batched map slots (slots x live_cap)
     unsigned int* d_live_full = nullptr;   // live-voxel list of the single-pivot paths (capacity N)
     ConeRec* d_recs = nullptr;             // cone records (kRecCap) and row tasks (kTaskCap)
@@ -240,7 +241,8 @@ constexpr int kCtrTiles = 1 + ST_COUNT;      // live count: full stream (+0), le
 constexpr int kCtrRT = kCtrTiles + 5;        // stage s: record count at +2s, task count at +2s+1
 constexpr int kCtrBricks = kCtrRT + 6;       // bricks kept by brick_test_kernel
 constexpr int kCtrSupers = kCtrBricks + 1;   // super-bricks kept (batched path)
-constexpr int kCtrWords = kCtrSupers + 1;
+constexpr int kCtrClear1 = kCtrSupers + 1;   // clear cells after level 0 (batched path, AM_OPT_L1_SPARSE)
+constexpr int kCtrWords = kCtrClear1 + 1;
 constexpr int kCtrAll = kCtrWords + ST_COUNT;  // + scratch stats of the clear-map levels
 constexpr int kCtrStride = kCtrAll;          // 64-bit words per slot
 constexpr int kMaxBatch = 64;                // pivots per layered batch launch (slots)
@@ -743,6 +745,8 @@ FusedParams fused_params(am_ctx* ctx, const float* pivot, uint32_t* gam) {
     F.lvl.task_cap = kTaskCap / 2;
     F.l1 = ctx->d_coarse + ctx->n_l0;
     F.l1subs = ctx->l1_subs ? ctx->d_l1subs : nullptr;
+    F.clear1 = ctx->l1_sparse > 0 ? ctx->d_ctr + kCtrClear1 : nullptr;
+    F.l1_sparse = ctx->l1_sparse;
     F.n0 = (unsigned int)ctx->n_l0;
     F.n1 = (unsigned int)(ctx->n_l1 - ctx->n_l0);
     F.rec1 = reinterpret_cast<unsigned int*>(ctx->d_ctr + kCtrRT + 2);
@@ -1924,6 +1928,10 @@ int am_set_option(am_ctx* ctx, int key, int64_t value) {
     case AM_OPT_L1_SUBS:
         if (value != 0 && value != 1) return fail(ctx, AM_EINVAL, "l1_subs must be 0 or 1");
         ctx->l1_subs = (int)value;
+        return AM_OK;
+    case AM_OPT_L1_SPARSE:
+        if (value < 0 || value > (1 << 20)) return fail(ctx, AM_EINVAL, "l1_sparse must be in [0, 2^20]");
+        ctx->l1_sparse = (int)value;
         return AM_OK;
     case AM_OPT_LIVE_CAP:
         if (value < 0 || value > INT32_MAX) return fail(ctx, AM_EINVAL, "live_cap must be in [0, 2^31-1]");

@@ -193,10 +193,19 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
     __shared__ FusedScratch sc;
     const int p = blockIdx.y;
     unsigned long long n;
-    {
+    unsigned int l1s = 1;  // level 1: every l1s-th voxel (AM_OPT_L1_SPARSE)
+    if constexpr (STAGE == BK_L1) {
+        // (the prologue's count: the clear cells the map after level 0 left, written by bk_map<true>)
+        const bool sparse = F.l1_sparse > 0 && F.clear1;
+        if (bk_prologue(sP, F, p, false, sparse ? (const void*)shift_bytes(F.clear1, p * F.ctr_stride) : nullptr, true,
+                        ~0ull, 0ull, true, n))
+            return;
+        l1s = (sparse && n <= (unsigned long long)F.l1_sparse) ? 2u : 1u;
+        n = (F.n1 + l1s - 1) / l1s;
+        if ((unsigned long long)blockIdx.x * blockDim.x >= n) return;  // CTA-uniform
+    } else {
         const void* cnt = STAGE == BK_LIVE ? (const void*)shift_bytes(F.main.live_count, p * F.ctr_stride) : nullptr;
-        const unsigned long long cap =
-            STAGE == BK_L0 ? ~0ull : (STAGE == BK_L1 ? (unsigned long long)F.n1 : (unsigned long long)F.main.live_cap);
+        const unsigned long long cap = STAGE == BK_L0 ? ~0ull : (unsigned long long)F.main.live_cap;
         if (bk_prologue(sP, F, p, STAGE == BK_L0, cnt, false, cap, (unsigned long long)blockIdx.x * blockDim.x,
                         STAGE != BK_L0, n))
             return;
@@ -251,13 +260,14 @@ __global__ void __launch_bounds__(kThreads, STAGE == 2 ? AM_LIVE_MIN_BLOCKS : AM
                 // (the warp's 32 voxels are one level-1 group: skipped together when the group's sphere
                 //  cannot reach a clear cell -- b0 is a multiple of blockDim, so the warp is group-aligned)
                 bool group = true;
-                if (F.l1subs) {
+                if (F.l1subs && l1s == 1) {
                     const float4 g = __ldg(F.l1subs + ((b0 + (threadIdx.x & ~31u)) >> 5));
                     group = !sphere_dropped(P, g.x - P.px, g.y - P.py, g.z - P.pz, g.w, F.cmapT1, F.texels1);
                 }
-                const float4 q = F.l1[e];
+                const unsigned long long el = e * l1s;
+                const float4 q = F.l1[el];
                 if (group && fast_filter(P, q, P.gam, F.cmapT1, F.texels1) == F_LIVE)
-                    nrows = cone_of_voxel<true>(P, q, 0x80000000u | (F.n0 + (unsigned int)e), r, counted, nullptr, -1,
+                    nrows = cone_of_voxel<true>(P, q, 0x80000000u | (F.n0 + (unsigned int)el), r, counted, nullptr, -1,
                                                 F.cmapT1, nullptr, F.texels1);
             } else {
                 const unsigned int vidx = P.live_idx[e];
@@ -359,6 +369,8 @@ __global__ void __launch_bounds__(kThreads, AM_MAP_MIN_BLOCKS) bk_map(const __gr
     const int total = clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
                                     const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x, false, !FIRST);
     if (total == 0 && blockIdx.x == 0 && threadIdx.x == 0) *P.early = 1ull;  // early exit (a7)
+    if (FIRST && F.clear1 && blockIdx.x == 0 && threadIdx.x == 0)  // (AM_OPT_L1_SPARSE: for bk_cones<L1>)
+        *shift_bytes(F.clear1, p * F.ctr_stride) = (unsigned long long)total;
 }
 
 // Super-brick test (P.supers set): super-bricks of 8 bricks whose bounding

@@ -44,6 +44,8 @@ struct FusedParams {
     StreamParams lvl;         // clear-map levels: scratch stats, stage-0 counters, vox = level-0 array
     const float4* l1;         // level-1 voxels (vox_coarse + n_l0, model order) and their count
     const float4* l1subs;     // bounding spheres of every 32 consecutive level-1 voxels (nullptr: not used)
+    unsigned long long* clear1;  // batched: clear cells after level 0 (slot 0's word; slot-shifted), or nullptr
+    int l1_sparse;            // batched: level 1 every 2nd voxel when at most this many cells are clear (0 = off)
     unsigned int n0, n1;
     unsigned int* rec1;       // stage-1 counters
     unsigned long long* task1;

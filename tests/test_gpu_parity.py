@@ -631,3 +631,24 @@ def test_live_list_overflow_is_exact(am, name):
     ctx.set_option(am.binding.OPT_FUSED, 0)
     assert np.array_equal(np.stack([ctx.compute(p)[0] for p in P[:4]]), ref[:4])
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["T_head", "T_imp", "C2"])
+def test_l1_sparse_same_maps(am, name):
+    """AM_OPT_L1_SPARSE: pivots whose map after level 0 is nearly full take every 2nd level-1 voxel (the
+    coarse levels only decide what is culled), from never to always: the same maps, with and without reuse."""
+    cfg = scenes.CONFIGS[name]
+    C, H = cfg.leaves()
+    ctx = _ctx(am, cfg, C, H)
+    ctx.set_option(am.binding.OPT_BATCH, 16)
+    for P in (cfg.pivots(16), cfg.toolpath(16)):
+        ctx.set_option(am.binding.OPT_L1_SPARSE, 0)
+        ref = ctx.compute_batch(P)
+        for th in (50, 1 << 20):
+            ctx.set_option(am.binding.OPT_L1_SPARSE, th)
+            assert np.array_equal(ctx.compute_batch(P), ref), th
+        ctx.set_option(am.binding.OPT_REUSE, 1)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        assert np.array_equal(ctx.compute_batch(P), ref)
+        ctx.set_option(am.binding.OPT_REUSE, 0)
+    ctx.close()
