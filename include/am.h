@@ -118,7 +118,7 @@ enum {
                                     CHECKICA before CHECKBOX (§4.3; 0..3,
                                     default 0 = CHECKBOX directly).  Same map outside the band  */
     AM_OPT_CMAP_T1 = 14,         /* resolution of the clear-direction map built after level 0,
-                                    which only filters level 1 (4..AM_OPT_CMAP_T, default 32).
+                                    which only filters level 1 (4..AM_OPT_CMAP_T, default 16).
                                     Same map                                                    */
     AM_OPT_CMAP_ROWSCAN = 15,    /* clear-direction map: with more clear cells than this -- and
                                     always with more than fit in shared memory (2048) -- each

@@ -71,7 +71,7 @@ constexpr int kMaxLanes = 8;
 #define AM_CMAP_FAR 100  // degrees (AM_OPT_CMAP_FAR; swept on B200: profiles/r5_sweeps.txt)
 #endif
 #ifndef AM_CMAP_T1
-#define AM_CMAP_T1 32
+#define AM_CMAP_T1 16  // (32 before; 16 equal or faster on every config, batched and single pivot: profiles/r5_sweeps.txt)
 #endif
 #ifndef AM_MAP1_WARP_BLOCKS
 #define AM_MAP1_WARP_BLOCKS 4

@@ -545,7 +545,7 @@ __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float*
     if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
         // (the far-block bound only for the final map: its blocks are small, rho ~ 4 deg at T = 96, where
-        //  the map after level 0, T1 = 32, would give up to 2 rho ~ 30 deg per texel)
+        //  the map after level 0, T1 = 16, would give up to 2 rho ~ 60 deg per texel)
         clear_map_blocks(texels, T, V, sDirs, total, gb * nwarps + warp, gn * nwarps, final_map ? g.far_cos : -2.f);
         return total;
     }
