@@ -73,6 +73,9 @@ constexpr int kMaxLanes = 8;
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 16  // (32 before; 16 equal or faster on every config, batched and single pivot: profiles/r5_sweeps.txt)
 #endif
+#ifndef AM_MAP1_WARP_TEXEL
+#define AM_MAP1_WARP_TEXEL 0
+#endif
 #ifndef AM_MAP1_WARP_BLOCKS
 #define AM_MAP1_WARP_BLOCKS 4
 #endif
@@ -1085,11 +1088,11 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             // (few texels, many clear cells after level 0: spread them over more CTAs -- one
             // warp per 4 x 4 coarse texel on the coarse-block path)
             const long long nt1 = 6ll * ctx->cmapT1 * ctx->cmapT1;
-            if ((rc = L(bk_map<true>,
-                        grid(std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32))), 1,
-                             1 << 16),
-                        ctx->smem_fused)))
-                return rc;
+            // (AM_MAP1_WARP_TEXEL: one warp per texel, <= 4 texels per warp -- clear_map_cta's warp_texel path)
+            const long long g1 = AM_MAP1_WARP_TEXEL
+                                     ? (nt1 + 4 * (kThreads / 32) - 1) / (4 * (kThreads / 32))
+                                     : std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32)));
+            if ((rc = L(bk_map<true>, grid(std::max(1ll, g1), 1, 1 << 16), ctx->smem_fused))) return rc;
         } else {
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
         }

@@ -35,6 +35,9 @@
 #ifndef AM_LEVEL_ROWS_MIN_BLOCKS
 #define AM_LEVEL_ROWS_MIN_BLOCKS 8
 #endif
+#ifndef AM_MAP1_WARP_TEXEL
+#define AM_MAP1_WARP_TEXEL 0  // the map after level 0: one warp per texel (1) or 8x8 texel blocks (0)
+#endif
 #ifndef AM_MAP_MIN_BLOCKS
 #define AM_MAP_MIN_BLOCKS 5  // (48 registers; 6 and 8 measured slower, profiles/r5_sweeps.txt)
 #endif
@@ -367,7 +370,8 @@ __global__ void __launch_bounds__(kThreads, AM_MAP_MIN_BLOCKS) bk_map(const __gr
     uint32_t* sAM = reinterpret_cast<uint32_t*>(smem_bm);
     float4* sDirs = reinterpret_cast<float4*>(smem_bm + fused_dirs_offset(P.grid.m, P.grid.W));
     const int total = clear_map_cta(P.gam, P.grid, P.tab, FIRST ? F.texels1 : F.texels, FIRST ? F.cmapT1 : P.cmapT,
-                                    const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x, false, !FIRST);
+                                    const_cast<float4*>(P.cmap), sAM, sDirs, &sN, blockIdx.x, gridDim.x,
+                                    FIRST && AM_MAP1_WARP_TEXEL, !FIRST);
     if (total == 0 && blockIdx.x == 0 && threadIdx.x == 0) *P.early = 1ull;  // early exit (a7)
     if (FIRST && F.clear1 && blockIdx.x == 0 && threadIdx.x == 0)  // (AM_OPT_L1_SPARSE: for bk_cones<L1>)
         *shift_bytes(F.clear1, p * F.ctr_stride) = (unsigned long long)total;
