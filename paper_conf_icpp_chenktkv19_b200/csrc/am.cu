@@ -1091,7 +1091,7 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             // (AM_MAP1_WARP_TEXEL: one warp per texel, <= 4 texels per warp -- clear_map_cta's warp_texel path)
             const long long g1 = AM_MAP1_WARP_TEXEL
                                      ? (nt1 + 4 * (kThreads / 32) - 1) / (4 * (kThreads / 32))
-                                     : std::max(nt1 / (4 * kThreads), nt1 / (16 * AM_MAP1_WARP_BLOCKS * (kThreads / 32)));
+                                     : std::max(nt1 / (4 * kThreads), nt1 / ((AM_MAP1_BLOCK4 ? 16 : 64) * AM_MAP1_WARP_BLOCKS / 4 * (kThreads / 32)));
             if ((rc = L(bk_map<true>, grid(std::max(1ll, g1), 1, 1 << 16), ctx->smem_fused))) return rc;
         } else {
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;

@@ -542,7 +542,10 @@ __device__ int clear_map_cta(const uint32_t* gam, const GridDev& g, const float*
         }
         return total;
     }
-    if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0) {
+#ifndef AM_MAP1_BLOCK4
+#define AM_MAP1_BLOCK4 1  // the map after level 0 (not final_map) by 4x4 texel blocks (r5_sweeps.txt)
+#endif
+    if (total > g.brute && total <= kMapDirs && g.cblock == 8 && (T & 7) == 0 && !(AM_MAP1_BLOCK4 && !final_map)) {
         compact_clear_dirs(sAM, g, tab, 0, MW, sDirs, sN);
         // (the far-block bound only for the final map: its blocks are small, rho ~ 4 deg at T = 96, where
         //  the map after level 0, T1 = 16, would give up to 2 rho ~ 60 deg per texel)
