@@ -73,6 +73,12 @@ constexpr int kMaxLanes = 8;
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 16  // (32 before; 16 equal or faster on every config, batched and single pivot: profiles/r5_sweeps.txt)
 #endif
+#ifndef AM_L0_PER_CTA
+#define AM_L0_PER_CTA 256
+#endif
+#ifndef AM_L0_CTAS
+#define AM_L0_CTAS 32
+#endif
 #ifndef AM_MAP1_WARP_TEXEL
 #define AM_MAP1_WARP_TEXEL 0
 #endif
@@ -1076,7 +1082,8 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
         AM_KM(AM_K_INIT);
         const long long n0e = ctx->n_l0 + (ctx->reuse ? ctx->grid.m * ctx->grid.n : 0);  // (+ reuse witnesses)
         if (ctx->stage_fusion & 1) {
-            if ((rc = L(bk_level0, grid(n0e, kThreads, 32), sm_rows))) return rc;  // (AM + row-full bits only)
+            // (AM + row-full bits only; AM_L0_PER_CTA level-0 voxels per CTA, their rows shared by its 256 threads)
+            if ((rc = L(bk_level0, grid(n0e, AM_L0_PER_CTA, AM_L0_CTAS), sm_rows))) return rc;
             AM_KM(AM_K_LEVEL0);
         } else {
             if ((rc = L(bk_cones<BK_L0>, grid(n0e, kThreads, 1 << 16), sm_rows))) return rc;
