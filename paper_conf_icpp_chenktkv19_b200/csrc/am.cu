@@ -73,6 +73,12 @@ constexpr int kMaxLanes = 8;
 #ifndef AM_CMAP_T1
 #define AM_CMAP_T1 16  // (32 before; 16 equal or faster on every config, batched and single pivot: profiles/r5_sweeps.txt)
 #endif
+#ifndef AM_FUSED_BRICKS
+#define AM_FUSED_BRICKS 1  // batched: bk_bricks_fused instead of bk_supers + bk_bricks (r5_sweeps.txt)
+#endif
+#ifndef AM_FUSED_BRICKS_SUPERS
+#define AM_FUSED_BRICKS_SUPERS 512  // super-bricks per CTA of bk_bricks_fused (2 per thread)
+#endif
 #ifndef AM_L0_PER_CTA
 #define AM_L0_PER_CTA 256
 #endif
@@ -1119,12 +1125,18 @@ int launch_batch_layers(am_ctx* ctx, const float* pivots, int64_t P, uint32_t* g
             if ((rc = L(bk_map<false>, grid(ntex, 4 * kThreads, map_cap), ctx->smem_fused))) return rc;
             AM_KM(AM_K_CLEAR_MAP);
         }
-        if (F.main.supers) {
-            if ((rc = L(bk_supers, grid((ctx->nbricks + 7) / 8, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
+        if (F.main.supers && AM_FUSED_BRICKS) {  // super-bricks -> bricks -> sub-bricks in one launch
+            if ((rc = L(bk_bricks_fused, grid((ctx->nbricks + 7) / 8, AM_FUSED_BRICKS_SUPERS, 1 << 16), 0))) return rc;
+            AM_KM(AM_K_BRICKS);
+        } else {
+            if (F.main.supers) {
+                if ((rc = L(bk_supers, grid((ctx->nbricks + 7) / 8, AM_BRICK_STEPS * kThreads, 1 << 16), 0))) return rc;
+                AM_KM(AM_K_BRICKS);
+            }
+            if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, F.main.supers ? AM_BRICKS_CTAS : (1 << 16)), 0)))
+                return rc;
             AM_KM(AM_K_BRICKS);
         }
-        if ((rc = L(bk_bricks, grid(ctx->nbricks, AM_BRICK_STEPS * kThreads, F.main.supers ? AM_BRICKS_CTAS : (1 << 16)), 0))) return rc;
-        AM_KM(AM_K_BRICKS);
         if (ctx->stage_fusion & 4) {
             if ((rc = L(bk_stream, grid(1 << 30, 1, ctx->bk_voxel_ctas), ctx->smem_fused))) return rc;
             AM_KM(AM_K_STREAM);

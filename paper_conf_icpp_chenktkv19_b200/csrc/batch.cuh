@@ -420,6 +420,36 @@ __global__ void __launch_bounds__(kThreads) bk_bricks(const __grid_constant__ Fu
     }
 }
 
+// AM_FUSED_BRICKS: super-bricks -> their bricks -> the kept bricks' sub-bricks in ONE launch (the
+// single-pivot kernel's P5): every warp tests 32 super-bricks dealt transposed over the pivot's warps (the
+// kept ones, a spatially clustered few, land on different warps), then the 8 bricks of each kept one,
+// 4 kept super-bricks x 8 lanes per pass (brick_test, which tests the sub-bricks of the kept bricks).
+__global__ void __launch_bounds__(kThreads) bk_bricks_fused(const __grid_constant__ FusedParams F) {
+    __shared__ StreamParams sP;
+    __shared__ unsigned int sKeptS[kWarps][32];
+    const int p = blockIdx.y;
+    unsigned long long unused;
+    if (bk_prologue(sP, F, p, false, nullptr, false, ~0ull, 0ull, true, unused)) return;
+    const StreamParams& P = sP;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const unsigned int nsup = (P.nbricks + 7) >> 3;
+    const unsigned int nw = gridDim.x * kWarps, gw = blockIdx.x * kWarps + warp;
+    for (unsigned int k0 = 0; k0 < nsup; k0 += nw * 32) {  // (uniform bound)
+        const unsigned int sp = k0 + lane * nw + gw;
+        const bool keep = sp < nsup && !node_dropped(P, P.supers, sp);
+        const unsigned int mk = __ballot_sync(0xffffffffu, keep);
+        if (keep) sKeptS[warp][__popc(mk & ((1u << lane) - 1u))] = sp;
+        __syncwarp();
+        const int n = __popc(mk);
+        for (int u = 0; u < n; u += 4) {  // 4 kept super-bricks x 8 bricks per pass
+            const int j = u + (lane >> 3);
+            const unsigned int b = j < n ? sKeptS[warp][j] * 8u + (lane & 7) : 0u;
+            brick_test(P, b, j < n);
+        }
+        __syncwarp();
+    }
+}
+
 // Kept sub-bricks' voxels through the filter; live voxels to the live list.
 __global__ void __launch_bounds__(kThreads) bk_voxels(const __grid_constant__ FusedParams F) {
     __shared__ StreamParams sP;

@@ -37,7 +37,7 @@ for w in $WHAT; do
       gzip -f $OUT/launches_$TAG.csv ;;
     full)
       for c in C3 C2 C4 C5; do
-        timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bk_ -s ${KSKIP:-24} -c ${KCOUNT:-12} \
+        timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bk_ -s ${KSKIP:-22} -c ${KCOUNT:-11} \
           -o $OUT/prof_${TAG}_$c -f python bench.py --config $c --steps 4 --warmup 3 --lanes 1 --no-cpu-baseline \
           --no-baseline --e2e-steps 1 --no-full-scan > $OUT/full_${TAG}_$c.log 2>&1
         echo "full $c rc=$?"

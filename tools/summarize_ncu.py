@@ -26,7 +26,7 @@ def base_name(k):
 
 _STAGES = {"bk_cones": ("l0_cones", "l1_cones", "live_cones"), "bk_rows": ("l0_rows", "l1_rows", "live_rows")}
 _PLAIN = {"am_latency_kernel": "fused_pipeline", "bk_init": "init", "bk_level0": "level0", "bk_level1": "level1",
-          "bk_stream": "stream", "bk_map": "clear_map", "bk_bricks": "bricks", "bk_voxels": "voxels", "bk_band": "band",
+          "bk_stream": "stream", "bk_map": "clear_map", "bk_bricks": "bricks", "bk_bricks_fused": "bricks", "bk_voxels": "voxels", "bk_band": "band",
           "am_pipeline_kernel": "fused_pipeline", "filter_kernel": "filter", "baseline_kernel": "baseline",
           "clear_map_kernel": "clear_map", "band_exact_kernel": "band", "brick_test_kernel": "bricks",
           "brick_voxels_kernel": "voxels"}
